@@ -1,0 +1,198 @@
+// dpx_peak.cu — measures the chip's min-plus relaxation rate on sm_100a.
+//
+// This is the roofline denominator for the FW phase-3 kernel:
+// one relaxation = c = min(c, a + b) (§II-A). Variants:
+//   s32     : __viaddmin_s32       -> SASS VIADDMNMX        (1 relax / instr)
+//   s16x2   : __viaddmin_s16x2     -> SASS VIADDMNMX.S16x2  (2 relax / instr)
+//   f32     : fminf(c, a + b)      -> SASS FADD + FMNMX     (1 relax / 2 instr)
+//   f32x2   : __fadd2_rn + 3-input min -> FADD2 + FMNMX3    (2 relax / 2 instr)
+// plus the host link (pinned H2D, D2H, both at once), used by the
+// out-of-core roofline. Prints one JSON object on stdout.
+#include <cuda_runtime.h>
+#include <cuda_fp16.h>
+#include <cstdio>
+#include <cstdlib>
+#include <cstdint>
+#include <vector>
+#include <algorithm>
+
+#define CK(x) do { cudaError_t e_ = (x); if (e_ != cudaSuccess) { \
+  fprintf(stderr, "%s:%d %s\n", __FILE__, __LINE__, cudaGetErrorString(e_)); exit(1); } } while (0)
+
+constexpr int CH = 16;  // independent chains per thread
+
+__global__ void k_s32(const int* __restrict__ in, int* __restrict__ out, int iters) {
+  int x[CH], acc[CH];
+#pragma unroll
+  for (int j = 0; j < CH; ++j) { x[j] = in[(threadIdx.x + j) & 255]; acc[j] = 1 << 29; }
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      int y = it * 8 + u;
+#pragma unroll
+      for (int j = 0; j < CH; ++j) acc[j] = __viaddmin_s32(x[j], y, acc[j]);
+    }
+  }
+  int s = 0;
+#pragma unroll
+  for (int j = 0; j < CH; ++j) s ^= acc[j];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+
+__global__ void k_s16x2(const int* __restrict__ in, int* __restrict__ out, int iters) {
+  unsigned x[CH], acc[CH];
+#pragma unroll
+  for (int j = 0; j < CH; ++j) { x[j] = (unsigned)in[(threadIdx.x + j) & 255]; acc[j] = 0x3fff3fffu; }
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      unsigned y = (unsigned)(it * 8 + u) * 0x00010001u;
+#pragma unroll
+      for (int j = 0; j < CH; ++j) acc[j] = __viaddmin_s16x2(x[j], y, acc[j]);
+    }
+  }
+  unsigned s = 0;
+#pragma unroll
+  for (int j = 0; j < CH; ++j) s ^= acc[j];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = (int)s;
+}
+
+__global__ void k_f32(const int* __restrict__ in, int* __restrict__ out, int iters) {
+  float x[CH], acc[CH];
+#pragma unroll
+  for (int j = 0; j < CH; ++j) { x[j] = (float)in[(threadIdx.x + j) & 255]; acc[j] = 1e30f; }
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      float y = (float)(it * 8 + u);
+#pragma unroll
+      for (int j = 0; j < CH; ++j) acc[j] = fminf(acc[j], x[j] + y);
+    }
+  }
+  float s = 0;
+#pragma unroll
+  for (int j = 0; j < CH; ++j) s += acc[j];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = (int)s;
+}
+
+// two relaxations per (FADD2, FMNMX3) pair: acc = min(acc, x.x + y.x, x.y + y.y)
+__global__ void k_f32x2(const int* __restrict__ in, int* __restrict__ out, int iters) {
+  float2 x[CH];
+  float acc[CH];
+#pragma unroll
+  for (int j = 0; j < CH; ++j) {
+    x[j] = make_float2((float)in[(threadIdx.x + j) & 255], (float)in[(threadIdx.x + j + 1) & 255]);
+    acc[j] = 1e30f;
+  }
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      float2 y = make_float2((float)(it * 8 + u), (float)(it * 8 + u + 1));
+#pragma unroll
+      for (int j = 0; j < CH; ++j) {
+        float2 s = __fadd2_rn(x[j], y);
+        acc[j] = fminf(fminf(acc[j], s.x), s.y);
+      }
+    }
+  }
+  float s = 0;
+#pragma unroll
+  for (int j = 0; j < CH; ++j) s += acc[j];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = (int)s;
+}
+
+typedef void (*kfn)(const int*, int*, int);
+
+static double run(kfn f, int blocks, int threads, int iters, const int* in, int* out, double relax_per_op) {
+  for (int w = 0; w < 2; ++w) f<<<blocks, threads>>>(in, out, iters);
+  CK(cudaDeviceSynchronize());
+  cudaEvent_t a, b;
+  CK(cudaEventCreate(&a)); CK(cudaEventCreate(&b));
+  float best = 1e30f;
+  for (int r = 0; r < 5; ++r) {
+    CK(cudaEventRecord(a));
+    f<<<blocks, threads>>>(in, out, iters);
+    CK(cudaEventRecord(b));
+    CK(cudaEventSynchronize(b));
+    float ms; CK(cudaEventElapsedTime(&ms, a, b));
+    best = std::min(best, ms);
+  }
+  double ops = (double)blocks * threads * iters * 8.0 * CH * relax_per_op;
+  return ops / (best * 1e-3);
+}
+
+static double link_bw(void* dst, const void* src, size_t bytes, cudaMemcpyKind kind, cudaStream_t s) {
+  cudaEvent_t a, b;
+  CK(cudaEventCreate(&a)); CK(cudaEventCreate(&b));
+  CK(cudaMemcpyAsync(dst, src, bytes, kind, s));
+  CK(cudaStreamSynchronize(s));
+  float best = 1e30f;
+  for (int r = 0; r < 3; ++r) {
+    CK(cudaEventRecord(a, s));
+    CK(cudaMemcpyAsync(dst, src, bytes, kind, s));
+    CK(cudaEventRecord(b, s));
+    CK(cudaEventSynchronize(b));
+    float ms; CK(cudaEventElapsedTime(&ms, a, b));
+    best = std::min(best, ms);
+  }
+  return bytes / (best * 1e-3) / 1e9;
+}
+
+int main(int argc, char** argv) {
+  int dev = 0;
+  CK(cudaSetDevice(dev));
+  cudaDeviceProp p; CK(cudaGetDeviceProperties(&p, dev));
+  int *in, *out;
+  CK(cudaMalloc(&in, 256 * sizeof(int)));
+  std::vector<int> h(256);
+  for (int i = 0; i < 256; ++i) h[i] = (i * 37) % 101;
+  CK(cudaMemcpy(in, h.data(), 256 * sizeof(int), cudaMemcpyHostToDevice));
+  const int iters = 4096;
+  printf("{\"gpu\": \"%s\", \"sms\": %d, \"cc\": \"%d.%d\"", p.name, p.multiProcessorCount, p.major, p.minor);
+  int cfgs[][2] = {{4, 256}, {8, 256}, {16, 128}, {4, 512}};
+  struct V { const char* name; kfn f; double rpo; } vs[] = {
+    {"s32", k_s32, 1.0}, {"s16x2", k_s16x2, 2.0}, {"f32", k_f32, 1.0}, {"f32x2", k_f32x2, 2.0}};
+  CK(cudaMalloc(&out, (size_t)p.multiProcessorCount * 16 * 512 * sizeof(int)));
+  for (auto& v : vs) {
+    double best = 0;
+    printf(", \"%s\": {", v.name);
+    for (int c = 0; c < 4; ++c) {
+      int blocks = p.multiProcessorCount * cfgs[c][0];
+      double r = run(v.f, blocks, cfgs[c][1], iters, in, out, v.rpo);
+      printf("%s\"%dx%d\": %.4e", c ? ", " : "", cfgs[c][0], cfgs[c][1], r);
+      best = std::max(best, r);
+    }
+    printf(", \"best_relax_per_s\": %.4e}", best);
+  }
+  // host link (pinned), 1 GiB
+  size_t bytes = (size_t)1 << 30;
+  void *hp, *hp2, *dp, *dp2;
+  CK(cudaHostAlloc(&hp, bytes, cudaHostAllocDefault));
+  CK(cudaHostAlloc(&hp2, bytes, cudaHostAllocDefault));
+  memset(hp, 1, bytes); memset(hp2, 2, bytes);
+  CK(cudaMalloc(&dp, bytes)); CK(cudaMalloc(&dp2, bytes));
+  cudaStream_t s1, s2; CK(cudaStreamCreate(&s1)); CK(cudaStreamCreate(&s2));
+  double h2d = link_bw(dp, hp, bytes, cudaMemcpyHostToDevice, s1);
+  double d2h = link_bw(hp2, dp2, bytes, cudaMemcpyDeviceToHost, s1);
+  // duplex
+  cudaEvent_t a, b, c2;
+  CK(cudaEventCreate(&a)); CK(cudaEventCreate(&b)); CK(cudaEventCreate(&c2));
+  float best = 1e30f;
+  for (int r = 0; r < 3; ++r) {
+    CK(cudaDeviceSynchronize());
+    CK(cudaEventRecord(a, s1));
+    CK(cudaStreamWaitEvent(s2, a));
+    CK(cudaMemcpyAsync(dp, hp, bytes, cudaMemcpyHostToDevice, s1));
+    CK(cudaMemcpyAsync(hp2, dp2, bytes, cudaMemcpyDeviceToHost, s2));
+    CK(cudaEventRecord(c2, s2));
+    CK(cudaStreamWaitEvent(s1, c2));
+    CK(cudaEventRecord(b, s1));
+    CK(cudaEventSynchronize(b));
+    float ms; CK(cudaEventElapsedTime(&ms, a, b));
+    best = std::min(best, ms);
+  }
+  printf(", \"link_gbs\": {\"h2d\": %.2f, \"d2h\": %.2f, \"duplex_each_dir\": %.2f}", h2d, d2h,
+         bytes / (best * 1e-3) / 1e9);
+  printf("}\n");
+  return 0;
+}
