@@ -1,0 +1,367 @@
+#!/usr/bin/env python
+"""Benchmark: blocked Floyd–Warshall APSP on B200 through the C ABI.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--workload NAME]
+
+Metric (BASELINE.json): APSP relaxations/s = n^3 / time (whole job, all ranks).
+One step = one pass of the whole hot path over the workload's graph with the
+CSR already resident in HBM: CSR->dense init (apsp_reinit) + all n/b rounds of
+phases 1-3 (apsp_fw_blocked; with N>1 ranks also the NCCL pivot-band broadcast).
+
+Default workload: N=1 -> cfg2_grid16384 (BASELINE.json configs[1]);
+N>1 -> cfg3_er65536 (configs[2], sharded 1-D block-row over N GPUs, strong scaling).
+Inputs are larger than L2 (n^2*4 B >= 1 GiB > 126 MB), so no explicit flush.
+
+`--impl reference` times the CPU oracle (oracle/, plain C + OpenMP) on a bounded
+sample of the same workload (the reference arm of this paper-only tier).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "APSP relaxations/s (n^3/time) at 1/2/4/8 B200; % of DPX min-plus peak"
+UNIT = "relax/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default=None)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle sample time")
+    return ap.parse_args()
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", str(rank)))
+    return world, rank, local
+
+
+def default_workload(n_gpus):
+    return "cfg2_grid16384" if n_gpus == 1 else "cfg3_er65536"
+
+
+def peaks():
+    """Roofline denominators: measured DPX min-plus rate (MEASURED_DPX.json, committed, from
+    build/dpx_peak) and the driver's MEASURED_PEAKS.json."""
+    out = {}
+    p = os.path.join(ROOT, "MEASURED_DPX.json")
+    if os.path.exists(p):
+        out["dpx"] = json.load(open(p))
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        out["driver"] = json.load(open(p))
+    return out
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device):
+        self.device = device
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.device), "--query-gpu=" + self.Q,
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        self.proc.terminate()
+        try:
+            out = self.proc.communicate(timeout=5)[0]
+        except Exception:
+            self.proc.kill()
+            out = ""
+        sms, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sms.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        if not sms:
+            return None
+        return {"sm_mhz": float(np.median(sms)), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sms)}
+
+
+def cpu_oracle_sample(g, target_s):
+    """Time the CPU oracle's plain FW (oracle.fw_dense_i64 / _f64) on this workload for a bounded
+    number of outer iterations k; each iteration does exactly n^2 relaxation checks,
+    so relax/s = k * n^2 / t. Returns (relax_per_s, cores, sample description)."""
+    import oracle
+    n = g.n
+    is_f = g.w.dtype.kind == "f"
+    t0 = time.time()
+    d = oracle.init_f64(g.row_ptr, g.col, g.w) if is_f else oracle.init_i64(g.row_ptr, g.col, g.w)
+    t_init = time.time() - t0
+    fw = oracle.fw_dense_f64 if is_f else oracle.fw_dense_i64
+    # calibrate on 2 iterations, then time a sample sized to ~target_s
+    t0 = time.time()
+    fw(d, 2)
+    per = max((time.time() - t0) / 2, 1e-6)
+    k = int(max(2, min(n, target_s / per)))
+    d2 = d.copy()
+    t0 = time.time()
+    fw(d2, k)
+    t = time.time() - t0
+    rate = k * float(n) ** 2 / t
+    return rate, oracle.threads(), "oracle plain FW (%s): first %d of %d outer iterations, n=%d (%.1f s; init %.1f s " \
+        "not counted); rate extrapolates since every iteration does n^2 checks" % (
+            "fp64" if is_f else "int64", k, n, n, t, t_init)
+
+
+def run_reference(args):
+    world, rank, _ = dist_env()
+    if rank != 0:
+        return 0
+    import graphgen as gg
+    wl = args.workload or default_workload(args.gpus)
+    g = gg.baseline_config(wl)
+    import oracle
+    oracle.build()
+    rates = []
+    per_step = max(2.0, min(args.cpu_seconds, 120.0 / max(1, args.steps + args.warmup)))
+    for i in range(args.warmup):
+        cpu_oracle_sample(g, per_step / 4)
+    sample = ""
+    cores = 0
+    t0 = time.time()
+    for i in range(args.steps):
+        r, cores, sample = cpu_oracle_sample(g, per_step)
+        rates.append(r)
+    wall = time.time() - t0
+    value = float(np.mean(rates))
+    n = g.n
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": float(n) ** 3 / value * 1e3, "higher_is_better": True,
+        "scaling": "strong" if args.gpus > 1 else "weak", "vs_baseline": None,
+        "dtype": "f64" if g.w.dtype.kind == "f" else "int64", "data": "synthetic",
+        "config": {"workload": wl, "n": n, "m": g.m, "desc": gg.BASELINE_CONFIGS[wl]},
+        "impl": "reference",
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        "wall_s": wall,
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    import graphgen as gg
+    import paper_conf_ipps_xia0ar22_b200 as apsp
+
+    world, rank, local = dist_env()
+    if world != args.gpus:
+        raise SystemExit("--gpus %d but WORLD_SIZE=%d" % (args.gpus, world))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    wl = args.workload or default_workload(args.gpus)
+    g = gg.baseline_config(wl)
+    n = g.n
+    is_f = g.w.dtype.kind == "f"
+    stream = torch.cuda.current_stream()
+
+    uid = None
+    if world > 1:
+        obj = [apsp.apsp_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+
+    def make_cfg(timing):
+        cfg = apsp.apsp_config_default(device=local, world_size=world, rank=rank, timing=timing)
+        cfg.stream = stream.cuda_stream
+        if uid is not None:
+            cfg._uid_buf = __import__("ctypes").create_string_buffer(uid, 128)
+            cfg.nccl_unique_id = __import__("ctypes").cast(cfg._uid_buf, __import__("ctypes").c_void_p)
+        return cfg
+
+    def barrier():
+        if world > 1:
+            dist.barrier(device_ids=[local])
+
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    # ---------------- device-resident timing (value) ------------------------
+    h = apsp.apsp_init_from_csr(n, g.row_ptr, g.col, g.w, cfg=make_cfg(1))
+    info = apsp.apsp_get_info(h)
+    for _ in range(args.warmup):
+        apsp.apsp_reinit(h)
+        apsp.apsp_fw_blocked(h)
+    torch.cuda.synchronize()
+    # phase stats of the timed steps only
+    st_acc = np.zeros((3, 4))
+    clk = ClockSampler(local)
+    barrier()
+    torch.cuda.synchronize()
+    clk.start()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(args.steps):
+        apsp.apsp_reinit(h)
+        apsp.apsp_fw_blocked(h)
+        s = apsp.apsp_get_phase_stats(h)
+        st_acc[0] += np.array(s.ms[:])
+        st_acc[1] += np.array(s.launches[:])
+        st_acc[2] += np.array(s.relax[:])
+    e1.record(stream)
+    torch.cuda.synchronize()
+    barrier()
+    clocks = clk.stop()
+    ms = max_over_ranks(e0.elapsed_time(e1))
+    ms_step = ms / args.steps
+    value = float(n) ** 3 / (ms_step * 1e-3)
+    launches_per_step = int(round((st_acc[1][:3].sum()) / args.steps)) + 1  # + init kernel
+    # sanity: relaxations performed per step must be n_pad^3 (whole job)
+    relax_local = st_acc[2][:3].sum() / args.steps
+
+    # ---------------- roofline of the dominant kernel (phase 3) --------------
+    pk = peaks()
+    p3_ms = st_acc[0][2] / max(1, st_acc[1][2])
+    p3_relax = st_acc[2][2] / max(1, st_acc[1][2])
+    achieved = p3_relax / (p3_ms * 1e-3)
+    dpx = pk.get("dpx", {})
+    if is_f:
+        peak = dpx.get("f32_relax_per_s")
+        peak_src = "measured fp32 FADD+FMNMX min-plus rate (MEASURED_DPX.json)"
+    else:
+        peak = dpx.get("s32_relax_per_s")
+        peak_src = "measured VIADDMNMX s32 rate (MEASURED_DPX.json)"
+    if not peak:
+        peak = 148 * 64 * 1.965e9
+        peak_src = "derived: 148 SMs x 64 lanes/clk x 1.965 GHz (no MEASURED_DPX.json)"
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "phase3_traffic.json")
+    if os.path.exists(tp):
+        try:
+            tj = json.load(open(tp))
+            if tj.get("workload") == wl:
+                traffic = tj.get("dram_bytes_per_launch")
+        except Exception:
+            pass
+    roofline = {"bound": "alu", "kernel": "minplus_kernel (phase 3)", "achieved": achieved / 1e12,
+                "peak": peak / 1e12, "unit": "Trelax/s", "frac": achieved / peak, "traffic": traffic,
+                "peak_source": peak_src, "avg_launch_ms": p3_ms, "relax_per_launch": p3_relax,
+                "share_of_step": (st_acc[0][2] / args.steps) / ms_step,
+                "hbm_gbs_algorithmic": None}
+    apsp.apsp_destroy(h)
+
+    # ---------------- end-to-end through the C ABI with host buffers ----------
+    e2e = None
+    if not args.no_e2e:
+        rb, rc = (0, n)
+        if world > 1:
+            _, rb, rc = apsp.apsp_partition(n, world, rank)
+        host_out = torch.empty((max(rc, 1), n), dtype=torch.float32 if is_f else torch.int32, pin_memory=True)
+        rp = torch.from_numpy(g.row_ptr).pin_memory().numpy()
+        cl = torch.from_numpy(g.col).pin_memory().numpy()
+        ww = torch.from_numpy(g.w).pin_memory().numpy()
+        h2d = rp.nbytes + cl.nbytes + ww.nbytes
+        d2h = rc * n * host_out.element_size()
+        k_e2e = max(1, min(args.steps, 3))
+        # warm once (allocator, NCCL comm)
+        he = apsp.apsp_init_from_csr(n, rp, cl, ww, cfg=make_cfg(0))
+        apsp.apsp_destroy(he)
+        barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(k_e2e):
+            he = apsp.apsp_init_from_csr(n, rp, cl, ww, cfg=make_cfg(0))
+            apsp.apsp_fw_blocked(he)
+            if rc > 0:
+                apsp.apsp_get_dist_ptr(he, rb, rc, host_out.data_ptr(), n)
+            apsp.apsp_destroy(he)
+        torch.cuda.synchronize()
+        el = time.perf_counter() - t0
+        el = max_over_ranks(el)
+        e2e = {"value": float(n) ** 3 / (el / k_e2e), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
+               "d2h_bytes_per_step": int(d2h), "steps": k_e2e,
+               "note": "apsp_init_from_csr(host CSR, pinned) + apsp_fw_blocked + apsp_get_dist(pinned host) + "
+                       "destroy, host wall clock (synchronous C-ABI calls)"}
+
+    # ---------------- CPU oracle baseline (rank 0, N=1 only) ------------------
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        r, cores, sample = cpu_oracle_sample(g, args.cpu_seconds)
+        cpu = {"value": r, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "scaling": "strong" if world > 1 else "weak", "vs_baseline": None,
+            "dtype": "f32" if is_f else "i32", "data": "synthetic",
+            "config": {"workload": wl, "n": n, "n_pad": int(info.n_pad), "m": g.m, "tile": 128,
+                       "desc": gg.BASELINE_CONFIGS[wl],
+                       "parallelism": "1-D block-row x%d, NCCL pivot-band broadcast" % world if world > 1
+                       else "single GPU",
+                       "l2": "inputs larger than L2 (dist = %.2f GB per step >> 126 MB L2); no flush" %
+                             (float(info.n_pad) ** 2 * 4 / 1e9),
+                       "step": "apsp_reinit (CSR->dense, CSR resident in HBM) + apsp_fw_blocked"},
+            "clocks": clocks,
+            "e2e": e2e,
+            "gpu_launches": launches_per_step * args.steps,
+            "roofline": roofline,
+            "cpu_baseline": cpu,
+            "relax_per_step_rank0": relax_local,
+            "phase_ms_per_step_rank0": {"phase1": st_acc[0][0] / args.steps, "phase2": st_acc[0][1] / args.steps,
+                                        "phase3": st_acc[0][2] / args.steps, "comm": st_acc[0][3] / args.steps},
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

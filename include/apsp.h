@@ -1,0 +1,211 @@
+/*
+ * apsp.h — C ABI of the B200 (sm_100a) blocked Floyd–Warshall APSP library
+ * (libapsp.so, built from paper_conf_ipps_xia0ar22_b200/csrc/).
+ *
+ * Problem (§II): G = (V, E), n = |V|, m = |E|, w[i][j] the weight
+ * of the arc from v_i to v_j; compute the n x n matrix dist where dist[i][j]
+ * is the shortest distance from v_i to v_j. The graph arrives as CSR (the
+ * paper's inputs are sparse adjacency matrices); the
+ * distance element type is int32 (the paper's `int`), with an
+ * fp32 instantiation for real weights (BASELINE.json config 4).
+ *
+ * Method (§II-A, and Algorithm 1, §III-A):
+ * blocked Floyd–Warshall. dist is split into b x b tiles A(i,j); round k runs
+ *   phase 1  A(k,k) := FW closure of A(k,k)
+ *   phase 2  A(k,j) := min(A(k,j), A(k,k) (x) A(k,j)),  A(i,k) := min(A(i,k), A(i,k) (x) A(k,k))
+ *   phase 3  A(i,j) := min(A(i,j), A(i,k) (x) A(k,j))   for i != k, j != k
+ * where (x) is the min-plus product (MinPlus Multiply). When
+ * n*n does not fit in device memory the library streams row bands from
+ * pinned host memory (out-of-core, Algorithm 1 and PAPER.md:197).
+ *
+ * Conventions for every call:
+ *  - Plain C; no exception crosses the boundary; every call returns
+ *    apsp_status and never aborts the process.
+ *  - Pointers are HOST pointers unless named *_device.
+ *  - Error behaviour: on a non-OK status apsp_last_error(h) (or
+ *    apsp_last_error(NULL) for failures before a handle exists) returns a
+ *    one-line message. After APSP_ECUDA or APSP_ENCCL the handle is
+ *    poisoned: only apsp_destroy is valid.
+ *  - A handle is not thread-safe; different handles may be used from
+ *    different threads on different devices.
+ *  - Multi-GPU (world_size > 1, one process per GPU): every rank makes the
+ *    same sequence of calls (init -> fw -> destroy), like an MPI collective.
+ */
+#ifndef APSP_H_
+#define APSP_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct apsp_handle apsp_handle; /* opaque, library-owned */
+
+typedef enum { APSP_I32 = 0, APSP_F32 = 1 } apsp_dtype;
+
+typedef enum {
+  APSP_OK = 0,
+  APSP_EINVAL = 1,     /* bad argument: NULL pointer, n < 0, row_ptr not monotone,
+                          col out of [0, n), non-finite fp32 weight, bad config */
+  APSP_ERANGE = 2,     /* int32 distances could reach APSP_INF_I32 (see init) */
+  APSP_ENOMEM = 3,     /* device or pinned host allocation failed */
+  APSP_ECUDA = 4,      /* CUDA runtime error (no device, launch failure ...) */
+  APSP_ENCCL = 5,      /* NCCL error (multi-GPU only) */
+  APSP_ENEGCYCLE = 6,  /* the graph holds a negative cycle; distances unspecified */
+  APSP_ESTATE = 7      /* call out of order (e.g. get_dist before fw_blocked) */
+} apsp_status;
+
+/* int32 "no path" value in the output (and the internal infinity):
+ * 2^30 - 1, so INF + INF still fits in int32 and the branch-free min-plus
+ * update (PAPER.md:60's infinity) never overflows. fp32 uses +INFINITY. */
+#define APSP_INF_I32 0x3FFFFFFF
+
+#define APSP_MODE_INCORE 0
+#define APSP_MODE_OUT_OF_CORE 1
+
+typedef struct {
+  int32_t struct_size;          /* = sizeof(apsp_config) (ABI versioning); 0 = defaults */
+  int32_t device;               /* CUDA ordinal; -1 = current device */
+  int32_t world_size;           /* number of ranks (1 = single GPU) */
+  int32_t rank;                 /* this process's rank, 0 <= rank < world_size */
+  const void* nccl_unique_id;   /* 128-byte ncclUniqueId from apsp_nccl_unique_id on
+                                   rank 0, broadcast by the caller (e.g. with
+                                   torch.distributed); NULL when world_size == 1 */
+  int32_t virtual_ranks;        /* 1 = run all world_size shards in THIS process on
+                                   one device, panel broadcast = device copy (tests the
+                                   sharded schedule on one GPU); rank is ignored */
+  int32_t tile;                 /* round depth b (tile edge); 0 = auto (128). Must be 128
+                                   in this build (the kernels' tile edge) */
+  void* stream;                 /* cudaStream_t to enqueue on; NULL = library stream */
+  int64_t device_budget_bytes;  /* 0 = use free device memory; smaller forces the
+                                   out-of-core path (tests) */
+  int32_t ooc_block;            /* out-of-core super-block (band height) B; 0 = auto;
+                                   multiple of the tile */
+  int32_t timing;               /* 1 = record CUDA events around every launch and
+                                   accumulate per-phase device times (apsp_phase_stats) */
+  int32_t force_out_of_core;    /* 1 = use the out-of-core path even if n*n fits */
+  int32_t reserved[7];
+} apsp_config;
+
+/* Fill *cfg with defaults (struct_size set, device -1, world 1, rank 0). */
+void apsp_config_default(apsp_config* cfg);
+
+/*
+ * apsp_init_from_csr — copy the graph to the device and build the initial
+ * distance matrix ("initializes the matrix dist with the input
+ * weights for the edges (which will be infinity when there are no edges)").
+ *
+ *   n         number of vertices, 0 <= n; vertices are 0..n-1
+ *   row_ptr   host int64[n+1], row_ptr[0] = 0, non-decreasing; arcs of source u
+ *             are e in [row_ptr[u], row_ptr[u+1])
+ *   col_idx   host int32[m], m = row_ptr[n]; destination of arc e, in [0, n)
+ *   weights   host int32[m] (APSP_I32) or float[m] (APSP_F32), finite
+ *   dtype     element type of weights and of the distance matrix
+ *   cfg       may be NULL (defaults)
+ *
+ * Semantics: dist[i][i] = 0; dist[u][v] = min over arcs u->v of w (duplicates
+ * keep the minimum; a self-loop gives min(0, w)); all other entries infinity.
+ * Ownership: the CSR arrays are read during the call only (copied).
+ * Errors: APSP_EINVAL (see enum), APSP_ERANGE for int32 when
+ * (n-1)*max|w| >= 2^28 with negative weights present or >= APSP_INF_I32 with
+ * all weights >= 0; APSP_ENOMEM; APSP_ECUDA; APSP_ENCCL.
+ * On success *out is a new handle (to be released with apsp_destroy).
+ * With world_size > 1 each rank initialises only its own block of rows.
+ */
+apsp_status apsp_init_from_csr(apsp_handle** out, int64_t n, const int64_t* row_ptr,
+                               const int32_t* col_idx, const void* weights, apsp_dtype dtype,
+                               const apsp_config* cfg);
+
+/*
+ * apsp_fw_blocked — run the whole blocked Floyd–Warshall (all n/b rounds,
+ * PAPER.md:62; out-of-core: Algorithm 1). Blocks until the
+ * device work is done. Returns APSP_ENEGCYCLE if a negative cycle exists
+ * (detected as a negative diagonal entry at the start of a phase-1 step; the
+ * distances are then unspecified), APSP_ESTATE if already run.
+ */
+apsp_status apsp_fw_blocked(apsp_handle* h);
+
+/*
+ * apsp_reinit — rebuild the initial distance matrix (same semantics as
+ * apsp_init_from_csr) from the device-resident copy of the CSR the handle
+ * keeps, so that apsp_fw_blocked can run again on the same graph without a
+ * host round trip (benchmark steps with inputs resident in HBM). Asynchronous
+ * on the handle's stream.
+ */
+apsp_status apsp_reinit(apsp_handle* h);
+
+/*
+ * apsp_fw_rounds — run rounds [k_begin, k_end) only (in-core mode). After
+ * rounds 0..K-1, dist[i][j] is the shortest path whose intermediates all lie
+ * in {0 .. K*b - 1}, i.e. the plain FW state after K*b outer iterations
+ * (PAPER.md:60). Used for per-round parity. Rounds must be run in order.
+ */
+apsp_status apsp_fw_rounds(apsp_handle* h, int64_t k_begin, int64_t k_end);
+
+/*
+ * apsp_get_dist — copy rows [row_begin, row_begin+row_count), columns [0, n),
+ * of dist into the caller's host buffer out (row_count x ld_out elements of
+ * dtype, ld_out >= n; pinned memory is faster). Unreachable pairs read
+ * APSP_INF_I32 (int32) or +INFINITY (fp32). With world_size > 1 (NCCL mode)
+ * the rows must lie in this rank's block (apsp_local_rows). Valid after
+ * apsp_init_from_csr (returns the initial matrix) and after apsp_fw_blocked.
+ */
+apsp_status apsp_get_dist(apsp_handle* h, int64_t row_begin, int64_t row_count, void* out,
+                          int64_t ld_out);
+
+/* Rows [*row_begin, *row_begin + *row_count) of dist held by this rank. */
+apsp_status apsp_local_rows(const apsp_handle* h, int64_t* row_begin, int64_t* row_count);
+
+/*
+ * apsp_partition — the 1-D block-row partition used for world_size ranks
+ * (host-only arithmetic, no device needed): n is padded to n_pad, a multiple
+ * of tile*world_size; rank r owns padded rows [r*n_pad/world, (r+1)*n_pad/world)
+ * and, of those, the real rows [*row_begin, *row_begin + *row_count).
+ * owner of round k = (k*tile) / (n_pad/world).
+ */
+apsp_status apsp_partition(int64_t n, int32_t tile, int32_t world_size, int32_t rank,
+                           int64_t* n_pad, int64_t* row_begin, int64_t* row_count);
+
+typedef struct {
+  int64_t n, n_pad;
+  int32_t tile, dtype, world_size, rank, mode; /* mode: APSP_MODE_* */
+  int32_t ooc_block;                           /* B when out-of-core, else 0 */
+  int64_t rounds;                              /* n_pad / tile */
+  int64_t device_bytes;                        /* device memory the handle holds */
+  int64_t host_bytes;                          /* pinned host memory (out-of-core) */
+  void* dist_device;                           /* in-core: device base of this rank's
+                                                  rows (row-major, ld = ld elements);
+                                                  NULL out-of-core */
+  int64_t ld;
+} apsp_info;
+
+apsp_status apsp_get_info(const apsp_handle* h, apsp_info* info);
+
+typedef struct {
+  double ms[4];          /* accumulated device time: [0] phase 1, [1] phase 2,
+                            [2] phase 3, [3] comm / host transfers */
+  int64_t launches[4];   /* kernel launches (or transfers) per class */
+  double relax[4];       /* relaxations performed per class */
+} apsp_phase_stats;
+
+/* Per-phase device times of the last apsp_fw_blocked (needs cfg.timing = 1). */
+apsp_status apsp_get_phase_stats(const apsp_handle* h, apsp_phase_stats* out);
+
+/* Rank-0 helper: write a fresh 128-byte ncclUniqueId into out128. */
+apsp_status apsp_nccl_unique_id(void* out128);
+
+/* Release everything the handle owns. NULL is allowed. */
+void apsp_destroy(apsp_handle* h);
+
+/* Last error message of h (thread-local message when h is NULL). Never NULL. */
+const char* apsp_last_error(const apsp_handle* h);
+
+/* Library version string, e.g. "apsp-b200 0.1 sm_100a". */
+const char* apsp_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* APSP_H_ */

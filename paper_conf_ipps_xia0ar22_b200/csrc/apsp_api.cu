@@ -1,0 +1,405 @@
+// apsp_api.cu — the C ABI (include/apsp.h) and the round schedulers.
+//
+//   in-core, 1 GPU        rounds k = 0 .. n_pad/b - 1 of the blocked FW
+//                         (PAPER.md:62): phase1 -> phase2 (row+col, one
+//                         launch) -> phase3, all on one stream.
+//   in-core, P ranks      1-D block-row shard (build extension; the paper is
+//                         single-GPU). Round k: the owner of row
+//                         band k runs phase 1 and the row panel, the band is
+//                         broadcast (NCCL over NVLink, or a device copy in
+//                         virtual-rank mode), then every rank updates its
+//                         column-panel tiles and its phase-3 tiles.
+//   out-of-core, 1 GPU    Algorithm 1 with super-blocks of
+//                         B rows streamed from pinned host memory
+//                         (apsp_ooc.cu).
+#include "apsp_internal.h"
+
+#include <cstdio>
+#include <cstring>
+#include <cmath>
+#include <cstdarg>
+#include <string>
+#include <vector>
+#include <algorithm>
+
+using namespace apsp;
+
+static thread_local std::string g_last_error = "";
+
+static apsp_status fail_global(apsp_status st, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_last_error = buf;
+  return st;
+}
+
+namespace apsp {
+
+apsp_status Handle::fail(apsp_status st, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  err = buf;
+  g_last_error = buf;
+  if (st == APSP_ECUDA || st == APSP_ENCCL) poisoned = true;
+  return st;
+}
+
+apsp_status Handle::cuda(cudaError_t e, const char* what) {
+  if (e == cudaSuccess) return APSP_OK;
+  return fail(e == cudaErrorMemoryAllocation ? APSP_ENOMEM : APSP_ECUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+void Handle::ev_begin(int cls) {
+  if (!timing) return;
+  TimedEvent te;
+  te.cls = cls;
+  cudaEventCreate(&te.a);
+  cudaEventCreate(&te.b);
+  cudaEventRecord(te.a, stream);
+  events.push_back(te);
+}
+
+void Handle::ev_end(double relax) {
+  if (!timing || events.empty()) return;
+  cudaEventRecord(events.back().b, stream);
+  events.back().relax = relax;
+}
+
+void Handle::collect_events() {
+  for (auto& te : events) {
+    float ms = 0.f;
+    if (cudaEventElapsedTime(&ms, te.a, te.b) == cudaSuccess) {
+      stats.ms[te.cls] += ms;
+      stats.launches[te.cls] += 1;
+      stats.relax[te.cls] += te.relax;
+    }
+    cudaEventDestroy(te.a);
+    cudaEventDestroy(te.b);
+  }
+  events.clear();
+}
+
+// --------------------------------------------------------- kernel helpers --
+
+template <typename T>
+static MinPlusDesc<T> mkdesc(T* Cout, const T* Cin, const T* A, const T* B, long long ldc, long long lda,
+                             long long ldb, int tiles_i, int tiles_j, int skip_i, int skip_j) {
+  MinPlusDesc<T> d;
+  d.Cout = Cout; d.Cin = Cin; d.A = A; d.B = B;
+  d.ldc_out = ldc; d.ldc_in = ldc; d.lda = lda; d.ldb = ldb;
+  d.tiles_i = tiles_i; d.tiles_j = tiles_j; d.skip_i = skip_i; d.skip_j = skip_j;
+  return d;
+}
+
+template <typename T>
+static double desc_relax(const MinPlusDesc<T>& d, int K) {
+  return (double)d.tiles_i * d.tiles_j * kTile * kTile * (double)K;
+}
+
+// One round k of the in-core blocked FW over this handle's shards.
+template <typename T>
+static apsp_status incore_round(Handle* h, long long k) {
+  const long long b = h->b, ld = h->ld, nb = h->n_pad / b;
+  const long long R = h->rows_per_rank;
+  const int owner = (int)((k * b) / R);
+  cudaStream_t s = h->stream;
+  apsp_status st;
+
+  // ---- owner: phase 1 (+ row panel) on its band -------------------------
+  Shard* own = nullptr;
+  for (auto& sh : h->shards)
+    if (sh.rank == owner) own = &sh;
+  T* band = nullptr;
+  if (own) {
+    band = static_cast<T*>(own->D) + (k * b - own->row_begin) * ld;
+    h->ev_begin(0);
+    if ((st = h->cuda(launch_phase1<T>(band + k * b, ld, h->d_flag, s), "phase1"))) return st;
+    h->ev_end((double)b * b * b);
+    if (h->world == 1) {
+      // phase 2: row panel A(k,j) and column panel A(i,k) in one launch
+      MinPlusDesc<T> d[2];
+      d[0] = mkdesc<T>(band, band, band + k * b, band, ld, ld, ld, 1, (int)(nb - 1), -1, (int)k);
+      T* D = static_cast<T*>(own->D);
+      d[1] = mkdesc<T>(D + k * b, D + k * b, D + k * b, band + k * b, ld, ld, ld, (int)(nb - 1), 1, (int)k, -1);
+      h->ev_begin(1);
+      if ((st = h->cuda(launch_minplus<T>(d, 2, (int)b, s), "phase2"))) return st;
+      h->ev_end(desc_relax(d[0], (int)b) + desc_relax(d[1], (int)b));
+      // phase 3
+      MinPlusDesc<T> p3 = mkdesc<T>(D, D, D + k * b, band, ld, ld, ld, (int)(nb - 1), (int)(nb - 1), (int)k, (int)k);
+      h->ev_begin(2);
+      if ((st = h->cuda(launch_minplus<T>(&p3, 1, (int)b, s), "phase3"))) return st;
+      h->ev_end(desc_relax(p3, (int)b));
+      return APSP_OK;
+    }
+    MinPlusDesc<T> dr = mkdesc<T>(band, band, band + k * b, band, ld, ld, ld, 1, (int)(nb - 1), -1, (int)k);
+    h->ev_begin(1);
+    if ((st = h->cuda(launch_minplus<T>(&dr, 1, (int)b, s), "phase2-row"))) return st;
+    h->ev_end(desc_relax(dr, (int)b));
+  }
+
+  // ---- pivot band to every shard ------------------------------------------
+  const T* panel = nullptr;
+  const size_t band_elems = (size_t)b * (size_t)h->n_pad;
+  h->ev_begin(3);
+  if (h->virt) {
+    if ((st = h->cuda(cudaMemcpyAsync(h->panel, band, band_elems * sizeof(T), cudaMemcpyDeviceToDevice, s),
+                      "panel copy")))
+      return st;
+    panel = static_cast<const T*>(h->panel);
+  } else {
+    if ((st = h->bcast(own ? (void*)band : h->panel, band_elems * sizeof(T), owner))) return st;
+    panel = own ? band : static_cast<const T*>(h->panel);
+  }
+  h->ev_end(0);
+
+  // ---- every shard: column panel, then phase 3 ----------------------------
+  for (auto& sh : h->shards) {
+    T* D = static_cast<T*>(sh.D);
+    const int local_tiles = (int)(R / b);
+    const int skip_i = (sh.rank == owner) ? (int)((k * b - sh.row_begin) / b) : -1;
+    const int tiles_i = local_tiles - (skip_i >= 0 ? 1 : 0);
+    MinPlusDesc<T> dc = mkdesc<T>(D + k * b, D + k * b, D + k * b, panel + k * b, ld, ld, ld, tiles_i, 1, skip_i, -1);
+    h->ev_begin(1);
+    if ((st = h->cuda(launch_minplus<T>(&dc, 1, (int)b, s), "phase2-col"))) return st;
+    h->ev_end(desc_relax(dc, (int)b));
+    MinPlusDesc<T> p3 = mkdesc<T>(D, D, D + k * b, panel, ld, ld, ld, tiles_i, (int)(nb - 1), skip_i, (int)k);
+    h->ev_begin(2);
+    if ((st = h->cuda(launch_minplus<T>(&p3, 1, (int)b, s), "phase3"))) return st;
+    h->ev_end(desc_relax(p3, (int)b));
+  }
+  return APSP_OK;
+}
+
+apsp_status run_incore_rounds(Handle* h, long long k0, long long k1) {
+  for (long long k = k0; k < k1; ++k) {
+    apsp_status st = (h->dtype == APSP_I32) ? incore_round<int>(h, k) : incore_round<float>(h, k);
+    if (st) return st;
+  }
+  return APSP_OK;
+}
+
+}  // namespace apsp
+
+// ======================================================================
+//                                C ABI
+// ======================================================================
+
+extern "C" {
+
+void apsp_config_default(apsp_config* cfg) {
+  if (!cfg) return;
+  memset(cfg, 0, sizeof(*cfg));
+  cfg->struct_size = (int32_t)sizeof(apsp_config);
+  cfg->device = -1;
+  cfg->world_size = 1;
+  cfg->rank = 0;
+}
+
+const char* apsp_version(void) { return "apsp-b200 0.1 sm_100a"; }
+
+const char* apsp_last_error(const apsp_handle* h) {
+  if (h) return reinterpret_cast<const Handle*>(h)->err.c_str();
+  return g_last_error.c_str();
+}
+
+apsp_status apsp_partition(int64_t n, int32_t tile, int32_t world_size, int32_t rank, int64_t* n_pad,
+                           int64_t* row_begin, int64_t* row_count) {
+  if (n < 0 || world_size < 1 || rank < 0 || rank >= world_size || !n_pad || !row_begin || !row_count)
+    return fail_global(APSP_EINVAL, "apsp_partition: bad arguments");
+  if (tile == 0) tile = kTile;
+  if (tile != kTile) return fail_global(APSP_EINVAL, "apsp_partition: tile must be %d", kTile);
+  const int64_t unit = (int64_t)tile * world_size;
+  int64_t np = ((n + unit - 1) / unit) * unit;
+  if (np == 0) np = unit;
+  const int64_t R = np / world_size;
+  const int64_t rb = (int64_t)rank * R;
+  *n_pad = np;
+  *row_begin = rb;
+  *row_count = std::max<int64_t>(0, std::min<int64_t>(rb + R, n) - rb);
+  return APSP_OK;
+}
+
+apsp_status apsp_nccl_unique_id(void* out128) {
+  if (!out128) return fail_global(APSP_EINVAL, "apsp_nccl_unique_id: NULL");
+  return nccl_unique_id(out128) ? APSP_OK : fail_global(APSP_ENCCL, "ncclGetUniqueId failed");
+}
+
+apsp_status apsp_init_from_csr(apsp_handle** out, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                               const void* weights, apsp_dtype dtype, const apsp_config* cfg_in) {
+  if (!out) return fail_global(APSP_EINVAL, "apsp_init_from_csr: out is NULL");
+  *out = nullptr;
+  apsp_config cfg;
+  apsp_config_default(&cfg);
+  if (cfg_in) {
+    if (cfg_in->struct_size != 0 && cfg_in->struct_size != (int32_t)sizeof(apsp_config))
+      return fail_global(APSP_EINVAL, "apsp_config.struct_size %d != %d", cfg_in->struct_size,
+                         (int)sizeof(apsp_config));
+    cfg = *cfg_in;
+  }
+  if (n < 0) return fail_global(APSP_EINVAL, "n < 0");
+  if (n > (int64_t)INT32_MAX) return fail_global(APSP_EINVAL, "n exceeds int32 vertex ids");
+  if (!row_ptr) return fail_global(APSP_EINVAL, "row_ptr is NULL");
+  if (dtype != APSP_I32 && dtype != APSP_F32) return fail_global(APSP_EINVAL, "bad dtype");
+  if (cfg.tile == 0) cfg.tile = kTile;
+  if (cfg.tile != kTile) return fail_global(APSP_EINVAL, "tile must be %d in this build", kTile);
+  if (cfg.world_size < 1 || cfg.rank < 0 || cfg.rank >= cfg.world_size)
+    return fail_global(APSP_EINVAL, "bad world_size/rank");
+  if (cfg.world_size > 1 && !cfg.virtual_ranks && !cfg.nccl_unique_id)
+    return fail_global(APSP_EINVAL, "world_size > 1 needs nccl_unique_id (or virtual_ranks)");
+
+  // ---- validate the CSR on the host (O(n + m)) -----------------------------
+  if (row_ptr[0] != 0) return fail_global(APSP_EINVAL, "row_ptr[0] != 0");
+  for (int64_t i = 0; i < n; ++i)
+    if (row_ptr[i + 1] < row_ptr[i]) return fail_global(APSP_EINVAL, "row_ptr not monotone at %lld", (long long)i);
+  const int64_t m = row_ptr[n];
+  if (m > 0 && (!col_idx || !weights)) return fail_global(APSP_EINVAL, "col_idx/weights NULL with m > 0");
+  for (int64_t e = 0; e < m; ++e)
+    if (col_idx[e] < 0 || col_idx[e] >= n) return fail_global(APSP_EINVAL, "col_idx[%lld] out of range", (long long)e);
+  bool has_neg = false;
+  if (dtype == APSP_I32) {
+    const int32_t* w = static_cast<const int32_t*>(weights);
+    int64_t maxabs = 0;
+    for (int64_t e = 0; e < m; ++e) {
+      int64_t v = w[e];
+      if (v < 0) has_neg = true;
+      maxabs = std::max<int64_t>(maxabs, v < 0 ? -v : v);
+    }
+    const int64_t bound = has_neg ? ((int64_t)1 << 28) : (int64_t)APSP_INF_I32;
+    if (n > 1 && (__int128)(n - 1) * maxabs >= bound)
+      return fail_global(APSP_ERANGE, "(n-1)*max|w| = %lld >= %lld: int32 distances could reach infinity",
+                         (long long)((n - 1) * maxabs), (long long)bound);
+  } else {
+    const float* w = static_cast<const float*>(weights);
+    for (int64_t e = 0; e < m; ++e) {
+      if (!std::isfinite(w[e])) return fail_global(APSP_EINVAL, "weight %lld is not finite", (long long)e);
+      if (w[e] < 0) has_neg = true;
+    }
+  }
+
+  Handle* h = new Handle();
+  h->n = n;
+  h->b = cfg.tile;
+  h->dtype = dtype;
+  h->world = cfg.world_size;
+  h->rank = cfg.virtual_ranks ? 0 : cfg.rank;
+  h->virt = cfg.virtual_ranks && cfg.world_size > 1;
+  h->timing = cfg.timing != 0;
+  h->has_neg = has_neg;
+  h->elem = sizeof(int32_t);
+
+  apsp_status st = init_handle(h, cfg, row_ptr, col_idx, weights);
+  if (st != APSP_OK) {
+    g_last_error = h->err;
+    delete_handle(h);
+    return st;
+  }
+  *out = reinterpret_cast<apsp_handle*>(h);
+  return APSP_OK;
+}
+
+apsp_status apsp_fw_rounds(apsp_handle* hh, int64_t k_begin, int64_t k_end) {
+  if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
+  Handle* h = reinterpret_cast<Handle*>(hh);
+  if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  if (h->mode != APSP_MODE_INCORE) return h->fail(APSP_ESTATE, "apsp_fw_rounds: in-core mode only");
+  const long long nb = h->n_pad / h->b;
+  if (k_begin != h->next_round || k_end < k_begin || k_end > nb)
+    return h->fail(APSP_ESTATE, "rounds must run in order: next is %lld of %lld", h->next_round, nb);
+  apsp_status st;
+  if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
+  if ((st = run_incore_rounds(h, k_begin, k_end))) return st;
+  h->next_round = k_end;
+  return finish_fw(h, k_end == nb);
+}
+
+apsp_status apsp_fw_blocked(apsp_handle* hh) {
+  if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
+  Handle* h = reinterpret_cast<Handle*>(hh);
+  if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  if (h->fw_done) return h->fail(APSP_ESTATE, "apsp_fw_blocked already ran");
+  apsp_status st;
+  if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
+  memset(&h->stats, 0, sizeof(h->stats));
+  if (h->mode == APSP_MODE_OUT_OF_CORE) {
+    if ((st = run_out_of_core(h))) return st;
+    return finish_fw(h, true);
+  }
+  const long long nb = h->n_pad / h->b;
+  if (h->next_round != 0) return h->fail(APSP_ESTATE, "apsp_fw_rounds already started");
+  if ((st = run_incore_rounds(h, 0, nb))) return st;
+  h->next_round = nb;
+  return finish_fw(h, true);
+}
+
+apsp_status apsp_reinit(apsp_handle* hh) {
+  if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
+  Handle* h = reinterpret_cast<Handle*>(hh);
+  if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  apsp_status st;
+  if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
+  if (h->mode == APSP_MODE_OUT_OF_CORE) return ooc_reinit(h);
+  return run_init(h);
+}
+
+apsp_status apsp_get_dist(apsp_handle* hh, int64_t row_begin, int64_t row_count, void* out, int64_t ld_out) {
+  if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
+  Handle* h = reinterpret_cast<Handle*>(hh);
+  if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  if (row_count < 0 || row_begin < 0 || row_begin + row_count > h->n || ld_out < h->n || (row_count > 0 && !out))
+    return h->fail(APSP_EINVAL, "get_dist: bad row range / ld_out / out");
+  if (row_count == 0) return APSP_OK;
+  apsp_status st;
+  if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
+  return get_rows(h, row_begin, row_count, out, ld_out);
+}
+
+apsp_status apsp_local_rows(const apsp_handle* hh, int64_t* row_begin, int64_t* row_count) {
+  if (!hh || !row_begin || !row_count) return fail_global(APSP_EINVAL, "NULL argument");
+  const Handle* h = reinterpret_cast<const Handle*>(hh);
+  if (h->virt || h->world == 1) {
+    *row_begin = 0;
+    *row_count = h->n;
+    return APSP_OK;
+  }
+  int64_t np;
+  return apsp_partition(h->n, h->b, h->world, h->rank, &np, row_begin, row_count);
+}
+
+apsp_status apsp_get_info(const apsp_handle* hh, apsp_info* info) {
+  if (!hh || !info) return fail_global(APSP_EINVAL, "NULL argument");
+  const Handle* h = reinterpret_cast<const Handle*>(hh);
+  memset(info, 0, sizeof(*info));
+  info->n = h->n;
+  info->n_pad = h->n_pad;
+  info->tile = h->b;
+  info->dtype = h->dtype;
+  info->world_size = h->world;
+  info->rank = h->rank;
+  info->mode = h->mode;
+  info->ooc_block = h->mode == APSP_MODE_OUT_OF_CORE ? (int32_t)h->ooc_B : 0;
+  info->rounds = h->n_pad / h->b;
+  info->device_bytes = h->device_bytes;
+  info->host_bytes = h->host_bytes;
+  info->dist_device = h->shards.empty() ? nullptr : h->shards[0].D;
+  info->ld = h->ld;
+  return APSP_OK;
+}
+
+apsp_status apsp_get_phase_stats(const apsp_handle* hh, apsp_phase_stats* out) {
+  if (!hh || !out) return fail_global(APSP_EINVAL, "NULL argument");
+  *out = reinterpret_cast<const Handle*>(hh)->stats;
+  return APSP_OK;
+}
+
+void apsp_destroy(apsp_handle* hh) {
+  if (!hh) return;
+  delete_handle(reinterpret_cast<Handle*>(hh));
+}
+
+}  // extern "C"

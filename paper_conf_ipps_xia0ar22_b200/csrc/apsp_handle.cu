@@ -1,0 +1,224 @@
+// apsp_handle.cu — handle lifetime: device selection, 1-D block-row
+// partition, allocation, NCCL communicator, CSR upload + init kernel
+// (PAPER.md:60), negative-cycle status, and result read-back (get_dist).
+#include "apsp_internal.h"
+
+#include <nccl.h>
+
+#include <algorithm>
+#include <cstring>
+
+namespace apsp {
+
+bool nccl_unique_id(void* out128) {
+  static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId is 128 bytes");
+  ncclUniqueId id;
+  if (ncclGetUniqueId(&id) != ncclSuccess) return false;
+  memcpy(out128, &id, sizeof(id));
+  return true;
+}
+
+apsp_status Handle::bcast(void* buf, size_t bytes, int root) {
+  ncclResult_t r = ncclBroadcast(buf, buf, bytes, ncclUint8, root, static_cast<ncclComm_t>(comm), stream);
+  if (r != ncclSuccess) return fail(APSP_ENCCL, "ncclBroadcast: %s", ncclGetErrorString(r));
+  return APSP_OK;
+}
+
+template <typename T>
+static apsp_status upload_csr(Handle* h, const int64_t* row_ptr, const int32_t* col, const void* w) {
+  apsp_status st;
+  for (auto& sh : h->shards) {
+    const long long R = h->rows_per_rank;
+    const long long real = std::max<long long>(0, std::min<long long>(R, h->n - sh.row_begin));
+    sh.real_rows = real;
+    if (real <= 0) continue;
+    const long long e0 = row_ptr[sh.row_begin];
+    const long long me = row_ptr[sh.row_begin + real] - e0;
+    sh.e0 = e0;
+    if ((st = h->cuda(cudaMalloc(&sh.d_rp, (real + 1) * sizeof(long long)), "cudaMalloc csr"))) return st;
+    if ((st = h->cuda(cudaMemcpyAsync(sh.d_rp, row_ptr + sh.row_begin, (real + 1) * sizeof(long long),
+                                      cudaMemcpyHostToDevice, h->stream), "H2D row_ptr")))
+      return st;
+    h->device_bytes += (real + 1) * sizeof(long long);
+    if (me > 0) {
+      if ((st = h->cuda(cudaMalloc(&sh.d_col, me * sizeof(int)), "cudaMalloc csr"))) return st;
+      if ((st = h->cuda(cudaMalloc(&sh.d_w, me * sizeof(T)), "cudaMalloc csr"))) return st;
+      if ((st = h->cuda(cudaMemcpyAsync(sh.d_col, col + e0, me * sizeof(int), cudaMemcpyHostToDevice, h->stream),
+                        "H2D col")))
+        return st;
+      if ((st = h->cuda(cudaMemcpyAsync(sh.d_w, static_cast<const T*>(w) + e0, me * sizeof(T),
+                                        cudaMemcpyHostToDevice, h->stream), "H2D w")))
+        return st;
+      h->device_bytes += me * (sizeof(int) + sizeof(T));
+    }
+  }
+  return APSP_OK;
+}
+
+// a1: CSR -> dense for every local shard, from the device CSR.
+apsp_status run_init(Handle* h) {
+  apsp_status st;
+  for (auto& sh : h->shards) {
+    cudaError_t e;
+    if (h->dtype == APSP_I32)
+      e = launch_init_rows<int>(static_cast<int*>(sh.D), h->ld, h->n_pad, sh.row_begin, h->rows_per_rank, h->n,
+                                sh.d_rp, sh.e0, sh.d_col, static_cast<const int*>(sh.d_w), h->stream);
+    else
+      e = launch_init_rows<float>(static_cast<float*>(sh.D), h->ld, h->n_pad, sh.row_begin, h->rows_per_rank, h->n,
+                                  sh.d_rp, sh.e0, sh.d_col, static_cast<const float*>(sh.d_w), h->stream);
+    if ((st = h->cuda(e, "init_rows"))) return st;
+  }
+  if ((st = h->cuda(cudaMemsetAsync(h->d_flag, 0, sizeof(int), h->stream), "memset flag"))) return st;
+  h->next_round = 0;
+  h->fw_done = false;
+  h->canonical = false;
+  return APSP_OK;
+}
+
+apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, const int32_t* col,
+                        const void* w) {
+  apsp_status st;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
+    return h->fail(APSP_ECUDA, "no CUDA device visible (the library has no CPU path)");
+  if (cfg.device >= 0) {
+    if (cfg.device >= ndev) return h->fail(APSP_EINVAL, "device %d >= device count %d", cfg.device, ndev);
+    h->device = cfg.device;
+  } else if ((st = h->cuda(cudaGetDevice(&h->device), "cudaGetDevice"))) {
+    return st;
+  }
+  if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
+  cudaDeviceProp prop;
+  if ((st = h->cuda(cudaGetDeviceProperties(&prop, h->device), "cudaGetDeviceProperties"))) return st;
+  if (prop.major < 10) return h->fail(APSP_ECUDA, "device %s is sm_%d%d; this library is built for sm_100a", prop.name,
+                                      prop.major, prop.minor);
+  if ((st = h->cuda(configure_kernels(), "configure_kernels"))) return st;
+  if (cfg.stream) {
+    h->stream = static_cast<cudaStream_t>(cfg.stream);
+  } else {
+    if ((st = h->cuda(cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking), "cudaStreamCreate"))) return st;
+    h->own_stream = true;
+  }
+
+  int64_t np, rb, rc;
+  if (apsp_partition(h->n, h->b, h->world, h->virt ? 0 : h->rank, &np, &rb, &rc) != APSP_OK)
+    return h->fail(APSP_EINVAL, "partition failed");
+  h->n_pad = np;
+  h->rows_per_rank = np / h->world;
+  h->ld = np;
+
+  if ((st = h->cuda(cudaMalloc(&h->d_flag, sizeof(int)), "cudaMalloc flag"))) return st;
+  if ((st = h->cuda(cudaMemsetAsync(h->d_flag, 0, sizeof(int), h->stream), "memset flag"))) return st;
+
+  // ---- in-core or out-of-core? ---------------------------------------------
+  const int nshards = h->virt ? h->world : 1;
+  const long long mat_bytes = (long long)nshards * h->rows_per_rank * h->ld * (long long)h->elem;
+  const long long panel_bytes = h->world > 1 ? (long long)h->b * h->ld * (long long)h->elem : 0;
+  size_t free_b = 0, total_b = 0;
+  if ((st = h->cuda(cudaMemGetInfo(&free_b, &total_b), "cudaMemGetInfo"))) return st;
+  long long budget = cfg.device_budget_bytes > 0 ? cfg.device_budget_bytes
+                                                 : (long long)free_b - (1ll << 30);  // keep 1 GiB headroom
+  const bool need_ooc = cfg.force_out_of_core || (mat_bytes + panel_bytes > budget);
+  if (need_ooc) {
+    if (h->world > 1) return h->fail(APSP_ENOMEM, "matrix shard (%lld B) exceeds the device budget (%lld B); "
+                                     "out-of-core x multi-GPU is not supported", mat_bytes, budget);
+    h->mode = APSP_MODE_OUT_OF_CORE;
+    return ooc_setup(h, cfg, budget, row_ptr, col, w);
+  }
+
+  if ((st = h->cuda(cudaMalloc(&h->d_base, mat_bytes), "cudaMalloc dist"))) return st;
+  h->device_bytes = mat_bytes;
+  if (panel_bytes) {
+    if ((st = h->cuda(cudaMalloc(&h->panel, panel_bytes), "cudaMalloc panel"))) return st;
+    h->device_bytes += panel_bytes;
+  }
+  for (int s = 0; s < nshards; ++s) {
+    Shard sh;
+    sh.rank = h->virt ? s : h->rank;
+    sh.row_begin = (long long)sh.rank * h->rows_per_rank;
+    sh.D = static_cast<char*>(h->d_base) + (size_t)s * h->rows_per_rank * h->ld * h->elem;
+    h->shards.push_back(sh);
+  }
+
+  if (h->world > 1 && !h->virt) {
+    ncclUniqueId id;
+    memcpy(&id, cfg.nccl_unique_id, sizeof(id));
+    ncclComm_t comm;
+    ncclResult_t r = ncclCommInitRank(&comm, h->world, id, h->rank);
+    if (r != ncclSuccess) return h->fail(APSP_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
+    h->comm = comm;
+  }
+
+  if ((st = h->dtype == APSP_I32 ? upload_csr<int>(h, row_ptr, col, w) : upload_csr<float>(h, row_ptr, col, w)))
+    return st;
+  if ((st = run_init(h))) return st;
+  return h->cuda(cudaStreamSynchronize(h->stream), "init sync");
+}
+
+void delete_handle(Handle* h) {
+  if (!h) return;
+  cudaSetDevice(h->device);
+  if (h->stream) cudaStreamSynchronize(h->stream);
+  for (auto& te : h->events) {
+    cudaEventDestroy(te.a);
+    cudaEventDestroy(te.b);
+  }
+  if (h->comm) ncclCommDestroy(static_cast<ncclComm_t>(h->comm));
+  ooc_free(h);
+  for (auto& sh : h->shards) {
+    cudaFree(sh.d_rp);
+    cudaFree(sh.d_col);
+    cudaFree(sh.d_w);
+  }
+  cudaFree(h->d_base);
+  cudaFree(h->panel);
+  cudaFree(h->d_flag);
+  if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
+  delete h;
+}
+
+apsp_status finish_fw(Handle* h, bool all_rounds) {
+  apsp_status st;
+  int flag = 0;
+  if (h->world > 1 && !h->virt) {
+    ncclResult_t r = ncclAllReduce(h->d_flag, h->d_flag, 1, ncclInt32, ncclMax, static_cast<ncclComm_t>(h->comm),
+                                   h->stream);
+    if (r != ncclSuccess) return h->fail(APSP_ENCCL, "ncclAllReduce(flag): %s", ncclGetErrorString(r));
+  }
+  if ((st = h->cuda(cudaMemcpyAsync(&flag, h->d_flag, sizeof(int), cudaMemcpyDeviceToHost, h->stream), "D2H flag")))
+    return st;
+  if ((st = h->cuda(cudaStreamSynchronize(h->stream), "fw sync"))) return st;
+  if (h->timing) h->collect_events();
+  h->canonical = false;
+  if (all_rounds) h->fw_done = true;
+  if (flag) return h->fail(APSP_ENEGCYCLE, "negative cycle detected: distances are unspecified");
+  return APSP_OK;
+}
+
+apsp_status get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out) {
+  if (h->mode == APSP_MODE_OUT_OF_CORE) return ooc_get_rows(h, r0, cnt, out, ld_out);
+  apsp_status st;
+  const char* base;
+  if (h->world > 1 && !h->virt) {
+    const long long rb = h->shards[0].row_begin;
+    if (r0 < rb || r0 + cnt > rb + h->rows_per_rank)
+      return h->fail(APSP_EINVAL, "rows [%lld, %lld) are not local to rank %d", r0, r0 + cnt, h->rank);
+    base = static_cast<const char*>(h->shards[0].D) + (size_t)(r0 - rb) * h->ld * h->elem;
+  } else {
+    base = static_cast<const char*>(h->d_base) + (size_t)r0 * h->ld * h->elem;
+  }
+  if (h->dtype == APSP_I32 && h->has_neg && !h->canonical) {
+    for (auto& sh : h->shards)
+      if ((st = h->cuda(launch_canonicalize_i32(static_cast<int*>(sh.D), h->ld, h->rows_per_rank, h->n_pad, h->stream),
+                        "canonicalize")))
+        return st;
+    h->canonical = true;
+  }
+  if ((st = h->cuda(cudaMemcpy2DAsync(out, (size_t)ld_out * h->elem, base, (size_t)h->ld * h->elem,
+                                      (size_t)h->n * h->elem, (size_t)cnt, cudaMemcpyDeviceToHost, h->stream),
+                    "D2H dist")))
+    return st;
+  return h->cuda(cudaStreamSynchronize(h->stream), "get_dist sync");
+}
+
+}  // namespace apsp

@@ -1,0 +1,90 @@
+// apsp_internal.h — handle state shared by the C ABI and the schedulers.
+#pragma once
+#include "../../include/apsp.h"
+#include "apsp_kernels.cuh"
+
+#include <cuda_runtime.h>
+#include <string>
+#include <vector>
+
+namespace apsp {
+
+// A block of rows of the (padded) distance matrix resident on the device.
+struct Shard {
+  int rank = 0;              // owner rank of these rows
+  long long row_begin = 0;   // first padded row
+  void* D = nullptr;         // rows_per_rank x ld elements, row-major
+  // device copy of this shard's CSR slice, kept for apsp_reinit
+  long long* d_rp = nullptr;
+  int* d_col = nullptr;
+  void* d_w = nullptr;
+  long long real_rows = 0, e0 = 0;
+};
+
+struct TimedEvent {
+  int cls = 0;
+  cudaEvent_t a = nullptr, b = nullptr;
+  double relax = 0;
+};
+
+struct Handle {
+  // problem
+  long long n = 0, n_pad = 0;
+  int b = kTile;
+  apsp_dtype dtype = APSP_I32;
+  size_t elem = 4;
+  bool has_neg = false;
+  // placement
+  int device = 0;
+  int world = 1, rank = 0;
+  bool virt = false;
+  long long rows_per_rank = 0, ld = 0;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  std::vector<Shard> shards;
+  void* d_base = nullptr;   // allocation behind the shards (in-core)
+  void* panel = nullptr;    // b x ld pivot band received from the owner
+  int* d_flag = nullptr;    // negative-cycle flag (device)
+  void* comm = nullptr;     // ncclComm_t
+  // out-of-core
+  int mode = APSP_MODE_INCORE;
+  long long ooc_B = 0;
+  void* h_dist = nullptr;   // pinned n_pad x n_pad host matrix
+  void* ooc_dev = nullptr;  // device arena for bands
+  void* ooc_streams[3] = {nullptr, nullptr, nullptr};
+  // bookkeeping
+  long long device_bytes = 0, host_bytes = 0;
+  long long next_round = 0;
+  bool fw_done = false, canonical = false, poisoned = false;
+  bool timing = false;
+  std::vector<TimedEvent> events;
+  apsp_phase_stats stats{};
+  std::string err;
+
+  apsp_status fail(apsp_status st, const char* fmt, ...);
+  apsp_status cuda(cudaError_t e, const char* what);
+  apsp_status bcast(void* buf, size_t bytes, int root);
+  // class: 0 phase1, 1 phase2, 2 phase3, 3 comm / host transfer
+  void ev_begin(int cls);
+  void ev_end(double relax);
+  void collect_events();
+};
+
+apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, const int32_t* col,
+                        const void* w);
+void delete_handle(Handle* h);
+apsp_status run_init(Handle* h);
+apsp_status run_incore_rounds(Handle* h, long long k0, long long k1);
+apsp_status finish_fw(Handle* h, bool all_rounds);
+apsp_status get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out);
+bool nccl_unique_id(void* out128);
+
+// out-of-core (apsp_ooc.cu)
+apsp_status ooc_setup(Handle* h, const apsp_config& cfg, long long budget, const int64_t* row_ptr,
+                      const int32_t* col, const void* w);
+apsp_status run_out_of_core(Handle* h);
+apsp_status ooc_get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out);
+void ooc_free(Handle* h);
+apsp_status ooc_reinit(Handle* h);
+
+}  // namespace apsp

@@ -1,0 +1,363 @@
+// apsp_kernels.cu — sm_100a kernels of the blocked Floyd–Warshall hot path.
+//
+//   init_rows      CSR -> dense distance rows
+//   phase1         FW closure of the pivot tile A(k,k) (PAPER.md:62 step 1;
+//                  Algorithm 1 line 3)
+//   minplus        C = min(C, A (x) B) on 128x128 output tiles — phase 2
+//                  (pivot row/column panels, PAPER.md:62 step 2, Alg. 1 l.7/11)
+//                  and phase 3 (all other tiles, PAPER.md:62 step 3, Alg. 1
+//                  l.17), and the depth-B products of the out-of-core path.
+//
+// The relaxation c = min(c, a + b) is one DPX instruction on
+// Blackwell: __viaddmin_s32 -> SASS VIADDMNMX (int32). fp32 uses FADD + FMNMX.
+// Tensor cores are not used: min-plus is not a multiply-add contraction.
+#include "apsp_kernels.cuh"
+
+#include <cuda_runtime.h>
+#include <cstdint>
+#include <cfloat>
+
+namespace apsp {
+
+// ----------------------------------------------------------------- values --
+
+template <typename T> struct Val;
+template <> struct Val<int> {
+  static __device__ __forceinline__ int inf() { return 0x3FFFFFFF; }  // = APSP_INF_I32
+  // min(c, a + b): VIADDMNMX on sm_90+/sm_100a
+  static __device__ __forceinline__ int relax(int a, int b, int c) { return __viaddmin_s32(a, b, c); }
+  static __device__ __forceinline__ int vmin(int a, int b) { return min(a, b); }
+};
+template <> struct Val<float> {
+  static __device__ __forceinline__ float inf() { return __int_as_float(0x7f800000); }
+  static __device__ __forceinline__ float relax(float a, float b, float c) { return fminf(c, __fadd_rn(a, b)); }
+  static __device__ __forceinline__ float vmin(float a, float b) { return fminf(a, b); }
+};
+
+template <typename T> struct Vec4;
+template <> struct Vec4<int> { using type = int4; };
+template <> struct Vec4<float> { using type = float4; };
+
+// ------------------------------------------------------------- cp.async --
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+  unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N)); }
+
+// ------------------------------------------------------------- min-plus --
+//
+// CTA: 256 threads, one 128x128 output tile, register-blocked 8x8 per thread
+// (two 4-row groups x two 4-col groups, 64 rows apart, so that every LDS is
+// a 16-byte vector and B reads of a warp are contiguous). The depth K is
+// streamed in chunks of 32 through a 3-stage cp.async pipeline:
+//   As[s][128 rows][32+4]  (A chunk, row-major as in HBM; +4 pad breaks the
+//                           bank aliasing of rows 4 apart)
+//   Bs[s][32][128]         (B chunk, row-major)
+// The accumulator starts as the C tile; C is written only after the whole
+// depth has been read, so phase 2 (where A or B aliases C) is out-of-place
+// per tile.
+
+constexpr int MP_BM = 128, MP_BN = 128, MP_BK = 32, MP_NT = 256, MP_STAGES = 3;
+constexpr int MP_ALD = MP_BK + 4;
+constexpr int MP_BLD = MP_BN;
+
+template <typename T>
+struct MinPlusArgs {
+  MinPlusDesc<T> d0, d1;
+  long long n0;  // tiles in d0 (blockIdx.x < n0 -> d0)
+  int K;
+};
+
+template <typename T>
+constexpr int minplus_smem_bytes() {
+  return MP_STAGES * (MP_BM * MP_ALD + MP_BK * MP_BLD) * (int)sizeof(T);
+}
+
+template <typename T>
+__global__ void __launch_bounds__(MP_NT, 2) minplus_kernel(const __grid_constant__ MinPlusArgs<T> args) {
+  using V4 = typename Vec4<T>::type;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  T* As = reinterpret_cast<T*>(smem_raw);
+  T* Bs = As + MP_STAGES * MP_BM * MP_ALD;
+
+  long long t = blockIdx.x;
+  const bool second = t >= args.n0;
+  const MinPlusDesc<T>& d = second ? args.d1 : args.d0;
+  if (second) t -= args.n0;
+  int ti = (int)(t / d.tiles_j);
+  int tj = (int)(t - (long long)ti * d.tiles_j);
+  if (d.skip_i >= 0 && ti >= d.skip_i) ++ti;
+  if (d.skip_j >= 0 && tj >= d.skip_j) ++tj;
+
+  const T* __restrict__ Cin = d.Cin + (long long)ti * MP_BM * d.ldc_in + (long long)tj * MP_BN;
+  T* __restrict__ Cout = d.Cout + (long long)ti * MP_BM * d.ldc_out + (long long)tj * MP_BN;
+  const T* __restrict__ A = d.A + (long long)ti * MP_BM * d.lda;
+  const T* __restrict__ B = d.B + (long long)tj * MP_BN;
+  const long long lda = d.lda, ldb = d.ldb, ldc_in = d.ldc_in, ldc_out = d.ldc_out;
+
+  const int tid = threadIdx.x;
+  const int tx = tid & 15, ty = tid >> 4;
+
+  auto load_chunk = [&](int stage, int chunk) {
+    const int k0 = chunk * MP_BK;
+    T* as = As + stage * MP_BM * MP_ALD;
+    T* bs = Bs + stage * MP_BK * MP_BLD;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      int idx = tid + q * MP_NT;        // 0..1023
+      int row = idx >> 3, ch = idx & 7;  // A: 128 rows x 8 x 16B
+      cp_async16(as + row * MP_ALD + ch * 4, A + row * lda + k0 + ch * 4);
+    }
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      int idx = tid + q * MP_NT;
+      int row = idx >> 5, ch = idx & 31;  // B: 32 rows x 32 x 16B
+      cp_async16(bs + row * MP_BLD + ch * 4, B + (long long)(k0 + row) * ldb + ch * 4);
+    }
+  };
+
+  const int nk = args.K / MP_BK;
+#pragma unroll
+  for (int s = 0; s < MP_STAGES - 1; ++s) {
+    if (s < nk) load_chunk(s, s);
+    cp_async_commit();
+  }
+
+  T acc[8][8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
+    V4 v0 = *reinterpret_cast<const V4*>(Cin + r * ldc_in + tx * 4);
+    V4 v1 = *reinterpret_cast<const V4*>(Cin + r * ldc_in + 64 + tx * 4);
+    acc[i][0] = v0.x; acc[i][1] = v0.y; acc[i][2] = v0.z; acc[i][3] = v0.w;
+    acc[i][4] = v1.x; acc[i][5] = v1.y; acc[i][6] = v1.z; acc[i][7] = v1.w;
+  }
+
+  for (int c = 0; c < nk; ++c) {
+    cp_async_wait<MP_STAGES - 2>();
+    __syncthreads();
+    {
+      int cn = c + MP_STAGES - 1;
+      if (cn < nk) load_chunk(cn % MP_STAGES, cn);
+      cp_async_commit();
+    }
+    const T* as = As + (c % MP_STAGES) * MP_BM * MP_ALD;
+    const T* bs = Bs + (c % MP_STAGES) * MP_BK * MP_BLD;
+#pragma unroll
+    for (int k2 = 0; k2 < MP_BK / 2; ++k2) {
+      T a[8][2];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
+        const T* ap = as + r * MP_ALD + k2 * 2;
+        a[i][0] = ap[0]; a[i][1] = ap[1];
+      }
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const T* brow = bs + (k2 * 2 + u) * MP_BLD;
+        V4 b0 = *reinterpret_cast<const V4*>(brow + tx * 4);
+        V4 b1 = *reinterpret_cast<const V4*>(brow + 64 + tx * 4);
+        const T b[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+          for (int j = 0; j < 8; ++j) acc[i][j] = Val<T>::relax(a[i][u], b[j], acc[i][j]);
+      }
+    }
+  }
+  cp_async_wait<0>();
+
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
+    V4 v0, v1;
+    v0.x = acc[i][0]; v0.y = acc[i][1]; v0.z = acc[i][2]; v0.w = acc[i][3];
+    v1.x = acc[i][4]; v1.y = acc[i][5]; v1.z = acc[i][6]; v1.w = acc[i][7];
+    *reinterpret_cast<V4*>(Cout + r * ldc_out + tx * 4) = v0;
+    *reinterpret_cast<V4*>(Cout + r * ldc_out + 64 + tx * 4) = v1;
+  }
+}
+
+template <typename T>
+static long long desc_tiles(const MinPlusDesc<T>& d) {
+  return (long long)d.tiles_i * (long long)d.tiles_j;
+}
+
+template <typename T>
+cudaError_t launch_minplus(const MinPlusDesc<T>* d, int ndesc, int K, cudaStream_t s) {
+  if (K <= 0 || K % MP_BK) return cudaErrorInvalidValue;
+  MinPlusArgs<T> a;
+  a.d0 = d[0];
+  a.d1 = ndesc > 1 ? d[1] : d[0];
+  a.n0 = desc_tiles(d[0]);
+  a.K = K;
+  long long total = a.n0 + (ndesc > 1 ? desc_tiles(d[1]) : 0);
+  if (total <= 0) return cudaSuccess;
+  if (ndesc > 1 && a.n0 == 0) { a.d0 = a.d1; a.n0 = total; }
+  constexpr int smem = minplus_smem_bytes<T>();
+  minplus_kernel<T><<<(unsigned)total, MP_NT, smem, s>>>(a);
+  return cudaGetLastError();
+}
+
+// --------------------------------------------------------------- phase 1 --
+//
+// One CTA of 1024 threads closes a 128x128 tile in place: thread t owns row
+// r = t/8, columns c0..c0+15 (c0 = 16*(t%8)) in registers. Step kk needs the
+// current row kk and column kk; their owners publish them to a double-
+// buffered shared copy, one barrier per step. In-place is exact because
+// row kk and column kk do not change in step kk when A[kk][kk] = 0
+// (A[kk][kk] < 0 is a negative cycle: flagged, result unspecified).
+
+template <typename T>
+__global__ void __launch_bounds__(1024) phase1_kernel(T* tile, long long ld, int* negflag) {
+  using V4 = typename Vec4<T>::type;
+  __shared__ __align__(16) T rowbuf[2][kTile];
+  __shared__ T colbuf[2][kTile];
+  const int t = threadIdx.x;
+  const int r = t >> 3, cb_own = t & 7, c0 = cb_own * 16;
+  T v[16];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    V4 x = *reinterpret_cast<const V4*>(tile + r * ld + c0 + 4 * q);
+    v[4 * q] = x.x; v[4 * q + 1] = x.y; v[4 * q + 2] = x.z; v[4 * q + 3] = x.w;
+  }
+  bool neg = false;
+  for (int cb = 0; cb < 8; ++cb) {
+#pragma unroll
+    for (int u = 0; u < 16; ++u) {
+      const int kk = cb * 16 + u;
+      const int p = kk & 1;
+      if (r == kk) {
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          V4 x;
+          x.x = v[4 * q]; x.y = v[4 * q + 1]; x.z = v[4 * q + 2]; x.w = v[4 * q + 3];
+          *reinterpret_cast<V4*>(&rowbuf[p][c0 + 4 * q]) = x;
+        }
+      }
+      if (cb_own == cb) colbuf[p][r] = v[u];
+      __syncthreads();
+      if (r == kk && cb_own == cb && v[u] < T(0)) neg = true;
+      const T dik = colbuf[p][r];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        V4 x = *reinterpret_cast<const V4*>(&rowbuf[p][c0 + 4 * q]);
+        v[4 * q] = Val<T>::relax(dik, x.x, v[4 * q]);
+        v[4 * q + 1] = Val<T>::relax(dik, x.y, v[4 * q + 1]);
+        v[4 * q + 2] = Val<T>::relax(dik, x.z, v[4 * q + 2]);
+        v[4 * q + 3] = Val<T>::relax(dik, x.w, v[4 * q + 3]);
+      }
+    }
+  }
+  if (neg) *negflag = 1;
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    V4 x;
+    x.x = v[4 * q]; x.y = v[4 * q + 1]; x.z = v[4 * q + 2]; x.w = v[4 * q + 3];
+    *reinterpret_cast<V4*>(tile + r * ld + c0 + 4 * q) = x;
+  }
+}
+
+template <typename T>
+cudaError_t launch_phase1(T* tile, long long ld, int* negflag, cudaStream_t s) {
+  phase1_kernel<T><<<1, 1024, 0, s>>>(tile, ld, negflag);
+  return cudaGetLastError();
+}
+
+// ------------------------------------------------------------------ init --
+//
+// One CTA per row: fill the row with infinity (16-byte stores, 0 on the
+// diagonal), barrier, then scatter-min the row's arcs (duplicate arcs keep
+// the minimum; a self-loop gives min(0, w)).
+
+__device__ __forceinline__ void atomic_min_t(int* p, int v) { atomicMin(p, v); }
+__device__ __forceinline__ void atomic_min_t(float* p, float v) {
+  int* ip = reinterpret_cast<int*>(p);
+  int old = *ip;
+  while (v < __int_as_float(old)) {
+    int prev = atomicCAS(ip, old, __float_as_int(v));
+    if (prev == old) break;
+    old = prev;
+  }
+}
+
+template <typename T>
+__global__ void __launch_bounds__(256) init_rows_kernel(T* D, long long ld, long long n_pad, long long row_begin,
+                                                        long long n, const long long* __restrict__ row_ptr,
+                                                        long long row_ptr_base, const int* __restrict__ col,
+                                                        const T* __restrict__ w) {
+  using V4 = typename Vec4<T>::type;
+  const long long lr = blockIdx.x;
+  const long long r = row_begin + lr;
+  T* row = D + lr * ld;
+  const T INF = Val<T>::inf();
+  const long long q4 = n_pad >> 2;
+  for (long long q = threadIdx.x; q < q4; q += blockDim.x) {
+    V4 x;
+    x.x = INF; x.y = INF; x.z = INF; x.w = INF;
+    const long long c = q * 4;
+    if (r >= c && r < c + 4) {
+      const int o = (int)(r - c);
+      if (o == 0) x.x = T(0); else if (o == 1) x.y = T(0); else if (o == 2) x.z = T(0); else x.w = T(0);
+    }
+    reinterpret_cast<V4*>(row)[q] = x;
+  }
+  __syncthreads();
+  if (r < n) {
+    const long long e0 = row_ptr[lr] - row_ptr_base, e1 = row_ptr[lr + 1] - row_ptr_base;
+    for (long long e = e0 + threadIdx.x; e < e1; e += blockDim.x) atomic_min_t(row + col[e], w[e]);
+  }
+}
+
+template <typename T>
+cudaError_t launch_init_rows(T* D, long long ld, long long n_pad, long long row_begin, long long rows, long long n,
+                             const long long* row_ptr, long long row_ptr_base, const int* col, const T* w,
+                             cudaStream_t s) {
+  if (rows <= 0) return cudaSuccess;
+  init_rows_kernel<T><<<(unsigned)rows, 256, 0, s>>>(D, ld, n_pad, row_begin, n, row_ptr, row_ptr_base, col, w);
+  return cudaGetLastError();
+}
+
+// ---------------------------------------------------------- canonicalize --
+
+__global__ void canonicalize_kernel(int* D, long long ld, long long rows, long long cols) {
+  const int INF = 0x3FFFFFFF;
+  const long long total = rows * cols;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
+       i += (long long)gridDim.x * blockDim.x) {
+    long long r = i / cols, c = i - r * cols;
+    int* p = D + r * ld + c;
+    if (*p >= INF / 2) *p = INF;
+  }
+}
+
+cudaError_t launch_canonicalize_i32(int* D, long long ld, long long rows, long long cols, cudaStream_t s) {
+  if (rows <= 0 || cols <= 0) return cudaSuccess;
+  canonicalize_kernel<<<148 * 8, 256, 0, s>>>(D, ld, rows, cols);
+  return cudaGetLastError();
+}
+
+// --------------------------------------------------------- instantiations --
+
+cudaError_t configure_kernels() {
+  cudaError_t e = cudaFuncSetAttribute(minplus_kernel<int>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       minplus_smem_bytes<int>());
+  if (e != cudaSuccess) return e;
+  return cudaFuncSetAttribute(minplus_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              minplus_smem_bytes<float>());
+}
+
+template cudaError_t launch_minplus<int>(const MinPlusDesc<int>*, int, int, cudaStream_t);
+template cudaError_t launch_minplus<float>(const MinPlusDesc<float>*, int, int, cudaStream_t);
+template cudaError_t launch_phase1<int>(int*, long long, int*, cudaStream_t);
+template cudaError_t launch_phase1<float>(float*, long long, int*, cudaStream_t);
+template cudaError_t launch_init_rows<int>(int*, long long, long long, long long, long long, long long,
+                                           const long long*, long long, const int*, const int*, cudaStream_t);
+template cudaError_t launch_init_rows<float>(float*, long long, long long, long long, long long, long long,
+                                             const long long*, long long, const int*, const float*, cudaStream_t);
+
+}  // namespace apsp

@@ -1,0 +1,56 @@
+// apsp_kernels.cuh — internal interface between the schedulers (apsp_api.cu)
+// and the sm_100a kernels (apsp_kernels.cu). Not part of the C ABI.
+#pragma once
+#include <cuda_runtime.h>
+#include <cstdint>
+
+namespace apsp {
+
+constexpr int kTile = 128;  // b: tile edge = round depth ("b x b" blocks)
+
+// One rectangular family of output tiles for the min-plus kernel:
+//   Cout(ti,tj) = min(Cin(ti,tj), A(ti, 0:K) (x) B(0:K, tj))
+// where tile (ti, tj) has its top-left element at
+//   Cin  + ti*128*ldc_in  + tj*128      (same for Cout with ldc_out)
+//   A    + ti*128*lda                    (128 rows x K, row-major, A already at column 0 of the depth)
+//   B    + tj*128                        (K rows x 128, row-major)
+// ti runs over tiles_i values skipping skip_i (>= 0) and tj over tiles_j
+// values skipping skip_j (>= 0): tiles_i / tiles_j count the tiles AFTER the
+// skip, so ti in [0, tiles_i + (skip_i>=0)).
+template <typename T>
+struct MinPlusDesc {
+  T* Cout;
+  const T* Cin;
+  const T* A;
+  const T* B;
+  long long ldc_out, ldc_in, lda, ldb;
+  int tiles_i, tiles_j, skip_i, skip_j;
+};
+
+// Phase 2 / phase 3 / out-of-core products: up to two tile families in one
+// launch (grid = total tiles). K must be a positive multiple of 32.
+template <typename T>
+cudaError_t launch_minplus(const MinPlusDesc<T>* d, int ndesc, int K, cudaStream_t s);
+
+// Phase 1: in-place FW closure of one 128x128 tile (ld elements per row).
+// Sets *negflag = 1 if a diagonal element is negative when its step starts.
+template <typename T>
+cudaError_t launch_phase1(T* tile, long long ld, int* negflag, cudaStream_t s);
+
+// CSR -> dense init of `rows` rows starting at global row row_begin into D
+// (ld elements per row, n_pad columns). row_ptr is the LOCAL slice
+// (rows+1 entries, absolute arc offsets minus row_ptr_base).
+template <typename T>
+cudaError_t launch_init_rows(T* D, long long ld, long long n_pad, long long row_begin, long long rows,
+                             long long n, const long long* row_ptr, long long row_ptr_base,
+                             const int* col, const T* w, cudaStream_t s);
+
+// int32 only: values >= INF/2 become INF (drifted infinities under negative
+// weights, reading R5). rows x cols block at ld.
+cudaError_t launch_canonicalize_i32(int* D, long long ld, long long rows, long long cols, cudaStream_t s);
+
+// Per-device kernel attributes (dynamic shared memory opt-in). Call once per
+// device before the first launch.
+cudaError_t configure_kernels();
+
+}  // namespace apsp

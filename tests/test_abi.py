@@ -1,0 +1,89 @@
+"""C-ABI boundary checks that need no GPU: the library loads, exports every symbol
+include/apsp.h declares, validates its inputs on the host, and fails loudly
+(APSP_ECUDA, no CPU fallback) when no device is visible."""
+import os
+import re
+
+import numpy as np
+import pytest
+
+import graphgen as gg
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def header_functions():
+    src = open(os.path.join(ROOT, "include", "apsp.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(apsp_[a-z0-9_]+)\s*\(", src)))
+
+
+def test_library_exports_every_declared_symbol(lib):
+    import ctypes
+    names = header_functions()
+    assert "apsp_init_from_csr" in names and "apsp_fw_blocked" in names and "apsp_get_dist" in names
+    so = ctypes.CDLL(lib.LIB_PATH)
+    for name in names:
+        assert hasattr(so, name), name
+    assert set(names) == set(lib.EXPORTED_SYMBOLS)
+    assert "sm_100a" in lib.apsp_version()
+
+
+def test_config_struct_layout(lib):
+    import ctypes
+    cfg = lib.apsp_config_default()
+    assert cfg.struct_size == ctypes.sizeof(lib.apsp_config)
+    assert cfg.device == -1 and cfg.world_size == 1 and cfg.rank == 0
+
+
+@pytest.mark.parametrize("n,world", [(0, 1), (1, 1), (127, 1), (128, 1), (129, 1), (1000, 2), (65536, 8),
+                                     (300, 4), (131072, 8)])
+def test_partition(lib, n, world):
+    rows = []
+    for r in range(world):
+        n_pad, rb, rc = lib.apsp_partition(n, world, r)
+        assert n_pad % (128 * world) == 0 and n_pad >= max(n, 1) and n_pad - n < 128 * world + (n == 0) * 128
+        assert rb == r * n_pad // world
+        assert rc == max(0, min(rb + n_pad // world, n) - rb)
+        rows += list(range(rb, rb + rc))
+    assert rows == list(range(n))
+
+
+def _bad(lib, n, rp, col, w, status, dtype=None):
+    with pytest.raises(lib.ApspError) as e:
+        lib.apsp_init_from_csr(n, rp, col, w, dtype=dtype)
+    assert e.value.status == status, str(e.value)
+    assert lib.apsp_last_error() != ""
+
+
+def test_input_validation(lib):
+    E = lib.APSP_EINVAL
+    _bad(lib, 3, [0, 1, 0, 1], [1], [1], E)             # row_ptr not monotone
+    _bad(lib, 3, [1, 1, 1, 1], [], [], E)               # row_ptr[0] != 0
+    _bad(lib, 3, [0, 1, 1, 1], [3], [1], E)             # col out of range
+    _bad(lib, 3, [0, 1, 1, 1], [-1], [1], E)            # negative col
+    _bad(lib, 2, [0, 1, 1], [1], [np.nan], E, lib.APSP_F32)
+    _bad(lib, 2, [0, 1, 1], [1], [np.inf], E, lib.APSP_F32)
+
+
+def test_erange(lib):
+    # (n-1)*max|w| >= 2^30-1 with non-negative weights
+    _bad(lib, 3, [0, 1, 1, 1], [1], [600_000_000], lib.APSP_ERANGE)
+    # negative weights tighten the bound to 2^28
+    _bad(lib, 3, [0, 2, 2, 2], [1, 2], [-1, 140_000_000], lib.APSP_ERANGE)
+
+
+def _has_gpu():
+    try:
+        import torch
+        return torch.cuda.is_available()
+    except Exception:
+        return False
+
+
+@pytest.mark.skipif(_has_gpu(), reason="checks the no-GPU failure mode")
+def test_no_gpu_fails_loudly(lib):
+    g = gg.erdos_renyi(50, 200, seed=1)
+    with pytest.raises(lib.ApspError) as e:
+        lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w)
+    assert e.value.status == lib.APSP_ECUDA
