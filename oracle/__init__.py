@@ -57,8 +57,8 @@ def _load():
         for name, args in [
             ("oracle_init_i64", [I64, P, P, P, P]),
             ("oracle_init_f64", [I64, P, P, P, P]),
-            ("oracle_fw_i64", [I64, P, I64]),
-            ("oracle_fw_f64", [I64, P, I64]),
+            ("oracle_fw_i64", [I64, P, I64, I64]),
+            ("oracle_fw_f64", [I64, P, I64, I64]),
             ("oracle_dijkstra_rows_i64", [I64, P, P, P, I64, P, P]),
             ("oracle_dijkstra_rows_f64", [I64, P, P, P, I64, P, P]),
             ("oracle_bellman_ford_row_i64", [I64, P, P, P, I64, P]),
@@ -106,19 +106,20 @@ def init_f64(row_ptr, col, w) -> np.ndarray:
     return d
 
 
-def fw_dense_i64(d: np.ndarray, k_iters: int | None = None):
-    """Plain FW in place on an int64 matrix; returns negcycle flag."""
+def fw_dense_i64(d: np.ndarray, k_iters: int | None = None, k_begin: int = 0):
+    """Plain FW in place on an int64 matrix, outer iterations
+    k_begin .. k_iters-1 (default: all); returns the negative-cycle flag."""
     assert d.dtype == np.int64 and d.flags.c_contiguous and d.shape[0] == d.shape[1]
     n = d.shape[0]
     k = n if k_iters is None else int(k_iters)
-    return bool(_load().oracle_fw_i64(n, _p(d), k))
+    return bool(_load().oracle_fw_i64(n, _p(d), int(k_begin), k))
 
 
-def fw_dense_f64(d: np.ndarray, k_iters: int | None = None):
+def fw_dense_f64(d: np.ndarray, k_iters: int | None = None, k_begin: int = 0):
     assert d.dtype == np.float64 and d.flags.c_contiguous and d.shape[0] == d.shape[1]
     n = d.shape[0]
     k = n if k_iters is None else int(k_iters)
-    return bool(_load().oracle_fw_f64(n, _p(d), k))
+    return bool(_load().oracle_fw_f64(n, _p(d), int(k_begin), k))
 
 
 def fw_i64(row_ptr, col, w, k_iters: int | None = None):

@@ -78,13 +78,14 @@ void oracle_init_f64(int64_t n, const int64_t* row_ptr, const int32_t* col,
 
 /* ------------------------------------------------------ Floyd–Warshall -- */
 
-/* Plain FW. Runs outer iterations k = 0 .. k_iters-1.
+/* Plain FW. Runs outer iterations k = k_begin .. k_end-1
+ * (k_begin > 0 continues an earlier call on the same matrix).
  * Returns 1 if a negative cycle was detected (dist unspecified), else 0.
  * The i-loop of one outer iteration is split over OpenMP threads: row k and
  * column k do not change during iteration k when dist[k][k] == 0, so the rows
  * are independent within an iteration. */
-int oracle_fw_i64(int64_t n, int64_t* dist, int64_t k_iters) {
-  for (int64_t k = 0; k < k_iters; ++k) {
+int oracle_fw_i64(int64_t n, int64_t* dist, int64_t k_begin, int64_t k_end) {
+  for (int64_t k = k_begin; k < k_end; ++k) {
     if (dist[k * n + k] < 0) return 1;
     const int64_t* rowk = dist + k * n;
 #pragma omp parallel for schedule(static)
@@ -102,8 +103,8 @@ int oracle_fw_i64(int64_t n, int64_t* dist, int64_t k_iters) {
   return 0;
 }
 
-int oracle_fw_f64(int64_t n, double* dist, int64_t k_iters) {
-  for (int64_t k = 0; k < k_iters; ++k) {
+int oracle_fw_f64(int64_t n, double* dist, int64_t k_begin, int64_t k_end) {
+  for (int64_t k = k_begin; k < k_end; ++k) {
     if (dist[k * n + k] < 0) return 1;
     const double* rowk = dist + k * n;
 #pragma omp parallel for schedule(static)

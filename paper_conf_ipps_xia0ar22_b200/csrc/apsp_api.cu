@@ -13,6 +13,7 @@
 //                         B rows streamed from pinned host memory
 //                         (apsp_ooc.cu).
 #include "apsp_internal.h"
+#include "apsp_sched.cuh"
 
 #include <cstdio>
 #include <cstring>
@@ -55,19 +56,19 @@ apsp_status Handle::cuda(cudaError_t e, const char* what) {
   return fail(e == cudaErrorMemoryAllocation ? APSP_ENOMEM : APSP_ECUDA, "%s: %s", what, cudaGetErrorString(e));
 }
 
-void Handle::ev_begin(int cls) {
+void Handle::ev_begin(int cls, cudaStream_t s) {
   if (!timing) return;
   TimedEvent te;
   te.cls = cls;
   cudaEventCreate(&te.a);
   cudaEventCreate(&te.b);
-  cudaEventRecord(te.a, stream);
+  cudaEventRecord(te.a, s);
   events.push_back(te);
 }
 
-void Handle::ev_end(double relax) {
+void Handle::ev_end(double relax, cudaStream_t s) {
   if (!timing || events.empty()) return;
-  cudaEventRecord(events.back().b, stream);
+  cudaEventRecord(events.back().b, s);
   events.back().relax = relax;
 }
 
@@ -83,23 +84,6 @@ void Handle::collect_events() {
     cudaEventDestroy(te.b);
   }
   events.clear();
-}
-
-// --------------------------------------------------------- kernel helpers --
-
-template <typename T>
-static MinPlusDesc<T> mkdesc(T* Cout, const T* Cin, const T* A, const T* B, long long ldc, long long lda,
-                             long long ldb, int tiles_i, int tiles_j, int skip_i, int skip_j) {
-  MinPlusDesc<T> d;
-  d.Cout = Cout; d.Cin = Cin; d.A = A; d.B = B;
-  d.ldc_out = ldc; d.ldc_in = ldc; d.lda = lda; d.ldb = ldb;
-  d.tiles_i = tiles_i; d.tiles_j = tiles_j; d.skip_i = skip_i; d.skip_j = skip_j;
-  return d;
-}
-
-template <typename T>
-static double desc_relax(const MinPlusDesc<T>& d, int K) {
-  return (double)d.tiles_i * d.tiles_j * kTile * kTile * (double)K;
 }
 
 // One round k of the in-core blocked FW over this handle's shards.
@@ -121,22 +105,6 @@ static apsp_status incore_round(Handle* h, long long k) {
     h->ev_begin(0);
     if ((st = h->cuda(launch_phase1<T>(band + k * b, ld, h->d_flag, s), "phase1"))) return st;
     h->ev_end((double)b * b * b);
-    if (h->world == 1) {
-      // phase 2: row panel A(k,j) and column panel A(i,k) in one launch
-      MinPlusDesc<T> d[2];
-      d[0] = mkdesc<T>(band, band, band + k * b, band, ld, ld, ld, 1, (int)(nb - 1), -1, (int)k);
-      T* D = static_cast<T*>(own->D);
-      d[1] = mkdesc<T>(D + k * b, D + k * b, D + k * b, band + k * b, ld, ld, ld, (int)(nb - 1), 1, (int)k, -1);
-      h->ev_begin(1);
-      if ((st = h->cuda(launch_minplus<T>(d, 2, (int)b, s), "phase2"))) return st;
-      h->ev_end(desc_relax(d[0], (int)b) + desc_relax(d[1], (int)b));
-      // phase 3
-      MinPlusDesc<T> p3 = mkdesc<T>(D, D, D + k * b, band, ld, ld, ld, (int)(nb - 1), (int)(nb - 1), (int)k, (int)k);
-      h->ev_begin(2);
-      if ((st = h->cuda(launch_minplus<T>(&p3, 1, (int)b, s), "phase3"))) return st;
-      h->ev_end(desc_relax(p3, (int)b));
-      return APSP_OK;
-    }
     MinPlusDesc<T> dr = mkdesc<T>(band, band, band + k * b, band, ld, ld, ld, 1, (int)(nb - 1), -1, (int)k);
     h->ev_begin(1);
     if ((st = h->cuda(launch_minplus<T>(&dr, 1, (int)b, s), "phase2-row"))) return st;
@@ -177,6 +145,11 @@ static apsp_status incore_round(Handle* h, long long k) {
 }
 
 apsp_status run_incore_rounds(Handle* h, long long k0, long long k1) {
+  if (h->world == 1) {  // single GPU: the whole closure, with lookahead
+    return h->dtype == APSP_I32
+               ? fw_closure<int>(h, static_cast<int*>(h->shards[0].D), h->ld, h->n_pad, k0, k1, h->stream)
+               : fw_closure<float>(h, static_cast<float*>(h->shards[0].D), h->ld, h->n_pad, k0, k1, h->stream);
+  }
   for (long long k = k0; k < k1; ++k) {
     apsp_status st = (h->dtype == APSP_I32) ? incore_round<int>(h, k) : incore_round<float>(h, k);
     if (st) return st;

@@ -99,6 +99,13 @@ apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_pt
     if ((st = h->cuda(cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking), "cudaStreamCreate"))) return st;
     h->own_stream = true;
   }
+  if (!cfg.reserved[1]) {  // reserved[1] = 1 disables the lookahead (tests / A-B timing)
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);
+    if ((st = h->cuda(cudaStreamCreateWithPriority(&h->side, cudaStreamNonBlocking, hi), "side stream"))) return st;
+    for (auto& e : h->ev_la)
+      if ((st = h->cuda(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event"))) return st;
+  }
 
   int64_t np, rb, rc;
   if (apsp_partition(h->n, h->b, h->world, h->virt ? 0 : h->rank, &np, &rb, &rc) != APSP_OK)
@@ -174,6 +181,12 @@ void delete_handle(Handle* h) {
   cudaFree(h->panel);
   cudaFree(h->d_flag);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
+  if (h->side) {
+    cudaStreamSynchronize(h->side);
+    cudaStreamDestroy(h->side);
+  }
+  for (auto& e : h->ev_la)
+    if (e) cudaEventDestroy(e);
   delete h;
 }
 

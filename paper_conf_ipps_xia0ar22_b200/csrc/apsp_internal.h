@@ -41,6 +41,8 @@ struct Handle {
   long long rows_per_rank = 0, ld = 0;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
+  cudaStream_t side = nullptr;        // high-priority stream for lookahead phases 1+2
+  cudaEvent_t ev_la[2] = {nullptr, nullptr};
   std::vector<Shard> shards;
   void* d_base = nullptr;   // allocation behind the shards (in-core)
   void* panel = nullptr;    // b x ld pivot band received from the owner
@@ -65,8 +67,10 @@ struct Handle {
   apsp_status cuda(cudaError_t e, const char* what);
   apsp_status bcast(void* buf, size_t bytes, int root);
   // class: 0 phase1, 1 phase2, 2 phase3, 3 comm / host transfer
-  void ev_begin(int cls);
-  void ev_end(double relax);
+  void ev_begin(int cls, cudaStream_t s);
+  void ev_end(double relax, cudaStream_t s);
+  void ev_begin(int cls) { ev_begin(cls, stream); }
+  void ev_end(double relax) { ev_end(relax, stream); }
   void collect_events();
 };
 

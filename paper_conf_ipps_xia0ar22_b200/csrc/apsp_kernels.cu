@@ -91,7 +91,9 @@ __global__ void __launch_bounds__(MP_NT, 2) minplus_kernel(const __grid_constant
   int ti = (int)(t / d.tiles_j);
   int tj = (int)(t - (long long)ti * d.tiles_j);
   if (d.skip_i >= 0 && ti >= d.skip_i) ++ti;
+  if (d.skip_i2 >= 0 && ti >= d.skip_i2) ++ti;
   if (d.skip_j >= 0 && tj >= d.skip_j) ++tj;
+  if (d.skip_j2 >= 0 && tj >= d.skip_j2) ++tj;
 
   const T* __restrict__ Cin = d.Cin + (long long)ti * MP_BM * d.ldc_in + (long long)tj * MP_BN;
   T* __restrict__ Cout = d.Cout + (long long)ti * MP_BM * d.ldc_out + (long long)tj * MP_BN;
@@ -205,66 +207,85 @@ cudaError_t launch_minplus(const MinPlusDesc<T>* d, int ndesc, int K, cudaStream
 
 // --------------------------------------------------------------- phase 1 --
 //
-// One CTA of 1024 threads closes a 128x128 tile in place: thread t owns row
-// r = t/8, columns c0..c0+15 (c0 = 16*(t%8)) in registers. Step kk needs the
-// current row kk and column kk; their owners publish them to a double-
-// buffered shared copy, one barrier per step. In-place is exact because
-// row kk and column kk do not change in step kk when A[kk][kk] = 0
-// (A[kk][kk] < 0 is a negative cycle: flagged, result unspecified).
+// One CTA of 256 threads closes a 128x128 tile in place with the plain FW
+// recurrence (PAPER.md:60 restricted to the tile). Thread (ty, tx) keeps the
+// same 8x8 register block as the min-plus kernel: rows {4ty..4ty+3,
+// 64+4ty..64+4ty+3} x columns {4tx..4tx+3, 64+4tx..64+4tx+3}. Step kk needs
+// column kk and row kk; their owners publish them (two 16-byte stores each)
+// to a double-buffered shared copy, then one barrier, then every thread does
+// 64 relaxations. In place is exact because row kk and column kk do not change
+// in step kk when A[kk][kk] = 0; A[kk][kk] < 0 at the start of step kk is a
+// negative cycle (flagged; the result is then unspecified).
 
 template <typename T>
-__global__ void __launch_bounds__(1024) phase1_kernel(T* tile, long long ld, int* negflag) {
+__global__ void __launch_bounds__(256) phase1_kernel(T* tile, long long ld, int* negflag) {
   using V4 = typename Vec4<T>::type;
   __shared__ __align__(16) T rowbuf[2][kTile];
-  __shared__ T colbuf[2][kTile];
-  const int t = threadIdx.x;
-  const int r = t >> 3, cb_own = t & 7, c0 = cb_own * 16;
-  T v[16];
+  __shared__ __align__(16) T colbuf[2][kTile];
+  const int tid = threadIdx.x;
+  const int tx = tid & 15, ty = tid >> 4;
+  T acc[8][8];
 #pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    V4 x = *reinterpret_cast<const V4*>(tile + r * ld + c0 + 4 * q);
-    v[4 * q] = x.x; v[4 * q + 1] = x.y; v[4 * q + 2] = x.z; v[4 * q + 3] = x.w;
+  for (int i = 0; i < 8; ++i) {
+    const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
+    V4 v0 = *reinterpret_cast<const V4*>(tile + r * ld + tx * 4);
+    V4 v1 = *reinterpret_cast<const V4*>(tile + r * ld + 64 + tx * 4);
+    acc[i][0] = v0.x; acc[i][1] = v0.y; acc[i][2] = v0.z; acc[i][3] = v0.w;
+    acc[i][4] = v1.x; acc[i][5] = v1.y; acc[i][6] = v1.z; acc[i][7] = v1.w;
   }
   bool neg = false;
-  for (int cb = 0; cb < 8; ++cb) {
 #pragma unroll
-    for (int u = 0; u < 16; ++u) {
-      const int kk = cb * 16 + u;
-      const int p = kk & 1;
-      if (r == kk) {
+  for (int half = 0; half < 2; ++half) {
+    for (int q = 0; q < 16; ++q) {
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-          V4 x;
-          x.x = v[4 * q]; x.y = v[4 * q + 1]; x.z = v[4 * q + 2]; x.w = v[4 * q + 3];
-          *reinterpret_cast<V4*>(&rowbuf[p][c0 + 4 * q]) = x;
+      for (int u = 0; u < 4; ++u) {
+        const int kk = half * 64 + q * 4 + u;
+        const int p = u & 1;  // kk & 1
+        const int io = half * 4 + u;  // register row / column of kk for its owners
+        if (ty == q) {  // row kk lives in this thread's rows: publish my 8 columns of it
+          V4 x0, x1;
+          x0.x = acc[io][0]; x0.y = acc[io][1]; x0.z = acc[io][2]; x0.w = acc[io][3];
+          x1.x = acc[io][4]; x1.y = acc[io][5]; x1.z = acc[io][6]; x1.w = acc[io][7];
+          *reinterpret_cast<V4*>(&rowbuf[p][tx * 4]) = x0;
+          *reinterpret_cast<V4*>(&rowbuf[p][64 + tx * 4]) = x1;
         }
-      }
-      if (cb_own == cb) colbuf[p][r] = v[u];
-      __syncthreads();
-      if (r == kk && cb_own == cb && v[u] < T(0)) neg = true;
-      const T dik = colbuf[p][r];
+        if (tx == q) {  // column kk: publish my 8 rows of it
+          V4 y0, y1;
+          y0.x = acc[0][io]; y0.y = acc[1][io]; y0.z = acc[2][io]; y0.w = acc[3][io];
+          y1.x = acc[4][io]; y1.y = acc[5][io]; y1.z = acc[6][io]; y1.w = acc[7][io];
+          *reinterpret_cast<V4*>(&colbuf[p][ty * 4]) = y0;
+          *reinterpret_cast<V4*>(&colbuf[p][64 + ty * 4]) = y1;
+        }
+        __syncthreads();
+        if (tid == 0 && rowbuf[p][kk] < T(0)) neg = true;
+        const V4 a0 = *reinterpret_cast<const V4*>(&colbuf[p][ty * 4]);
+        const V4 a1 = *reinterpret_cast<const V4*>(&colbuf[p][64 + ty * 4]);
+        const V4 b0 = *reinterpret_cast<const V4*>(&rowbuf[p][tx * 4]);
+        const V4 b1 = *reinterpret_cast<const V4*>(&rowbuf[p][64 + tx * 4]);
+        const T a[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+        const T bb[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
 #pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        V4 x = *reinterpret_cast<const V4*>(&rowbuf[p][c0 + 4 * q]);
-        v[4 * q] = Val<T>::relax(dik, x.x, v[4 * q]);
-        v[4 * q + 1] = Val<T>::relax(dik, x.y, v[4 * q + 1]);
-        v[4 * q + 2] = Val<T>::relax(dik, x.z, v[4 * q + 2]);
-        v[4 * q + 3] = Val<T>::relax(dik, x.w, v[4 * q + 3]);
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+          for (int j = 0; j < 8; ++j) acc[i][j] = Val<T>::relax(a[i], bb[j], acc[i][j]);
       }
     }
   }
   if (neg) *negflag = 1;
 #pragma unroll
-  for (int q = 0; q < 4; ++q) {
-    V4 x;
-    x.x = v[4 * q]; x.y = v[4 * q + 1]; x.z = v[4 * q + 2]; x.w = v[4 * q + 3];
-    *reinterpret_cast<V4*>(tile + r * ld + c0 + 4 * q) = x;
+  for (int i = 0; i < 8; ++i) {
+    const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
+    V4 v0, v1;
+    v0.x = acc[i][0]; v0.y = acc[i][1]; v0.z = acc[i][2]; v0.w = acc[i][3];
+    v1.x = acc[i][4]; v1.y = acc[i][5]; v1.z = acc[i][6]; v1.w = acc[i][7];
+    *reinterpret_cast<V4*>(tile + r * ld + tx * 4) = v0;
+    *reinterpret_cast<V4*>(tile + r * ld + 64 + tx * 4) = v1;
   }
 }
 
 template <typename T>
 cudaError_t launch_phase1(T* tile, long long ld, int* negflag, cudaStream_t s) {
-  phase1_kernel<T><<<1, 1024, 0, s>>>(tile, ld, negflag);
+  phase1_kernel<T><<<1, 256, 0, s>>>(tile, ld, negflag);
   return cudaGetLastError();
 }
 

@@ -25,6 +25,7 @@ struct MinPlusDesc {
   const T* B;
   long long ldc_out, ldc_in, lda, ldb;
   int tiles_i, tiles_j, skip_i, skip_j;
+  int skip_i2 = -1, skip_j2 = -1;  // optional second skipped index, > skip_i / skip_j
 };
 
 // Phase 2 / phase 3 / out-of-core products: up to two tile families in one

@@ -1,0 +1,89 @@
+"""Out-of-core path (Algorithm 1) at small n, forced by a device
+budget / force_out_of_core, bit-exact against the oracle (and vs the in-core path)."""
+import numpy as np
+import pytest
+
+import graphgen as gg
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+INF32 = 0x3FFFFFFF
+
+
+def ooc_cfg(lib, block, budget_mb=0, stream_all=True):
+    c = lib.apsp_config_default(device=0, force_out_of_core=1, ooc_block=block, timing=1)
+    if budget_mb:
+        c.device_budget_bytes = int(budget_mb * 2 ** 20)
+    if stream_all:
+        c.reserved[0] = 1
+    return c
+
+
+def oracle_i32(g):
+    d, neg = oracle.fw_i64(g.row_ptr, g.col, g.w)
+    return np.where(d == oracle.INF_I64, INF32, d), neg
+
+
+@pytest.mark.parametrize("n,block", [(1000, 256), (700, 128), (1536, 512), (300, 128)])
+def test_ooc_int32_bit_exact(lib, n, block):
+    g = gg.grid_2d(max(2, n // 25), 25, seed=n) if n % 2 == 0 else gg.erdos_renyi(n, 4 * n, seed=n)
+    with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=ooc_cfg(lib, block)) as h:
+        info = lib.apsp_get_info(h)
+        assert info.mode == lib.APSP_MODE_OUT_OF_CORE and info.ooc_block == block
+        assert info.host_bytes > 0
+        lib.apsp_fw_blocked(h)
+        got = lib.apsp_get_dist(h)
+        st = lib.apsp_get_phase_stats(h)
+    want, _ = oracle_i32(g)
+    assert np.array_equal(got.astype(np.int64), want)
+    assert st.launches[3] > 0  # host transfers happened
+    assert abs(sum(st.relax[:3]) - float(info.n_pad) ** 3) < 1
+
+
+def test_ooc_with_resident_bands(lib):
+    g = gg.erdos_renyi(1024, 6000, seed=3)
+    # n_pad=1024, B=256: band = 1 MiB; budget leaves room for 2 resident bands
+    with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w,
+                                cfg=ooc_cfg(lib, 256, budget_mb=6.5, stream_all=False)) as h:
+        info = lib.apsp_get_info(h)
+        assert info.mode == lib.APSP_MODE_OUT_OF_CORE
+        assert 0 < info.host_bytes < 1024 * 1024 * 4
+        lib.apsp_fw_blocked(h)
+        got = lib.apsp_get_dist(h)
+        part = lib.apsp_get_dist(h, 200, 300)
+    want, _ = oracle_i32(g)
+    assert np.array_equal(got.astype(np.int64), want)
+    assert np.array_equal(part.astype(np.int64), want[200:500])
+
+
+def test_ooc_negative_weights_and_cycle(lib):
+    rng = np.random.default_rng(0)
+    g0 = gg.erdos_renyi(640, 3000, seed=1)
+    p = rng.integers(-300, 300, size=g0.n)
+    s, t, w = g0.arcs()
+    g = gg.csr_from_arcs(g0.n, s, t, (w.astype(np.int64) + p[s] - p[t]).astype(np.int32))
+    with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=ooc_cfg(lib, 128)) as h:
+        lib.apsp_fw_blocked(h)
+        got = lib.apsp_get_dist(h)
+    want, _ = oracle_i32(g)
+    assert np.array_equal(got.astype(np.int64), want)
+    gc = gg.with_arcs(g0, [500, 20], [20, 500], [-200, 50])
+    with lib.apsp_init_from_csr(gc.n, gc.row_ptr, gc.col, gc.w, cfg=ooc_cfg(lib, 128)) as h:
+        with pytest.raises(lib.NegativeCycleError):
+            lib.apsp_fw_blocked(h)
+
+
+def test_ooc_f32_and_reinit(lib):
+    g = gg.erdos_renyi(800, 8000, seed=5, dtype="f32")
+    with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=ooc_cfg(lib, 256)) as h:
+        lib.apsp_fw_blocked(h)
+        a = lib.apsp_get_dist(h)
+        lib.apsp_reinit(h)
+        lib.apsp_fw_blocked(h)
+        b = lib.apsp_get_dist(h)
+    assert np.array_equal(a, b)
+    want, _ = oracle.fw_f64(g.row_ptr, g.col, g.w)
+    fin = np.isfinite(want)
+    assert np.array_equal(np.isfinite(a), fin)
+    assert np.all(np.abs(a[fin] - want[fin]) <= 1e-5 * np.abs(want[fin]))

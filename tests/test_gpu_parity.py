@@ -82,6 +82,17 @@ def test_fw_int32_bit_exact(lib, n):
         assert_i32_equal(got, want)
 
 
+@pytest.mark.parametrize("n", [384, 640, 1000])
+def test_fw_without_lookahead(lib, n):
+    """reserved[1] = 1 runs phases 1-3 strictly in order on one stream (no split phase 3)."""
+    for name, g in graphs_for(n, seed=n + 7):
+        c = cfg(lib)
+        c.reserved[1] = 1
+        got = lib.solve(g, cfg=c)
+        want, _ = oracle_i32(g)
+        assert_i32_equal(got, want)
+
+
 @pytest.mark.parametrize("seed", [0, 1, 2])
 def test_fw_negative_weights_reweighted(lib, seed):
     """Potential-reweighted arcs are negative but no cycle is; INF must stay canonical."""

@@ -201,6 +201,9 @@ def test_partial_fw_restricted_intermediates(seed):
         d, _ = oracle.fw_i64(g.row_ptr, g.col, g.w, k_iters=K)
         bf, _ = brute_force(n, arcs, allowed_mid=set(range(K)))
         assert np.array_equal(d, bf), K
+        # continuing from iteration K reaches the full result
+        oracle.fw_dense_i64(d, n, k_begin=K)
+        assert np.array_equal(d, brute_force(n, arcs)[0]), K
 
 
 # --------------------------------------------------- independent algorithms
