@@ -145,7 +145,7 @@ static apsp_status incore_round(Handle* h, long long k) {
 }
 
 apsp_status run_incore_rounds(Handle* h, long long k0, long long k1) {
-  if (h->world == 1) {  // single GPU: the whole closure, with lookahead
+  if (h->world == 1 && !h->use_comm) {  // single GPU: the whole closure, with lookahead
     return h->dtype == APSP_I32
                ? fw_closure<int>(h, static_cast<int*>(h->shards[0].D), h->ld, h->n_pad, k0, k1, h->stream)
                : fw_closure<float>(h, static_cast<float*>(h->shards[0].D), h->ld, h->n_pad, k0, k1, h->stream);

@@ -147,9 +147,18 @@ apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_pt
     h->shards.push_back(sh);
   }
 
-  if (h->world > 1 && !h->virt) {
+  // reserved[2] = 1: run the sharded schedule with a 1-rank NCCL communicator even
+  // at world_size 1, so a single GPU exercises the broadcast / all-reduce path
+  h->use_comm = (h->world > 1 && !h->virt) || (h->world == 1 && cfg.reserved[2] == 1);
+  if (h->use_comm) {
     ncclUniqueId id;
-    memcpy(&id, cfg.nccl_unique_id, sizeof(id));
+    if (cfg.nccl_unique_id) {
+      memcpy(&id, cfg.nccl_unique_id, sizeof(id));
+    } else if (h->world == 1) {
+      if (ncclGetUniqueId(&id) != ncclSuccess) return h->fail(APSP_ENCCL, "ncclGetUniqueId failed");
+    } else {
+      return h->fail(APSP_EINVAL, "nccl_unique_id is NULL");
+    }
     ncclComm_t comm;
     ncclResult_t r = ncclCommInitRank(&comm, h->world, id, h->rank);
     if (r != ncclSuccess) return h->fail(APSP_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
@@ -193,7 +202,7 @@ void delete_handle(Handle* h) {
 apsp_status finish_fw(Handle* h, bool all_rounds) {
   apsp_status st;
   int flag = 0;
-  if (h->world > 1 && !h->virt) {
+  if (h->use_comm) {
     ncclResult_t r = ncclAllReduce(h->d_flag, h->d_flag, 1, ncclInt32, ncclMax, static_cast<ncclComm_t>(h->comm),
                                    h->stream);
     if (r != ncclSuccess) return h->fail(APSP_ENCCL, "ncclAllReduce(flag): %s", ncclGetErrorString(r));

@@ -38,6 +38,7 @@ struct Handle {
   int device = 0;
   int world = 1, rank = 0;
   bool virt = false;
+  bool use_comm = false;    // NCCL communicator present (world > 1, or forced at world 1)
   long long rows_per_rank = 0, ld = 0;
   cudaStream_t stream = nullptr;
   bool own_stream = false;

@@ -64,6 +64,9 @@ __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_gr
 constexpr int MP_BM = 128, MP_BN = 128, MP_BK = 32, MP_NT = 256, MP_STAGES = 3;
 constexpr int MP_ALD = MP_BK + 4;
 constexpr int MP_BLD = MP_BN;
+constexpr int MP_STAGE_ELEMS = MP_BM * MP_ALD + MP_BK * MP_BLD;  // 8704 words = 34 KB
+constexpr int MP_CLD = MP_BN + 4;  // C tile rows staged in smem (64 rows per stage)
+static_assert(64 * MP_CLD <= MP_STAGE_ELEMS, "half a C tile must fit one stage");
 
 template <typename T>
 struct MinPlusArgs {
@@ -74,15 +77,15 @@ struct MinPlusArgs {
 
 template <typename T>
 constexpr int minplus_smem_bytes() {
-  return MP_STAGES * (MP_BM * MP_ALD + MP_BK * MP_BLD) * (int)sizeof(T);
+  return MP_STAGES * MP_STAGE_ELEMS * (int)sizeof(T);
 }
 
 template <typename T>
 __global__ void __launch_bounds__(MP_NT, 2) minplus_kernel(const __grid_constant__ MinPlusArgs<T> args) {
   using V4 = typename Vec4<T>::type;
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  T* As = reinterpret_cast<T*>(smem_raw);
-  T* Bs = As + MP_STAGES * MP_BM * MP_ALD;
+  // stage s = [A chunk 128 x 36][B chunk 32 x 128], contiguous
+  T* const stage0 = reinterpret_cast<T*>(smem_raw);
 
   long long t = blockIdx.x;
   const bool second = t >= args.n0;
@@ -104,22 +107,20 @@ __global__ void __launch_bounds__(MP_NT, 2) minplus_kernel(const __grid_constant
   const int tid = threadIdx.x;
   const int tx = tid & 15, ty = tid >> 4;
 
+  // per-thread copy coordinates: A chunk = 128 rows x 8 x 16B (rows tid/8 + 32q),
+  // B chunk = 32 rows x 32 x 16B (rows tid/32 + 8q)
+  const T* const a_src = A + (tid >> 3) * lda + (tid & 7) * 4;
+  const T* const b_src = B + (tid >> 5) * ldb + (tid & 31) * 4;
+  const int a_dst = (tid >> 3) * MP_ALD + (tid & 7) * 4;
+  const int b_dst = MP_BM * MP_ALD + (tid >> 5) * MP_BLD + (tid & 31) * 4;
   auto load_chunk = [&](int stage, int chunk) {
-    const int k0 = chunk * MP_BK;
-    T* as = As + stage * MP_BM * MP_ALD;
-    T* bs = Bs + stage * MP_BK * MP_BLD;
+    T* st = stage0 + stage * MP_STAGE_ELEMS;
+    const T* ag = a_src + chunk * MP_BK;
+    const T* bg = b_src + (long long)chunk * MP_BK * ldb;
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      int idx = tid + q * MP_NT;        // 0..1023
-      int row = idx >> 3, ch = idx & 7;  // A: 128 rows x 8 x 16B
-      cp_async16(as + row * MP_ALD + ch * 4, A + row * lda + k0 + ch * 4);
-    }
+    for (int q = 0; q < 4; ++q) cp_async16(st + a_dst + q * 32 * MP_ALD, ag + q * 32 * lda);
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      int idx = tid + q * MP_NT;
-      int row = idx >> 5, ch = idx & 31;  // B: 32 rows x 32 x 16B
-      cp_async16(bs + row * MP_BLD + ch * 4, B + (long long)(k0 + row) * ldb + ch * 4);
-    }
+    for (int q = 0; q < 4; ++q) cp_async16(st + b_dst + q * 8 * MP_BLD, bg + q * 8 * ldb);
   };
 
   const int nk = args.K / MP_BK;
@@ -129,15 +130,17 @@ __global__ void __launch_bounds__(MP_NT, 2) minplus_kernel(const __grid_constant
     cp_async_commit();
   }
 
+  // The accumulators start at +infinity and C is folded in at the end:
+  // min is exact, so min(C, min_kk(a + b)) equals the in-order update. C is
+  // fetched by cp.async into the two stages that are free during the last
+  // chunk, so its HBM latency hides behind that chunk's relaxations.
   T acc[8][8];
 #pragma unroll
-  for (int i = 0; i < 8; ++i) {
-    const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
-    V4 v0 = *reinterpret_cast<const V4*>(Cin + r * ldc_in + tx * 4);
-    V4 v1 = *reinterpret_cast<const V4*>(Cin + r * ldc_in + 64 + tx * 4);
-    acc[i][0] = v0.x; acc[i][1] = v0.y; acc[i][2] = v0.z; acc[i][3] = v0.w;
-    acc[i][4] = v1.x; acc[i][5] = v1.y; acc[i][6] = v1.z; acc[i][7] = v1.w;
-  }
+  for (int i = 0; i < 8; ++i)
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[i][j] = Val<T>::inf();
+  T* const cs_lo = stage0 + (nk % MP_STAGES) * MP_STAGE_ELEMS;        // C rows 0..63
+  T* const cs_hi = stage0 + ((nk + 1) % MP_STAGES) * MP_STAGE_ELEMS;  // C rows 64..127
 
   for (int c = 0; c < nk; ++c) {
     cp_async_wait<MP_STAGES - 2>();
@@ -145,10 +148,18 @@ __global__ void __launch_bounds__(MP_NT, 2) minplus_kernel(const __grid_constant
     {
       int cn = c + MP_STAGES - 1;
       if (cn < nk) load_chunk(cn % MP_STAGES, cn);
+      if (c == nk - 1) {  // C tile: 128 rows x 32 x 16B, rows tid/32 + 8q
+        const T* cg = Cin + (tid >> 5) * ldc_in + (tid & 31) * 4;
+        const int cd = (tid >> 5) * MP_CLD + (tid & 31) * 4;
+#pragma unroll
+        for (int q = 0; q < 8; ++q) cp_async16(cs_lo + cd + q * 8 * MP_CLD, cg + q * 8 * ldc_in);
+#pragma unroll
+        for (int q = 0; q < 8; ++q) cp_async16(cs_hi + cd + q * 8 * MP_CLD, cg + (64 + q * 8) * ldc_in);
+      }
       cp_async_commit();
     }
-    const T* as = As + (c % MP_STAGES) * MP_BM * MP_ALD;
-    const T* bs = Bs + (c % MP_STAGES) * MP_BK * MP_BLD;
+    const T* as = stage0 + (c % MP_STAGES) * MP_STAGE_ELEMS;
+    const T* bs = as + MP_BM * MP_ALD;
 #pragma unroll
     for (int k2 = 0; k2 < MP_BK / 2; ++k2) {
       T a[8][2];
@@ -172,13 +183,19 @@ __global__ void __launch_bounds__(MP_NT, 2) minplus_kernel(const __grid_constant
     }
   }
   cp_async_wait<0>();
+  __syncthreads();
 
 #pragma unroll
   for (int i = 0; i < 8; ++i) {
     const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
+    const T* crow = (i < 4 ? cs_lo : cs_hi) + (ty * 4 + (i & 3)) * MP_CLD;
+    V4 c0 = *reinterpret_cast<const V4*>(crow + tx * 4);
+    V4 c1 = *reinterpret_cast<const V4*>(crow + 64 + tx * 4);
     V4 v0, v1;
-    v0.x = acc[i][0]; v0.y = acc[i][1]; v0.z = acc[i][2]; v0.w = acc[i][3];
-    v1.x = acc[i][4]; v1.y = acc[i][5]; v1.z = acc[i][6]; v1.w = acc[i][7];
+    v0.x = Val<T>::vmin(acc[i][0], c0.x); v0.y = Val<T>::vmin(acc[i][1], c0.y);
+    v0.z = Val<T>::vmin(acc[i][2], c0.z); v0.w = Val<T>::vmin(acc[i][3], c0.w);
+    v1.x = Val<T>::vmin(acc[i][4], c1.x); v1.y = Val<T>::vmin(acc[i][5], c1.y);
+    v1.z = Val<T>::vmin(acc[i][6], c1.z); v1.w = Val<T>::vmin(acc[i][7], c1.w);
     *reinterpret_cast<V4*>(Cout + r * ldc_out + tx * 4) = v0;
     *reinterpret_cast<V4*>(Cout + r * ldc_out + 64 + tx * 4) = v1;
   }

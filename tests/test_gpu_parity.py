@@ -219,6 +219,23 @@ def test_virtual_ranks_match_oracle(lib, world):
         assert_i32_equal(got, want)
 
 
+def test_nccl_path_single_rank(lib):
+    """reserved[2] = 1: the sharded schedule with a real 1-rank NCCL communicator
+    (ncclBroadcast of the pivot band every round, ncclAllReduce of the status flag)."""
+    for g in [gg.grid_2d(17, 31, seed=1), gg.erdos_renyi(700, 2800, seed=2)]:
+        c = cfg(lib)
+        c.reserved[2] = 1
+        got = lib.solve(g, cfg=c)
+        want, _ = oracle_i32(g)
+        assert_i32_equal(got, want)
+    g = gg.with_arcs(gg.erdos_renyi(300, 900, seed=3), [10, 290], [290, 10], [-100, 20])
+    c = cfg(lib)
+    c.reserved[2] = 1
+    with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
+        with pytest.raises(lib.NegativeCycleError):
+            lib.apsp_fw_blocked(h)
+
+
 def test_virtual_ranks_negative_cycle(lib):
     g = gg.with_arcs(gg.erdos_renyi(700, 2500, seed=5), [600, 650], [650, 600], [-300, 100])
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=cfg(lib, world_size=4, virtual_ranks=1)) as h:
@@ -235,4 +252,6 @@ def test_phase_stats_count_all_relaxations(lib):
         st = lib.apsp_get_phase_stats(h)
         n_pad = lib.apsp_get_info(h).n_pad
     assert sum(st.relax[:3]) == float(n_pad) ** 3
-    assert st.launches[2] == n_pad // 128 and st.ms[2] > 0
+    nb = n_pad // 128
+    # phase 3 = one launch in the last round, two (3A + 3B, lookahead split) before it
+    assert st.launches[0] == nb and st.launches[2] == 2 * (nb - 1) + 1 and st.ms[2] > 0
