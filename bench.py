@@ -42,6 +42,11 @@ def parse():
     ap.add_argument("--workload", default=None)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--force-ooc", action="store_true", help="use the out-of-core path (experiments)")
+    ap.add_argument("--ooc-block", type=int, default=0, help="out-of-core band height B (0 = auto)")
+    ap.add_argument("--stream-all", action="store_true", help="out-of-core: keep no band resident")
+    ap.add_argument("--no-lookahead", action="store_true", help="in-core: no phase-3 split / overlap")
+    ap.add_argument("--minplus-v1", action="store_true", help="cp.async min-plus kernel instead of TMA (A/B)")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle sample time")
     return ap.parse_args()
 
@@ -210,6 +215,15 @@ def run_ours(args):
     def make_cfg(timing):
         cfg = apsp.apsp_config_default(device=local, world_size=world, rank=rank, timing=timing)
         cfg.stream = stream.cuda_stream
+        if args.force_ooc:
+            cfg.force_out_of_core = 1
+            cfg.ooc_block = args.ooc_block
+            if args.stream_all:
+                cfg.reserved[0] = 1
+        if args.no_lookahead:
+            cfg.reserved[1] = 1
+        if args.minplus_v1:
+            cfg.reserved[3] = 1
         if uid is not None:
             cfg._uid_buf = __import__("ctypes").create_string_buffer(uid, 128)
             cfg.nccl_unique_id = __import__("ctypes").cast(cfg._uid_buf, __import__("ctypes").c_void_p)

@@ -206,8 +206,11 @@ static long long desc_tiles(const MinPlusDesc<T>& d) {
   return (long long)d.tiles_i * (long long)d.tiles_j;
 }
 
+int g_minplus_variant = 0;
+
 template <typename T>
 cudaError_t launch_minplus(const MinPlusDesc<T>* d, int ndesc, int K, cudaStream_t s) {
+  if (g_minplus_variant == 0) return launch_minplus_tma<T>(d, ndesc, K, s);
   if (K <= 0 || K % MP_BK) return cudaErrorInvalidValue;
   MinPlusArgs<T> a;
   a.d0 = d[0];
@@ -385,8 +388,10 @@ cudaError_t configure_kernels() {
   cudaError_t e = cudaFuncSetAttribute(minplus_kernel<int>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        minplus_smem_bytes<int>());
   if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(minplus_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                              minplus_smem_bytes<float>());
+  e = cudaFuncSetAttribute(minplus_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           minplus_smem_bytes<float>());
+  if (e != cudaSuccess) return e;
+  return configure_tma_kernels();
 }
 
 template cudaError_t launch_minplus<int>(const MinPlusDesc<int>*, int, int, cudaStream_t);

@@ -54,4 +54,12 @@ cudaError_t launch_canonicalize_i32(int* D, long long ld, long long rows, long l
 // device before the first launch.
 cudaError_t configure_kernels();
 
+// The TMA + mbarrier persistent variant of launch_minplus (apsp_minplus_tma.cu),
+// the default. g_minplus_variant = 1 selects the cp.async kernel instead
+// (A/B timing and parity of both; set from apsp_config.reserved[3]).
+template <typename T>
+cudaError_t launch_minplus_tma(const MinPlusDesc<T>* d, int ndesc, int K, cudaStream_t s);
+cudaError_t configure_tma_kernels();
+extern int g_minplus_variant;
+
 }  // namespace apsp

@@ -82,6 +82,21 @@ def test_fw_int32_bit_exact(lib, n):
         assert_i32_equal(got, want)
 
 
+@pytest.mark.parametrize("n", [129, 640, 1000])
+def test_fw_cp_async_minplus_variant(lib, n):
+    """reserved[3] = 1 selects the cp.async min-plus kernel (the TMA kernel is the default)."""
+    for name, g in graphs_for(n, seed=n + 3):
+        c = cfg(lib)
+        c.reserved[3] = 1
+        got = lib.solve(g, cfg=c)
+        want, _ = oracle_i32(g)
+        assert_i32_equal(got, want)
+    gf = gg.erdos_renyi(n, 6 * n, seed=n, dtype="f32")
+    c = cfg(lib)
+    c.reserved[3] = 1
+    assert_f32_close(lib.solve(gf, cfg=c), oracle.fw_f64(gf.row_ptr, gf.col, gf.w)[0])
+
+
 @pytest.mark.parametrize("n", [384, 640, 1000])
 def test_fw_without_lookahead(lib, n):
     """reserved[1] = 1 runs phases 1-3 strictly in order on one stream (no split phase 3)."""
