@@ -93,7 +93,7 @@ apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_pt
   if (prop.major < 10) return h->fail(APSP_ECUDA, "device %s is sm_%d%d; this library is built for sm_100a", prop.name,
                                       prop.major, prop.minor);
   if ((st = h->cuda(configure_kernels(), "configure_kernels"))) return st;
-  g_minplus_variant = cfg.reserved[3] == 1 ? 1 : 0;  // test hook: 1 = cp.async min-plus kernel
+  g_minplus_variant = cfg.reserved[3];  // test hook: 0 = cp.async (default), 2 = TMA min-plus kernel
   if (cfg.stream) {
     h->stream = static_cast<cudaStream_t>(cfg.stream);
   } else {

@@ -210,7 +210,7 @@ int g_minplus_variant = 0;
 
 template <typename T>
 cudaError_t launch_minplus(const MinPlusDesc<T>* d, int ndesc, int K, cudaStream_t s) {
-  if (g_minplus_variant == 0) return launch_minplus_tma<T>(d, ndesc, K, s);
+  if (g_minplus_variant == 2) return launch_minplus_tma<T>(d, ndesc, K, s);
   if (K <= 0 || K % MP_BK) return cudaErrorInvalidValue;
   MinPlusArgs<T> a;
   a.d0 = d[0];

@@ -54,9 +54,10 @@ cudaError_t launch_canonicalize_i32(int* D, long long ld, long long rows, long l
 // device before the first launch.
 cudaError_t configure_kernels();
 
-// The TMA + mbarrier persistent variant of launch_minplus (apsp_minplus_tma.cu),
-// the default. g_minplus_variant = 1 selects the cp.async kernel instead
-// (A/B timing and parity of both; set from apsp_config.reserved[3]).
+// The TMA + mbarrier persistent variant of launch_minplus (apsp_minplus_tma.cu).
+// g_minplus_variant (set from apsp_config.reserved[3]): 0 = cp.async kernel
+// (default), 2 = TMA persistent kernel (measured slower in round 1: its
+// persistent grid also blocks the lookahead phases 1+2).
 template <typename T>
 cudaError_t launch_minplus_tma(const MinPlusDesc<T>* d, int ndesc, int K, cudaStream_t s);
 cudaError_t configure_tma_kernels();

@@ -83,17 +83,17 @@ def test_fw_int32_bit_exact(lib, n):
 
 
 @pytest.mark.parametrize("n", [129, 640, 1000])
-def test_fw_cp_async_minplus_variant(lib, n):
-    """reserved[3] = 1 selects the cp.async min-plus kernel (the TMA kernel is the default)."""
+def test_fw_tma_minplus_variant(lib, n):
+    """reserved[3] = 2 selects the TMA + mbarrier persistent min-plus kernel (cp.async is the default)."""
     for name, g in graphs_for(n, seed=n + 3):
         c = cfg(lib)
-        c.reserved[3] = 1
+        c.reserved[3] = 2
         got = lib.solve(g, cfg=c)
         want, _ = oracle_i32(g)
         assert_i32_equal(got, want)
     gf = gg.erdos_renyi(n, 6 * n, seed=n, dtype="f32")
     c = cfg(lib)
-    c.reserved[3] = 1
+    c.reserved[3] = 2
     assert_f32_close(lib.solve(gf, cfg=c), oracle.fw_f64(gf.row_ptr, gf.col, gf.w)[0])
 
 
