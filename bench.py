@@ -47,6 +47,8 @@ def parse():
     ap.add_argument("--stream-all", action="store_true", help="out-of-core: keep no band resident")
     ap.add_argument("--no-lookahead", action="store_true", help="in-core: no phase-3 split / overlap")
     ap.add_argument("--minplus-tma", action="store_true", help="TMA persistent min-plus kernel (A/B)")
+    ap.add_argument("--packed16", action="store_true",
+                    help="packed int16 arithmetic (VIADDMNMX.S16x2) when exact, int32 otherwise")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle sample time")
     return ap.parse_args()
 
@@ -224,6 +226,8 @@ def run_ours(args):
             cfg.reserved[1] = 1
         if args.minplus_tma:
             cfg.reserved[3] = 2
+        if args.packed16:
+            cfg.packed16 = 1
         if uid is not None:
             cfg._uid_buf = __import__("ctypes").create_string_buffer(uid, 128)
             cfg.nccl_unique_id = __import__("ctypes").cast(cfg._uid_buf, __import__("ctypes").c_void_p)
@@ -279,9 +283,13 @@ def run_ours(args):
     p3_relax = st_acc[2][2] / max(1, st_acc[1][2])
     achieved = p3_relax / (p3_ms * 1e-3)
     dpx = pk.get("dpx", {})
+    arith = apsp.ARITH_NAMES[apsp.apsp_get_info(h).arith]
     if is_f:
         peak = dpx.get("f32_relax_per_s")
         peak_src = "measured fp32 FADD+FMNMX min-plus rate (MEASURED_DPX.json)"
+    elif arith == "s16x2":
+        peak = dpx.get("s16x2_relax_per_s")
+        peak_src = "measured VIADDMNMX.S16x2 rate, 2 relaxations/instruction (MEASURED_DPX.json)"
     else:
         peak = dpx.get("s32_relax_per_s")
         peak_src = "measured VIADDMNMX s32 rate (MEASURED_DPX.json)"
@@ -293,7 +301,7 @@ def run_ours(args):
     if os.path.exists(tp):
         try:
             tj = json.load(open(tp))
-            if tj.get("workload") == wl:
+            if tj.get("workload") == wl and tj.get("arith", "i32") == arith and not args.force_ooc:
                 # measured DRAM bytes per relaxation (ncu capture) x this run's relax per launch
                 traffic = tj["dram_bytes_per_relax"] * p3_relax
         except Exception:
@@ -303,7 +311,8 @@ def run_ours(args):
                 "peak_source": peak_src, "avg_launch_ms": p3_ms, "relax_per_launch": p3_relax,
                 "share_of_step": (st_acc[0][2] / args.steps) / ms_step,
                 "traffic_unit": "bytes per launch (DRAM read+write)",
-                "algorithmic_bytes_per_launch": p3_relax * 2 * 65536 / 128 ** 3 if not args.force_ooc else None}
+                "algorithmic_bytes_per_launch": (p3_relax * 2 * 128 * 128 * (2 if arith == "s16x2" else 4) / 128 ** 3
+                                                 if not args.force_ooc else None)}
     apsp.apsp_destroy(h)
 
     # ---------------- end-to-end through the C ABI with host buffers ----------
@@ -350,7 +359,7 @@ def run_ours(args):
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
             "scaling": "strong" if world > 1 else "weak", "vs_baseline": None,
-            "dtype": "f32" if is_f else "i32", "data": "synthetic",
+            "dtype": arith, "data": "synthetic",
             "config": {"workload": wl, "n": n, "n_pad": int(info.n_pad), "m": g.m, "tile": 128,
                        "desc": gg.BASELINE_CONFIGS[wl],
                        "parallelism": "1-D block-row x%d, NCCL pivot-band broadcast" % world if world > 1

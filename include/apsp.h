@@ -85,7 +85,17 @@ typedef struct {
   int32_t timing;               /* 1 = record CUDA events around every launch and
                                    accumulate per-phase device times (apsp_phase_stats) */
   int32_t force_out_of_core;    /* 1 = use the out-of-core path even if n*n fits */
-  int32_t reserved[7];
+  int32_t packed16;             /* 1 = int32 inputs whose weights lie in [0, 8191]
+                                   are solved in packed int16 pairs (VIADDMNMX.S16x2,
+                                   two relaxations per DPX instruction). The result is
+                                   checked (max finite entry < 8192 proves it exact,
+                                   DESIGN.md R16) and recomputed in int32 otherwise, so
+                                   the output is always the exact int32 APSP. Single-GPU
+                                   in-core only; ignored elsewhere. apsp_info.arith
+                                   reports which arithmetic produced the result */
+  int32_t reserved[6];          /* test hooks: [0] out-of-core streams every band,
+                                   [1] no lookahead, [2] NCCL at world 1,
+                                   [3] min-plus kernel variant; otherwise 0 */
 } apsp_config;
 
 /* Fill *cfg with defaults (struct_size set, device -1, world 1, rank 0). */
@@ -175,10 +185,18 @@ typedef struct {
   int64_t device_bytes;                        /* device memory the handle holds */
   int64_t host_bytes;                          /* pinned host memory (out-of-core) */
   void* dist_device;                           /* in-core: device base of this rank's
-                                                  rows (row-major, ld = ld elements);
+                                                  rows (row-major, ld = ld elements,
+                                                  int16 when arith == APSP_ARITH_S16X2);
                                                   NULL out-of-core */
   int64_t ld;
+  int32_t arith;                               /* APSP_ARITH_*: arithmetic of the current
+                                                  result (or of the next run) */
+  int32_t packed16_eligible;                   /* packed16 requested and the input allows it */
 } apsp_info;
+
+#define APSP_ARITH_I32 0   /* VIADDMNMX (int32 DPX), 1 relaxation / instruction */
+#define APSP_ARITH_S16X2 1 /* VIADDMNMX.S16x2, 2 relaxations / instruction, verified exact */
+#define APSP_ARITH_F32 2   /* FADD + FMNMX */
 
 apsp_status apsp_get_info(const apsp_handle* h, apsp_info* info);
 

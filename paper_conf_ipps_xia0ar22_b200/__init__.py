@@ -50,7 +50,8 @@ class apsp_config(ctypes.Structure):
         ("ooc_block", ctypes.c_int32),
         ("timing", ctypes.c_int32),
         ("force_out_of_core", ctypes.c_int32),
-        ("reserved", ctypes.c_int32 * 7),
+        ("packed16", ctypes.c_int32),
+        ("reserved", ctypes.c_int32 * 6),
     ]
 
 
@@ -61,7 +62,12 @@ class apsp_info(ctypes.Structure):
         ("rank", ctypes.c_int32), ("mode", ctypes.c_int32), ("ooc_block", ctypes.c_int32),
         ("rounds", ctypes.c_int64), ("device_bytes", ctypes.c_int64), ("host_bytes", ctypes.c_int64),
         ("dist_device", ctypes.c_void_p), ("ld", ctypes.c_int64),
+        ("arith", ctypes.c_int32), ("packed16_eligible", ctypes.c_int32),
     ]
+
+
+APSP_ARITH_I32, APSP_ARITH_S16X2, APSP_ARITH_F32 = 0, 1, 2
+ARITH_NAMES = {0: "i32", 1: "s16x2", 2: "f32"}
 
 
 class apsp_phase_stats(ctypes.Structure):

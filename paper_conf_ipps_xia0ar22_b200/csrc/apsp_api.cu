@@ -235,9 +235,9 @@ apsp_status apsp_init_from_csr(apsp_handle** out, int64_t n, const int64_t* row_
   for (int64_t e = 0; e < m; ++e)
     if (col_idx[e] < 0 || col_idx[e] >= n) return fail_global(APSP_EINVAL, "col_idx[%lld] out of range", (long long)e);
   bool has_neg = false;
+  int64_t maxabs = 0;
   if (dtype == APSP_I32) {
     const int32_t* w = static_cast<const int32_t*>(weights);
-    int64_t maxabs = 0;
     for (int64_t e = 0; e < m; ++e) {
       int64_t v = w[e];
       if (v < 0) has_neg = true;
@@ -264,6 +264,8 @@ apsp_status apsp_init_from_csr(apsp_handle** out, int64_t n, const int64_t* row_
   h->virt = cfg.virtual_ranks && cfg.world_size > 1;
   h->timing = cfg.timing != 0;
   h->has_neg = has_neg;
+  h->max_abs_w = maxabs;
+  h->arith = dtype == APSP_F32 ? APSP_ARITH_F32 : APSP_ARITH_I32;
   h->elem = sizeof(int32_t);
 
   apsp_status st = init_handle(h, cfg, row_ptr, col_idx, weights);
@@ -281,6 +283,7 @@ apsp_status apsp_fw_rounds(apsp_handle* hh, int64_t k_begin, int64_t k_end) {
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
   if (h->mode != APSP_MODE_INCORE) return h->fail(APSP_ESTATE, "apsp_fw_rounds: in-core mode only");
+  if (h->mode16) return h->fail(APSP_ESTATE, "apsp_fw_rounds: not available with packed16");
   const long long nb = h->n_pad / h->b;
   if (k_begin != h->next_round || k_end < k_begin || k_end > nb)
     return h->fail(APSP_ESTATE, "rounds must run in order: next is %lld of %lld", h->next_round, nb);
@@ -305,6 +308,11 @@ apsp_status apsp_fw_blocked(apsp_handle* hh) {
   }
   const long long nb = h->n_pad / h->b;
   if (h->next_round != 0) return h->fail(APSP_ESTATE, "apsp_fw_rounds already started");
+  if (h->mode16) {
+    if ((st = run_fw16(h))) return st;
+    h->next_round = nb;
+    return finish_fw(h, true);
+  }
   if ((st = run_incore_rounds(h, 0, nb))) return st;
   h->next_round = nb;
   return finish_fw(h, true);
@@ -361,6 +369,9 @@ apsp_status apsp_get_info(const apsp_handle* hh, apsp_info* info) {
   info->host_bytes = h->host_bytes;
   info->dist_device = h->shards.empty() ? nullptr : h->shards[0].D;
   info->ld = h->ld;
+  info->arith = h->arith;
+  info->packed16_eligible = h->mode16 ? 1 : 0;
+  if (h->result16) info->dist_device = h->d16;
   return APSP_OK;
 }
 

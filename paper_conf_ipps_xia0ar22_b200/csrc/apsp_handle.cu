@@ -2,6 +2,7 @@
 // partition, allocation, NCCL communicator, CSR upload + init kernel
 // (PAPER.md:60), negative-cycle status, and result read-back (get_dist).
 #include "apsp_internal.h"
+#include "apsp_sched.cuh"
 
 #include <nccl.h>
 
@@ -58,7 +59,17 @@ static apsp_status upload_csr(Handle* h, const int64_t* row_ptr, const int32_t* 
 // a1: CSR -> dense for every local shard, from the device CSR.
 apsp_status run_init(Handle* h) {
   apsp_status st;
+  h->result16 = false;
+  if (h->mode16 && !h->fell_back16) {
+    const Shard& sh = h->shards[0];
+    if ((st = h->cuda(launch_init16(h->d16, h->ld, h->n_pad, h->n_pad, h->n, sh.d_rp, sh.d_col,
+                                    static_cast<const int*>(sh.d_w), h->stream),
+                      "init16")))
+      return st;
+    h->arith = APSP_ARITH_S16X2;
+  }
   for (auto& sh : h->shards) {
+    if (!sh.D) continue;
     cudaError_t e;
     if (h->dtype == APSP_I32)
       e = launch_init_rows<int>(static_cast<int*>(sh.D), h->ld, h->n_pad, sh.row_begin, h->rows_per_rank, h->n,
@@ -134,6 +145,21 @@ apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_pt
     return ooc_setup(h, cfg, budget, row_ptr, col, w);
   }
 
+  // packed int16 (R16): single GPU, in core, int32 weights in [0, 8191]
+  h->mode16 = cfg.packed16 == 1 && h->dtype == APSP_I32 && !h->has_neg && h->max_abs_w <= 8191 &&
+              h->world == 1 && !h->virt && cfg.reserved[2] != 1;
+  if (h->mode16) {
+    const long long b16 = h->n_pad * h->n_pad * 2;
+    if ((st = h->cuda(cudaMalloc(&h->d16, b16), "cudaMalloc dist16"))) return st;
+    if ((st = h->cuda(cudaMalloc(&h->d_max16, sizeof(int)), "cudaMalloc"))) return st;
+    h->device_bytes = b16;
+    Shard sh;  // the int32 matrix is allocated only if the int16 result must be redone
+    h->shards.push_back(sh);
+    if ((st = upload_csr<int>(h, row_ptr, col, w))) return st;
+    if ((st = run_init(h))) return st;
+    return h->cuda(cudaStreamSynchronize(h->stream), "init sync");
+  }
+
   if ((st = h->cuda(cudaMalloc(&h->d_base, mat_bytes), "cudaMalloc dist"))) return st;
   h->device_bytes = mat_bytes;
   if (panel_bytes) {
@@ -172,6 +198,42 @@ apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_pt
   return h->cuda(cudaStreamSynchronize(h->stream), "init sync");
 }
 
+// Packed int16 closure (VIADDMNMX.S16x2) with exactness check; int32 redo if the
+// largest finite distance reaches 8192 (R16).
+apsp_status run_fw16(Handle* h) {
+  apsp_status st;
+  const long long nb = h->n_pad / h->b;
+  if (!h->fell_back16) {
+    if ((st = fw_closure<short>(h, h->d16, h->ld, h->n_pad, 0, nb, h->stream))) return st;
+    int mx = 0;
+    if ((st = h->cuda(launch_max_finite16(h->d16, h->ld, h->n_pad, h->n_pad, h->d_max16, h->stream), "max16")))
+      return st;
+    if ((st = h->cuda(cudaMemcpyAsync(&mx, h->d_max16, sizeof(int), cudaMemcpyDeviceToHost, h->stream), "D2H max")))
+      return st;
+    if ((st = h->cuda(cudaStreamSynchronize(h->stream), "fw16 sync"))) return st;
+    if (mx < 8192) {
+      h->result16 = true;
+      h->arith = APSP_ARITH_S16X2;
+      return APSP_OK;
+    }
+    h->fell_back16 = true;  // distances too long for int16: redo (and from now on run) in int32
+  }
+  Shard& sh = h->shards[0];
+  if (!sh.D) {
+    const long long mat_bytes = h->n_pad * h->ld * 4;
+    if ((st = h->cuda(cudaMalloc(&h->d_base, mat_bytes), "cudaMalloc dist (int32 fallback)"))) return st;
+    h->device_bytes += mat_bytes;
+    sh.D = h->d_base;
+  }
+  if ((st = h->cuda(launch_init_rows<int>(static_cast<int*>(sh.D), h->ld, h->n_pad, 0, h->n_pad, h->n, sh.d_rp,
+                                          sh.e0, sh.d_col, static_cast<const int*>(sh.d_w), h->stream),
+                    "init_rows")))
+    return st;
+  h->result16 = false;
+  h->arith = APSP_ARITH_I32;
+  return fw_closure<int>(h, static_cast<int*>(sh.D), h->ld, h->n_pad, 0, nb, h->stream);
+}
+
 void delete_handle(Handle* h) {
   if (!h) return;
   cudaSetDevice(h->device);
@@ -188,6 +250,9 @@ void delete_handle(Handle* h) {
     cudaFree(sh.d_w);
   }
   cudaFree(h->d_base);
+  cudaFree(h->d16);
+  cudaFree(h->d_max16);
+  cudaFree(h->d_widen);
   cudaFree(h->panel);
   cudaFree(h->d_flag);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
@@ -221,6 +286,29 @@ apsp_status finish_fw(Handle* h, bool all_rounds) {
 apsp_status get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out) {
   if (h->mode == APSP_MODE_OUT_OF_CORE) return ooc_get_rows(h, r0, cnt, out, ld_out);
   apsp_status st;
+  if (h->mode16 && !h->shards[0].D && !h->result16)
+    return h->fail(APSP_ESTATE, "no int32 matrix yet");
+  if (h->result16) {
+    // widen int16 rows to int32 on the device (INF16 -> APSP_INF_I32), then D2H, in blocks
+    const long long blk = std::max<long long>(1, std::min<long long>(cnt, (64ll << 20) / (h->n * 4)));
+    if (h->widen_rows < blk) {
+      cudaFree(h->d_widen);
+      h->d_widen = nullptr;
+      if ((st = h->cuda(cudaMalloc(&h->d_widen, blk * h->n * 4), "cudaMalloc widen"))) return st;
+      h->widen_rows = blk;
+    }
+    for (long long r = r0; r < r0 + cnt; r += blk) {
+      const long long rr = std::min(blk, r0 + cnt - r);
+      if ((st = h->cuda(launch_widen16(h->d16 + r * h->ld, h->ld, h->d_widen, h->n, rr, h->n, h->stream), "widen16")))
+        return st;
+      if ((st = h->cuda(cudaMemcpy2DAsync(static_cast<int*>(out) + (r - r0) * ld_out, (size_t)ld_out * 4, h->d_widen,
+                                          (size_t)h->n * 4, (size_t)h->n * 4, (size_t)rr, cudaMemcpyDeviceToHost,
+                                          h->stream),
+                        "D2H dist")))
+        return st;
+    }
+    return h->cuda(cudaStreamSynchronize(h->stream), "get_dist sync");
+  }
   const char* base;
   if (h->world > 1 && !h->virt) {
     const long long rb = h->shards[0].row_begin;

@@ -34,6 +34,16 @@ struct Handle {
   apsp_dtype dtype = APSP_I32;
   size_t elem = 4;
   bool has_neg = false;
+  long long max_abs_w = 0;
+  // packed int16 path (apsp_kernels16.cu)
+  bool mode16 = false;      // requested and eligible: try int16 first
+  bool result16 = false;    // the current result lives in d16
+  bool fell_back16 = false; // this graph needed int32: later runs go straight to int32
+  short* d16 = nullptr;     // n_pad x n_pad int16 matrix (single GPU, in core)
+  int* d_max16 = nullptr;
+  int* d_widen = nullptr;   // staging for get_dist of an int16 result
+  long long widen_rows = 0;
+  int arith = APSP_ARITH_I32;
   // placement
   int device = 0;
   int world = 1, rank = 0;
@@ -79,6 +89,7 @@ apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_pt
                         const void* w);
 void delete_handle(Handle* h);
 apsp_status run_init(Handle* h);
+apsp_status run_fw16(Handle* h);  // packed int16 closure, verify, int32 fallback
 apsp_status run_incore_rounds(Handle* h, long long k0, long long k1);
 apsp_status finish_fw(Handle* h, bool all_rounds);
 apsp_status get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out);

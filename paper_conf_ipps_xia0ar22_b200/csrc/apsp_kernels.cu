@@ -391,6 +391,7 @@ cudaError_t configure_kernels() {
   e = cudaFuncSetAttribute(minplus_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                            minplus_smem_bytes<float>());
   if (e != cudaSuccess) return e;
+  if ((e = configure_kernels16()) != cudaSuccess) return e;
   return configure_tma_kernels();
 }
 

@@ -54,6 +54,23 @@ cudaError_t launch_canonicalize_i32(int* D, long long ld, long long rows, long l
 // device before the first launch.
 cudaError_t configure_kernels();
 
+// ---- packed int16 path (apsp_kernels16.cu): VIADDMNMX.S16x2, 2 relax/instr ----
+template <>
+cudaError_t launch_minplus<short>(const MinPlusDesc<short>* d, int ndesc, int K, cudaStream_t s);
+template <>
+cudaError_t launch_phase1<short>(short* tile, long long ld, int* negflag, cudaStream_t s);
+// rows 0..rows-1 (global = local, single GPU) of the int16 matrix from a CSR
+// with absolute offsets; INF16 = 16383; weights must lie in [0, 8191]
+cudaError_t launch_init16(short* D, long long ld, long long n_pad, long long rows, long long n,
+                          const long long* row_ptr, const int* col, const int* w, cudaStream_t s);
+// *out = max entry < INF16 (or -1)
+cudaError_t launch_max_finite16(const short* D, long long ld, long long rows, long long cols, int* out,
+                                cudaStream_t s);
+// int16 rows -> int32 rows, INF16 -> APSP_INF_I32
+cudaError_t launch_widen16(const short* S, long long lds, int* D, long long ldd, long long rows, long long cols,
+                           cudaStream_t s);
+cudaError_t configure_kernels16();
+
 // The TMA + mbarrier persistent variant of launch_minplus (apsp_minplus_tma.cu).
 // g_minplus_variant (set from apsp_config.reserved[3]): 0 = cp.async kernel
 // (default), 2 = TMA persistent kernel (measured slower in round 1: its
