@@ -18,6 +18,7 @@ sample of the same workload (the reference arm of this paper-only tier).
 from __future__ import annotations
 
 import argparse
+import ctypes
 import json
 import os
 import subprocess
@@ -47,6 +48,7 @@ def parse():
     ap.add_argument("--stream-all", action="store_true", help="out-of-core: keep no band resident")
     ap.add_argument("--no-lookahead", action="store_true", help="in-core: no phase-3 split / overlap")
     ap.add_argument("--minplus-tma", action="store_true", help="TMA persistent min-plus kernel (A/B)")
+    ap.add_argument("--no-packed16", action="store_true", help="skip the packed-int16 alternative measurement")
     ap.add_argument("--packed16", action="store_true",
                     help="packed int16 arithmetic (VIADDMNMX.S16x2) when exact, int32 otherwise")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle sample time")
@@ -214,7 +216,7 @@ def run_ours(args):
         dist.broadcast_object_list(obj, src=0)
         uid = obj[0]
 
-    def make_cfg(timing):
+    def make_cfg(timing, packed16):
         cfg = apsp.apsp_config_default(device=local, world_size=world, rank=rank, timing=timing)
         cfg.stream = stream.cuda_stream
         if args.force_ooc:
@@ -226,11 +228,11 @@ def run_ours(args):
             cfg.reserved[1] = 1
         if args.minplus_tma:
             cfg.reserved[3] = 2
-        if args.packed16:
+        if packed16:
             cfg.packed16 = 1
         if uid is not None:
-            cfg._uid_buf = __import__("ctypes").create_string_buffer(uid, 128)
-            cfg.nccl_unique_id = __import__("ctypes").cast(cfg._uid_buf, __import__("ctypes").c_void_p)
+            cfg._uid_buf = ctypes.create_string_buffer(uid, 128)
+            cfg.nccl_unique_id = ctypes.cast(cfg._uid_buf, ctypes.c_void_p)
         return cfg
 
     def barrier():
@@ -244,80 +246,85 @@ def run_ours(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
-    # ---------------- device-resident timing (value) ------------------------
-    h = apsp.apsp_init_from_csr(n, g.row_ptr, g.col, g.w, cfg=make_cfg(1))
-    info = apsp.apsp_get_info(h)
-    for _ in range(args.warmup):
-        apsp.apsp_reinit(h)
-        apsp.apsp_fw_blocked(h)
-    torch.cuda.synchronize()
-    # phase stats of the timed steps only
-    st_acc = np.zeros((3, 4))
-    clk = ClockSampler(local)
-    barrier()
-    torch.cuda.synchronize()
-    clk.start()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    for _ in range(args.steps):
-        apsp.apsp_reinit(h)
-        apsp.apsp_fw_blocked(h)
-        s = apsp.apsp_get_phase_stats(h)
-        st_acc[0] += np.array(s.ms[:])
-        st_acc[1] += np.array(s.launches[:])
-        st_acc[2] += np.array(s.relax[:])
-    e1.record(stream)
-    torch.cuda.synchronize()
-    barrier()
-    clocks = clk.stop()
-    ms = max_over_ranks(e0.elapsed_time(e1))
-    ms_step = ms / args.steps
-    value = float(n) ** 3 / (ms_step * 1e-3)
-    launches_per_step = int(round((st_acc[1][:3].sum()) / args.steps)) + 1  # + init kernel
-    # sanity: relaxations performed per step must be n_pad^3 (whole job)
-    relax_local = st_acc[2][:3].sum() / args.steps
-
-    # ---------------- roofline of the dominant kernel (phase 3) --------------
     pk = peaks()
-    p3_ms = st_acc[0][2] / max(1, st_acc[1][2])
-    p3_relax = st_acc[2][2] / max(1, st_acc[1][2])
-    achieved = p3_relax / (p3_ms * 1e-3)
-    dpx = pk.get("dpx", {})
-    arith = apsp.ARITH_NAMES[apsp.apsp_get_info(h).arith]
-    if is_f:
-        peak = dpx.get("f32_relax_per_s")
-        peak_src = "measured fp32 FADD+FMNMX min-plus rate (MEASURED_DPX.json)"
-    elif arith == "s16x2":
-        peak = dpx.get("s16x2_relax_per_s")
-        peak_src = "measured VIADDMNMX.S16x2 rate, 2 relaxations/instruction (MEASURED_DPX.json)"
-    else:
-        peak = dpx.get("s32_relax_per_s")
-        peak_src = "measured VIADDMNMX s32 rate (MEASURED_DPX.json)"
-    if not peak:
-        peak = 148 * 64 * 1.965e9
-        peak_src = "derived: 148 SMs x 64 lanes/clk x 1.965 GHz (no MEASURED_DPX.json)"
-    traffic = None
-    tp = os.path.join(ROOT, "profiles", "phase3_traffic.json")
-    if os.path.exists(tp):
-        try:
-            tj = json.load(open(tp))
-            if tj.get("workload") == wl and tj.get("arith", "i32") == arith and not args.force_ooc:
-                # measured DRAM bytes per relaxation (ncu capture) x this run's relax per launch
-                traffic = tj["dram_bytes_per_relax"] * p3_relax
-        except Exception:
-            pass
-    roofline = {"bound": "alu", "kernel": "minplus_kernel (phase 3)", "achieved": achieved / 1e12,
-                "peak": peak / 1e12, "unit": "Trelax/s", "frac": achieved / peak, "traffic": traffic,
-                "peak_source": peak_src, "avg_launch_ms": p3_ms, "relax_per_launch": p3_relax,
-                "share_of_step": (st_acc[0][2] / args.steps) / ms_step,
-                "traffic_unit": "bytes per launch (DRAM read+write)",
-                "algorithmic_bytes_per_launch": (p3_relax * 2 * 128 * 128 * (2 if arith == "s16x2" else 4) / 128 ** 3
-                                                 if not args.force_ooc else None)}
-    apsp.apsp_destroy(h)
 
-    # ---------------- end-to-end through the C ABI with host buffers ----------
-    e2e = None
-    if not args.no_e2e:
+    def device_timed(packed16):
+        """W warm-up + K timed steps (apsp_reinit + apsp_fw_blocked, CSR resident in HBM),
+        CUDA events on the library's stream, max over ranks; roofline of phase 3."""
+        h = apsp.apsp_init_from_csr(n, g.row_ptr, g.col, g.w, cfg=make_cfg(1, packed16))
+        info = apsp.apsp_get_info(h)
+        for _ in range(args.warmup):
+            apsp.apsp_reinit(h)
+            apsp.apsp_fw_blocked(h)
+        torch.cuda.synchronize()
+        st_acc = np.zeros((3, 4))
+        clk = ClockSampler(local)
+        barrier()
+        torch.cuda.synchronize()
+        clk.start()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            apsp.apsp_reinit(h)
+            apsp.apsp_fw_blocked(h)
+            s = apsp.apsp_get_phase_stats(h)
+            st_acc[0] += np.array(s.ms[:])
+            st_acc[1] += np.array(s.launches[:])
+            st_acc[2] += np.array(s.relax[:])
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        clocks = clk.stop()
+        ms_step = max_over_ranks(e0.elapsed_time(e1)) / args.steps
+        value = float(n) ** 3 / (ms_step * 1e-3)
+        arith = apsp.ARITH_NAMES[apsp.apsp_get_info(h).arith]
+        apsp.apsp_destroy(h)
+        # roofline of the dominant kernel: phase-3 min-plus launches
+        p3_ms = st_acc[0][2] / max(1, st_acc[1][2])
+        p3_relax = st_acc[2][2] / max(1, st_acc[1][2])
+        achieved = p3_relax / (p3_ms * 1e-3)
+        dpx = pk.get("dpx", {})
+        if is_f:
+            peak = dpx.get("f32_relax_per_s")
+            peak_src = "measured fp32 FADD+FMNMX min-plus rate (MEASURED_DPX.json)"
+        elif arith == "s16x2":
+            peak = dpx.get("s16x2_relax_per_s")
+            peak_src = "measured VIADDMNMX.S16x2 rate, 2 relaxations/instruction (MEASURED_DPX.json)"
+        else:
+            peak = dpx.get("s32_relax_per_s")
+            peak_src = "measured VIADDMNMX s32 rate (MEASURED_DPX.json)"
+        if not peak:
+            peak = 148 * 64 * 1.965e9 * (2 if arith == "s16x2" else 1)
+            peak_src = "derived: 148 SMs x 64 lanes/clk x 1.965 GHz (no MEASURED_DPX.json)"
+        elem = 2 if arith == "s16x2" else 4
+        traffic = None
+        tp = os.path.join(ROOT, "profiles", "phase3_traffic.json")
+        if os.path.exists(tp) and not args.force_ooc:
+            try:
+                for tj in json.load(open(tp)).get("captures", []):
+                    if tj.get("workload") == wl and tj.get("arith") == arith:
+                        # measured DRAM bytes per relaxation (ncu capture) x this run's relax per launch
+                        traffic = tj["dram_bytes_per_relax"] * p3_relax
+            except Exception:
+                pass
+        roofline = {"bound": "alu", "kernel": "phase-3 min-plus (%s)" % arith, "achieved": achieved / 1e12,
+                    "peak": peak / 1e12, "unit": "Trelax/s", "frac": achieved / peak, "traffic": traffic,
+                    "traffic_unit": "bytes per launch (DRAM read+write)",
+                    "algorithmic_bytes_per_launch": (p3_relax * 2 * 128 * 128 * elem / 128 ** 3
+                                                     if not args.force_ooc else None),
+                    "peak_source": peak_src, "avg_launch_ms": p3_ms, "relax_per_launch": p3_relax,
+                    "share_of_step": (st_acc[0][2] / args.steps) / ms_step}
+        return {"value": value, "ms_per_step": ms_step, "arith": arith, "clocks": clocks, "roofline": roofline,
+                "launches_per_step": int(round(st_acc[1][:3].sum() / args.steps)) + 1,  # + init kernel
+                "relax_per_step_rank0": st_acc[2][:3].sum() / args.steps, "n_pad": int(info.n_pad),
+                "phase_ms_per_step_rank0": {"phase1": st_acc[0][0] / args.steps,
+                                            "phase2": st_acc[0][1] / args.steps,
+                                            "phase3": st_acc[0][2] / args.steps,
+                                            "comm": st_acc[0][3] / args.steps}}
+
+    def end_to_end(packed16):
+        """Same metric through the C ABI with host buffers: apsp_init_from_csr (pinned host
+        CSR, H2D inside) + apsp_fw_blocked + apsp_get_dist into pinned host memory + destroy."""
         rb, rc = (0, n)
         if world > 1:
             _, rb, rc = apsp.apsp_partition(n, world, rank)
@@ -328,25 +335,38 @@ def run_ours(args):
         h2d = rp.nbytes + cl.nbytes + ww.nbytes
         d2h = rc * n * host_out.element_size()
         k_e2e = max(1, min(args.steps, 3))
-        # warm once (allocator, NCCL comm)
-        he = apsp.apsp_init_from_csr(n, rp, cl, ww, cfg=make_cfg(0))
+        he = apsp.apsp_init_from_csr(n, rp, cl, ww, cfg=make_cfg(0, packed16))  # warm (allocator, comm)
         apsp.apsp_destroy(he)
         barrier()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
         for _ in range(k_e2e):
-            he = apsp.apsp_init_from_csr(n, rp, cl, ww, cfg=make_cfg(0))
+            he = apsp.apsp_init_from_csr(n, rp, cl, ww, cfg=make_cfg(0, packed16))
             apsp.apsp_fw_blocked(he)
             if rc > 0:
                 apsp.apsp_get_dist_ptr(he, rb, rc, host_out.data_ptr(), n)
             apsp.apsp_destroy(he)
         torch.cuda.synchronize()
-        el = time.perf_counter() - t0
-        el = max_over_ranks(el)
-        e2e = {"value": float(n) ** 3 / (el / k_e2e), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
-               "d2h_bytes_per_step": int(d2h), "steps": k_e2e,
-               "note": "apsp_init_from_csr(host CSR, pinned) + apsp_fw_blocked + apsp_get_dist(pinned host) + "
-                       "destroy, host wall clock (synchronous C-ABI calls)"}
+        el = max_over_ranks(time.perf_counter() - t0)
+        return {"value": float(n) ** 3 / (el / k_e2e), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
+                "d2h_bytes_per_step": int(d2h), "steps": k_e2e,
+                "note": "apsp_init_from_csr(host CSR, pinned) + apsp_fw_blocked + apsp_get_dist(pinned host) + "
+                        "destroy, host wall clock (synchronous C-ABI calls)"}
+
+    main_run = device_timed(args.packed16)
+    e2e = None if args.no_e2e else end_to_end(args.packed16)
+
+    # the packed int16 alternative (exact, verified; R16), single GPU int32 inputs
+    alt16 = None
+    if world == 1 and not is_f and not args.packed16 and not args.no_packed16 and not args.force_ooc:
+        r16 = device_timed(True)
+        alt16 = {"value": r16["value"], "ms_per_step": r16["ms_per_step"], "dtype": r16["arith"],
+                 "roofline": r16["roofline"], "clocks": r16["clocks"],
+                 "e2e": None if args.no_e2e else end_to_end(True),
+                 "note": "same workload, apsp_config.packed16=1: VIADDMNMX.S16x2 (2 relaxations per DPX "
+                         "instruction) with the exactness check of DESIGN.md R16; the result is the exact int32 "
+                         "APSP (bit-exact in tests/test_gpu_packed16.py); falls back to int32 when distances "
+                         "reach 8192 (dtype then reads i32)"}
 
     # ---------------- CPU oracle baseline (rank 0, N=1 only) ------------------
     cpu = None
@@ -356,25 +376,25 @@ def run_ours(args):
 
     if rank == 0:
         line = {
-            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True,
+            "metric": METRIC, "value": main_run["value"], "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": main_run["ms_per_step"], "higher_is_better": True,
             "scaling": "strong" if world > 1 else "weak", "vs_baseline": None,
-            "dtype": arith, "data": "synthetic",
-            "config": {"workload": wl, "n": n, "n_pad": int(info.n_pad), "m": g.m, "tile": 128,
+            "dtype": main_run["arith"], "data": "synthetic",
+            "config": {"workload": wl, "n": n, "n_pad": main_run["n_pad"], "m": g.m, "tile": 128,
                        "desc": gg.BASELINE_CONFIGS[wl],
                        "parallelism": "1-D block-row x%d, NCCL pivot-band broadcast" % world if world > 1
                        else "single GPU",
                        "l2": "inputs larger than L2 (dist = %.2f GB per step >> 126 MB L2); no flush" %
-                             (float(info.n_pad) ** 2 * 4 / 1e9),
+                             (float(main_run["n_pad"]) ** 2 * (2 if main_run["arith"] == "s16x2" else 4) / 1e9),
                        "step": "apsp_reinit (CSR->dense, CSR resident in HBM) + apsp_fw_blocked"},
-            "clocks": clocks,
+            "clocks": main_run["clocks"],
             "e2e": e2e,
-            "gpu_launches": launches_per_step * args.steps,
-            "roofline": roofline,
+            "gpu_launches": main_run["launches_per_step"] * args.steps,
+            "roofline": main_run["roofline"],
             "cpu_baseline": cpu,
-            "relax_per_step_rank0": relax_local,
-            "phase_ms_per_step_rank0": {"phase1": st_acc[0][0] / args.steps, "phase2": st_acc[0][1] / args.steps,
-                                        "phase3": st_acc[0][2] / args.steps, "comm": st_acc[0][3] / args.steps},
+            "packed16": alt16,
+            "relax_per_step_rank0": main_run["relax_per_step_rank0"],
+            "phase_ms_per_step_rank0": main_run["phase_ms_per_step_rank0"],
         }
         print(json.dumps(line), flush=True)
     if world > 1:

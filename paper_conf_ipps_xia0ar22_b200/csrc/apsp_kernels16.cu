@@ -137,6 +137,10 @@ __global__ void __launch_bounds__(S_NT, 2) minplus16_kernel(const __grid_constan
   for (int i = 0; i < 8; ++i)
 #pragma unroll
     for (int p = 0; p < 4; ++p) acc[i][p] = 0x7FFF7FFFu;
+  // C (128 rows x 256 B) is fetched during the last chunk into the two stages
+  // that are then free: rows 0..63 -> stage nk%3, rows 64..127 -> stage (nk+1)%3
+  unsigned short* const c_lo = reinterpret_cast<unsigned short*>(smem_raw + (nk % S_ST) * S_STAGE_BYTES);
+  unsigned short* const c_hi = reinterpret_cast<unsigned short*>(smem_raw + ((nk + 1) % S_ST) * S_STAGE_BYTES);
 
   for (int c = 0; c < nk; ++c) {
     wait_group<S_ST - 2>();
@@ -146,6 +150,14 @@ __global__ void __launch_bounds__(S_NT, 2) minplus16_kernel(const __grid_constan
     if (cn < nk) {
       load_b(cn % S_ST, cn);
       load_a_regs(cn, ra0, ra1);
+    }
+    if (c == nk - 1) {
+      const int cr = tid >> 4, cc = (tid & 15) * 8;
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        cp_async16b(c_lo + (cr + 16 * q) * 128 + cc, Cin + (cr + 16 * q) * d.ldc_in + cc);
+        cp_async16b(c_hi + (cr + 16 * q) * 128 + cc, Cin + (64 + cr + 16 * q) * d.ldc_in + cc);
+      }
     }
     commit();
     const unsigned* as = stageA(c % S_ST);
@@ -173,11 +185,12 @@ __global__ void __launch_bounds__(S_NT, 2) minplus16_kernel(const __grid_constan
     if (cn < nk) store_a(cn % S_ST, ra0, ra1);
   }
   wait_group<0>();
+  __syncthreads();
 
 #pragma unroll
   for (int i = 0; i < 8; ++i) {
     const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
-    const uint4 cv = *reinterpret_cast<const uint4*>(Cin + r * d.ldc_in + tx * 8);
+    const uint4 cv = *reinterpret_cast<const uint4*>((i < 4 ? c_lo : c_hi) + (ty * 4 + (i & 3)) * 128 + tx * 8);
     uint4 o;
     o.x = __vmins2(acc[i][0], cv.x);
     o.y = __vmins2(acc[i][1], cv.y);

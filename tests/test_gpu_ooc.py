@@ -74,6 +74,25 @@ def test_ooc_negative_weights_and_cycle(lib):
             lib.apsp_fw_blocked(h)
 
 
+def test_ooc_config2_size_mixed_residency(lib):
+    """BASELINE config 2's graph (n=16384) through the out-of-core scheduler with
+    B=2048 (8 bands) and a budget that keeps 3 bands resident and streams 5 through
+    pinned host memory; sampled rows vs the oracle's Dijkstra, bit-exact."""
+    g = gg.baseline_config("cfg2_grid16384")
+    bb = 2048 * 16384 * 4
+    c = ooc_cfg(lib, 2048, stream_all=False)
+    c.device_budget_bytes = 4 * bb + 2048 * 2048 * 4 + 3 * bb + (1 << 20)
+    with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
+        info = lib.apsp_get_info(h)
+        assert info.mode == lib.APSP_MODE_OUT_OF_CORE and info.host_bytes == 5 * bb
+        lib.apsp_fw_blocked(h)
+        srcs = np.array([0, 1, 2047, 2048, 5000, 8191, 12000, 16383])
+        want = oracle.dijkstra_rows_i64(g.row_ptr, g.col, g.w, srcs)
+        for i, s in enumerate(srcs):
+            got = lib.apsp_get_dist(h, int(s), 1)[0]
+            assert np.array_equal(got.astype(np.int64), want[i]), s
+
+
 def test_ooc_f32_and_reinit(lib):
     g = gg.erdos_renyi(800, 8000, seed=5, dtype="f32")
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=ooc_cfg(lib, 256)) as h:
