@@ -47,7 +47,9 @@ def parse():
     ap.add_argument("--ooc-block", type=int, default=0, help="out-of-core band height B (0 = auto)")
     ap.add_argument("--stream-all", action="store_true", help="out-of-core: keep no band resident")
     ap.add_argument("--no-lookahead", action="store_true", help="in-core: no phase-3 split / overlap")
-    ap.add_argument("--minplus-tma", action="store_true", help="TMA persistent min-plus kernel (A/B)")
+    ap.add_argument("--minplus-variant", type=int, default=0,
+                    help="min-plus kernel for A/B: 0 cp.async + CTA barrier (default), 2 TMA persistent, "
+                         "3 cp.async + mbarrier pipeline")
     ap.add_argument("--no-packed16", action="store_true", help="skip the packed-int16 alternative measurement")
     ap.add_argument("--packed16", action="store_true",
                     help="packed int16 arithmetic (VIADDMNMX.S16x2) when exact, int32 otherwise")
@@ -226,8 +228,7 @@ def run_ours(args):
                 cfg.reserved[0] = 1
         if args.no_lookahead:
             cfg.reserved[1] = 1
-        if args.minplus_tma:
-            cfg.reserved[3] = 2
+        cfg.reserved[3] = args.minplus_variant
         if packed16:
             cfg.packed16 = 1
         if uid is not None:
@@ -339,17 +340,25 @@ def run_ours(args):
         apsp.apsp_destroy(he)
         barrier()
         torch.cuda.synchronize()
+        parts = np.zeros(4)
         t0 = time.perf_counter()
         for _ in range(k_e2e):
+            ta = time.perf_counter()
             he = apsp.apsp_init_from_csr(n, rp, cl, ww, cfg=make_cfg(0, packed16))
+            tb = time.perf_counter()
             apsp.apsp_fw_blocked(he)
+            tc = time.perf_counter()
             if rc > 0:
                 apsp.apsp_get_dist_ptr(he, rb, rc, host_out.data_ptr(), n)
+            td = time.perf_counter()
             apsp.apsp_destroy(he)
+            parts += np.array([tb - ta, tc - tb, td - tc, time.perf_counter() - td])
         torch.cuda.synchronize()
         el = max_over_ranks(time.perf_counter() - t0)
         return {"value": float(n) ** 3 / (el / k_e2e), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                 "d2h_bytes_per_step": int(d2h), "steps": k_e2e,
+                "ms_per_step_parts": dict(zip(["init", "fw", "get_dist", "destroy"],
+                                              (parts / k_e2e * 1e3).round(2).tolist())),
                 "note": "apsp_init_from_csr(host CSR, pinned) + apsp_fw_blocked + apsp_get_dist(pinned host) + "
                         "destroy, host wall clock (synchronous C-ABI calls)"}
 

@@ -252,6 +252,12 @@ void delete_handle(Handle* h) {
   cudaFree(h->d_base);
   cudaFree(h->d16);
   cudaFree(h->d_max16);
+  if (h->copy_stream) {
+    cudaStreamSynchronize(h->copy_stream);
+    cudaStreamDestroy(h->copy_stream);
+  }
+  for (auto& e : h->copy_ev)
+    if (e) cudaEventDestroy(e);
   cudaFree(h->d_widen);
   cudaFree(h->panel);
   cudaFree(h->d_flag);
@@ -289,25 +295,39 @@ apsp_status get_rows(Handle* h, long long r0, long long cnt, void* out, long lon
   if (h->mode16 && !h->shards[0].D && !h->result16)
     return h->fail(APSP_ESTATE, "no int32 matrix yet");
   if (h->result16) {
-    // widen int16 rows to int32 on the device (INF16 -> APSP_INF_I32), then D2H, in blocks
-    const long long blk = std::max<long long>(1, std::min<long long>(cnt, (64ll << 20) / (h->n * 4)));
+    // widen int16 rows to int32 on the device (INF16 -> APSP_INF_I32) into two
+    // alternating staging blocks; the D2H of one block overlaps the widening of the next
+    const long long ldw = (h->n + 7) / 8 * 8;
+    const long long blk = std::max<long long>(1, std::min<long long>(cnt, (64ll << 20) / (ldw * 4)));
     if (h->widen_rows < blk) {
       cudaFree(h->d_widen);
       h->d_widen = nullptr;
-      if ((st = h->cuda(cudaMalloc(&h->d_widen, blk * h->n * 4), "cudaMalloc widen"))) return st;
+      if ((st = h->cuda(cudaMalloc(&h->d_widen, 2 * blk * ldw * 4), "cudaMalloc widen"))) return st;
       h->widen_rows = blk;
     }
-    for (long long r = r0; r < r0 + cnt; r += blk) {
+    if (!h->copy_stream) {
+      if ((st = h->cuda(cudaStreamCreateWithFlags(&h->copy_stream, cudaStreamNonBlocking), "stream"))) return st;
+      for (auto& e : h->copy_ev)
+        if ((st = h->cuda(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event"))) return st;
+    }
+    int b = 0;
+    for (long long r = r0; r < r0 + cnt; r += blk, b ^= 1) {
       const long long rr = std::min(blk, r0 + cnt - r);
-      if ((st = h->cuda(launch_widen16(h->d16 + r * h->ld, h->ld, h->d_widen, h->n, rr, h->n, h->stream), "widen16")))
+      int* stage = h->d_widen + (size_t)b * h->widen_rows * ldw;
+      // the D2H that last read this staging block must be done before it is rewritten
+      if ((st = h->cuda(cudaStreamWaitEvent(h->stream, h->copy_ev[2 + b], 0), "wait"))) return st;
+      if ((st = h->cuda(launch_widen16(h->d16 + r * h->ld, h->ld, stage, ldw, rr, h->n, h->stream), "widen16")))
         return st;
-      if ((st = h->cuda(cudaMemcpy2DAsync(static_cast<int*>(out) + (r - r0) * ld_out, (size_t)ld_out * 4, h->d_widen,
-                                          (size_t)h->n * 4, (size_t)h->n * 4, (size_t)rr, cudaMemcpyDeviceToHost,
-                                          h->stream),
+      if ((st = h->cuda(cudaEventRecord(h->copy_ev[b], h->stream), "event"))) return st;
+      if ((st = h->cuda(cudaStreamWaitEvent(h->copy_stream, h->copy_ev[b], 0), "wait"))) return st;
+      if ((st = h->cuda(cudaMemcpy2DAsync(static_cast<int*>(out) + (r - r0) * ld_out, (size_t)ld_out * 4, stage,
+                                          (size_t)ldw * 4, (size_t)h->n * 4, (size_t)rr, cudaMemcpyDeviceToHost,
+                                          h->copy_stream),
                         "D2H dist")))
         return st;
+      if ((st = h->cuda(cudaEventRecord(h->copy_ev[2 + b], h->copy_stream), "event"))) return st;
     }
-    return h->cuda(cudaStreamSynchronize(h->stream), "get_dist sync");
+    return h->cuda(cudaStreamSynchronize(h->copy_stream), "get_dist sync");
   }
   const char* base;
   if (h->world > 1 && !h->virt) {

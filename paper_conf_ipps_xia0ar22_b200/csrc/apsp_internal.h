@@ -41,8 +41,10 @@ struct Handle {
   bool fell_back16 = false; // this graph needed int32: later runs go straight to int32
   short* d16 = nullptr;     // n_pad x n_pad int16 matrix (single GPU, in core)
   int* d_max16 = nullptr;
-  int* d_widen = nullptr;   // staging for get_dist of an int16 result
+  int* d_widen = nullptr;   // 2 staging blocks for get_dist of an int16 result
   long long widen_rows = 0;
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t copy_ev[4] = {nullptr, nullptr, nullptr, nullptr};  // widened[2], copied[2]
   int arith = APSP_ARITH_I32;
   // placement
   int device = 0;

@@ -201,6 +201,175 @@ __global__ void __launch_bounds__(MP_NT, 2) minplus_kernel(const __grid_constant
   }
 }
 
+// ------------------------------------------------ min-plus, mbarrier pipeline --
+//
+// Same tiling and shared layout as minplus_kernel, but the 3-stage pipeline is
+// synchronised with mbarriers instead of a CTA barrier per chunk:
+//   full[s]  (256 arrivals): each thread's cp.async.mbarrier.arrive.noinc fires
+//            when ITS copies into stage s have landed, so the stage becomes
+//            readable without any thread having to reach a sync point;
+//   empty[s] (8 arrivals): each warp arrives after its last read of stage s.
+// A warp refills the stage of chunk c-1 with its share of chunk c+2 after it
+// finished chunk c and the stage's empty barrier shows every warp is past c-1,
+// so warps may drift by about a chunk without stalling each other. The C tile
+// is fetched into the two stages that are free during the last chunk after one
+// CTA barrier (the only one per tile besides the epilogue's).
+
+__device__ __forceinline__ unsigned smem_addr(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mb_init(unsigned bar, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count));
+}
+__device__ __forceinline__ void mb_arrive(unsigned bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mb_cp_arrive(unsigned bar) {
+  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mb_wait(unsigned bar, unsigned parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "MBW_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra MBW_%=;\n"
+      "}\n" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+
+template <typename T>
+__global__ void __launch_bounds__(MP_NT, 2) minplus_mbar_kernel(const __grid_constant__ MinPlusArgs<T> args) {
+  using V4 = typename Vec4<T>::type;
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  T* const stage0 = reinterpret_cast<T*>(smem_raw);
+  __shared__ __align__(8) unsigned long long bars[2 * MP_STAGES];
+  const unsigned full0 = smem_addr(bars), empty0 = full0 + 8 * MP_STAGES;
+
+  long long t = blockIdx.x;
+  const bool second = t >= args.n0;
+  const MinPlusDesc<T>& d = second ? args.d1 : args.d0;
+  if (second) t -= args.n0;
+  int ti = (int)(t / d.tiles_j);
+  int tj = (int)(t - (long long)ti * d.tiles_j);
+  if (d.skip_i >= 0 && ti >= d.skip_i) ++ti;
+  if (d.skip_i2 >= 0 && ti >= d.skip_i2) ++ti;
+  if (d.skip_j >= 0 && tj >= d.skip_j) ++tj;
+  if (d.skip_j2 >= 0 && tj >= d.skip_j2) ++tj;
+
+  const T* __restrict__ Cin = d.Cin + (long long)ti * MP_BM * d.ldc_in + (long long)tj * MP_BN;
+  T* __restrict__ Cout = d.Cout + (long long)ti * MP_BM * d.ldc_out + (long long)tj * MP_BN;
+  const T* __restrict__ A = d.A + (long long)ti * MP_BM * d.lda;
+  const T* __restrict__ B = d.B + (long long)tj * MP_BN;
+  const long long lda = d.lda, ldb = d.ldb, ldc_in = d.ldc_in, ldc_out = d.ldc_out;
+
+  const int tid = threadIdx.x;
+  const int lane = tid & 31;
+  const int tx = tid & 15, ty = tid >> 4;
+  if (tid == 0) {
+    for (int s = 0; s < MP_STAGES; ++s) {
+      mb_init(full0 + 8 * s, MP_NT);
+      mb_init(empty0 + 8 * s, MP_NT / 32);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+
+  const T* const a_src = A + (tid >> 3) * lda + (tid & 7) * 4;
+  const T* const b_src = B + (tid >> 5) * ldb + (tid & 31) * 4;
+  const int a_dst = (tid >> 3) * MP_ALD + (tid & 7) * 4;
+  const int b_dst = MP_BM * MP_ALD + (tid >> 5) * MP_BLD + (tid & 31) * 4;
+  auto load_chunk = [&](int stage, int chunk) {
+    T* st = stage0 + stage * MP_STAGE_ELEMS;
+    const T* ag = a_src + chunk * MP_BK;
+    const T* bg = b_src + (long long)chunk * MP_BK * ldb;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) cp_async16(st + a_dst + q * 32 * MP_ALD, ag + q * 32 * lda);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) cp_async16(st + b_dst + q * 8 * MP_BLD, bg + q * 8 * ldb);
+    mb_cp_arrive(full0 + 8 * stage);
+  };
+
+  const int nk = args.K / MP_BK;
+  for (int s = 0; s < MP_STAGES - 1 && s < nk; ++s) load_chunk(s, s);
+
+  T acc[8][8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[i][j] = Val<T>::inf();
+  T* const cs_lo = stage0 + (nk % MP_STAGES) * MP_STAGE_ELEMS;
+  T* const cs_hi = stage0 + ((nk + 1) % MP_STAGES) * MP_STAGE_ELEMS;
+
+  int s = 0, ph = 0;  // stage of chunk c and its use parity
+  for (int c = 0; c < nk; ++c) {
+    if (c == nk - 1) {
+      // every warp is past chunk nk-2: the two other stages are free for C
+      __syncthreads();
+      const T* cg = Cin + (tid >> 5) * ldc_in + (tid & 31) * 4;
+      const int cd = (tid >> 5) * MP_CLD + (tid & 31) * 4;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) cp_async16(cs_lo + cd + q * 8 * MP_CLD, cg + q * 8 * ldc_in);
+#pragma unroll
+      for (int q = 0; q < 8; ++q) cp_async16(cs_hi + cd + q * 8 * MP_CLD, cg + (64 + q * 8) * ldc_in);
+      cp_async_commit();
+    }
+    mb_wait(full0 + 8 * s, (unsigned)ph);
+    const T* as = stage0 + s * MP_STAGE_ELEMS;
+    const T* bs = as + MP_BM * MP_ALD;
+#pragma unroll
+    for (int k2 = 0; k2 < MP_BK / 2; ++k2) {
+      T a[8][2];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
+        const T* ap = as + r * MP_ALD + k2 * 2;
+        a[i][0] = ap[0]; a[i][1] = ap[1];
+      }
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const T* brow = bs + (k2 * 2 + u) * MP_BLD;
+        V4 b0 = *reinterpret_cast<const V4*>(brow + tx * 4);
+        V4 b1 = *reinterpret_cast<const V4*>(brow + 64 + tx * 4);
+        const T b[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+          for (int j = 0; j < 8; ++j) acc[i][j] = Val<T>::relax(a[i][u], b[j], acc[i][j]);
+      }
+    }
+    __syncwarp();
+    if (lane == 0) mb_arrive(empty0 + 8 * s);
+    // refill the stage of chunk c-1 with this thread's share of chunk c+2
+    const int cn = c + MP_STAGES - 1;
+    if (cn < nk) {
+      const int sn = cn % MP_STAGES;  // == (c - 1) % 3
+      if (c >= 1) mb_wait(empty0 + 8 * sn, (unsigned)(((c - 1) / MP_STAGES) & 1));
+      load_chunk(sn, cn);
+    }
+    if (++s == MP_STAGES) {
+      s = 0;
+      ph ^= 1;
+    }
+  }
+  cp_async_wait<0>();
+  __syncthreads();
+
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
+    const T* crow = (i < 4 ? cs_lo : cs_hi) + (ty * 4 + (i & 3)) * MP_CLD;
+    V4 c0 = *reinterpret_cast<const V4*>(crow + tx * 4);
+    V4 c1 = *reinterpret_cast<const V4*>(crow + 64 + tx * 4);
+    V4 v0, v1;
+    v0.x = Val<T>::vmin(acc[i][0], c0.x); v0.y = Val<T>::vmin(acc[i][1], c0.y);
+    v0.z = Val<T>::vmin(acc[i][2], c0.z); v0.w = Val<T>::vmin(acc[i][3], c0.w);
+    v1.x = Val<T>::vmin(acc[i][4], c1.x); v1.y = Val<T>::vmin(acc[i][5], c1.y);
+    v1.z = Val<T>::vmin(acc[i][6], c1.z); v1.w = Val<T>::vmin(acc[i][7], c1.w);
+    *reinterpret_cast<V4*>(Cout + r * ldc_out + tx * 4) = v0;
+    *reinterpret_cast<V4*>(Cout + r * ldc_out + 64 + tx * 4) = v1;
+  }
+}
+
 template <typename T>
 static long long desc_tiles(const MinPlusDesc<T>& d) {
   return (long long)d.tiles_i * (long long)d.tiles_j;
@@ -221,7 +390,10 @@ cudaError_t launch_minplus(const MinPlusDesc<T>* d, int ndesc, int K, cudaStream
   if (total <= 0) return cudaSuccess;
   if (ndesc > 1 && a.n0 == 0) { a.d0 = a.d1; a.n0 = total; }
   constexpr int smem = minplus_smem_bytes<T>();
-  minplus_kernel<T><<<(unsigned)total, MP_NT, smem, s>>>(a);
+  if (g_minplus_variant == 3)
+    minplus_mbar_kernel<T><<<(unsigned)total, MP_NT, smem, s>>>(a);
+  else
+    minplus_kernel<T><<<(unsigned)total, MP_NT, smem, s>>>(a);
   return cudaGetLastError();
 }
 
@@ -385,7 +557,13 @@ cudaError_t launch_canonicalize_i32(int* D, long long ld, long long rows, long l
 // --------------------------------------------------------- instantiations --
 
 cudaError_t configure_kernels() {
-  cudaError_t e = cudaFuncSetAttribute(minplus_kernel<int>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  cudaError_t e = cudaFuncSetAttribute(minplus_mbar_kernel<int>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       minplus_smem_bytes<int>());
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(minplus_mbar_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           minplus_smem_bytes<float>());
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(minplus_kernel<int>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                        minplus_smem_bytes<int>());
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(minplus_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize,

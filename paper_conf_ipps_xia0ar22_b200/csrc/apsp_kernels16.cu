@@ -315,14 +315,27 @@ __global__ void max_finite16_kernel(const short* D, long long ld, long long rows
   if ((threadIdx.x & 31) == 0) atomicMax(out, m);
 }
 
-// int16 rows -> int32 rows (INF16 -> APSP_INF_I32)
-__global__ void widen16_kernel(const short* S, long long lds, int* D, long long ldd, long long rows, long long cols) {
-  const long long total = rows * cols;
-  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < total;
-       i += (long long)gridDim.x * blockDim.x) {
-    const long long r = i / cols, c = i - r * cols;
-    const short v = S[r * lds + c];
-    D[r * ldd + c] = v >= INF16 ? 0x3FFFFFFF : (int)v;
+// int16 rows -> int32 rows (INF16 -> APSP_INF_I32); one CTA per row, 8 values per step
+__global__ void widen16_kernel(const short* S, long long lds, int* D, long long ldd, long long cols) {
+  const short* src = S + blockIdx.x * lds;
+  int* dst = D + blockIdx.x * ldd;
+  const long long c8 = cols >> 3;
+  for (long long q = threadIdx.x; q < c8; q += blockDim.x) {
+    const uint4 v = *reinterpret_cast<const uint4*>(src + q * 8);
+    const unsigned w[4] = {v.x, v.y, v.z, v.w};
+    int o[8];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+      const short lo = (short)(w[k] & 0xFFFF), hi = (short)(w[k] >> 16);
+      o[2 * k] = lo >= INF16 ? 0x3FFFFFFF : (int)lo;
+      o[2 * k + 1] = hi >= INF16 ? 0x3FFFFFFF : (int)hi;
+    }
+    *reinterpret_cast<int4*>(dst + q * 8) = make_int4(o[0], o[1], o[2], o[3]);
+    *reinterpret_cast<int4*>(dst + q * 8 + 4) = make_int4(o[4], o[5], o[6], o[7]);
+  }
+  for (long long c = c8 * 8 + threadIdx.x; c < cols; c += blockDim.x) {
+    const short v = src[c];
+    dst[c] = v >= INF16 ? 0x3FFFFFFF : (int)v;
   }
 }
 
@@ -370,7 +383,7 @@ cudaError_t launch_max_finite16(const short* D, long long ld, long long rows, lo
 cudaError_t launch_widen16(const short* S, long long lds, int* D, long long ldd, long long rows, long long cols,
                            cudaStream_t s) {
   if (rows <= 0 || cols <= 0) return cudaSuccess;
-  widen16_kernel<<<148 * 8, 256, 0, s>>>(S, lds, D, ldd, rows, cols);
+  widen16_kernel<<<(unsigned)rows, 256, 0, s>>>(S, lds, D, ldd, cols);
   return cudaGetLastError();
 }
 

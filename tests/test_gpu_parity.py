@@ -82,18 +82,20 @@ def test_fw_int32_bit_exact(lib, n):
         assert_i32_equal(got, want)
 
 
+@pytest.mark.parametrize("variant", [2, 3])
 @pytest.mark.parametrize("n", [129, 640, 1000])
-def test_fw_tma_minplus_variant(lib, n):
-    """reserved[3] = 2 selects the TMA + mbarrier persistent min-plus kernel (cp.async is the default)."""
+def test_fw_minplus_variants(lib, n, variant):
+    """reserved[3] selects the min-plus kernel: 2 = TMA + mbarrier persistent,
+    3 = cp.async + mbarrier pipeline (0, the cp.async + CTA-barrier kernel, is the default)."""
     for name, g in graphs_for(n, seed=n + 3):
         c = cfg(lib)
-        c.reserved[3] = 2
+        c.reserved[3] = variant
         got = lib.solve(g, cfg=c)
         want, _ = oracle_i32(g)
         assert_i32_equal(got, want)
     gf = gg.erdos_renyi(n, 6 * n, seed=n, dtype="f32")
     c = cfg(lib)
-    c.reserved[3] = 2
+    c.reserved[3] = variant
     assert_f32_close(lib.solve(gf, cfg=c), oracle.fw_f64(gf.row_ptr, gf.col, gf.w)[0])
 
 
