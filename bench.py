@@ -48,8 +48,8 @@ def parse():
     ap.add_argument("--stream-all", action="store_true", help="out-of-core: keep no band resident")
     ap.add_argument("--no-lookahead", action="store_true", help="in-core: no phase-3 split / overlap")
     ap.add_argument("--minplus-variant", type=int, default=0,
-                    help="min-plus kernel for A/B: 0 cp.async + CTA barrier (default), 2 TMA persistent, "
-                         "3 cp.async + mbarrier pipeline")
+                    help="min-plus kernel for A/B: 0 cp.async + mbarrier pipeline (default), "
+                         "1 cp.async + CTA barrier per chunk, 2 TMA persistent")
     ap.add_argument("--no-packed16", action="store_true", help="skip the packed-int16 alternative measurement")
     ap.add_argument("--packed16", action="store_true",
                     help="packed int16 arithmetic (VIADDMNMX.S16x2) when exact, int32 otherwise")

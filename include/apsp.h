@@ -213,8 +213,13 @@ apsp_status apsp_get_phase_stats(const apsp_handle* h, apsp_phase_stats* out);
 /* Rank-0 helper: write a fresh 128-byte ncclUniqueId into out128. */
 apsp_status apsp_nccl_unique_id(void* out128);
 
-/* Release everything the handle owns. NULL is allowed. */
+/* Release everything the handle owns. NULL is allowed. The large device
+ * buffers come from the device's stream-ordered memory pool (cudaMallocAsync),
+ * which keeps freed memory cached for the next handle (no driver round trip). */
 void apsp_destroy(apsp_handle* h);
+
+/* Return the cached pool memory of `device` (-1 = current) to the driver. */
+apsp_status apsp_trim_memory(int32_t device);
 
 /* Last error message of h (thread-local message when h is NULL). Never NULL. */
 const char* apsp_last_error(const apsp_handle* h);

@@ -93,6 +93,7 @@ _sig = {
     "apsp_get_phase_stats": (ctypes.c_int, [_H, ctypes.POINTER(apsp_phase_stats)]),
     "apsp_nccl_unique_id": (ctypes.c_int, [_P]),
     "apsp_destroy": (None, [_H]),
+    "apsp_trim_memory": (ctypes.c_int, [_I32]),
     "apsp_last_error": (ctypes.c_char_p, [_H]),
     "apsp_version": (ctypes.c_char_p, []),
 }
@@ -250,6 +251,10 @@ def apsp_get_phase_stats(h: Handle) -> apsp_phase_stats:
 
 def apsp_destroy(h: Handle) -> None:
     h.close()
+
+
+def apsp_trim_memory(device: int = -1) -> None:
+    _check(_lib.apsp_trim_memory(device))
 
 
 def apsp_last_error(h: Handle | None = None) -> str:

@@ -121,7 +121,7 @@ static apsp_status incore_round(Handle* h, long long k) {
       return st;
     panel = static_cast<const T*>(h->panel);
   } else {
-    if ((st = h->bcast(own ? (void*)band : h->panel, band_elems * sizeof(T), owner))) return st;
+    if ((st = h->bcast(own ? (void*)band : h->panel, band_elems * sizeof(T), owner, s))) return st;
     panel = own ? band : static_cast<const T*>(h->panel);
   }
   h->ev_end(0);
@@ -144,12 +144,123 @@ static apsp_status incore_round(Handle* h, long long k) {
   return APSP_OK;
 }
 
+// All rounds of the sharded (1-D block-row) schedule with lookahead:
+//   side stream X: pivot(k) = owner's phase 1 + row panel of band k, then the
+//                  band broadcast (NCCL) / device copy into panel[k & 1];
+//   main stream S: round k = every shard's column-panel tiles, then phase 3.
+// During round k the owner of band k+1 first updates its band-(k+1) tiles, so
+// pivot(k+1) — including its broadcast over NVLink — runs on X while S does the
+// rest of round k's phase 3. A panel buffer is rewritten only after the phase 3
+// that read it (two rounds earlier) has finished. All ranks issue the
+// broadcasts in the same order (k = 0, 1, ...) on X.
+template <typename T>
+static apsp_status sharded_lookahead(Handle* h) {
+  const long long b = h->b, ld = h->ld, nb = h->n_pad / b;
+  const long long R = h->rows_per_rank;
+  const int local_tiles = (int)(R / b);
+  cudaStream_t S = h->stream, X = h->side;
+  const size_t band_elems = (size_t)b * (size_t)h->n_pad;
+  T* panels[2] = {static_cast<T*>(h->panel), static_cast<T*>(h->panel) + band_elems};
+  apsp_status st;
+  for (auto& e : h->ev_sh)
+    if (!e && (st = h->cuda(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event"))) return st;
+  cudaEvent_t ev_bcast = h->ev_sh[0], ev_band = h->ev_sh[1], ev_p3 = h->ev_sh[2];
+
+  auto owner_of = [&](long long k) { return (int)((k * b) / R); };
+  auto shard_of = [&](int rank) -> Shard* {
+    for (auto& sh : h->shards)
+      if (sh.rank == rank) return &sh;
+    return nullptr;
+  };
+  auto local_tile = [&](const Shard* sh, long long k) { return (int)((k * b - sh->row_begin) / b); };
+  auto Dp = [&](const Shard* sh) { return static_cast<T*>(sh->D); };
+
+  // pivot(k) on X; returns the panel round k reads
+  auto pivot = [&](long long k, const T*& panel_k) -> apsp_status {
+    Shard* own = shard_of(owner_of(k));
+    T* band = own ? Dp(own) + (long long)local_tile(own, k) * b * ld : nullptr;
+    if (own) {
+      h->ev_begin(0, X);
+      if ((st = h->cuda(launch_phase1<T>(band + k * b, ld, h->d_flag, X), "phase1"))) return st;
+      h->ev_end((double)b * b * b, X);
+      MinPlusDesc<T> dr = mkdesc<T>(band, band, band + k * b, band, ld, ld, ld, 1, (int)(nb - 1), -1, (int)k);
+      h->ev_begin(1, X);
+      if ((st = h->cuda(launch_minplus<T>(&dr, 1, (int)b, X), "phase2-row"))) return st;
+      h->ev_end(desc_relax(dr, (int)b), X);
+    }
+    // panel[k & 1] was last read by round k-2, whose end is ev_p3's latest record
+    if (k >= 2 && (st = h->cuda(cudaStreamWaitEvent(X, ev_p3, 0), "wait"))) return st;
+    T* dst = panels[k & 1];
+    h->ev_begin(3, X);
+    if (h->virt) {
+      if ((st = h->cuda(cudaMemcpyAsync(dst, band, band_elems * sizeof(T), cudaMemcpyDeviceToDevice, X), "panel")))
+        return st;
+      panel_k = dst;
+    } else {
+      if ((st = h->bcast(own ? (void*)band : (void*)dst, band_elems * sizeof(T), owner_of(k), X))) return st;
+      panel_k = own ? band : dst;
+    }
+    h->ev_end(0, X);
+    return h->cuda(cudaEventRecord(ev_bcast, X), "event");
+  };
+
+  const T* next_panel = nullptr;
+  if ((st = h->cuda(cudaEventRecord(ev_p3, S), "event"))) return st;  // X must not run ahead of prior S work
+  if ((st = h->cuda(cudaStreamWaitEvent(X, ev_p3, 0), "wait"))) return st;
+  if ((st = pivot(0, next_panel))) return st;
+  for (long long k = 0; k < nb; ++k) {
+    const T* panel = next_panel;
+    if ((st = h->cuda(cudaStreamWaitEvent(S, ev_bcast, 0), "wait"))) return st;
+    // column-panel tiles of every shard
+    for (auto& sh : h->shards) {
+      const int skip = sh.rank == owner_of(k) ? local_tile(&sh, k) : -1;
+      T* D = Dp(&sh);
+      MinPlusDesc<T> dc = mkdesc<T>(D + k * b, D + k * b, D + k * b, panel + k * b, ld, ld, ld,
+                                    local_tiles - (skip >= 0), 1, skip, -1);
+      h->ev_begin(1, S);
+      if ((st = h->cuda(launch_minplus<T>(&dc, 1, (int)b, S), "phase2-col"))) return st;
+      h->ev_end(desc_relax(dc, (int)b), S);
+    }
+    const long long k1 = k + 1;
+    Shard* own1 = k1 < nb ? shard_of(owner_of(k1)) : nullptr;
+    if (own1) {  // band k+1 first, then its pivot can start on X
+      T* D = Dp(own1);
+      T* row = D + (long long)local_tile(own1, k1) * b * ld;
+      MinPlusDesc<T> pa = mkdesc<T>(row, row, row + k * b, panel, ld, ld, ld, 1, (int)(nb - 1), -1, (int)k);
+      h->ev_begin(2, S);
+      if ((st = h->cuda(launch_minplus<T>(&pa, 1, (int)b, S), "phase3a"))) return st;
+      h->ev_end(desc_relax(pa, (int)b), S);
+      if ((st = h->cuda(cudaEventRecord(ev_band, S), "event"))) return st;
+      if ((st = h->cuda(cudaStreamWaitEvent(X, ev_band, 0), "wait"))) return st;
+    }
+    if (k1 < nb && (st = pivot(k1, next_panel))) return st;
+    // the rest of phase 3
+    for (auto& sh : h->shards) {
+      int s0 = sh.rank == owner_of(k) ? local_tile(&sh, k) : -1;
+      int s1 = (own1 == &sh) ? local_tile(&sh, k1) : -1;
+      if (s0 < 0) std::swap(s0, s1);
+      const int tiles_i = local_tiles - (s0 >= 0) - (s1 >= 0);
+      if (tiles_i <= 0) continue;
+      T* D = Dp(&sh);
+      MinPlusDesc<T> p3 = mkdesc<T>(D, D, D + k * b, panel, ld, ld, ld, tiles_i, (int)(nb - 1), s0, (int)k);
+      p3.skip_i2 = s1;
+      h->ev_begin(2, S);
+      if ((st = h->cuda(launch_minplus<T>(&p3, 1, (int)b, S), "phase3"))) return st;
+      h->ev_end(desc_relax(p3, (int)b), S);
+    }
+    if ((st = h->cuda(cudaEventRecord(ev_p3, S), "event"))) return st;
+  }
+  return APSP_OK;
+}
+
 apsp_status run_incore_rounds(Handle* h, long long k0, long long k1) {
   if (h->world == 1 && !h->use_comm) {  // single GPU: the whole closure, with lookahead
     return h->dtype == APSP_I32
                ? fw_closure<int>(h, static_cast<int*>(h->shards[0].D), h->ld, h->n_pad, k0, k1, h->stream)
                : fw_closure<float>(h, static_cast<float*>(h->shards[0].D), h->ld, h->n_pad, k0, k1, h->stream);
   }
+  if (h->side && k0 == 0 && k1 == h->n_pad / h->b)
+    return h->dtype == APSP_I32 ? sharded_lookahead<int>(h) : sharded_lookahead<float>(h);
   for (long long k = k0; k < k1; ++k) {
     apsp_status st = (h->dtype == APSP_I32) ? incore_round<int>(h, k) : incore_round<float>(h, k);
     if (st) return st;
@@ -384,6 +495,16 @@ apsp_status apsp_get_phase_stats(const apsp_handle* hh, apsp_phase_stats* out) {
 void apsp_destroy(apsp_handle* hh) {
   if (!hh) return;
   delete_handle(reinterpret_cast<Handle*>(hh));
+}
+
+apsp_status apsp_trim_memory(int32_t device) {
+  int dev = device;
+  if (dev < 0 && cudaGetDevice(&dev) != cudaSuccess) return fail_global(APSP_ECUDA, "no CUDA device");
+  cudaMemPool_t pool;
+  if (cudaDeviceGetDefaultMemPool(&pool, dev) != cudaSuccess) return fail_global(APSP_ECUDA, "no memory pool");
+  if (cudaDeviceSynchronize() != cudaSuccess || cudaMemPoolTrimTo(pool, 0) != cudaSuccess)
+    return fail_global(APSP_ECUDA, "cudaMemPoolTrimTo failed");
+  return APSP_OK;
 }
 
 }  // extern "C"

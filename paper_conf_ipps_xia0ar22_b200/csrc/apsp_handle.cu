@@ -19,8 +19,8 @@ bool nccl_unique_id(void* out128) {
   return true;
 }
 
-apsp_status Handle::bcast(void* buf, size_t bytes, int root) {
-  ncclResult_t r = ncclBroadcast(buf, buf, bytes, ncclUint8, root, static_cast<ncclComm_t>(comm), stream);
+apsp_status Handle::bcast(void* buf, size_t bytes, int root, cudaStream_t s) {
+  ncclResult_t r = ncclBroadcast(buf, buf, bytes, ncclUint8, root, static_cast<ncclComm_t>(comm), s);
   if (r != ncclSuccess) return fail(APSP_ENCCL, "ncclBroadcast: %s", ncclGetErrorString(r));
   return APSP_OK;
 }
@@ -104,7 +104,15 @@ apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_pt
   if (prop.major < 10) return h->fail(APSP_ECUDA, "device %s is sm_%d%d; this library is built for sm_100a", prop.name,
                                       prop.major, prop.minor);
   if ((st = h->cuda(configure_kernels(), "configure_kernels"))) return st;
-  g_minplus_variant = cfg.reserved[3];  // test hook: 0 = cp.async (default), 2 = TMA min-plus kernel
+  {
+    // keep freed pool memory cached (apsp_trim_memory releases it)
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, h->device) == cudaSuccess) {
+      unsigned long long thr = ~0ull;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  }
+  g_minplus_variant = cfg.reserved[3];  // test hook: min-plus kernel variant (apsp_kernels.cuh)
   if (cfg.stream) {
     h->stream = static_cast<cudaStream_t>(cfg.stream);
   } else {
@@ -132,7 +140,12 @@ apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_pt
   // ---- in-core or out-of-core? ---------------------------------------------
   const int nshards = h->virt ? h->world : 1;
   const long long mat_bytes = (long long)nshards * h->rows_per_rank * h->ld * (long long)h->elem;
-  const long long panel_bytes = h->world > 1 ? (long long)h->b * h->ld * (long long)h->elem : 0;
+  // reserved[2] = 1: run the sharded schedule with a 1-rank NCCL communicator even
+  // at world_size 1, so a single GPU exercises the broadcast / all-reduce path
+  h->use_comm = (h->world > 1 && !h->virt) || (h->world == 1 && cfg.reserved[2] == 1);
+  // two pivot-band panels (double-buffered by round parity)
+  const long long panel_bytes =
+      (h->world > 1 || h->use_comm) ? 2 * (long long)h->b * h->ld * (long long)h->elem : 0;
   size_t free_b = 0, total_b = 0;
   if ((st = h->cuda(cudaMemGetInfo(&free_b, &total_b), "cudaMemGetInfo"))) return st;
   long long budget = cfg.device_budget_bytes > 0 ? cfg.device_budget_bytes
@@ -150,7 +163,8 @@ apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_pt
               h->world == 1 && !h->virt && cfg.reserved[2] != 1;
   if (h->mode16) {
     const long long b16 = h->n_pad * h->n_pad * 2;
-    if ((st = h->cuda(cudaMalloc(&h->d16, b16), "cudaMalloc dist16"))) return st;
+    if ((st = h->cuda(cudaMallocAsync(reinterpret_cast<void**>(&h->d16), b16, h->stream), "cudaMalloc dist16")))
+      return st;
     if ((st = h->cuda(cudaMalloc(&h->d_max16, sizeof(int)), "cudaMalloc"))) return st;
     h->device_bytes = b16;
     Shard sh;  // the int32 matrix is allocated only if the int16 result must be redone
@@ -160,10 +174,10 @@ apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_pt
     return h->cuda(cudaStreamSynchronize(h->stream), "init sync");
   }
 
-  if ((st = h->cuda(cudaMalloc(&h->d_base, mat_bytes), "cudaMalloc dist"))) return st;
+  if ((st = h->cuda(cudaMallocAsync(&h->d_base, mat_bytes, h->stream), "cudaMalloc dist"))) return st;
   h->device_bytes = mat_bytes;
   if (panel_bytes) {
-    if ((st = h->cuda(cudaMalloc(&h->panel, panel_bytes), "cudaMalloc panel"))) return st;
+    if ((st = h->cuda(cudaMallocAsync(&h->panel, panel_bytes, h->stream), "cudaMalloc panel"))) return st;
     h->device_bytes += panel_bytes;
   }
   for (int s = 0; s < nshards; ++s) {
@@ -174,9 +188,6 @@ apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_pt
     h->shards.push_back(sh);
   }
 
-  // reserved[2] = 1: run the sharded schedule with a 1-rank NCCL communicator even
-  // at world_size 1, so a single GPU exercises the broadcast / all-reduce path
-  h->use_comm = (h->world > 1 && !h->virt) || (h->world == 1 && cfg.reserved[2] == 1);
   if (h->use_comm) {
     ncclUniqueId id;
     if (cfg.nccl_unique_id) {
@@ -221,7 +232,8 @@ apsp_status run_fw16(Handle* h) {
   Shard& sh = h->shards[0];
   if (!sh.D) {
     const long long mat_bytes = h->n_pad * h->ld * 4;
-    if ((st = h->cuda(cudaMalloc(&h->d_base, mat_bytes), "cudaMalloc dist (int32 fallback)"))) return st;
+    if ((st = h->cuda(cudaMallocAsync(&h->d_base, mat_bytes, h->stream), "cudaMalloc dist (int32 fallback)")))
+      return st;
     h->device_bytes += mat_bytes;
     sh.D = h->d_base;
   }
@@ -237,7 +249,18 @@ apsp_status run_fw16(Handle* h) {
 void delete_handle(Handle* h) {
   if (!h) return;
   cudaSetDevice(h->device);
-  if (h->stream) cudaStreamSynchronize(h->stream);
+  if (h->side) cudaStreamSynchronize(h->side);
+  if (h->copy_stream) cudaStreamSynchronize(h->copy_stream);
+  if (h->stream) {
+    // large buffers come from the device's stream-ordered pool (cudaMallocAsync); the
+    // pool keeps them for the next handle instead of returning them to the driver
+    if (h->d_base) cudaFreeAsync(h->d_base, h->stream);
+    if (h->d16) cudaFreeAsync(h->d16, h->stream);
+    if (h->panel) cudaFreeAsync(h->panel, h->stream);
+    h->d_base = h->panel = nullptr;
+    h->d16 = nullptr;
+    cudaStreamSynchronize(h->stream);
+  }
   for (auto& te : h->events) {
     cudaEventDestroy(te.a);
     cudaEventDestroy(te.b);
@@ -249,8 +272,6 @@ void delete_handle(Handle* h) {
     cudaFree(sh.d_col);
     cudaFree(sh.d_w);
   }
-  cudaFree(h->d_base);
-  cudaFree(h->d16);
   cudaFree(h->d_max16);
   if (h->copy_stream) {
     cudaStreamSynchronize(h->copy_stream);
@@ -259,7 +280,6 @@ void delete_handle(Handle* h) {
   for (auto& e : h->copy_ev)
     if (e) cudaEventDestroy(e);
   cudaFree(h->d_widen);
-  cudaFree(h->panel);
   cudaFree(h->d_flag);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
   if (h->side) {
@@ -267,6 +287,8 @@ void delete_handle(Handle* h) {
     cudaStreamDestroy(h->side);
   }
   for (auto& e : h->ev_la)
+    if (e) cudaEventDestroy(e);
+  for (auto& e : h->ev_sh)
     if (e) cudaEventDestroy(e);
   delete h;
 }

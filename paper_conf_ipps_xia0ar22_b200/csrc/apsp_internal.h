@@ -78,7 +78,8 @@ struct Handle {
 
   apsp_status fail(apsp_status st, const char* fmt, ...);
   apsp_status cuda(cudaError_t e, const char* what);
-  apsp_status bcast(void* buf, size_t bytes, int root);
+  apsp_status bcast(void* buf, size_t bytes, int root, cudaStream_t s);
+  cudaEvent_t ev_sh[3] = {nullptr, nullptr, nullptr};  // sharded lookahead: bcast, band, p3
   // class: 0 phase1, 1 phase2, 2 phase3, 3 comm / host transfer
   void ev_begin(int cls, cudaStream_t s);
   void ev_end(double relax, cudaStream_t s);

@@ -390,10 +390,10 @@ cudaError_t launch_minplus(const MinPlusDesc<T>* d, int ndesc, int K, cudaStream
   if (total <= 0) return cudaSuccess;
   if (ndesc > 1 && a.n0 == 0) { a.d0 = a.d1; a.n0 = total; }
   constexpr int smem = minplus_smem_bytes<T>();
-  if (g_minplus_variant == 3)
-    minplus_mbar_kernel<T><<<(unsigned)total, MP_NT, smem, s>>>(a);
-  else
+  if (g_minplus_variant == 1)
     minplus_kernel<T><<<(unsigned)total, MP_NT, smem, s>>>(a);
+  else
+    minplus_mbar_kernel<T><<<(unsigned)total, MP_NT, smem, s>>>(a);
   return cudaGetLastError();
 }
 

@@ -72,9 +72,10 @@ cudaError_t launch_widen16(const short* S, long long lds, int* D, long long ldd,
 cudaError_t configure_kernels16();
 
 // The TMA + mbarrier persistent variant of launch_minplus (apsp_minplus_tma.cu).
-// g_minplus_variant (set from apsp_config.reserved[3]): 0 = cp.async kernel
-// (default), 2 = TMA persistent kernel (measured slower in round 1: its
-// persistent grid also blocks the lookahead phases 1+2).
+// g_minplus_variant (set from apsp_config.reserved[3]): 0 = cp.async +
+// mbarrier pipeline (default), 1 = cp.async + one CTA barrier per chunk,
+// 2 = TMA persistent kernel (measured slower in round 1: its persistent grid
+// also blocks the lookahead phases 1+2).
 template <typename T>
 cudaError_t launch_minplus_tma(const MinPlusDesc<T>* d, int ndesc, int K, cudaStream_t s);
 cudaError_t configure_tma_kernels();
