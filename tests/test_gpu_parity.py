@@ -236,6 +236,21 @@ def test_virtual_ranks_match_oracle(lib, world):
         assert_i32_equal(got, want)
 
 
+@pytest.mark.parametrize("world", [2, 4])
+def test_virtual_ranks_without_lookahead(lib, world):
+    """reserved[1] = 1: the sharded schedule round by round on one stream (no pivot lookahead)."""
+    for g in [gg.grid_2d(20, 33, seed=world + 7), gg.erdos_renyi(1100, 4000, seed=world + 7)]:
+        c = cfg(lib, world_size=world, virtual_ranks=1)
+        c.reserved[1] = 1
+        assert_i32_equal(lib.solve(g, cfg=c), oracle_i32(g)[0])
+
+
+def test_virtual_ranks_f32(lib):
+    g = gg.erdos_renyi(800, 6400, seed=8, dtype="f32")
+    got = lib.solve(g, cfg=cfg(lib, world_size=3, virtual_ranks=1))
+    assert_f32_close(got, oracle.fw_f64(g.row_ptr, g.col, g.w)[0])
+
+
 def test_nccl_path_single_rank(lib):
     """reserved[2] = 1: the sharded schedule with a real 1-rank NCCL communicator
     (ncclBroadcast of the pivot band every round, ncclAllReduce of the status flag)."""
