@@ -117,48 +117,17 @@ __global__ void __launch_bounds__(S_NT, 2) minplus16_kernel(const __grid_constan
     *reinterpret_cast<uint4*>(p1 + 4) = make_uint4(d1[4], d1[5], d1[6], d1[7]);
   };
 
-  // mbarrier pipeline (as minplus_mbar_kernel): full[s] completes when every
-  // thread's B copies have landed (cp.async arrive.noinc) AND every thread has
-  // stored its duplicated A values (plain arrive after the STS); empty[s] when
-  // all 8 warps are done reading stage s
-  __shared__ __align__(8) unsigned long long bars16[2 * S_ST];
-  const unsigned full0 = (unsigned)__cvta_generic_to_shared(bars16), empty0 = full0 + 8 * S_ST;
-  if (tid == 0) {
-    for (int s = 0; s < S_ST; ++s) {
-      asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(full0 + 8 * s), "r"(2 * S_NT));
-      asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(empty0 + 8 * s), "r"(S_NT / 32));
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  auto arrive = [](unsigned bar) { asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory"); };
-  auto cp_arrive = [](unsigned bar) {
-    asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bar) : "memory");
-  };
-  auto wait = [](unsigned bar, unsigned parity) {
-    asm volatile(
-        "{\n"
-        ".reg .pred p;\n"
-        "W16_%=:\n"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-        "@!p bra W16_%=;\n"
-        "}\n" ::"r"(bar),
-        "r"(parity)
-        : "memory");
-  };
-
   const int nk = args.K / S_BK;
   // prologue: chunks 0 and 1
 #pragma unroll
   for (int s = 0; s < S_ST - 1; ++s) {
     if (s < nk) {
       load_b(s, s);
-      cp_arrive(full0 + 8 * s);
       uint4 r0, r1;
       load_a_regs(s, r0, r1);
       store_a(s, r0, r1);
-      arrive(full0 + 8 * s);
     }
+    commit();
   }
 
   unsigned acc[8][4];
@@ -171,25 +140,26 @@ __global__ void __launch_bounds__(S_NT, 2) minplus16_kernel(const __grid_constan
   unsigned short* const c_lo = reinterpret_cast<unsigned short*>(smem_raw + (nk % S_ST) * S_STAGE_BYTES);
   unsigned short* const c_hi = reinterpret_cast<unsigned short*>(smem_raw + ((nk + 1) % S_ST) * S_STAGE_BYTES);
 
-  int st = 0, ph = 0;  // stage of chunk c and its use parity
   for (int c = 0; c < nk; ++c) {
+    wait_group<S_ST - 2>();
+    __syncthreads();
+    const int cn = c + S_ST - 1;
+    uint4 ra0, ra1;
+    if (cn < nk) {
+      load_b(cn % S_ST, cn);
+      load_a_regs(cn, ra0, ra1);
+    }
     if (c == nk - 1) {
-      // every warp is past chunk nk-2: the two other stages are free for C
-      __syncthreads();
       const int cr = tid >> 4, cc = (tid & 15) * 8;
 #pragma unroll
       for (int q = 0; q < 4; ++q) {
         cp_async16b(c_lo + (cr + 16 * q) * 128 + cc, Cin + (cr + 16 * q) * d.ldc_in + cc);
         cp_async16b(c_hi + (cr + 16 * q) * 128 + cc, Cin + (64 + cr + 16 * q) * d.ldc_in + cc);
       }
-      commit();
     }
-    const int cn = c + S_ST - 1;
-    uint4 ra0, ra1;
-    if (cn < nk) load_a_regs(cn, ra0, ra1);  // A of chunk c+2 into registers, in flight during chunk c
-    wait(full0 + 8 * st, (unsigned)ph);
-    const unsigned* as = stageA(st);
-    const unsigned short* bs = stageB(st);
+    commit();
+    const unsigned* as = stageA(c % S_ST);
+    const unsigned short* bs = stageB(c % S_ST);
 #pragma unroll
     for (int k4 = 0; k4 < S_BK / 4; ++k4) {
       unsigned a[8][4];
@@ -209,21 +179,8 @@ __global__ void __launch_bounds__(S_NT, 2) minplus16_kernel(const __grid_constan
           for (int p = 0; p < 4; ++p) acc[i][p] = __viaddmin_s16x2(a[i][u], b[p], acc[i][p]);
       }
     }
-    __syncwarp();
-    if ((tid & 31) == 0) arrive(empty0 + 8 * st);
-    // refill the stage of chunk c-1 with this thread's share of chunk c+2
-    if (cn < nk) {
-      const int sn = cn % S_ST;
-      if (c >= 1) wait(empty0 + 8 * sn, (unsigned)(((c - 1) / S_ST) & 1));
-      load_b(sn, cn);
-      cp_arrive(full0 + 8 * sn);
-      store_a(sn, ra0, ra1);
-      arrive(full0 + 8 * sn);
-    }
-    if (++st == S_ST) {
-      st = 0;
-      ph ^= 1;
-    }
+    // stage cn was last read in chunk c-1; every thread passed this chunk's barrier
+    if (cn < nk) store_a(cn % S_ST, ra0, ra1);
   }
   wait_group<0>();
   __syncthreads();
