@@ -29,6 +29,7 @@ class CSR:
     col: np.ndarray  # int32 [m]
     w: np.ndarray  # int32 or float32 [m]
     name: str = ""
+    meta: dict | None = None  # generator facts (grid: rows, cols, perm)
 
     @property
     def m(self) -> int:
@@ -117,11 +118,36 @@ def grid_2d(rows: int, cols: int, seed: int, dtype: str = "i32", permute: bool =
     else:
         w = draw_weights(rng, u.size, dtype, lo, hi)
     n = rows * cols
+    perm = np.arange(n, dtype=np.int64)
     if permute:
         perm = rng.permutation(n).astype(np.int64)
         u, v = perm[u], perm[v]
-    return csr_from_arcs(n, np.concatenate([u, v]), np.concatenate([v, u]),
-                         np.concatenate([w, w]), name or f"grid_{rows}x{cols}")
+    g = csr_from_arcs(n, np.concatenate([u, v]), np.concatenate([v, u]),
+                      np.concatenate([w, w]), name or f"grid_{rows}x{cols}")
+    g.meta = {"rows": rows, "cols": cols, "perm": perm}  # vertex (r, c) has id perm[r*cols + c]
+    return g
+
+
+def grid_block_partition(g: CSR, block_rows: int, block_cols: int):
+    """Geometric partition of a grid_2d graph into block_rows x block_cols rectangles of
+    cells (the stand-in for the paper's METIS k-way partition, on mesh-like
+    graphs). Returns (comp int32[n], k)."""
+    rows, cols, perm = g.meta["rows"], g.meta["cols"], g.meta["perm"]
+    old = np.empty(g.n, dtype=np.int64)
+    old[perm] = np.arange(g.n)
+    r, c = old // cols, old % cols
+    bh = -(-rows // block_rows)
+    bw = -(-cols // block_cols)
+    comp = (r // bh) * block_cols + (c // bw)
+    return comp.astype(np.int32), block_rows * block_cols
+
+
+def random_partition(n: int, k: int, seed: int):
+    """Balanced random partition (many boundary nodes: a stress case, not a small separator)."""
+    rng = np.random.default_rng(seed)
+    comp = np.arange(n) % k
+    rng.shuffle(comp)
+    return comp.astype(np.int32), k
 
 
 def relabel(g: CSR, perm) -> CSR:

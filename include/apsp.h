@@ -63,6 +63,7 @@ typedef enum {
 
 #define APSP_MODE_INCORE 0
 #define APSP_MODE_OUT_OF_CORE 1
+#define APSP_MODE_BOUNDARY 2
 
 typedef struct {
   int32_t struct_size;          /* = sizeof(apsp_config) (ABI versioning); 0 = defaults */
@@ -126,6 +127,33 @@ void apsp_config_default(apsp_config* cfg);
 apsp_status apsp_init_from_csr(apsp_handle** out, int64_t n, const int64_t* row_ptr,
                                const int32_t* col_idx, const void* weights, apsp_dtype dtype,
                                const apsp_config* cfg);
+
+/*
+ * apsp_init_boundary — set up the boundary algorithm (Djidjev et al.,
+ * PAPER.md:139-150, eq. (1); Algorithm 3) for a graph with a
+ * small separator. Same CSR arguments and semantics as apsp_init_from_csr,
+ * plus a partition of the vertices (the paper uses METIS; the caller
+ * provides it here):
+ *   comp      host int32[n], component of each vertex, in [0, k)
+ *   k         number of components, >= 1
+ * A vertex with an arc to another component is a boundary node. Work
+ * is O(k s^3 + NB^3 + n * NB * s) for components of size s and NB boundary
+ * nodes instead of n^3. Single GPU, in core (the n x n result must fit in
+ * device memory). Run with apsp_solve; apsp_get_dist as usual.
+ * Errors: as apsp_init_from_csr; APSP_EINVAL for a bad comp / k; APSP_ENOMEM
+ * when the result does not fit.
+ */
+apsp_status apsp_init_boundary(apsp_handle** out, int64_t n, const int64_t* row_ptr,
+                               const int32_t* col_idx, const void* weights, apsp_dtype dtype,
+                               const int32_t* comp, int32_t k, const apsp_config* cfg);
+
+/*
+ * apsp_solve — run the method the handle was created for: the blocked
+ * Floyd–Warshall (apsp_init_from_csr, same as apsp_fw_blocked) or the boundary
+ * algorithm (apsp_init_boundary). Blocks until done; APSP_ENEGCYCLE as
+ * apsp_fw_blocked.
+ */
+apsp_status apsp_solve(apsp_handle* h);
 
 /*
  * apsp_fw_blocked — run the whole blocked Floyd–Warshall (all n/b rounds,
@@ -192,6 +220,7 @@ typedef struct {
   int32_t arith;                               /* APSP_ARITH_*: arithmetic of the current
                                                   result (or of the next run) */
   int32_t packed16_eligible;                   /* packed16 requested and the input allows it */
+  int64_t boundary_nodes;                      /* boundary algorithm: boundary nodes, else 0 */
 } apsp_info;
 
 #define APSP_ARITH_I32 0   /* VIADDMNMX (int32 DPX), 1 relaxation / instruction */

@@ -63,6 +63,7 @@ class apsp_info(ctypes.Structure):
         ("rounds", ctypes.c_int64), ("device_bytes", ctypes.c_int64), ("host_bytes", ctypes.c_int64),
         ("dist_device", ctypes.c_void_p), ("ld", ctypes.c_int64),
         ("arith", ctypes.c_int32), ("packed16_eligible", ctypes.c_int32),
+        ("boundary_nodes", ctypes.c_int64),
     ]
 
 
@@ -83,6 +84,9 @@ _sig = {
     "apsp_init_from_csr": (ctypes.c_int, [ctypes.POINTER(_H), _I64, _P, _P, _P, ctypes.c_int,
                                           ctypes.POINTER(apsp_config)]),
     "apsp_fw_blocked": (ctypes.c_int, [_H]),
+    "apsp_init_boundary": (ctypes.c_int, [ctypes.POINTER(_H), _I64, _P, _P, _P, ctypes.c_int, _P, _I32,
+                                          ctypes.POINTER(apsp_config)]),
+    "apsp_solve": (ctypes.c_int, [_H]),
     "apsp_reinit": (ctypes.c_int, [_H]),
     "apsp_fw_rounds": (ctypes.c_int, [_H, _I64, _I64]),
     "apsp_get_dist": (ctypes.c_int, [_H, _I64, _I64, _P, _I64]),
@@ -207,6 +211,30 @@ def apsp_fw_blocked(h: Handle) -> None:
     _check(_lib.apsp_fw_blocked(h.raw), h.raw)
 
 
+def apsp_init_boundary(n: int, row_ptr, col_idx, weights, comp, k: int, dtype: int | None = None,
+                       cfg: apsp_config | None = None) -> Handle:
+    """Boundary algorithm with the caller's partition comp[v] in [0, k)."""
+    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
+    comp = np.ascontiguousarray(comp, dtype=np.int32)
+    w = np.asarray(weights)
+    if dtype is None:
+        dtype = APSP_F32 if w.dtype.kind == "f" else APSP_I32
+    w = np.ascontiguousarray(w, dtype=np.int32 if dtype == APSP_I32 else np.float32)
+    if row_ptr.shape[0] != n + 1 or comp.shape[0] != n:
+        raise ApspError(APSP_EINVAL, "row_ptr must have n+1 entries and comp n")
+    if cfg is None:
+        cfg = apsp_config_default()
+    raw = ctypes.c_void_p()
+    _check(_lib.apsp_init_boundary(ctypes.byref(raw), n, _ptr(row_ptr), _ptr(col_idx), _ptr(w), dtype, _ptr(comp),
+                                   k, ctypes.byref(cfg)))
+    return Handle(raw, dtype, n, (cfg,))
+
+
+def apsp_solve(h: Handle) -> None:
+    _check(_lib.apsp_solve(h.raw), h.raw)
+
+
 def apsp_reinit(h: Handle) -> None:
     _check(_lib.apsp_reinit(h.raw), h.raw)
 
@@ -267,4 +295,11 @@ def solve(g, cfg: apsp_config | None = None, dtype: int | None = None) -> np.nda
     """Full APSP of a ``graphgen.CSR``-like object (n, row_ptr, col, w) -> n x n host array."""
     with apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, dtype=dtype, cfg=cfg) as h:
         apsp_fw_blocked(h)
+        return apsp_get_dist(h)
+
+
+def solve_boundary(g, comp, k: int, cfg: apsp_config | None = None) -> np.ndarray:
+    """Full APSP by the boundary algorithm with partition comp (k components)."""
+    with apsp_init_boundary(g.n, g.row_ptr, g.col, g.w, comp, k, cfg=cfg) as h:
+        apsp_solve(h)
         return apsp_get_dist(h)

@@ -314,30 +314,9 @@ apsp_status apsp_nccl_unique_id(void* out128) {
   return nccl_unique_id(out128) ? APSP_OK : fail_global(APSP_ENCCL, "ncclGetUniqueId failed");
 }
 
-apsp_status apsp_init_from_csr(apsp_handle** out, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
-                               const void* weights, apsp_dtype dtype, const apsp_config* cfg_in) {
-  if (!out) return fail_global(APSP_EINVAL, "apsp_init_from_csr: out is NULL");
-  *out = nullptr;
-  apsp_config cfg;
-  apsp_config_default(&cfg);
-  if (cfg_in) {
-    if (cfg_in->struct_size != 0 && cfg_in->struct_size != (int32_t)sizeof(apsp_config))
-      return fail_global(APSP_EINVAL, "apsp_config.struct_size %d != %d", cfg_in->struct_size,
-                         (int)sizeof(apsp_config));
-    cfg = *cfg_in;
-  }
-  if (n < 0) return fail_global(APSP_EINVAL, "n < 0");
-  if (n > (int64_t)INT32_MAX) return fail_global(APSP_EINVAL, "n exceeds int32 vertex ids");
-  if (!row_ptr) return fail_global(APSP_EINVAL, "row_ptr is NULL");
-  if (dtype != APSP_I32 && dtype != APSP_F32) return fail_global(APSP_EINVAL, "bad dtype");
-  if (cfg.tile == 0) cfg.tile = kTile;
-  if (cfg.tile != kTile) return fail_global(APSP_EINVAL, "tile must be %d in this build", kTile);
-  if (cfg.world_size < 1 || cfg.rank < 0 || cfg.rank >= cfg.world_size)
-    return fail_global(APSP_EINVAL, "bad world_size/rank");
-  if (cfg.world_size > 1 && !cfg.virtual_ranks && !cfg.nccl_unique_id)
-    return fail_global(APSP_EINVAL, "world_size > 1 needs nccl_unique_id (or virtual_ranks)");
-
-  // ---- validate the CSR on the host (O(n + m)) -----------------------------
+// Host validation of a CSR graph (O(n + m)) and the int32 range rule (R5).
+static apsp_status validate_csr(int64_t n, const int64_t* row_ptr, const int32_t* col_idx, const void* weights,
+                                apsp_dtype dtype, bool* has_neg_out, int64_t* maxabs_out) {
   if (row_ptr[0] != 0) return fail_global(APSP_EINVAL, "row_ptr[0] != 0");
   for (int64_t i = 0; i < n; ++i)
     if (row_ptr[i + 1] < row_ptr[i]) return fail_global(APSP_EINVAL, "row_ptr not monotone at %lld", (long long)i);
@@ -365,6 +344,38 @@ apsp_status apsp_init_from_csr(apsp_handle** out, int64_t n, const int64_t* row_
       if (w[e] < 0) has_neg = true;
     }
   }
+  *has_neg_out = has_neg;
+  *maxabs_out = maxabs;
+  return APSP_OK;
+}
+
+apsp_status apsp_init_from_csr(apsp_handle** out, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                               const void* weights, apsp_dtype dtype, const apsp_config* cfg_in) {
+  if (!out) return fail_global(APSP_EINVAL, "apsp_init_from_csr: out is NULL");
+  *out = nullptr;
+  apsp_config cfg;
+  apsp_config_default(&cfg);
+  if (cfg_in) {
+    if (cfg_in->struct_size != 0 && cfg_in->struct_size != (int32_t)sizeof(apsp_config))
+      return fail_global(APSP_EINVAL, "apsp_config.struct_size %d != %d", cfg_in->struct_size,
+                         (int)sizeof(apsp_config));
+    cfg = *cfg_in;
+  }
+  if (n < 0) return fail_global(APSP_EINVAL, "n < 0");
+  if (n > (int64_t)INT32_MAX) return fail_global(APSP_EINVAL, "n exceeds int32 vertex ids");
+  if (!row_ptr) return fail_global(APSP_EINVAL, "row_ptr is NULL");
+  if (dtype != APSP_I32 && dtype != APSP_F32) return fail_global(APSP_EINVAL, "bad dtype");
+  if (cfg.tile == 0) cfg.tile = kTile;
+  if (cfg.tile != kTile) return fail_global(APSP_EINVAL, "tile must be %d in this build", kTile);
+  if (cfg.world_size < 1 || cfg.rank < 0 || cfg.rank >= cfg.world_size)
+    return fail_global(APSP_EINVAL, "bad world_size/rank");
+  if (cfg.world_size > 1 && !cfg.virtual_ranks && !cfg.nccl_unique_id)
+    return fail_global(APSP_EINVAL, "world_size > 1 needs nccl_unique_id (or virtual_ranks)");
+
+  bool has_neg = false;
+  int64_t maxabs = 0;
+  apsp_status vst = validate_csr(n, row_ptr, col_idx, weights, dtype, &has_neg, &maxabs);
+  if (vst != APSP_OK) return vst;
 
   Handle* h = new Handle();
   h->n = n;
@@ -389,6 +400,64 @@ apsp_status apsp_init_from_csr(apsp_handle** out, int64_t n, const int64_t* row_
   return APSP_OK;
 }
 
+apsp_status apsp_init_boundary(apsp_handle** out, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                               const void* weights, apsp_dtype dtype, const int32_t* comp, int32_t k,
+                               const apsp_config* cfg_in) {
+  if (!out) return fail_global(APSP_EINVAL, "apsp_init_boundary: out is NULL");
+  *out = nullptr;
+  apsp_config cfg;
+  apsp_config_default(&cfg);
+  if (cfg_in) {
+    if (cfg_in->struct_size != 0 && cfg_in->struct_size != (int32_t)sizeof(apsp_config))
+      return fail_global(APSP_EINVAL, "apsp_config.struct_size %d != %d", cfg_in->struct_size,
+                         (int)sizeof(apsp_config));
+    cfg = *cfg_in;
+  }
+  if (n < 1 || n > (int64_t)INT32_MAX) return fail_global(APSP_EINVAL, "bad n");
+  if (!row_ptr || !comp) return fail_global(APSP_EINVAL, "row_ptr / comp is NULL");
+  if (dtype != APSP_I32 && dtype != APSP_F32) return fail_global(APSP_EINVAL, "bad dtype");
+  if (k < 1) return fail_global(APSP_EINVAL, "k < 1");
+  if (cfg.world_size != 1) return fail_global(APSP_EINVAL, "the boundary algorithm runs on one GPU");
+  for (int64_t v = 0; v < n; ++v)
+    if (comp[v] < 0 || comp[v] >= k) return fail_global(APSP_EINVAL, "comp[%lld] out of [0, k)", (long long)v);
+  bool has_neg = false;
+  int64_t maxabs = 0;
+  apsp_status vst = validate_csr(n, row_ptr, col_idx, weights, dtype, &has_neg, &maxabs);
+  if (vst != APSP_OK) return vst;
+
+  Handle* h = new Handle();
+  h->n = n;
+  h->dtype = dtype;
+  h->timing = cfg.timing != 0;
+  h->has_neg = has_neg;
+  h->max_abs_w = maxabs;
+  h->arith = dtype == APSP_F32 ? APSP_ARITH_F32 : APSP_ARITH_I32;
+  h->elem = 4;
+  h->mode = APSP_MODE_BOUNDARY;
+  apsp_status st = setup_device(h, cfg);
+  if (!st) st = bnd_setup(h, row_ptr, col_idx, weights, comp, k);
+  if (st != APSP_OK) {
+    g_last_error = h->err;
+    delete_handle(h);
+    return st;
+  }
+  *out = reinterpret_cast<apsp_handle*>(h);
+  return APSP_OK;
+}
+
+apsp_status apsp_solve(apsp_handle* hh) {
+  if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
+  Handle* h = reinterpret_cast<Handle*>(hh);
+  if (h->mode != APSP_MODE_BOUNDARY) return apsp_fw_blocked(hh);
+  if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  if (h->fw_done) return h->fail(APSP_ESTATE, "apsp_solve already ran (apsp_reinit first)");
+  apsp_status st;
+  if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
+  memset(&h->stats, 0, sizeof(h->stats));
+  if ((st = bnd_run(h))) return st;
+  return finish_fw(h, true);
+}
+
 apsp_status apsp_fw_rounds(apsp_handle* hh, int64_t k_begin, int64_t k_end) {
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
@@ -410,6 +479,7 @@ apsp_status apsp_fw_blocked(apsp_handle* hh) {
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
   if (h->fw_done) return h->fail(APSP_ESTATE, "apsp_fw_blocked already ran");
+  if (h->mode == APSP_MODE_BOUNDARY) return h->fail(APSP_ESTATE, "boundary-algorithm handle: use apsp_solve");
   apsp_status st;
   if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
   memset(&h->stats, 0, sizeof(h->stats));
@@ -436,6 +506,7 @@ apsp_status apsp_reinit(apsp_handle* hh) {
   apsp_status st;
   if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
   if (h->mode == APSP_MODE_OUT_OF_CORE) return ooc_reinit(h);
+  if (h->mode == APSP_MODE_BOUNDARY) return bnd_reinit(h);
   return run_init(h);
 }
 
@@ -483,6 +554,7 @@ apsp_status apsp_get_info(const apsp_handle* hh, apsp_info* info) {
   info->arith = h->arith;
   info->packed16_eligible = h->mode16 ? 1 : 0;
   if (h->result16) info->dist_device = h->d16;
+  info->boundary_nodes = bnd_boundary_nodes(h);
   return APSP_OK;
 }
 

@@ -86,8 +86,27 @@ apsp_status run_init(Handle* h) {
   return APSP_OK;
 }
 
+static apsp_status init_placement(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, const int32_t* col,
+                                  const void* w);
+
 apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, const int32_t* col,
                         const void* w) {
+  apsp_status st;
+  if ((st = setup_device(h, cfg))) return st;
+
+  int64_t np, rb, rc;
+  if (apsp_partition(h->n, h->b, h->world, h->virt ? 0 : h->rank, &np, &rb, &rc) != APSP_OK)
+    return h->fail(APSP_EINVAL, "partition failed");
+  h->n_pad = np;
+  h->rows_per_rank = np / h->world;
+  h->ld = np;
+
+  // ---- in-core or out-of-core? ---------------------------------------------
+  return init_placement(h, cfg, row_ptr, col, w);
+}
+
+// Device selection, kernel attributes, pool policy, streams, status flag.
+apsp_status setup_device(Handle* h, const apsp_config& cfg) {
   apsp_status st;
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
@@ -126,18 +145,14 @@ apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_pt
     for (auto& e : h->ev_la)
       if ((st = h->cuda(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event"))) return st;
   }
-
-  int64_t np, rb, rc;
-  if (apsp_partition(h->n, h->b, h->world, h->virt ? 0 : h->rank, &np, &rb, &rc) != APSP_OK)
-    return h->fail(APSP_EINVAL, "partition failed");
-  h->n_pad = np;
-  h->rows_per_rank = np / h->world;
-  h->ld = np;
-
   if ((st = h->cuda(cudaMalloc(&h->d_flag, sizeof(int)), "cudaMalloc flag"))) return st;
-  if ((st = h->cuda(cudaMemsetAsync(h->d_flag, 0, sizeof(int), h->stream), "memset flag"))) return st;
+  return h->cuda(cudaMemsetAsync(h->d_flag, 0, sizeof(int), h->stream), "memset flag");
+}
 
-  // ---- in-core or out-of-core? ---------------------------------------------
+// In-core (1-D block-row shards, packed int16) or out-of-core placement + init.
+static apsp_status init_placement(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, const int32_t* col,
+                                  const void* w) {
+  apsp_status st;
   const int nshards = h->virt ? h->world : 1;
   const long long mat_bytes = (long long)nshards * h->rows_per_rank * h->ld * (long long)h->elem;
   // reserved[2] = 1: run the sharded schedule with a 1-rank NCCL communicator even
@@ -267,6 +282,7 @@ void delete_handle(Handle* h) {
   }
   if (h->comm) ncclCommDestroy(static_cast<ncclComm_t>(h->comm));
   ooc_free(h);
+  bnd_free(h);
   for (auto& sh : h->shards) {
     cudaFree(sh.d_rp);
     cudaFree(sh.d_col);
@@ -313,6 +329,7 @@ apsp_status finish_fw(Handle* h, bool all_rounds) {
 
 apsp_status get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out) {
   if (h->mode == APSP_MODE_OUT_OF_CORE) return ooc_get_rows(h, r0, cnt, out, ld_out);
+  if (h->mode == APSP_MODE_BOUNDARY) return bnd_get_rows(h, r0, cnt, out, ld_out);
   apsp_status st;
   if (h->mode16 && !h->shards[0].D && !h->result16)
     return h->fail(APSP_ESTATE, "no int32 matrix yet");

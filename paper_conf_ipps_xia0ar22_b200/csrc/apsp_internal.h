@@ -67,6 +67,8 @@ struct Handle {
   void* h_dist = nullptr;   // pinned n_pad x n_pad host matrix
   void* ooc_dev = nullptr;  // device arena for bands
   void* ooc_streams[3] = {nullptr, nullptr, nullptr};
+  // boundary algorithm (apsp_boundary.cu)
+  void* bnd = nullptr;
   // bookkeeping
   long long device_bytes = 0, host_bytes = 0;
   long long next_round = 0;
@@ -105,5 +107,16 @@ apsp_status run_out_of_core(Handle* h);
 apsp_status ooc_get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out);
 void ooc_free(Handle* h);
 apsp_status ooc_reinit(Handle* h);
+
+// boundary algorithm (apsp_boundary.cu)
+apsp_status bnd_setup(Handle* h, const int64_t* row_ptr, const int32_t* col, const void* w, const int32_t* comp,
+                      int k);
+apsp_status bnd_reinit(Handle* h);
+apsp_status bnd_run(Handle* h);
+apsp_status bnd_get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out);
+long long bnd_boundary_nodes(const Handle* h);
+void bnd_free(Handle* h);
+// common device / stream setup of a handle (apsp_handle.cu)
+apsp_status setup_device(Handle* h, const apsp_config& cfg);
 
 }  // namespace apsp

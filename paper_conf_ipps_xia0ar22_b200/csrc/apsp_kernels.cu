@@ -238,23 +238,65 @@ __device__ __forceinline__ void mb_wait(unsigned bar, unsigned parity) {
 }
 
 template <typename T>
-__global__ void __launch_bounds__(MP_NT, 2) minplus_mbar_kernel(const __grid_constant__ MinPlusArgs<T> args) {
-  using V4 = typename Vec4<T>::type;
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  T* const stage0 = reinterpret_cast<T*>(smem_raw);
-  __shared__ __align__(8) unsigned long long bars[2 * MP_STAGES];
-  const unsigned full0 = smem_addr(bars), empty0 = full0 + 8 * MP_STAGES;
-
-  long long t = blockIdx.x;
-  const bool second = t >= args.n0;
-  const MinPlusDesc<T>& d = second ? args.d1 : args.d0;
-  if (second) t -= args.n0;
-  int ti = (int)(t / d.tiles_j);
-  int tj = (int)(t - (long long)ti * d.tiles_j);
+__device__ __forceinline__ void tile_of(const MinPlusDesc<T>& d, long long t, int& ti, int& tj) {
+  ti = (int)(t / d.tiles_j);
+  tj = (int)(t - (long long)ti * d.tiles_j);
   if (d.skip_i >= 0 && ti >= d.skip_i) ++ti;
   if (d.skip_i2 >= 0 && ti >= d.skip_i2) ++ti;
   if (d.skip_j >= 0 && tj >= d.skip_j) ++tj;
   if (d.skip_j2 >= 0 && tj >= d.skip_j2) ++tj;
+}
+
+template <typename T>
+__device__ __forceinline__ void minplus_mbar_tile(const MinPlusDesc<T>& d, int ti, int tj, int K,
+                                                  unsigned char* smem_raw, unsigned long long* bars);
+
+template <typename T>
+__global__ void __launch_bounds__(MP_NT, 2) minplus_mbar_kernel(const __grid_constant__ MinPlusArgs<T> args) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  __shared__ __align__(8) unsigned long long bars[2 * MP_STAGES];
+  long long t = blockIdx.x;
+  const bool second = t >= args.n0;
+  const MinPlusDesc<T>& d = second ? args.d1 : args.d0;
+  if (second) t -= args.n0;
+  int ti, tj;
+  tile_of(d, t, ti, tj);
+  minplus_mbar_tile<T>(d, ti, tj, args.K, smem_raw, bars);
+}
+
+// Many tile families in one launch (the boundary algorithm's products, one
+// family per component pair): descs[f] in device memory, prefix[f] = first
+// CTA of family f (prefix[nf] = grid), depth per family in desc.K.
+template <typename T>
+__global__ void __launch_bounds__(MP_NT, 2) minplus_batched_kernel(const MinPlusDesc<T>* __restrict__ descs,
+                                                                   const long long* __restrict__ prefix, int nf) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  __shared__ __align__(8) unsigned long long bars[2 * MP_STAGES];
+  __shared__ MinPlusDesc<T> sd;
+  __shared__ long long st0;
+  if (threadIdx.x == 0) {
+    const long long t = blockIdx.x;
+    int lo = 0, hi = nf - 1;  // last f with prefix[f] <= t
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (prefix[mid] <= t) lo = mid; else hi = mid - 1;
+    }
+    sd = descs[lo];
+    st0 = prefix[lo];
+  }
+  __syncthreads();
+  const MinPlusDesc<T> d = sd;
+  int ti, tj;
+  tile_of(d, (long long)blockIdx.x - st0, ti, tj);
+  minplus_mbar_tile<T>(d, ti, tj, d.K, smem_raw, bars);
+}
+
+template <typename T>
+__device__ __forceinline__ void minplus_mbar_tile(const MinPlusDesc<T>& d, int ti, int tj, int K,
+                                                  unsigned char* smem_raw, unsigned long long* bars) {
+  using V4 = typename Vec4<T>::type;
+  T* const stage0 = reinterpret_cast<T*>(smem_raw);
+  const unsigned full0 = smem_addr(bars), empty0 = full0 + 8 * MP_STAGES;
 
   const T* __restrict__ Cin = d.Cin + (long long)ti * MP_BM * d.ldc_in + (long long)tj * MP_BN;
   T* __restrict__ Cout = d.Cout + (long long)ti * MP_BM * d.ldc_out + (long long)tj * MP_BN;
@@ -289,7 +331,7 @@ __global__ void __launch_bounds__(MP_NT, 2) minplus_mbar_kernel(const __grid_con
     mb_cp_arrive(full0 + 8 * stage);
   };
 
-  const int nk = args.K / MP_BK;
+  const int nk = K / MP_BK;
   for (int s = 0; s < MP_STAGES - 1 && s < nk; ++s) load_chunk(s, s);
 
   T acc[8][8];
@@ -410,7 +452,21 @@ cudaError_t launch_minplus(const MinPlusDesc<T>* d, int ndesc, int K, cudaStream
 // negative cycle (flagged; the result is then unspecified).
 
 template <typename T>
+__device__ __forceinline__ void phase1_body(T* tile, long long ld, int* negflag);
+
+template <typename T>
 __global__ void __launch_bounds__(256) phase1_kernel(T* tile, long long ld, int* negflag) {
+  phase1_body<T>(tile, ld, negflag);
+}
+
+// one pivot tile per CTA (the boundary algorithm closes all components' tiles of a round at once)
+template <typename T>
+__global__ void __launch_bounds__(256) phase1_batched_kernel(T* const* tiles, long long ld, int* negflag) {
+  phase1_body<T>(tiles[blockIdx.x], ld, negflag);
+}
+
+template <typename T>
+__device__ __forceinline__ void phase1_body(T* tile, long long ld, int* negflag) {
   using V4 = typename Vec4<T>::type;
   __shared__ __align__(16) T rowbuf[2][kTile];
   __shared__ __align__(16) T colbuf[2][kTile];
@@ -480,6 +536,15 @@ cudaError_t launch_phase1(T* tile, long long ld, int* negflag, cudaStream_t s) {
   phase1_kernel<T><<<1, 256, 0, s>>>(tile, ld, negflag);
   return cudaGetLastError();
 }
+
+template <typename T>
+cudaError_t launch_phase1_batched(T* const* tiles, int count, long long ld, int* negflag, cudaStream_t s) {
+  if (count <= 0) return cudaSuccess;
+  phase1_batched_kernel<T><<<count, 256, 0, s>>>(tiles, ld, negflag);
+  return cudaGetLastError();
+}
+template cudaError_t launch_phase1_batched<int>(int* const*, int, long long, int*, cudaStream_t);
+template cudaError_t launch_phase1_batched<float>(float* const*, int, long long, int*, cudaStream_t);
 
 // ------------------------------------------------------------------ init --
 //
@@ -554,6 +619,82 @@ cudaError_t launch_canonicalize_i32(int* D, long long ld, long long rows, long l
   return cudaGetLastError();
 }
 
+// ------------------------------------------------------ batched min-plus --
+
+template <typename T>
+cudaError_t launch_minplus_batched(const MinPlusDesc<T>* descs, const long long* prefix, int nf, long long total,
+                                   cudaStream_t s) {
+  if (nf <= 0 || total <= 0) return cudaSuccess;
+  minplus_batched_kernel<T><<<(unsigned)total, MP_NT, minplus_smem_bytes<T>(), s>>>(descs, prefix, nf);
+  return cudaGetLastError();
+}
+
+// --------------------------------------------------------------- helpers --
+
+template <typename T>
+__global__ void fill_kernel(T* p, long long count, T v) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < count;
+       i += (long long)gridDim.x * blockDim.x)
+    p[i] = v;
+}
+
+template <typename T>
+cudaError_t launch_fill(T* p, long long count, T value, cudaStream_t s) {
+  if (count <= 0) return cudaSuccess;
+  fill_kernel<T><<<148 * 4, 256, 0, s>>>(p, count, value);
+  return cudaGetLastError();
+}
+
+template <typename T>
+__global__ void min_into_kernel(T* dst, long long ldd, const T* src, long long lds, long long cols) {
+  T* d = dst + blockIdx.x * ldd;
+  const T* q = src + blockIdx.x * lds;
+  for (long long c = threadIdx.x; c < cols; c += blockDim.x) d[c] = Val<T>::vmin(d[c], q[c]);
+}
+
+template <typename T>
+cudaError_t launch_min_into(T* dst, long long ldd, const T* src, long long lds, long long rows, long long cols,
+                            cudaStream_t s) {
+  if (rows <= 0 || cols <= 0) return cudaSuccess;
+  min_into_kernel<T><<<(unsigned)rows, 256, 0, s>>>(dst, ldd, src, lds, cols);
+  return cudaGetLastError();
+}
+
+template <typename T>
+__device__ __forceinline__ T canon_inf(T v) { return v; }
+template <>
+__device__ __forceinline__ int canon_inf<int>(int v) { return v >= 0x3FFFFFFF / 2 ? 0x3FFFFFFF : v; }
+
+template <typename T>
+__global__ void gather_kernel(const T* D, long long ld, const int* rowmap, const int* colmap, T* out, long long ldo,
+                              long long ncols) {
+  const T* src = D + (long long)rowmap[blockIdx.x] * ld;
+  T* dst = out + blockIdx.x * ldo;
+  for (long long c = threadIdx.x; c < ncols; c += blockDim.x) dst[c] = canon_inf<T>(src[colmap[c]]);
+}
+
+template <typename T>
+cudaError_t launch_gather(const T* D, long long ld, const int* rowmap, const int* colmap, T* out, long long ldo,
+                          long long cnt, long long ncols, cudaStream_t s) {
+  if (cnt <= 0 || ncols <= 0) return cudaSuccess;
+  gather_kernel<T><<<(unsigned)cnt, 256, 0, s>>>(D, ld, rowmap, colmap, out, ldo, ncols);
+  return cudaGetLastError();
+}
+
+template cudaError_t launch_minplus_batched<int>(const MinPlusDesc<int>*, const long long*, int, long long,
+                                                 cudaStream_t);
+template cudaError_t launch_minplus_batched<float>(const MinPlusDesc<float>*, const long long*, int, long long,
+                                                   cudaStream_t);
+template cudaError_t launch_fill<int>(int*, long long, int, cudaStream_t);
+template cudaError_t launch_fill<float>(float*, long long, float, cudaStream_t);
+template cudaError_t launch_min_into<int>(int*, long long, const int*, long long, long long, long long, cudaStream_t);
+template cudaError_t launch_min_into<float>(float*, long long, const float*, long long, long long, long long,
+                                            cudaStream_t);
+template cudaError_t launch_gather<int>(const int*, long long, const int*, const int*, int*, long long, long long,
+                                        long long, cudaStream_t);
+template cudaError_t launch_gather<float>(const float*, long long, const int*, const int*, float*, long long,
+                                          long long, long long, cudaStream_t);
+
 // --------------------------------------------------------- instantiations --
 
 cudaError_t configure_kernels() {
@@ -561,6 +702,12 @@ cudaError_t configure_kernels() {
                                        minplus_smem_bytes<int>());
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(minplus_mbar_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           minplus_smem_bytes<float>());
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(minplus_batched_kernel<int>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           minplus_smem_bytes<int>());
+  if (e != cudaSuccess) return e;
+  e = cudaFuncSetAttribute(minplus_batched_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                            minplus_smem_bytes<float>());
   if (e != cudaSuccess) return e;
   e = cudaFuncSetAttribute(minplus_kernel<int>, cudaFuncAttributeMaxDynamicSharedMemorySize,

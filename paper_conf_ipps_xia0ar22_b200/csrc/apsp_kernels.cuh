@@ -26,7 +26,31 @@ struct MinPlusDesc {
   long long ldc_out, ldc_in, lda, ldb;
   int tiles_i, tiles_j, skip_i, skip_j;
   int skip_i2 = -1, skip_j2 = -1;  // optional second skipped index, > skip_i / skip_j
+  int K = 0;                       // depth, used by launch_minplus_batched only
 };
+
+// Many tile families in one launch: descs / prefix are DEVICE arrays of nf
+// descriptors (each with its own K, a multiple of 32) and nf+1 CTA offsets
+// (prefix[0] = 0, prefix[nf] = total tiles).
+template <typename T>
+cudaError_t launch_minplus_batched(const MinPlusDesc<T>* descs, const long long* prefix, int nf, long long total,
+                                   cudaStream_t s);
+
+// phase 1 on `count` tiles (device array of tile pointers, same ld), one CTA each
+template <typename T>
+cudaError_t launch_phase1_batched(T* const* tiles, int count, long long ld, int* negflag, cudaStream_t s);
+
+// small helpers (boundary algorithm)
+template <typename T>
+cudaError_t launch_fill(T* p, long long count, T value, cudaStream_t s);
+// dst = min(dst, src) on a rows x cols block
+template <typename T>
+cudaError_t launch_min_into(T* dst, long long ldd, const T* src, long long lds, long long rows, long long cols,
+                            cudaStream_t s);
+// out[r][c] = D[rowmap[r]][colmap[c]] for r < cnt, c < ncols (int32: values >= INF/2 -> INF)
+template <typename T>
+cudaError_t launch_gather(const T* D, long long ld, const int* rowmap, const int* colmap, T* out, long long ldo,
+                          long long cnt, long long ncols, cudaStream_t s);
 
 // Phase 2 / phase 3 / out-of-core products: up to two tile families in one
 // launch (grid = total tiles). K must be a positive multiple of 32.
