@@ -32,7 +32,7 @@ APSP_OK, APSP_EINVAL, APSP_ERANGE, APSP_ENOMEM, APSP_ECUDA, APSP_ENCCL, APSP_ENE
 STATUS_NAMES = ["APSP_OK", "APSP_EINVAL", "APSP_ERANGE", "APSP_ENOMEM", "APSP_ECUDA", "APSP_ENCCL",
                 "APSP_ENEGCYCLE", "APSP_ESTATE"]
 APSP_INF_I32 = 0x3FFFFFFF
-APSP_MODE_INCORE, APSP_MODE_OUT_OF_CORE = 0, 1
+APSP_MODE_INCORE, APSP_MODE_OUT_OF_CORE, APSP_MODE_BOUNDARY = 0, 1, 2
 TILE = 128
 
 

@@ -87,3 +87,28 @@ def test_no_gpu_fails_loudly(lib):
     with pytest.raises(lib.ApspError) as e:
         lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w)
     assert e.value.status == lib.APSP_ECUDA
+
+
+def test_binding_constants_match_header(lib):
+    """Every `#define APSP_*` integer constant and `apsp_status` / `apsp_dtype` enumerator in
+    include/apsp.h has the same value in the Python binding."""
+    src = open(os.path.join(ROOT, "include", "apsp.h")).read()
+    src_nc = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    consts = {k: int(v, 0) for k, v in re.findall(r"#define\s+(APSP_[A-Z0-9_]+)\s+(0x[0-9A-Fa-f]+|\d+)\b", src_nc)}
+    for body in re.findall(r"typedef\s+enum\s*\{(.*?)\}", src_nc, flags=re.S):
+        nxt = 0
+        for item in body.split(","):
+            item = item.strip()
+            if not item:
+                continue
+            if "=" in item:
+                name, val = (s.strip() for s in item.split("="))
+                nxt = int(val, 0)
+            else:
+                name = item
+            consts[name] = nxt
+            nxt += 1
+    assert "APSP_MODE_BOUNDARY" in consts and "APSP_ENEGCYCLE" in consts
+    for name, val in consts.items():
+        if name.startswith("APSP_") and not name.endswith("_H"):
+            assert getattr(lib, name) == val, name
