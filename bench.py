@@ -47,6 +47,9 @@ def parse():
     ap.add_argument("--ooc-block", type=int, default=0, help="out-of-core band height B (0 = auto)")
     ap.add_argument("--stream-all", action="store_true", help="out-of-core: keep no band resident")
     ap.add_argument("--no-lookahead", action="store_true", help="in-core: no phase-3 split / overlap")
+    ap.add_argument("--legacy", action="store_true",
+                    help="single GPU: launch-per-phase schedule instead of the persistent dataflow kernel")
+    ap.add_argument("--df-delay", type=int, default=0, help="dataflow kernel queue delay (0 = auto)")
     ap.add_argument("--minplus-variant", type=int, default=0,
                     help="min-plus kernel for A/B: 0 cp.async + mbarrier pipeline (default), "
                          "1 cp.async + CTA barrier per chunk, 2 TMA persistent")
@@ -229,6 +232,9 @@ def run_ours(args):
         if args.no_lookahead:
             cfg.reserved[1] = 1
         cfg.reserved[3] = args.minplus_variant
+        if args.legacy:
+            cfg.reserved[4] = 1
+        cfg.reserved[5] = args.df_delay
         if packed16:
             cfg.packed16 = 1
         if uid is not None:
@@ -308,7 +314,10 @@ def run_ours(args):
                         traffic = tj["dram_bytes_per_relax"] * p3_relax
             except Exception:
                 pass
-        roofline = {"bound": "alu", "kernel": "phase-3 min-plus (%s)" % arith, "achieved": achieved / 1e12,
+        dataflow = st_acc[1][0] == 0 and st_acc[1][2] == args.steps  # one launch per step, no phase-1 launches
+        kname = ("fw_dataflow_kernel: all rounds and phases 1-3 in one persistent launch (%s)" % arith if dataflow
+                 else "phase-3 min-plus (%s)" % arith)
+        roofline = {"bound": "alu", "kernel": kname, "achieved": achieved / 1e12,
                     "peak": peak / 1e12, "unit": "Trelax/s", "frac": achieved / peak, "traffic": traffic,
                     "traffic_unit": "bytes per launch (DRAM read+write)",
                     "algorithmic_bytes_per_launch": (p3_relax * 2 * 128 * 128 * elem / 128 ** 3

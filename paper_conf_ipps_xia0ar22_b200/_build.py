@@ -53,6 +53,7 @@ def build_lib(force: bool = False, verbose: bool = False) -> str:
     newest_hdr = max(os.path.getmtime(h) for h in headers)
     common = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC,-O2",
               "-I", os.path.join(ROOT, "include"), "-I", inc]
+    common += os.environ.get("APSP_NVCC_EXTRA", "").split()  # experiments (pass force=True)
     procs, objs = [], []
     for s in srcs:
         o = os.path.join(BUILD, os.path.basename(s) + ".o")

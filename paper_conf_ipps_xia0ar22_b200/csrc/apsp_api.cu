@@ -13,6 +13,8 @@
 //                         B rows streamed from pinned host memory
 //                         (apsp_ooc.cu).
 #include "apsp_internal.h"
+
+#include <cstdlib>
 #include "apsp_sched.cuh"
 
 #include <cstdio>
@@ -253,7 +255,55 @@ static apsp_status sharded_lookahead(Handle* h) {
   return APSP_OK;
 }
 
+// All rounds of a single-GPU in-core closure in one persistent dataflow launch
+// (apsp_fw_dataflow.cu). The phases are not separable in time, so the launch
+// is timed as one event of class 2 carrying all n_pad^3 relaxations.
+template <typename T>
+static apsp_status run_dataflow(Handle* h) {
+  const int nb = (int)(h->n_pad / h->b);
+  apsp_status st;
+  if (!h->df_work) {
+    if ((st = h->cuda(cudaMallocAsync(&h->df_work, fw_dataflow_work_bytes(nb, sizeof(T)), h->stream),
+                      "cudaMalloc dataflow")))
+      return st;
+    h->device_bytes += fw_dataflow_work_bytes(nb, sizeof(T));
+  }
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const long long delay = h->df_delay > 0 ? h->df_delay : 8ll * sms;
+  long long stagger = 0;
+  if (const char* e = getenv("APSP_DF_STAGGER")) stagger = atoll(e);  // tuning experiments only
+  // APSP_DF_PROFILE=1: per-group cycle counters printed to stderr (tuning experiments only)
+  unsigned long long* prof = nullptr;
+  const bool want_prof = getenv("APSP_DF_PROFILE") != nullptr;
+  const size_t prof_bytes = (size_t)sms * 2 * 8 * sizeof(unsigned long long);  // 2 groups per SM
+  if (want_prof && (st = h->cuda(cudaMalloc(&prof, prof_bytes), "cudaMalloc prof"))) return st;
+  h->ev_begin(2);
+  if ((st = h->cuda(launch_fw_dataflow<T>(static_cast<T*>(h->shards[0].D), h->ld, nb, h->df_work, h->d_flag, delay,
+                                          stagger, h->stream, prof),
+                    "fw_dataflow")))
+    return st;
+  h->ev_end((double)h->n_pad * h->n_pad * h->n_pad);
+  if (want_prof) {
+    std::vector<unsigned long long> hp(prof_bytes / 8);
+    cudaStreamSynchronize(h->stream);
+    cudaMemcpy(hp.data(), prof, prof_bytes, cudaMemcpyDeviceToHost);
+    cudaFree(prof);
+    double tot[6] = {0, 0, 0, 0, 0, 0};
+    for (int i = 0; i < sms * 2; ++i)
+      for (int j = 0; j < 6; ++j) tot[j] += (double)hp[(size_t)i * 8 + j];
+    const double all = tot[0] + tot[1] + tot[2];
+    fprintf(stderr, "[df] groups %d: wait %.2f%% body %.2f%% tail %.2f%% | tasks %.0f blocked %.0f p1 %.2f%% | "
+            "body/task %.0f cyc\n", sms * 2, 100 * tot[0] / all, 100 * tot[1] / all, 100 * tot[2] / all, tot[3],
+            tot[5], 100 * tot[4] / all, (tot[1] - tot[4]) / (tot[3] - nb));
+  }
+  return APSP_OK;
+}
+
 apsp_status run_incore_rounds(Handle* h, long long k0, long long k1) {
+  if (h->world == 1 && !h->use_comm && !h->virt && h->dataflow && k0 == 0 && k1 == h->n_pad / h->b)
+    return h->dtype == APSP_I32 ? run_dataflow<int>(h) : run_dataflow<float>(h);
   if (h->world == 1 && !h->use_comm) {  // single GPU: the whole closure, with lookahead
     return h->dtype == APSP_I32
                ? fw_closure<int>(h, static_cast<int*>(h->shards[0].D), h->ld, h->n_pad, k0, k1, h->stream)

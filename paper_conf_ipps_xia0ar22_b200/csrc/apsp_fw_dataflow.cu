@@ -1,0 +1,709 @@
+// apsp_fw_dataflow.cu — the whole single-GPU blocked Floyd–Warshall (every
+// round, all three phases of PAPER.md:62) as ONE persistent dataflow kernel.
+//
+// Why: with one launch per phase the chip idles at every launch boundary
+// (wave tail, the partial wave of the next round's panels, launch gaps) and
+// the two CTAs that share an SM start and finish their tiles in lockstep, so
+// the prologue of every tile (first chunks in flight) leaves the SM idle.
+// Here each SM runs one CTA of two independent 256-thread "groups"; every
+// group pulls tasks (one 128x128 tile update each) from a global queue in a
+// fixed dependency-respecting order and waits on per-tile flags, so rounds
+// overlap (round k+1's panels are computed while round k's phase 3 drains)
+// and group 1 starts half a tile after group 0, so one group's prologue and
+// epilogue run under the other's relaxations.
+//
+// Tasks of round k (nb = n/128 tile rows):
+//   P1(k)       closure of A(k,k) (phase 1, Alg. 1 l.3)
+//   P2(k; k,j)  A(k,j) = D (x) A(k,j), j != k  (phase 2 row panel, Alg. 1 l.7)
+//   P2(k; i,k)  A(i,k) = A(i,k) (x) D, i != k  (phase 2 column panel, l.11)
+//   P3(k; i,j)  A(i,j) = min(A(i,j), A(i,k) (x) A(k,j)), i,j != k  (phase 3, l.17)
+// P1 and P2 also write their result to a panel buffer pbuf[k % 2] (diagonal,
+// row-panel and column-panel tiles, 128x128 each, ld 128); P2 and P3 read the
+// panels from there, so a later round may update A(i,k) in place while round
+// k's readers still run (write-after-read on the matrix never arises).
+//
+// Flags (device ints, monotone within one solve, zeroed before the launch):
+//   ver[i*nb+j]      rounds applied to tile (i,j)
+//   diagready[p]     k+1 once P1(k) wrote pbuf[p] (p = k % 2)
+//   rowready[p][j]   k+1 once P2(k; k,j) wrote pbuf[p]
+//   colready[p][i]   k+1 once P2(k; i,k) wrote pbuf[p]
+//   done2[k], done3[k]  completed P2 / P3 tasks of round k
+// Dependencies: P1(k): ver(k,k) >= k and (k >= 2) done2[k-2] complete (pbuf
+// diagonal reuse); P2(k): ver >= k, diagready >= k+1, (k >= 2) done3[k-2]
+// complete (pbuf panel reuse); P3(k): ver >= k, rowready/colready >= k+1.
+//
+// Queue order (one global counter): P1(0), seg(0), ..., seg(nb-1), tail, where
+//   seg(k) = [G3R(k-1)[0:delay], G2(k), G3R(k-1)[delay:], G3L(k)[0], P1(k+1), G3L(k)[1:]]
+//   G2(k)  = the 2(nb-1) panel tasks of round k
+//   G3L(k) = round-k phase 3 on row/column k+1, tile (k+1,k+1) first
+//   G3R(k) = the other round-k phase-3 tiles, row/column k+2 first
+//   tail   = G3R(nb-1)  (the last round's whole phase 3)
+// Every task's dependencies are earlier in this order and a group finishes a
+// task before it takes the next one, so the task with the smallest index
+// that is not done always has its dependencies met and a running group:
+// the kernel cannot deadlock, whatever the number of resident CTAs.
+//
+// The tile engine is the min-plus kernel's (apsp_kernels.cu): 8x8 outputs per
+// thread, 32-deep chunks through a 3-stage cp.async pipeline with full/empty
+// mbarriers; here the chunk stream of a group is continuous across its tasks
+// (stage and barrier parity carry over), and the C tile is fetched into the
+// two free stages during the last chunk.
+#include "apsp_kernels.cuh"
+
+#include <cuda_runtime.h>
+#include <climits>
+#include <cstdint>
+
+namespace apsp {
+namespace {
+
+#ifndef DF_GROUPS
+#define DF_GROUPS 1
+#endif
+constexpr int BM = 128, BN = 128, BK = 32, GNT = 256, GROUPS = DF_GROUPS, STAGES = 3;
+constexpr int CTAS_PER_SM = 2 / GROUPS;  // two groups per SM either way
+constexpr int ALD = BK + 4, BLD = BN, CLD = BN + 4;
+constexpr int STAGE_ELEMS = BM * ALD + BK * BLD;  // 8704 words
+constexpr int TILE_ELEMS = BM * BN;
+// Bookkeeping is spread over lanes 0 of three warps of a group, so no warp
+// carries more than one latency (a warp that lags delays the group's barriers):
+constexpr int SIG = 32;  // publishes the group's finished task (release fence + flags)
+constexpr int SCH = 64;  // dequeues the next task, decodes it, reads its flags, fills its slot
+static_assert(64 * CLD <= STAGE_ELEMS, "half a C tile must fit one stage");
+
+template <typename T> struct DV;
+template <> struct DV<int> {
+  using V4 = int4;
+  static __device__ __forceinline__ int inf() { return 0x3FFFFFFF; }
+  static __device__ __forceinline__ int relax(int a, int b, int c) { return __viaddmin_s32(a, b, c); }
+  static __device__ __forceinline__ int vmin(int a, int b) { return min(a, b); }
+};
+template <> struct DV<float> {
+  using V4 = float4;
+  static __device__ __forceinline__ float inf() { return __int_as_float(0x7f800000); }
+  static __device__ __forceinline__ float relax(float a, float b, float c) { return fminf(c, __fadd_rn(a, b)); }
+  static __device__ __forceinline__ float vmin(float a, float b) { return fminf(a, b); }
+};
+
+__device__ __forceinline__ unsigned saddr(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void cp16(void* smem, const void* gmem) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(saddr(smem)), "l"(gmem));
+}
+__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+__device__ __forceinline__ void cp_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::); }
+__device__ __forceinline__ void mb_init(unsigned bar, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count));
+}
+__device__ __forceinline__ void mb_arrive(unsigned bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mb_cp_arrive(unsigned bar) {
+  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mb_wait(unsigned bar, unsigned parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "DFW_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra DFW_%=;\n"
+      "}\n" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+// named barrier of one 256-thread group (id 0 is __syncthreads)
+__device__ __forceinline__ void gbar(int g) { asm volatile("bar.sync %0, %1;" ::"r"(g + 1), "r"(GNT) : "memory"); }
+
+__device__ __forceinline__ int ld_relaxed(const int* p) {
+  int v;
+  asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed(int* p, int v) {
+  asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void red_relaxed_add(int* p, int v) {
+  asm volatile("red.relaxed.gpu.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+template <typename T>
+struct DFArgs {
+  T* D;            // n_pad x n_pad, row-major, ld
+  long long ld;
+  int nb;
+  T* pbuf;         // 2 x (2nb+1) tiles of 128x128: [p][0] diagonal, [p][1+j] row panel, [p][1+nb+i] column panel
+  int* ver;        // nb*nb
+  int* diagready;  // [2]
+  int* rowready;   // [2][nb]
+  int* colready;   // [2][nb]
+  int* done2;      // [nb]
+  int* done3;      // [nb]
+  unsigned long long* counter;
+  int* negflag;
+  long long total;   // nb^3 tasks
+  long long delay;   // G3R tasks placed before G2 in a segment
+  long long stagger; // clock cycles group 1 waits before its first task
+  unsigned long long* prof;  // optional [CTAs x GROUPS x 8] cycle counters (thread 0 of each group)
+};
+
+enum { T_P1 = 0, T_P2R = 1, T_P2C = 2, T_P3 = 3 };
+struct Task {
+  int type, k, i, j;
+};
+
+// i-th value of [0, nb) without the excluded values s0 < s1 < s2 (-1 = none)
+__device__ __forceinline__ int skip3(int x, int s0, int s1, int s2) {
+  if (s0 >= 0 && x >= s0) ++x;
+  if (s1 >= 0 && x >= s1) ++x;
+  if (s2 >= 0 && x >= s2) ++x;
+  return x;
+}
+
+__device__ __forceinline__ Task p2_task(int nb, int k, long long x) {
+  Task t;
+  t.k = k;
+  if (x < nb - 1) {
+    t.type = T_P2R; t.i = k; t.j = skip3((int)x, k, -1, -1);
+  } else {
+    t.type = T_P2C; t.i = skip3((int)(x - (nb - 1)), k, -1, -1); t.j = k;
+  }
+  return t;
+}
+// G3L(k): (k+1,k+1), row k+1 (j not in {k,k+1}), column k+1 (i not in {k,k+1})
+__device__ __forceinline__ Task g3l_task(int nb, int k, long long x) {
+  Task t;
+  t.type = T_P3; t.k = k;
+  if (x == 0) { t.i = k + 1; t.j = k + 1; return t; }
+  x -= 1;
+  if (x < nb - 2) { t.i = k + 1; t.j = skip3((int)x, k, k + 1, -1); return t; }
+  x -= nb - 2;
+  t.i = skip3((int)x, k, k + 1, -1); t.j = k + 1;
+  return t;
+}
+// G3R(k), k <= nb-2: tiles with i,j not in {k,k+1}; row k+2, column k+2 first
+__device__ __forceinline__ Task g3r_task(int nb, int k, long long x) {
+  Task t;
+  t.type = T_P3; t.k = k;
+  if (k + 2 < nb) {
+    if (x < nb - 2) { t.i = k + 2; t.j = skip3((int)x, k, k + 1, -1); return t; }
+    x -= nb - 2;
+    if (x < nb - 3) { t.i = skip3((int)x, k, k + 1, k + 2); t.j = k + 2; return t; }
+    x -= nb - 3;
+    const int w = nb - 3;
+    t.i = skip3((int)(x / w), k, k + 1, k + 2);
+    t.j = skip3((int)(x % w), k, k + 1, k + 2);
+    return t;
+  }
+  const int w = nb - 2;
+  t.i = skip3((int)(x / w), k, k + 1, -1);
+  t.j = skip3((int)(x % w), k, k + 1, -1);
+  return t;
+}
+
+__device__ Task decode(long long g, int nb, long long delay) {
+  Task t;
+  if (g == 0) { t.type = T_P1; t.k = 0; t.i = t.j = 0; return t; }
+  g -= 1;
+  const long long n1 = nb - 1, n2 = nb - 2;
+  const long long s0 = 4 * n1;  // seg(0) = G2(0) + G3L(0) + P1(1)
+  if (g < s0) {
+    if (g < 2 * n1) return p2_task(nb, 0, g);
+    g -= 2 * n1;
+    if (g == 0) return g3l_task(nb, 0, 0);
+    if (g == 1) { t.type = T_P1; t.k = 1; t.i = t.j = 1; return t; }
+    return g3l_task(nb, 0, g - 1);
+  }
+  g -= s0;
+  int k;
+  long long r3;  // segment k: G3R(k-1) size r3
+  const long long mid = (long long)(nb - 2) * nb * nb;  // segments 1..nb-2 are nb^2 tasks each
+  if (g < mid) {
+    k = 1 + (int)(g / ((long long)nb * nb));
+    g -= (long long)(k - 1) * nb * nb;
+    r3 = n2 * n2;
+
+  } else {
+    g -= mid;
+    const long long last = n2 * n2 + 2 * n1;  // seg(nb-1) = G3R(nb-2) + G2(nb-1)
+    if (g >= last) {                           // tail: G3R(nb-1), all (i,j) != nb-1
+      g -= last;
+      t.type = T_P3; t.k = nb - 1;
+      t.i = (int)(g / n1); t.j = (int)(g % n1);
+      return t;
+    }
+    k = nb - 1;
+    r3 = n2 * n2;
+
+  }
+  const long long d = delay < r3 ? delay : r3;
+  if (g < d) return g3r_task(nb, k - 1, g);
+  g -= d;
+  if (g < 2 * n1) return p2_task(nb, k, g);
+  g -= 2 * n1;
+  if (g < r3 - d) return g3r_task(nb, k - 1, d + g);
+  g -= r3 - d;
+
+  if (g == 0) return g3l_task(nb, k, 0);
+  if (g == 1) { t.type = T_P1; t.k = k + 1; t.i = t.j = k + 1; return t; }
+  return g3l_task(nb, k, g - 1);
+}
+
+template <typename T>
+__device__ __forceinline__ T* pb_diag(const DFArgs<T>& a, int k) {
+  return a.pbuf + (long long)(k & 1) * (2 * a.nb + 1) * TILE_ELEMS;
+}
+template <typename T>
+__device__ __forceinline__ T* pb_row(const DFArgs<T>& a, int k, int j) {
+  return pb_diag(a, k) + (long long)(1 + j) * TILE_ELEMS;
+}
+template <typename T>
+__device__ __forceinline__ T* pb_col(const DFArgs<T>& a, int k, int i) {
+  return pb_diag(a, k) + (long long)(1 + a.nb + i) * TILE_ELEMS;
+}
+
+// Dependency test of task t (one thread): up to three flags, read with
+// independent relaxed loads (one round trip), then an acquire fence once met.
+template <typename T>
+__device__ bool deps_met(const DFArgs<T>& a, const Task& t) {
+  const int nb = a.nb, k = t.k, p = k & 1;
+  const int* f0 = a.ver + (long long)t.i * nb + t.j;
+  const int* f1;
+  const int* f2;
+  int v1, v2;
+  const int v0 = k;
+  if (t.type == T_P1) {
+    f1 = a.done2 + (k >= 2 ? k - 2 : 0); v1 = k >= 2 ? 2 * (nb - 1) : INT_MIN;
+    f2 = f1; v2 = v1;
+  } else if (t.type == T_P3) {
+    f1 = a.rowready + p * nb + t.j; v1 = k + 1;
+    f2 = a.colready + p * nb + t.i; v2 = k + 1;
+  } else {
+    f1 = a.diagready + p; v1 = k + 1;
+    f2 = a.done3 + (k >= 2 ? k - 2 : 0); v2 = k >= 2 ? (nb - 1) * (nb - 1) : INT_MIN;
+  }
+  const int x0 = ld_relaxed(f0), x1 = ld_relaxed(f1), x2 = ld_relaxed(f2);
+  if (x0 >= v0 && x1 >= v1 && x2 >= v2) {
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+    return true;
+  }
+  return false;
+}
+
+// Publish task t (one thread, after a group barrier that follows every
+// thread's stores of t): one release fence, then the flags.
+template <typename T>
+__device__ void signal_done(const DFArgs<T>& a, const Task& t) {
+  const int nb = a.nb, k = t.k, p = k & 1;
+  asm volatile("fence.acq_rel.gpu;" ::: "memory");
+  st_relaxed(a.ver + (long long)t.i * nb + t.j, k + 1);
+  switch (t.type) {
+    case T_P1: st_relaxed(a.diagready + p, k + 1); break;
+    case T_P2R: st_relaxed(a.rowready + p * nb + t.j, k + 1); red_relaxed_add(a.done2 + k, 1); break;
+    case T_P2C: st_relaxed(a.colready + p * nb + t.i, k + 1); red_relaxed_add(a.done2 + k, 1); break;
+    default: red_relaxed_add(a.done3 + k, 1); break;
+  }
+}
+
+// Phase 1 inside a group: in-place FW closure of one 128x128 tile (the same
+// register blocking as phase1_kernel in apsp_kernels.cu); result also to out2.
+template <typename T>
+__device__ __noinline__ void group_phase1(T* tile, long long ld, T* out2, int* negflag, T* scratch, int g, int gtid) {
+  using V4 = typename DV<T>::V4;
+  T* rowbuf = scratch;            // [2][128]
+  T* colbuf = scratch + 2 * 128;  // [2][128]
+  const int tx = gtid & 15, ty = gtid >> 4;
+  T acc[8][8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
+    const V4 v0 = __ldcg(reinterpret_cast<const V4*>(tile + r * ld + tx * 4));
+    const V4 v1 = __ldcg(reinterpret_cast<const V4*>(tile + r * ld + 64 + tx * 4));
+    acc[i][0] = v0.x; acc[i][1] = v0.y; acc[i][2] = v0.z; acc[i][3] = v0.w;
+    acc[i][4] = v1.x; acc[i][5] = v1.y; acc[i][6] = v1.z; acc[i][7] = v1.w;
+  }
+  bool neg = false;
+#pragma unroll
+  for (int half = 0; half < 2; ++half) {
+    for (int q = 0; q < 16; ++q) {
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int kk = half * 64 + q * 4 + u;
+        const int p = u & 1;
+        const int io = half * 4 + u;
+        if (ty == q) {
+          V4 x0, x1;
+          x0.x = acc[io][0]; x0.y = acc[io][1]; x0.z = acc[io][2]; x0.w = acc[io][3];
+          x1.x = acc[io][4]; x1.y = acc[io][5]; x1.z = acc[io][6]; x1.w = acc[io][7];
+          *reinterpret_cast<V4*>(&rowbuf[p * 128 + tx * 4]) = x0;
+          *reinterpret_cast<V4*>(&rowbuf[p * 128 + 64 + tx * 4]) = x1;
+        }
+        if (tx == q) {
+          V4 y0, y1;
+          y0.x = acc[0][io]; y0.y = acc[1][io]; y0.z = acc[2][io]; y0.w = acc[3][io];
+          y1.x = acc[4][io]; y1.y = acc[5][io]; y1.z = acc[6][io]; y1.w = acc[7][io];
+          *reinterpret_cast<V4*>(&colbuf[p * 128 + ty * 4]) = y0;
+          *reinterpret_cast<V4*>(&colbuf[p * 128 + 64 + ty * 4]) = y1;
+        }
+        gbar(g);
+        if (gtid == 0 && rowbuf[p * 128 + kk] < T(0)) neg = true;
+        const V4 a0 = *reinterpret_cast<const V4*>(&colbuf[p * 128 + ty * 4]);
+        const V4 a1 = *reinterpret_cast<const V4*>(&colbuf[p * 128 + 64 + ty * 4]);
+        const V4 b0 = *reinterpret_cast<const V4*>(&rowbuf[p * 128 + tx * 4]);
+        const V4 b1 = *reinterpret_cast<const V4*>(&rowbuf[p * 128 + 64 + tx * 4]);
+        const T av[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+        const T bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+          for (int j = 0; j < 8; ++j) acc[i][j] = DV<T>::relax(av[i], bv[j], acc[i][j]);
+      }
+    }
+  }
+  if (neg) *negflag = 1;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
+    V4 v0, v1;
+    v0.x = acc[i][0]; v0.y = acc[i][1]; v0.z = acc[i][2]; v0.w = acc[i][3];
+    v1.x = acc[i][4]; v1.y = acc[i][5]; v1.z = acc[i][6]; v1.w = acc[i][7];
+    *reinterpret_cast<V4*>(tile + r * ld + tx * 4) = v0;
+    *reinterpret_cast<V4*>(tile + r * ld + 64 + tx * 4) = v1;
+    *reinterpret_cast<V4*>(out2 + r * BN + tx * 4) = v0;
+    *reinterpret_cast<V4*>(out2 + r * BN + 64 + tx * 4) = v1;
+  }
+}
+
+// Operands of a group's current min-plus task, written by the group's thread 0
+// before the task-start barrier (kept in shared memory, not in registers).
+template <typename T>
+struct GDesc {
+  const T* A;
+  const T* B;
+  const T* Cin;
+  T* Cout;
+  T* Cout2;  // panel copy (ld 128) or nullptr
+  int lda, ldb, ldc;
+};
+
+__device__ __forceinline__ int ld_acquire(const int* p) {
+  int v;
+  asm volatile("ld.acquire.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// flags (and the values they must reach) that task t waits for
+template <typename T>
+__device__ __forceinline__ void dep_flags(const DFArgs<T>& a, const Task& t, const int* (&f)[3], int (&v)[3]) {
+  const int nb = a.nb, k = t.k, p = k & 1;
+  f[0] = a.ver + (long long)t.i * nb + t.j;
+  v[0] = k;
+  if (t.type == T_P1) {
+    f[1] = a.done2 + (k >= 2 ? k - 2 : 0); v[1] = k >= 2 ? 2 * (nb - 1) : INT_MIN;
+    f[2] = f[1]; v[2] = v[1];
+  } else if (t.type == T_P3) {
+    f[1] = a.rowready + p * nb + t.j; v[1] = k + 1;
+    f[2] = a.colready + p * nb + t.i; v[2] = k + 1;
+  } else {
+    f[1] = a.diagready + p; v[1] = k + 1;
+    f[2] = a.done3 + (k >= 2 ? k - 2 : 0); v[2] = k >= 2 ? (nb - 1) * (nb - 1) : INT_MIN;
+  }
+}
+
+// A group's task slot (shared memory, double-buffered by iteration parity):
+// the task index, its decoded form, the operands of a min-plus task and
+// whether its dependencies were already seen met. Thread 0 fills the slot of
+// the next iteration while the current task runs.
+template <typename T>
+struct Slot {
+  long long t;
+  Task tk;
+  GDesc<T> d;
+  int ready;
+};
+
+template <typename T>
+__device__ void fill_desc(const DFArgs<T>& a, const Task& tk, GDesc<T>& d) {
+  const int k = tk.k;
+  T* const tile = a.D + (long long)tk.i * BM * a.ld + (long long)tk.j * BN;
+  d.Cin = tile; d.Cout = tile; d.ldc = (int)a.ld;
+  if (tk.type == T_P2R) {         // A(k,j) = D (x) A(k,j)
+    d.A = pb_diag(a, k); d.lda = BN; d.B = tile; d.ldb = (int)a.ld; d.Cout2 = pb_row(a, k, tk.j);
+  } else if (tk.type == T_P2C) {  // A(i,k) = A(i,k) (x) D
+    d.A = tile; d.lda = (int)a.ld; d.B = pb_diag(a, k); d.ldb = BN; d.Cout2 = pb_col(a, k, tk.i);
+  } else {                        // A(i,j) = min(A(i,j), A(i,k) (x) A(k,j)) from the panel copies
+    d.A = pb_col(a, k, tk.i); d.lda = BN; d.B = pb_row(a, k, tk.j); d.ldb = BN; d.Cout2 = nullptr;
+  }
+}
+
+// One 128x128 min-plus tile update of depth 128 by a group:
+//   Cout = min(Cin, A (x) B)  (and Cout2 = the same, ld 128, if non-null)
+// `c0` is the group's running chunk counter (stage = chunk % 3, barrier
+// parity = (chunk / 3) & 1); the task uses chunks c0 .. c0+3.
+// Thread 0 of the group also (a) publishes the group's previous task `pend`
+// once this task's first loads are issued, and (b) prepares the slot of the
+// next task `nxt`: decoded and its flags read (acquire) during chunk 2, its
+// readiness evaluated and its operands written after the epilogue.
+template <typename T>
+__device__ __noinline__ void group_minplus(const GDesc<T>* d, T* stage0, unsigned full0, unsigned empty0, unsigned c0,
+                                           int gtid, int g, const DFArgs<T>* args, const Task* pend,
+                                           long long nxt, Slot<T>* ns) {
+  using V4 = typename DV<T>::V4;
+  constexpr int NK = BM / BK;  // 4 chunks of depth 32
+  const int lane = gtid & 31;
+  const int tx = gtid & 15, ty = gtid >> 4;
+  auto load_chunk = [&](int stage, int c) {
+    T* st = stage0 + stage * STAGE_ELEMS;
+    const int lda = d->lda, ldb = d->ldb;
+    const T* ag = d->A + (gtid >> 3) * lda + (gtid & 7) * 4 + c * BK;
+    const T* bg = d->B + ((gtid >> 5) + c * BK) * (long long)ldb + (gtid & 31) * 4;
+    const int a_dst = (gtid >> 3) * ALD + (gtid & 7) * 4;
+    const int b_dst = BM * ALD + (gtid >> 5) * BLD + (gtid & 31) * 4;
+#pragma unroll
+    for (int q = 0; q < 4; ++q) cp16(st + a_dst + q * 32 * ALD, ag + q * 32 * lda);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) cp16(st + b_dst + q * 8 * BLD, bg + q * 8 * ldb);
+    mb_cp_arrive(full0 + 8 * stage);
+  };
+  load_chunk((int)(c0 % STAGES), 0);
+  load_chunk((int)((c0 + 1) % STAGES), 1);
+  // the previous task's completion is published here, under this task's first loads
+  if (pend && gtid == SIG) signal_done(*args, *pend);
+
+  T acc[8][8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
+#pragma unroll
+    for (int j = 0; j < 8; ++j) acc[i][j] = DV<T>::inf();
+  const int s_lo = (int)((c0 + 1) % STAGES), s_hi = (int)((c0 + 2) % STAGES);
+
+#pragma unroll 1
+  for (int c = 0; c < NK; ++c) {
+    const unsigned G = c0 + c;
+    const int s = (int)(G % STAGES);
+    if (c == NK - 1) {
+      // C goes to the stages of chunks c0+1 and c0+2 once every warp released them
+      mb_wait(empty0 + 8 * s_lo, ((c0 + 1) / STAGES) & 1);
+      mb_wait(empty0 + 8 * s_hi, ((c0 + 2) / STAGES) & 1);
+      const int ldc = d->ldc;
+      const T* cg = d->Cin + (gtid >> 5) * ldc + (gtid & 31) * 4;
+      const int cd = (gtid >> 5) * CLD + (gtid & 31) * 4;
+      T* const cs_lo = stage0 + s_lo * STAGE_ELEMS;
+      T* const cs_hi = stage0 + s_hi * STAGE_ELEMS;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) cp16(cs_lo + cd + q * 8 * CLD, cg + q * 8 * ldc);
+#pragma unroll
+      for (int q = 0; q < 8; ++q) cp16(cs_hi + cd + q * 8 * CLD, cg + (64 + q * 8) * ldc);
+      cp_commit();
+    }
+    if (c == 1 && gtid == SCH) {  // decode the next task, fill its slot and read its flags
+      ns->t = nxt;
+      if (nxt < args->total) {
+        const Task tn = decode(nxt, args->nb, args->delay);
+        ns->tk = tn;
+        if (tn.type != T_P1) fill_desc(*args, tn, ns->d);
+        ns->ready = deps_met(*args, tn) ? 1 : 0;
+      }
+    }
+    mb_wait(full0 + 8 * s, (G / STAGES) & 1);
+    const T* as = stage0 + s * STAGE_ELEMS;
+    const T* bs = as + BM * ALD;
+#pragma unroll
+    for (int k2 = 0; k2 < BK / 2; ++k2) {
+      T av[8][2];
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
+        const T* ap = as + r * ALD + k2 * 2;
+        av[i][0] = ap[0]; av[i][1] = ap[1];
+      }
+#pragma unroll
+      for (int u = 0; u < 2; ++u) {
+        const T* brow = bs + (k2 * 2 + u) * BLD;
+        const V4 b0 = *reinterpret_cast<const V4*>(brow + tx * 4);
+        const V4 b1 = *reinterpret_cast<const V4*>(brow + 64 + tx * 4);
+        const T bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+          for (int j = 0; j < 8; ++j) acc[i][j] = DV<T>::relax(av[i][u], bv[j], acc[i][j]);
+      }
+    }
+    __syncwarp();
+    if (lane == 0) mb_arrive(empty0 + 8 * s);
+    if (c + 2 < NK) {  // refill the stage of chunk G-1 with chunk c+2
+      const unsigned Gn = G + 2;
+      const int sn = (int)(Gn % STAGES);
+      if (Gn >= STAGES) mb_wait(empty0 + 8 * sn, ((Gn - STAGES) / STAGES) & 1);
+      load_chunk(sn, c + 2);
+    }
+  }
+  cp_wait_all();
+  gbar(g);
+  {
+    T* const Cout = d->Cout;
+    T* const Cout2 = d->Cout2;
+    const int ldc = d->ldc;
+    const T* const cs_lo = stage0 + s_lo * STAGE_ELEMS;
+    const T* const cs_hi = stage0 + s_hi * STAGE_ELEMS;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
+      const T* crow = (i < 4 ? cs_lo : cs_hi) + (ty * 4 + (i & 3)) * CLD;
+      const V4 x0 = *reinterpret_cast<const V4*>(crow + tx * 4);
+      const V4 x1 = *reinterpret_cast<const V4*>(crow + 64 + tx * 4);
+      V4 v0, v1;
+      v0.x = DV<T>::vmin(acc[i][0], x0.x); v0.y = DV<T>::vmin(acc[i][1], x0.y);
+      v0.z = DV<T>::vmin(acc[i][2], x0.z); v0.w = DV<T>::vmin(acc[i][3], x0.w);
+      v1.x = DV<T>::vmin(acc[i][4], x1.x); v1.y = DV<T>::vmin(acc[i][5], x1.y);
+      v1.z = DV<T>::vmin(acc[i][6], x1.z); v1.w = DV<T>::vmin(acc[i][7], x1.w);
+      *reinterpret_cast<V4*>(Cout + (long long)r * ldc + tx * 4) = v0;
+      *reinterpret_cast<V4*>(Cout + (long long)r * ldc + 64 + tx * 4) = v1;
+      if (Cout2) {
+        *reinterpret_cast<V4*>(Cout2 + r * BN + tx * 4) = v0;
+        *reinterpret_cast<V4*>(Cout2 + r * BN + 64 + tx * 4) = v1;
+      }
+    }
+  }
+}
+
+template <typename T>
+__global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(const __grid_constant__ DFArgs<T> a) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  __shared__ __align__(8) unsigned long long bars[GROUPS][2 * STAGES];
+  __shared__ Slot<T> slots[GROUPS][2];
+  const int g = threadIdx.x / GNT, gtid = threadIdx.x % GNT;
+  T* const stage0 = reinterpret_cast<T*>(smem_raw) + g * STAGES * STAGE_ELEMS;
+  const unsigned full0 = saddr(&bars[g][0]), empty0 = full0 + 8 * STAGES;
+  if (gtid == 0) {
+    for (int s = 0; s < STAGES; ++s) {
+      mb_init(full0 + 8 * s, GNT);
+      mb_init(empty0 + 8 * s, GNT / 32);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (gtid == SCH) {
+    if ((GROUPS > 1 ? g > 0 : blockIdx.x >= gridDim.x / 2) && a.stagger > 0) {  // half the groups start later
+      const long long t0 = clock64();
+      while (clock64() - t0 < a.stagger) __nanosleep(256);
+    }
+    Slot<T>& s0 = slots[g][0];
+    s0.t = (long long)atomicAdd(a.counter, 1ull);
+    s0.ready = 0;
+    if (s0.t < a.total) {
+      s0.tk = decode(s0.t, a.nb, a.delay);
+      if (s0.tk.type != T_P1) fill_desc(a, s0.tk, s0.d);
+    }
+  }
+  gbar(g);
+  unsigned chunk = 0;
+  // The completion of a group's task is published after the next task's first
+  // loads are issued (the fence then overlaps their latency); at once when the
+  // next task cannot start yet (it may depend on it); and before the group exits.
+  Task pend{};
+  bool has_pend = false;  // (only thread 0 publishes; the flag is per thread)
+  unsigned long long pr[6] = {0, 0, 0, 0, 0, 0};  // wait, body, tail, tasks, p1 cycles, waits that blocked
+  long long tc0 = clock64();
+  for (int it = 0;; ++it) {
+    Slot<T>& S = slots[g][it & 1];
+    Slot<T>* N = &slots[g][(it + 1) & 1];
+    const long long t = S.t;
+    if (t >= a.total) break;
+    const Task tk = S.tk;
+    if (!S.ready) {  // uniform: the slot was published by the last barrier
+      // the task may depend on the group's own previous task: publish that first
+      if (gtid == SIG && has_pend) signal_done(a, pend);
+      has_pend = false;
+      if (gtid == SCH && !deps_met(a, tk)) {
+        while (!deps_met(a, tk)) __nanosleep(64);
+        pr[5]++;
+      }
+      gbar(g);
+    }
+    long long nxt = 0;
+    if (gtid == SCH) nxt = (long long)atomicAdd(a.counter, 1ull);  // the result is needed in chunk 1
+    const Task* pp = has_pend ? &pend : nullptr;
+    const long long tc1 = clock64();
+    pr[0] += tc1 - tc0;
+    if (tk.type == T_P1) {
+      if (pp && gtid == SIG) signal_done(a, *pp);
+      T* const tile = a.D + (long long)tk.i * BM * a.ld + (long long)tk.j * BN;
+      group_phase1<T>(tile, a.ld, pb_diag(a, tk.k), a.negflag, stage0, g, gtid);
+      if (gtid == SCH) {
+        N->t = nxt;
+        if (nxt < a.total) {
+          N->tk = decode(nxt, a.nb, a.delay);
+          N->ready = 0;
+          if (N->tk.type != T_P1) fill_desc(a, N->tk, N->d);
+        }
+      }
+    } else {
+      group_minplus<T>(&S.d, stage0, full0, empty0, chunk, gtid, g, &a, pp, nxt, N);
+      chunk += BM / BK;
+    }
+    const long long tc2 = clock64();
+    pr[1] += tc2 - tc1;
+    if (tk.type == T_P1) pr[4] += tc2 - tc1;
+    pr[3]++;
+    pend = tk;
+    has_pend = true;
+    gbar(g);  // every thread's stores of this task are issued; the next slot is published
+    tc0 = clock64();
+    pr[2] += tc0 - tc2;
+  }
+  if (has_pend && gtid == SIG) signal_done(a, pend);
+  if (a.prof && gtid == SCH) {
+    unsigned long long* o = a.prof + ((long long)blockIdx.x * GROUPS + g) * 8;
+    for (int i = 0; i < 6; ++i) o[i] = pr[i];
+  }
+}
+
+}  // namespace
+
+template <typename T>
+cudaError_t launch_fw_dataflow(T* D, long long ld, int nb, void* work, int* negflag, long long delay,
+                               long long stagger, cudaStream_t s, unsigned long long* prof) {
+  if (nb <= 0) return cudaSuccess;
+  const int smem = GROUPS * STAGES * STAGE_ELEMS * (int)sizeof(T);
+  cudaError_t e = cudaFuncSetAttribute(fw_dataflow_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return e;
+  int dev = 0, sms = 0;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+  if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
+  DFArgs<T> a;
+  a.D = D; a.ld = ld; a.nb = nb;
+  a.pbuf = static_cast<T*>(work);
+  int* f = reinterpret_cast<int*>(static_cast<char*>(work) + fw_dataflow_pbuf_bytes(nb, sizeof(T)));
+  a.counter = reinterpret_cast<unsigned long long*>(f); f += 2;  // first: 8-byte aligned
+  a.ver = f; f += (long long)nb * nb;
+  a.diagready = f; f += 2;
+  a.rowready = f; f += 2 * nb;
+  a.colready = f; f += 2 * nb;
+  a.done2 = f; f += nb;
+  a.done3 = f; f += nb;
+  a.negflag = negflag;
+  a.total = (long long)nb * nb * nb;
+  a.delay = delay;
+  a.stagger = stagger;
+  a.prof = prof;
+  e = cudaMemsetAsync(a.counter, 0, fw_dataflow_flag_bytes(nb), s);
+  if (e != cudaSuccess) return e;
+  long long grid = (long long)sms * CTAS_PER_SM;
+  if (grid > a.total) grid = a.total;
+  fw_dataflow_kernel<T><<<(unsigned)grid, GNT * GROUPS, smem, s>>>(a);
+  return cudaGetLastError();
+}
+
+long long fw_dataflow_pbuf_bytes(int nb, size_t elem) {
+  return 2ll * (2 * nb + 1) * TILE_ELEMS * (long long)elem;  // (kept a multiple of 8 bytes)
+}
+long long fw_dataflow_flag_bytes(int nb) { return ((long long)nb * nb + 6ll * nb + 4) * 4; }
+long long fw_dataflow_work_bytes(int nb, size_t elem) {
+  return fw_dataflow_pbuf_bytes(nb, elem) + fw_dataflow_flag_bytes(nb);
+}
+
+template cudaError_t launch_fw_dataflow<int>(int*, long long, int, void*, int*, long long, long long, cudaStream_t,
+                                             unsigned long long*);
+template cudaError_t launch_fw_dataflow<float>(float*, long long, int, void*, int*, long long, long long,
+                                               cudaStream_t, unsigned long long*);
+
+}  // namespace apsp

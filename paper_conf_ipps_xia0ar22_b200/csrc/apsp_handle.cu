@@ -132,6 +132,8 @@ apsp_status setup_device(Handle* h, const apsp_config& cfg) {
     }
   }
   g_minplus_variant = cfg.reserved[3];  // test hook: min-plus kernel variant (apsp_kernels.cuh)
+  h->dataflow = cfg.reserved[4] == 0;   // reserved[4] = 1: launch-per-phase schedule instead of the dataflow kernel
+  h->df_delay = cfg.reserved[5];
   if (cfg.stream) {
     h->stream = static_cast<cudaStream_t>(cfg.stream);
   } else {
@@ -272,7 +274,8 @@ void delete_handle(Handle* h) {
     if (h->d_base) cudaFreeAsync(h->d_base, h->stream);
     if (h->d16) cudaFreeAsync(h->d16, h->stream);
     if (h->panel) cudaFreeAsync(h->panel, h->stream);
-    h->d_base = h->panel = nullptr;
+    if (h->df_work) cudaFreeAsync(h->df_work, h->stream);
+    h->d_base = h->panel = h->df_work = nullptr;
     h->d16 = nullptr;
     cudaStreamSynchronize(h->stream);
   }

@@ -69,6 +69,10 @@ struct Handle {
   void* ooc_streams[3] = {nullptr, nullptr, nullptr};
   // boundary algorithm (apsp_boundary.cu)
   void* bnd = nullptr;
+  // single-GPU in-core dataflow kernel (apsp_fw_dataflow.cu)
+  bool dataflow = true;     // apsp_config.reserved[4] = 1 selects the launch-per-phase schedule
+  long long df_delay = 0;   // reserved[5] (0 = auto)
+  void* df_work = nullptr;
   // bookkeeping
   long long device_bytes = 0, host_bytes = 0;
   long long next_round = 0;

@@ -105,4 +105,17 @@ cudaError_t launch_minplus_tma(const MinPlusDesc<T>* d, int ndesc, int K, cudaSt
 cudaError_t configure_tma_kernels();
 extern int g_minplus_variant;
 
+// The whole single-GPU blocked FW (all nb rounds, phases 1-3) as one
+// persistent dataflow kernel (apsp_fw_dataflow.cu). `work` is a device buffer
+// of fw_dataflow_work_bytes(nb, sizeof(T)) bytes (panel copies + flags; the
+// flags are zeroed by the launch). delay: phase-3 tasks queued between a
+// round's phase-1 task and its phase-2 tasks; stagger: cycles the second
+// group of every CTA waits before its first task.
+template <typename T>
+cudaError_t launch_fw_dataflow(T* D, long long ld, int nb, void* work, int* negflag, long long delay,
+                               long long stagger, cudaStream_t s, unsigned long long* prof = nullptr);
+long long fw_dataflow_pbuf_bytes(int nb, size_t elem);
+long long fw_dataflow_flag_bytes(int nb);
+long long fw_dataflow_work_bytes(int nb, size_t elem);
+
 }  // namespace apsp

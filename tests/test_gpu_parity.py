@@ -90,12 +90,14 @@ def test_fw_minplus_variants(lib, n, variant):
     for name, g in graphs_for(n, seed=n + 3):
         c = cfg(lib)
         c.reserved[3] = variant
+        c.reserved[4] = 1  # launch-per-phase schedule (the min-plus launches take the variant)
         got = lib.solve(g, cfg=c)
         want, _ = oracle_i32(g)
         assert_i32_equal(got, want)
     gf = gg.erdos_renyi(n, 6 * n, seed=n, dtype="f32")
     c = cfg(lib)
     c.reserved[3] = variant
+    c.reserved[4] = 1
     assert_f32_close(lib.solve(gf, cfg=c), oracle.fw_f64(gf.row_ptr, gf.col, gf.w)[0])
 
 
@@ -105,6 +107,7 @@ def test_fw_without_lookahead(lib, n):
     for name, g in graphs_for(n, seed=n + 7):
         c = cfg(lib)
         c.reserved[1] = 1
+        c.reserved[4] = 1
         got = lib.solve(g, cfg=c)
         want, _ = oracle_i32(g)
         assert_i32_equal(got, want)
@@ -279,7 +282,9 @@ def test_virtual_ranks_negative_cycle(lib):
 
 def test_phase_stats_count_all_relaxations(lib):
     g = gg.erdos_renyi(1000, 5000, seed=1)
-    with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=cfg(lib, timing=1)) as h:
+    c = cfg(lib, timing=1)
+    c.reserved[4] = 1  # launch-per-phase schedule
+    with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
         lib.apsp_fw_blocked(h)
         st = lib.apsp_get_phase_stats(h)
         n_pad = lib.apsp_get_info(h).n_pad
