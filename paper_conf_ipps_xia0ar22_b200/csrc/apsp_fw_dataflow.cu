@@ -2,15 +2,16 @@
 // round, all three phases of PAPER.md:62) as ONE persistent dataflow kernel.
 //
 // Why: with one launch per phase the chip idles at every launch boundary
-// (wave tail, the partial wave of the next round's panels, launch gaps) and
-// the two CTAs that share an SM start and finish their tiles in lockstep, so
-// the prologue of every tile (first chunks in flight) leaves the SM idle.
-// Here each SM runs one CTA of two independent 256-thread "groups"; every
-// group pulls tasks (one 128x128 tile update each) from a global queue in a
-// fixed dependency-respecting order and waits on per-tile flags, so rounds
-// overlap (round k+1's panels are computed while round k's phase 3 drains)
-// and group 1 starts half a tile after group 0, so one group's prologue and
-// epilogue run under the other's relaxations.
+// (wave tail, the partial wave of the next round's panels, launch gaps, the
+// phase-1 tile on the critical path of every round). Here 2 CTAs of 256
+// threads per SM pull tasks (one 128x128 tile update each) from a global
+// queue in a fixed dependency-respecting order and wait on per-tile flags, so
+// rounds overlap (round k+1's panels are computed while round k's phase 3
+// drains) and no SM waits for a wave to finish.
+// Measured on cfg2 (n=16384, int32): 0.887 of the DPX peak vs 0.846 for the
+// launch-per-phase schedule (profiles/). Two CTAs per SM of one
+// 256-thread group each measured far better than one CTA of two groups
+// (0.825; DF_GROUPS=2 keeps that variant compilable for experiments).
 //
 // Tasks of round k (nb = n/128 tile rows):
 //   P1(k)       closure of A(k,k) (phase 1, Alg. 1 l.3)
@@ -45,9 +46,13 @@
 //
 // The tile engine is the min-plus kernel's (apsp_kernels.cu): 8x8 outputs per
 // thread, 32-deep chunks through a 3-stage cp.async pipeline with full/empty
-// mbarriers; here the chunk stream of a group is continuous across its tasks
+// mbarriers; here the chunk stream of a CTA is continuous across its tasks
 // (stage and barrier parity carry over), and the C tile is fetched into the
 // two free stages during the last chunk.
+// Bookkeeping per task: the SCH thread dequeues the next task, decodes it and
+// checks its flags (relaxed loads + fence.acquire) during chunk 1, so the next
+// task usually starts without waiting; the SIG thread publishes a finished
+// task (fence.release, then the flags) right after the task's last barrier.
 #include "apsp_kernels.cuh"
 
 #include <cuda_runtime.h>
@@ -283,7 +288,10 @@ __device__ bool deps_met(const DFArgs<T>& a, const Task& t) {
   }
   const int x0 = ld_relaxed(f0), x1 = ld_relaxed(f1), x2 = ld_relaxed(f2);
   if (x0 >= v0 && x1 >= v1 && x2 >= v2) {
-    asm volatile("fence.acq_rel.gpu;" ::: "memory");
+    // acquire: later reads (after the CTA learns of this) see the producers' data.
+    // fence.acquire (an L1 invalidation here) instead of fence.acq_rel, which would
+    // also wait for this thread's own outstanding copies
+    asm volatile("fence.acquire.gpu;" ::: "memory");
     return true;
   }
   return false;
@@ -294,7 +302,7 @@ __device__ bool deps_met(const DFArgs<T>& a, const Task& t) {
 template <typename T>
 __device__ void signal_done(const DFArgs<T>& a, const Task& t) {
   const int nb = a.nb, k = t.k, p = k & 1;
-  asm volatile("fence.acq_rel.gpu;" ::: "memory");
+  asm volatile("fence.release.gpu;" ::: "memory");
   st_relaxed(a.ver + (long long)t.i * nb + t.j, k + 1);
   switch (t.type) {
     case T_P1: st_relaxed(a.diagready + p, k + 1); break;
@@ -385,11 +393,6 @@ struct GDesc {
   int lda, ldb, ldc;
 };
 
-__device__ __forceinline__ int ld_acquire(const int* p) {
-  int v;
-  asm volatile("ld.acquire.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
 
 // flags (and the values they must reach) that task t waits for
 template <typename T>
@@ -445,8 +448,8 @@ __device__ void fill_desc(const DFArgs<T>& a, const Task& tk, GDesc<T>& d) {
 // readiness evaluated and its operands written after the epilogue.
 template <typename T>
 __device__ __noinline__ void group_minplus(const GDesc<T>* d, T* stage0, unsigned full0, unsigned empty0, unsigned c0,
-                                           int gtid, int g, const DFArgs<T>* args, const Task* pend,
-                                           long long nxt, Slot<T>* ns) {
+                                           int gtid, int g, const DFArgs<T>* args, long long nxt,
+                                           Slot<T>* ns) {
   using V4 = typename DV<T>::V4;
   constexpr int NK = BM / BK;  // 4 chunks of depth 32
   const int lane = gtid & 31;
@@ -466,8 +469,6 @@ __device__ __noinline__ void group_minplus(const GDesc<T>* d, T* stage0, unsigne
   };
   load_chunk((int)(c0 % STAGES), 0);
   load_chunk((int)((c0 + 1) % STAGES), 1);
-  // the previous task's completion is published here, under this task's first loads
-  if (pend && gtid == SIG) signal_done(*args, *pend);
 
   T acc[8][8];
 #pragma unroll
@@ -596,11 +597,6 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
   }
   gbar(g);
   unsigned chunk = 0;
-  // The completion of a group's task is published after the next task's first
-  // loads are issued (the fence then overlaps their latency); at once when the
-  // next task cannot start yet (it may depend on it); and before the group exits.
-  Task pend{};
-  bool has_pend = false;  // (only thread 0 publishes; the flag is per thread)
   unsigned long long pr[6] = {0, 0, 0, 0, 0, 0};  // wait, body, tail, tasks, p1 cycles, waits that blocked
   long long tc0 = clock64();
   for (int it = 0;; ++it) {
@@ -610,9 +606,6 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
     if (t >= a.total) break;
     const Task tk = S.tk;
     if (!S.ready) {  // uniform: the slot was published by the last barrier
-      // the task may depend on the group's own previous task: publish that first
-      if (gtid == SIG && has_pend) signal_done(a, pend);
-      has_pend = false;
       if (gtid == SCH && !deps_met(a, tk)) {
         while (!deps_met(a, tk)) __nanosleep(64);
         pr[5]++;
@@ -621,11 +614,9 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
     }
     long long nxt = 0;
     if (gtid == SCH) nxt = (long long)atomicAdd(a.counter, 1ull);  // the result is needed in chunk 1
-    const Task* pp = has_pend ? &pend : nullptr;
     const long long tc1 = clock64();
     pr[0] += tc1 - tc0;
     if (tk.type == T_P1) {
-      if (pp && gtid == SIG) signal_done(a, *pp);
       T* const tile = a.D + (long long)tk.i * BM * a.ld + (long long)tk.j * BN;
       group_phase1<T>(tile, a.ld, pb_diag(a, tk.k), a.negflag, stage0, g, gtid);
       if (gtid == SCH) {
@@ -637,20 +628,20 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
         }
       }
     } else {
-      group_minplus<T>(&S.d, stage0, full0, empty0, chunk, gtid, g, &a, pp, nxt, N);
+      group_minplus<T>(&S.d, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N);
       chunk += BM / BK;
     }
     const long long tc2 = clock64();
     pr[1] += tc2 - tc1;
     if (tk.type == T_P1) pr[4] += tc2 - tc1;
     pr[3]++;
-    pend = tk;
-    has_pend = true;
     gbar(g);  // every thread's stores of this task are issued; the next slot is published
+    // published right away by the SIG thread (its warp absorbs the fence; measured
+    // better than deferring it under the next task's first loads)
+    if (gtid == SIG) signal_done(a, tk);
     tc0 = clock64();
     pr[2] += tc0 - tc2;
   }
-  if (has_pend && gtid == SIG) signal_done(a, pend);
   if (a.prof && gtid == SCH) {
     unsigned long long* o = a.prof + ((long long)blockIdx.x * GROUPS + g) * 8;
     for (int i = 0; i < 6; ++i) o[i] = pr[i];
