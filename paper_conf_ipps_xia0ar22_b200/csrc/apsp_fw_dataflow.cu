@@ -67,8 +67,11 @@ namespace {
 #endif
 constexpr int BM = 128, BN = 128, BK = 32, GNT = 256, GROUPS = DF_GROUPS, STAGES = 3;
 constexpr int CTAS_PER_SM = 2 / GROUPS;  // two groups per SM either way
-constexpr int ALD = BK + 4, BLD = BN, CLD = BN + 4;
-constexpr int STAGE_ELEMS = BM * ALD + BK * BLD;  // 8704 words
+// Stage = A chunk stored transposed, As[kk][r] (32 x 128), then B chunk
+// Bs[kk][c] (32 x 128): every operand read is one 16-byte vector per 4 rows or
+// columns (4 shared loads per 64 relaxations); a C half-tile (64 x 128) fits too.
+constexpr int ALD = BM, BLD = BN, CLD = BN;
+constexpr int STAGE_ELEMS = BK * ALD + BK * BLD;  // 8192 words
 constexpr int TILE_ELEMS = BM * BN;
 // Bookkeeping is spread over lanes 0 of three warps of a group, so no warp
 // carries more than one latency (a warp that lags delays the group's barriers):
@@ -102,9 +105,6 @@ __device__ __forceinline__ void mb_init(unsigned bar, unsigned count) {
 __device__ __forceinline__ void mb_arrive(unsigned bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
-__device__ __forceinline__ void mb_cp_arrive(unsigned bar) {
-  asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(bar) : "memory");
-}
 __device__ __forceinline__ void mb_wait(unsigned bar, unsigned parity) {
   asm volatile(
       "{\n"
@@ -115,6 +115,17 @@ __device__ __forceinline__ void mb_wait(unsigned bar, unsigned parity) {
       "}\n" ::"r"(bar),
       "r"(parity)
       : "memory");
+}
+__device__ __forceinline__ void mb_expect_tx(unsigned bar, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(unsigned dst, const void* src, unsigned bytes, unsigned bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(bar)
+               : "memory");
+}
+__device__ __forceinline__ void mb_cp_arrive_inc(unsigned bar) {  // counts +1 then -1: no net arrival
+  asm volatile("cp.async.mbarrier.arrive.shared::cta.b64 [%0];" ::"r"(bar) : "memory");
 }
 // named barrier of one 256-thread group (id 0 is __syncthreads)
 __device__ __forceinline__ void gbar(int g) { asm volatile("bar.sync %0, %1;" ::"r"(g + 1), "r"(GNT) : "memory"); }
@@ -253,17 +264,23 @@ __device__ Task decode(long long g, int nb, long long delay) {
   return g3l_task(nb, k, g - 1);
 }
 
+// panel copies of round k (parity k % 2), 128x128 tiles with ld 128:
+//   D = A(k,k) closed, D^T, row panel A(k,j), column panel A(i,k) transposed
 template <typename T>
 __device__ __forceinline__ T* pb_diag(const DFArgs<T>& a, int k) {
-  return a.pbuf + (long long)(k & 1) * (2 * a.nb + 1) * TILE_ELEMS;
+  return a.pbuf + (long long)(k & 1) * (2 * a.nb + 2) * TILE_ELEMS;
+}
+template <typename T>
+__device__ __forceinline__ T* pb_diagT(const DFArgs<T>& a, int k) {
+  return pb_diag(a, k) + TILE_ELEMS;
 }
 template <typename T>
 __device__ __forceinline__ T* pb_row(const DFArgs<T>& a, int k, int j) {
-  return pb_diag(a, k) + (long long)(1 + j) * TILE_ELEMS;
+  return pb_diag(a, k) + (long long)(2 + j) * TILE_ELEMS;
 }
 template <typename T>
-__device__ __forceinline__ T* pb_col(const DFArgs<T>& a, int k, int i) {
-  return pb_diag(a, k) + (long long)(1 + a.nb + i) * TILE_ELEMS;
+__device__ __forceinline__ T* pb_colT(const DFArgs<T>& a, int k, int i) {
+  return pb_diag(a, k) + (long long)(2 + a.nb + i) * TILE_ELEMS;
 }
 
 // Dependency test of task t (one thread): up to three flags, read with
@@ -315,7 +332,8 @@ __device__ void signal_done(const DFArgs<T>& a, const Task& t) {
 // Phase 1 inside a group: in-place FW closure of one 128x128 tile (the same
 // register blocking as phase1_kernel in apsp_kernels.cu); result also to out2.
 template <typename T>
-__device__ __noinline__ void group_phase1(T* tile, long long ld, T* out2, int* negflag, T* scratch, int g, int gtid) {
+__device__ __noinline__ void group_phase1(T* tile, long long ld, T* out2, T* out2t, int* negflag, T* scratch, int g,
+                                         int gtid) {
   using V4 = typename DV<T>::V4;
   T* rowbuf = scratch;            // [2][128]
   T* colbuf = scratch + 2 * 128;  // [2][128]
@@ -379,18 +397,29 @@ __device__ __noinline__ void group_phase1(T* tile, long long ld, T* out2, int* n
     *reinterpret_cast<V4*>(out2 + r * BN + tx * 4) = v0;
     *reinterpret_cast<V4*>(out2 + r * BN + 64 + tx * 4) = v1;
   }
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {  // D^T: column c of the block = 4 + 4 consecutive rows
+    const int c = (j < 4) ? (tx * 4 + j) : (64 + tx * 4 + j - 4);
+    V4 w0, w1;
+    w0.x = acc[0][j]; w0.y = acc[1][j]; w0.z = acc[2][j]; w0.w = acc[3][j];
+    w1.x = acc[4][j]; w1.y = acc[5][j]; w1.z = acc[6][j]; w1.w = acc[7][j];
+    *reinterpret_cast<V4*>(out2t + c * BM + ty * 4) = w0;
+    *reinterpret_cast<V4*>(out2t + c * BM + 64 + ty * 4) = w1;
+  }
 }
 
 // Operands of a group's current min-plus task, written by the group's thread 0
 // before the task-start barrier (kept in shared memory, not in registers).
 template <typename T>
 struct GDesc {
-  const T* A;
-  const T* B;
+  const T* A;  // a_rows = 0: A^T as 128 rows kk of 128 r (ld lda); 1: A itself, rows r (transposed on load)
+  const T* B;  // rows kk of 128 c (ld ldb)
   const T* Cin;
   T* Cout;
-  T* Cout2;  // panel copy (ld 128) or nullptr
+  T* Cout2;  // panel copy (ld 128) or nullptr; c2t = 1: written transposed
   int lda, ldb, ldc;
+  int a_rows, c2t;
+  int bulk;  // 1: A and B chunks are contiguous 16 KB blocks (panel copies): one thread copies them
 };
 
 
@@ -429,12 +458,17 @@ __device__ void fill_desc(const DFArgs<T>& a, const Task& tk, GDesc<T>& d) {
   const int k = tk.k;
   T* const tile = a.D + (long long)tk.i * BM * a.ld + (long long)tk.j * BN;
   d.Cin = tile; d.Cout = tile; d.ldc = (int)a.ld;
+  d.a_rows = 0; d.c2t = 0; d.bulk = 0;
   if (tk.type == T_P2R) {         // A(k,j) = D (x) A(k,j)
-    d.A = pb_diag(a, k); d.lda = BN; d.B = tile; d.ldb = (int)a.ld; d.Cout2 = pb_row(a, k, tk.j);
-  } else if (tk.type == T_P2C) {  // A(i,k) = A(i,k) (x) D
-    d.A = tile; d.lda = (int)a.ld; d.B = pb_diag(a, k); d.ldb = BN; d.Cout2 = pb_col(a, k, tk.i);
+    d.A = pb_diagT(a, k); d.lda = BM; d.B = tile; d.ldb = (int)a.ld; d.Cout2 = pb_row(a, k, tk.j);
+  } else if (tk.type == T_P2C) {  // A(i,k) = A(i,k) (x) D; the copy goes to the transposed column panel
+    d.A = tile; d.lda = (int)a.ld; d.a_rows = 1; d.B = pb_diag(a, k); d.ldb = BN;
+    d.Cout2 = pb_colT(a, k, tk.i); d.c2t = 1;
   } else {                        // A(i,j) = min(A(i,j), A(i,k) (x) A(k,j)) from the panel copies
-    d.A = pb_col(a, k, tk.i); d.lda = BN; d.B = pb_row(a, k, tk.j); d.ldb = BN; d.Cout2 = nullptr;
+    d.A = pb_colT(a, k, tk.i); d.lda = BM; d.B = pb_row(a, k, tk.j); d.ldb = BN; d.Cout2 = nullptr;
+#ifndef DF_NOBULK
+    d.bulk = 1;
+#endif
   }
 }
 
@@ -442,10 +476,8 @@ __device__ void fill_desc(const DFArgs<T>& a, const Task& tk, GDesc<T>& d) {
 //   Cout = min(Cin, A (x) B)  (and Cout2 = the same, ld 128, if non-null)
 // `c0` is the group's running chunk counter (stage = chunk % 3, barrier
 // parity = (chunk / 3) & 1); the task uses chunks c0 .. c0+3.
-// Thread 0 of the group also (a) publishes the group's previous task `pend`
-// once this task's first loads are issued, and (b) prepares the slot of the
-// next task `nxt`: decoded and its flags read (acquire) during chunk 2, its
-// readiness evaluated and its operands written after the epilogue.
+// The SCH thread also prepares the slot of the next task `nxt` during chunk 1:
+// decoded, operands filled, dependencies checked once.
 template <typename T>
 __device__ __noinline__ void group_minplus(const GDesc<T>* d, T* stage0, unsigned full0, unsigned empty0, unsigned c0,
                                            int gtid, int g, const DFArgs<T>* args, long long nxt,
@@ -454,21 +486,63 @@ __device__ __noinline__ void group_minplus(const GDesc<T>* d, T* stage0, unsigne
   constexpr int NK = BM / BK;  // 4 chunks of depth 32
   const int lane = gtid & 31;
   const int tx = gtid & 15, ty = gtid >> 4;
-  auto load_chunk = [&](int stage, int c) {
+  // Chunk c of A and B into stage `stage`, completing one phase of full[stage]
+  // (one arrival + transaction bytes). Panel-copy tasks (phase 3, 62 in 64
+  // tasks): thread 0 issues two 16 KB bulk copies, after waiting for the
+  // stage's previous chunk to be released (wait_G: that chunk, or -1). Phase-2
+  // tasks: every thread copies its share (the column-panel task transposes A
+  // through registers), then one barrier and one arrival.
+  const bool bulk = d->bulk;
+  auto load_chunk = [&](int stage, int c, long long wait_G) {
     T* st = stage0 + stage * STAGE_ELEMS;
-    const int lda = d->lda, ldb = d->ldb;
-    const T* ag = d->A + (gtid >> 3) * lda + (gtid & 7) * 4 + c * BK;
+    if (bulk) {
+      if (gtid == 0) {
+        if (wait_G >= 0) mb_wait(empty0 + 8 * stage, ((unsigned)wait_G / STAGES) & 1);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        const unsigned bytes = BK * BM * (unsigned)sizeof(T);
+        mb_expect_tx(full0 + 8 * stage, 2 * bytes);
+        bulk_g2s(saddr(st), d->A + (long long)c * BK * BM, bytes, full0 + 8 * stage);
+        bulk_g2s(saddr(st + BK * ALD), d->B + (long long)c * BK * BN, bytes, full0 + 8 * stage);
+      }
+      return;
+    }
+    if (wait_G >= 0) mb_wait(empty0 + 8 * stage, ((unsigned)wait_G / STAGES) & 1);
+    const int ldb = d->ldb;
     const T* bg = d->B + ((gtid >> 5) + c * BK) * (long long)ldb + (gtid & 31) * 4;
-    const int a_dst = (gtid >> 3) * ALD + (gtid & 7) * 4;
-    const int b_dst = BM * ALD + (gtid >> 5) * BLD + (gtid & 31) * 4;
+    T* const bdst = st + BK * ALD + (gtid >> 5) * BLD + (gtid & 31) * 4;
+    if (!d->a_rows) {  // A^T rows (panel copies): a 32 x 128 block, like B
+      const int lda = d->lda;
+      const T* ag = d->A + ((gtid >> 5) + c * BK) * (long long)lda + (gtid & 31) * 4;
+      T* const adst = st + (gtid >> 5) * ALD + (gtid & 31) * 4;
 #pragma unroll
-    for (int q = 0; q < 4; ++q) cp16(st + a_dst + q * 32 * ALD, ag + q * 32 * lda);
+      for (int q = 0; q < 4; ++q) cp16(adst + q * 8 * ALD, ag + q * 8 * lda);
 #pragma unroll
-    for (int q = 0; q < 4; ++q) cp16(st + b_dst + q * 8 * BLD, bg + q * 8 * ldb);
-    mb_cp_arrive(full0 + 8 * stage);
+      for (int q = 0; q < 4; ++q) cp16(bdst + q * 8 * BLD, bg + q * 8 * ldb);
+      mb_cp_arrive_inc(full0 + 8 * stage);  // the phase also waits for these copies
+    } else {  // A rows r (column-panel tasks): transpose through registers
+      const int r = gtid & (BM - 1), h = gtid >> 7;
+      const T* ag = d->A + (long long)r * d->lda + c * BK + h * 16;
+      V4 v[4];
+#pragma unroll
+      for (int m = 0; m < 4; ++m) v[m] = __ldcg(reinterpret_cast<const V4*>(ag + 4 * m));
+      V4 w[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) w[q] = __ldcg(reinterpret_cast<const V4*>(bg + q * 8 * ldb));
+#pragma unroll
+      for (int m = 0; m < 4; ++m) {
+        st[(h * 16 + 4 * m + 0) * ALD + r] = v[m].x;
+        st[(h * 16 + 4 * m + 1) * ALD + r] = v[m].y;
+        st[(h * 16 + 4 * m + 2) * ALD + r] = v[m].z;
+        st[(h * 16 + 4 * m + 3) * ALD + r] = v[m].w;
+      }
+#pragma unroll
+      for (int q = 0; q < 4; ++q) *reinterpret_cast<V4*>(bdst + q * 8 * BLD) = w[q];
+    }
+    gbar(g);
+    if (gtid == 0) mb_arrive(full0 + 8 * stage);
   };
-  load_chunk((int)(c0 % STAGES), 0);
-  load_chunk((int)((c0 + 1) % STAGES), 1);
+  load_chunk((int)(c0 % STAGES), 0, -1);  // (the previous task ended with a barrier)
+  load_chunk((int)((c0 + 1) % STAGES), 1, -1);
 
   T acc[8][8];
 #pragma unroll
@@ -496,7 +570,7 @@ __device__ __noinline__ void group_minplus(const GDesc<T>* d, T* stage0, unsigne
       for (int q = 0; q < 8; ++q) cp16(cs_hi + cd + q * 8 * CLD, cg + (64 + q * 8) * ldc);
       cp_commit();
     }
-    if (c == 1 && gtid == SCH) {  // decode the next task, fill its slot and read its flags
+    if (c == 1 && gtid == SCH) {  // the next task's slot
       ns->t = nxt;
       if (nxt < args->total) {
         const Task tn = decode(nxt, args->nb, args->delay);
@@ -506,36 +580,26 @@ __device__ __noinline__ void group_minplus(const GDesc<T>* d, T* stage0, unsigne
       }
     }
     mb_wait(full0 + 8 * s, (G / STAGES) & 1);
-    const T* as = stage0 + s * STAGE_ELEMS;
-    const T* bs = as + BM * ALD;
+    const T* as = stage0 + s * STAGE_ELEMS;  // As[kk][r]
+    const T* bs = as + BK * ALD;             // Bs[kk][c]
 #pragma unroll
-    for (int k2 = 0; k2 < BK / 2; ++k2) {
-      T av[8][2];
+    for (int kk = 0; kk < BK; ++kk) {
+      const V4 a0 = *reinterpret_cast<const V4*>(as + kk * ALD + ty * 4);
+      const V4 a1 = *reinterpret_cast<const V4*>(as + kk * ALD + 64 + ty * 4);
+      const V4 b0 = *reinterpret_cast<const V4*>(bs + kk * BLD + tx * 4);
+      const V4 b1 = *reinterpret_cast<const V4*>(bs + kk * BLD + 64 + tx * 4);
+      const T av[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+      const T bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
 #pragma unroll
-      for (int i = 0; i < 8; ++i) {
-        const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
-        const T* ap = as + r * ALD + k2 * 2;
-        av[i][0] = ap[0]; av[i][1] = ap[1];
-      }
+      for (int i = 0; i < 8; ++i)
 #pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const T* brow = bs + (k2 * 2 + u) * BLD;
-        const V4 b0 = *reinterpret_cast<const V4*>(brow + tx * 4);
-        const V4 b1 = *reinterpret_cast<const V4*>(brow + 64 + tx * 4);
-        const T bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
-#pragma unroll
-        for (int i = 0; i < 8; ++i)
-#pragma unroll
-          for (int j = 0; j < 8; ++j) acc[i][j] = DV<T>::relax(av[i][u], bv[j], acc[i][j]);
-      }
+        for (int j = 0; j < 8; ++j) acc[i][j] = DV<T>::relax(av[i], bv[j], acc[i][j]);
     }
     __syncwarp();
     if (lane == 0) mb_arrive(empty0 + 8 * s);
     if (c + 2 < NK) {  // refill the stage of chunk G-1 with chunk c+2
       const unsigned Gn = G + 2;
-      const int sn = (int)(Gn % STAGES);
-      if (Gn >= STAGES) mb_wait(empty0 + 8 * sn, ((Gn - STAGES) / STAGES) & 1);
-      load_chunk(sn, c + 2);
+      load_chunk((int)(Gn % STAGES), c + 2, Gn >= STAGES ? (long long)(Gn - STAGES) : -1ll);
     }
   }
   cp_wait_all();
@@ -552,16 +616,29 @@ __device__ __noinline__ void group_minplus(const GDesc<T>* d, T* stage0, unsigne
       const T* crow = (i < 4 ? cs_lo : cs_hi) + (ty * 4 + (i & 3)) * CLD;
       const V4 x0 = *reinterpret_cast<const V4*>(crow + tx * 4);
       const V4 x1 = *reinterpret_cast<const V4*>(crow + 64 + tx * 4);
+      acc[i][0] = DV<T>::vmin(acc[i][0], x0.x); acc[i][1] = DV<T>::vmin(acc[i][1], x0.y);
+      acc[i][2] = DV<T>::vmin(acc[i][2], x0.z); acc[i][3] = DV<T>::vmin(acc[i][3], x0.w);
+      acc[i][4] = DV<T>::vmin(acc[i][4], x1.x); acc[i][5] = DV<T>::vmin(acc[i][5], x1.y);
+      acc[i][6] = DV<T>::vmin(acc[i][6], x1.z); acc[i][7] = DV<T>::vmin(acc[i][7], x1.w);
       V4 v0, v1;
-      v0.x = DV<T>::vmin(acc[i][0], x0.x); v0.y = DV<T>::vmin(acc[i][1], x0.y);
-      v0.z = DV<T>::vmin(acc[i][2], x0.z); v0.w = DV<T>::vmin(acc[i][3], x0.w);
-      v1.x = DV<T>::vmin(acc[i][4], x1.x); v1.y = DV<T>::vmin(acc[i][5], x1.y);
-      v1.z = DV<T>::vmin(acc[i][6], x1.z); v1.w = DV<T>::vmin(acc[i][7], x1.w);
+      v0.x = acc[i][0]; v0.y = acc[i][1]; v0.z = acc[i][2]; v0.w = acc[i][3];
+      v1.x = acc[i][4]; v1.y = acc[i][5]; v1.z = acc[i][6]; v1.w = acc[i][7];
       *reinterpret_cast<V4*>(Cout + (long long)r * ldc + tx * 4) = v0;
       *reinterpret_cast<V4*>(Cout + (long long)r * ldc + 64 + tx * 4) = v1;
-      if (Cout2) {
+      if (Cout2 && !d->c2t) {
         *reinterpret_cast<V4*>(Cout2 + r * BN + tx * 4) = v0;
         *reinterpret_cast<V4*>(Cout2 + r * BN + 64 + tx * 4) = v1;
+      }
+    }
+    if (Cout2 && d->c2t) {  // transposed copy: column c of the block = 4 + 4 consecutive rows
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        const int cc = (j < 4) ? (tx * 4 + j) : (64 + tx * 4 + j - 4);
+        V4 w0, w1;
+        w0.x = acc[0][j]; w0.y = acc[1][j]; w0.z = acc[2][j]; w0.w = acc[3][j];
+        w1.x = acc[4][j]; w1.y = acc[5][j]; w1.z = acc[6][j]; w1.w = acc[7][j];
+        *reinterpret_cast<V4*>(Cout2 + cc * BM + ty * 4) = w0;
+        *reinterpret_cast<V4*>(Cout2 + cc * BM + 64 + ty * 4) = w1;
       }
     }
   }
@@ -577,7 +654,7 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
   const unsigned full0 = saddr(&bars[g][0]), empty0 = full0 + 8 * STAGES;
   if (gtid == 0) {
     for (int s = 0; s < STAGES; ++s) {
-      mb_init(full0 + 8 * s, GNT);
+      mb_init(full0 + 8 * s, 1);  // one arrival per chunk (+ transaction bytes of bulk copies)
       mb_init(empty0 + 8 * s, GNT / 32);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -618,7 +695,7 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
     pr[0] += tc1 - tc0;
     if (tk.type == T_P1) {
       T* const tile = a.D + (long long)tk.i * BM * a.ld + (long long)tk.j * BN;
-      group_phase1<T>(tile, a.ld, pb_diag(a, tk.k), a.negflag, stage0, g, gtid);
+      group_phase1<T>(tile, a.ld, pb_diag(a, tk.k), pb_diagT(a, tk.k), a.negflag, stage0, g, gtid);
       if (gtid == SCH) {
         N->t = nxt;
         if (nxt < a.total) {
@@ -685,7 +762,7 @@ cudaError_t launch_fw_dataflow(T* D, long long ld, int nb, void* work, int* negf
 }
 
 long long fw_dataflow_pbuf_bytes(int nb, size_t elem) {
-  return 2ll * (2 * nb + 1) * TILE_ELEMS * (long long)elem;  // (kept a multiple of 8 bytes)
+  return 2ll * (2 * nb + 2) * TILE_ELEMS * (long long)elem;  // (kept a multiple of 8 bytes)
 }
 long long fw_dataflow_flag_bytes(int nb) { return ((long long)nb * nb + 6ll * nb + 4) * 4; }
 long long fw_dataflow_work_bytes(int nb, size_t elem) {
