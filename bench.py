@@ -303,18 +303,20 @@ def run_ours(args):
         if not peak:
             peak = 148 * 64 * 1.965e9 * (2 if arith == "s16x2" else 1)
             peak_src = "derived: 148 SMs x 64 lanes/clk x 1.965 GHz (no MEASURED_DPX.json)"
+        dataflow = st_acc[1][0] == 0 and st_acc[1][2] == args.steps  # one launch per step, no phase-1 launches
         elem = 2 if arith == "s16x2" else 4
         traffic = None
         tp = os.path.join(ROOT, "profiles", "phase3_traffic.json")
         if os.path.exists(tp) and not args.force_ooc:
             try:
+                sched = "dataflow" if dataflow else "legacy"
                 for tj in json.load(open(tp)).get("captures", []):
-                    if tj.get("workload") == wl and tj.get("arith") == arith:
+                    if (tj.get("workload") == wl and tj.get("arith") == arith
+                            and tj.get("schedule", "legacy") == sched):
                         # measured DRAM bytes per relaxation (ncu capture) x this run's relax per launch
                         traffic = tj["dram_bytes_per_relax"] * p3_relax
             except Exception:
                 pass
-        dataflow = st_acc[1][0] == 0 and st_acc[1][2] == args.steps  # one launch per step, no phase-1 launches
         kname = ("fw_dataflow_kernel: all rounds and phases 1-3 in one persistent launch (%s)" % arith if dataflow
                  else "phase-3 min-plus (%s)" % arith)
         roofline = {"bound": "alu", "kernel": kname, "achieved": achieved / 1e12,
