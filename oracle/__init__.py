@@ -66,6 +66,8 @@ def _load():
             f = getattr(lib, name)
             f.argtypes = args
             f.restype = ctypes.c_int
+        lib.oracle_certify_rows_i32.argtypes = [I64, P, P, P, I64, I64, P, I64, ctypes.c_int32, P]
+        lib.oracle_certify_rows_i32.restype = I64
         lib.oracle_omp_max_threads.restype = ctypes.c_int
         lib.oracle_omp_max_threads.argtypes = []
         _lib = lib
@@ -165,3 +167,19 @@ def bellman_ford_row_i64(row_ptr, col, w, src: int):
     out = np.empty(n, dtype=np.int64)
     neg = _load().oracle_bellman_ford_row_i64(n, _p(row_ptr), _p(col), _p(w), int(src), _p(out))
     return out, bool(neg)
+
+
+def certify_rows_i32(row_ptr, col, w, r0: int, rows: np.ndarray, inf: int):
+    """Optimality certificate (apsp_oracle.c: oracle_certify_rows_i32) for claimed
+    int32 distance rows dist[r0 .. r0+len(rows)) of a graph with weights > 0.
+    `rows` may be a strided 2-D view (C-contiguous rows). Returns (n_bad, first_bad_source)."""
+    n, row_ptr, col, w = _csr(row_ptr, col, w, np.int64)
+    assert rows.dtype == np.int32 and rows.ndim == 2 and rows.strides[1] == 4
+    assert rows.shape[1] >= n
+    ld = rows.strides[0] // 4
+    first = np.zeros(1, dtype=np.int64)
+    bad = _load().oracle_certify_rows_i32(n, _p(row_ptr), _p(col), _p(w), int(r0), rows.shape[0],
+                                          rows.ctypes.data_as(ctypes.c_void_p), ld, int(inf), _p(first))
+    if bad < 0:
+        raise ValueError("certificate needs strictly positive weights")
+    return int(bad), int(first[0])

@@ -37,6 +37,11 @@
  *                     independent pin of oracle_fw_* on small graphs.
  *   oracle_bellman_ford_row_i64  PAPER.md:68 (§II-B) Bellman–Ford, one source,
  *                     any weights; returns 1 on a reachable negative cycle.
+ *   oracle_certify_rows_i32  the shortest-path optimality conditions (Bellman
+ *                     equations of the single-source problem)
+ *                     as an O(m)-per-row exactness certificate for claimed
+ *                     int32 rows with strictly positive weights; checks every
+ *                     row of the full-size (n=262144) results.
  *
  * Parity pins (tests/test_oracle.py, -m "not gpu"): closed forms (grid =
  * Manhattan distance, directed ring, weighted path, complete graph, disjoint
@@ -269,6 +274,67 @@ int oracle_bellman_ford_row_i64(int64_t n, const int64_t* row_ptr, const int32_t
     if (round == n - 1) return 1;
   }
   return 0;
+}
+
+/* --------------------------------------------- optimality certificate -- */
+
+/* Shortest-path optimality certificate for claimed distance rows (SURVEY.md
+ * §8(c) "full-scale exactness"; the Bellman equations of PAPER.md:66-68's
+ * single-source problem). For a graph whose arc weights are all STRICTLY
+ * positive, a row d = D[s][.] equals the true shortest distances from s iff
+ *   (i)   d[s] = 0;
+ *   (ii)  every arc (u,v,w) with d[u] finite has d[v] <= d[u] + w
+ *         (an "unreachable" d[v] violates it);
+ *   (iii) every v != s with d[v] finite has an arc (u,v,w) with d[u] finite
+ *         and d[v] = d[u] + w.
+ * Proof: (ii) along a shortest s->v path gives d[v] <= dist(s,v) (and finite
+ * whenever v is reachable); following (iii) backwards from v gives a walk
+ * into v of length d[v] whose d-values strictly decrease (w > 0), so it
+ * cannot repeat a vertex and must end at the only vertex with no tight arc
+ * required, s: d[v] >= dist(s,v). Cost O(m) per row, no triple loop, so it
+ * checks every row of the n=262144 result.
+ *
+ * rows: cnt rows of an int32 matrix (row i is source s = r0 + i), ld elements
+ * apart, `inf` the value that marks "no path". Integers are compared in int64.
+ * Returns the number of rows that fail; -1 if some weight is <= 0. If fail_row
+ * is non-NULL it receives the first failing source (or -1). */
+int64_t oracle_certify_rows_i32(int64_t n, const int64_t* row_ptr, const int32_t* col,
+                                const int64_t* w, int64_t r0, int64_t cnt,
+                                const int32_t* rows, int64_t ld, int32_t inf,
+                                int64_t* fail_row) {
+  for (int64_t e = 0; e < row_ptr[n]; ++e)
+    if (w[e] <= 0) return -1;
+  int64_t bad = 0, first = -1;
+#pragma omp parallel
+  {
+    unsigned char* tight = (unsigned char*)malloc((size_t)(n > 0 ? n : 1));
+#pragma omp for schedule(dynamic, 16) reduction(+ : bad)
+    for (int64_t i = 0; i < cnt; ++i) {
+      const int32_t* d = rows + i * ld;
+      const int64_t s = r0 + i;
+      int ok = (d[s] == 0);
+      memset(tight, 0, (size_t)n);
+      for (int64_t u = 0; u < n && ok; ++u) {
+        if (d[u] == inf) continue;
+        for (int64_t e = row_ptr[u]; e < row_ptr[u + 1]; ++e) {
+          const int64_t v = col[e];
+          const int64_t via = (int64_t)d[u] + w[e];
+          if (d[v] == inf || (int64_t)d[v] > via) { ok = 0; break; }   /* (ii) */
+          if ((int64_t)d[v] == via) tight[v] = 1;
+        }
+      }
+      for (int64_t v = 0; v < n && ok; ++v)
+        if (v != s && d[v] != inf && !tight[v]) ok = 0;                /* (iii) */
+      if (!ok) {
+        bad += 1;
+#pragma omp critical
+        if (first < 0 || s < first) first = s;
+      }
+    }
+    free(tight);
+  }
+  if (fail_row) *fail_row = first;
+  return bad;
 }
 
 int oracle_omp_max_threads(void) {

@@ -2,7 +2,8 @@
 (default config, one handle, apsp_reinit + apsp_fw_blocked), on outputs the oracle
 computes one by one: sampled full rows by the oracle's Dijkstra compared
 bit-exactly, plus properties that hold at any size (zero diagonal, symmetry of an
-undirected graph, D[u][v] <= w(u,v))."""
+undirected graph, D[u][v] <= w(u,v)), and EVERY row checked by the oracle's optimality
+certificate (oracle.certify_rows_i32, exact for strictly positive weights)."""
 import numpy as np
 import pytest
 
@@ -50,6 +51,7 @@ def test_config2_grid16384_full_size(lib):
         s, t, w = g.arcs()
         assert np.all(d[s, t] <= w)
         assert np.all(d < INF32)  # connected grid
+        assert oracle.certify_rows_i32(g.row_ptr, g.col, g.w, 0, d, INF32) == (0, -1)
     finally:
         h.close()
 
@@ -59,6 +61,9 @@ def test_config3_er65536_full_size(lib):
     h = run_like_bench(lib, g)
     try:
         check_sampled_rows(lib, h, g, n_rows=24, seed=3)
+        for r0 in range(0, g.n, 8192):  # whole 17 GB result, 2 GB at a time
+            rows = lib.apsp_get_dist(h, r0, 8192)
+            assert oracle.certify_rows_i32(g.row_ptr, g.col, g.w, r0, rows, INF32) == (0, -1)
     finally:
         h.close()
 

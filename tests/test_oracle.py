@@ -347,3 +347,64 @@ def test_graphgen_shapes():
     g1 = gg.erdos_renyi(500, 3000, seed=11)
     g2 = gg.erdos_renyi(500, 3000, seed=11)
     assert np.array_equal(g1.col, g2.col) and np.array_equal(g1.w, g2.w)
+
+
+# ------------------------------------------------- optimality certificate
+
+INF32 = 0x3FFFFFFF  # the int32 output's "no path" value (include/apsp.h, R1)
+
+
+def _as_i32(d):
+    return np.where(d == oracle.INF_I64, INF32, d).astype(np.int32)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_certificate_accepts_apsp_and_rejects_every_single_perturbation(seed):
+    """The certificate (Bellman optimality conditions) accepts the true APSP rows
+    (brute force on tiny graphs) and rejects ANY single-entry change: +1, -1, a
+    finite entry made unreachable, an unreachable one made finite."""
+    rng = np.random.default_rng(100 + seed)
+    n = 7
+    arcs = random_arcs(rng, n, 12, 1, 9)
+    bf, _ = brute_force(n, arcs)
+    g = csr_of(n, arcs)
+    d = _as_i32(bf)
+    assert oracle.certify_rows_i32(g.row_ptr, g.col, g.w, 0, d, INF32) == (0, -1)
+    for s in range(n):
+        for v in range(n):
+            for new in (d[s, v] + 1, d[s, v] - 1, INF32, 5):
+                if new == d[s, v]:
+                    continue
+                e = d.copy()
+                e[s, v] = new
+                bad, first = oracle.certify_rows_i32(g.row_ptr, g.col, g.w, 0, e, INF32)
+                assert bad == 1 and first == s, (s, v, new)
+
+
+def test_certificate_on_row_slices_and_strided_rows():
+    g = gg.grid_2d(20, 30, seed=7)
+    d, _ = oracle.fw_i64(g.row_ptr, g.col, g.w)
+    d32 = _as_i32(d)
+    wide = np.full((g.n, g.n + 40), -7, dtype=np.int32)
+    wide[:, :g.n] = d32
+    assert oracle.certify_rows_i32(g.row_ptr, g.col, g.w, 100, wide[100:300], INF32) == (0, -1)
+    wide[250, 3] += 1
+    assert oracle.certify_rows_i32(g.row_ptr, g.col, g.w, 100, wide[100:300], INF32) == (1, 250)
+    # a row certified against the wrong source fails (d[s][s] != 0)
+    assert oracle.certify_rows_i32(g.row_ptr, g.col, g.w, 101, wide[100:101], INF32)[0] == 1
+
+
+def test_certificate_disconnected_and_rejects_zero_weights():
+    a = gg.grid_2d(4, 4, seed=1)
+    arcs = list(zip(*[x.tolist() for x in a.arcs()]))
+    arcs += [(16 + u, 16 + v, w) for (u, v, w) in arcs]
+    g = csr_of(32, arcs)
+    d, _ = oracle.fw_i64(g.row_ptr, g.col, g.w)
+    d32 = _as_i32(d)
+    assert oracle.certify_rows_i32(g.row_ptr, g.col, g.w, 0, d32, INF32) == (0, -1)
+    e = d32.copy()
+    e[0, 20] = 1000  # finite entry for an unreachable vertex: no tight arc can support it
+    assert oracle.certify_rows_i32(g.row_ptr, g.col, g.w, 0, e, INF32)[0] == 1
+    z = csr_of(3, [(0, 1, 0), (1, 2, 4)])
+    with pytest.raises(ValueError):
+        oracle.certify_rows_i32(z.row_ptr, z.col, z.w, 0, np.zeros((3, 3), np.int32), INF32)
