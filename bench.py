@@ -352,6 +352,7 @@ def run_ours(args):
         barrier()
         torch.cuda.synchronize()
         parts = np.zeros(4)
+        per_step = []
         t0 = time.perf_counter()
         for _ in range(k_e2e):
             ta = time.perf_counter()
@@ -363,13 +364,15 @@ def run_ours(args):
                 apsp.apsp_get_dist_ptr(he, rb, rc, host_out.data_ptr(), n)
             td = time.perf_counter()
             apsp.apsp_destroy(he)
-            parts += np.array([tb - ta, tc - tb, td - tc, time.perf_counter() - td])
+            per_step.append([tb - ta, tc - tb, td - tc, time.perf_counter() - td])
+            parts += np.array(per_step[-1])
         torch.cuda.synchronize()
         el = max_over_ranks(time.perf_counter() - t0)
         return {"value": float(n) ** 3 / (el / k_e2e), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                 "d2h_bytes_per_step": int(d2h), "steps": k_e2e,
                 "ms_per_step_parts": dict(zip(["init", "fw", "get_dist", "destroy"],
                                               (parts / k_e2e * 1e3).round(2).tolist())),
+                "ms_parts_each_step": (np.array(per_step) * 1e3).round(2).tolist(),
                 "note": "apsp_init_from_csr(host CSR, pinned) + apsp_fw_blocked + apsp_get_dist(pinned host) + "
                         "destroy, host wall clock (synchronous C-ABI calls)"}
 
