@@ -64,6 +64,7 @@ typedef enum {
 #define APSP_MODE_INCORE 0
 #define APSP_MODE_OUT_OF_CORE 1
 #define APSP_MODE_BOUNDARY 2
+#define APSP_MODE_JOHNSON 3
 
 typedef struct {
   int32_t struct_size;          /* = sizeof(apsp_config) (ABI versioning); 0 = defaults */
@@ -148,10 +149,35 @@ apsp_status apsp_init_boundary(apsp_handle** out, int64_t n, const int64_t* row_
                                const int32_t* comp, int32_t k, const apsp_config* cfg);
 
 /*
+ * apsp_init_johnson — set up Johnson's algorithm (§II-B): one
+ * single-source shortest-path run per source vertex, each by the Near-Far
+ * method in ONE thread block, a persistent grid of blocks walking the
+ * sources (Algorithm 2). Same CSR arguments, semantics and errors
+ * as apsp_init_from_csr, plus:
+ *   delta     the Near-Far bucket width Delta in weight units; 0 = auto
+ *             (4 x the mean |weight|). Any delta > 0 gives the same distances
+ *   batch     sources per batch when the result does not fit in device
+ *             memory (Algorithm 2's `bat`; rows of a finished batch go
+ *             to a pinned host matrix while the next batch runs); 0 = auto
+ * Work is O(n * m * (re-expansions)) instead of n^3, so it wins on sparse
+ * graphs (the paper's selection finding). The n x n result stays
+ * in device memory when it fits the budget (cfg->device_budget_bytes, else
+ * free memory), otherwise in pinned host memory (cfg->force_out_of_core = 1
+ * forces this). Negative int32 weights are reweighted (Johnson: Bellman–Ford
+ * potentials); a negative cycle makes apsp_solve return
+ * APSP_ENEGCYCLE. fp32 weights must be >= 0 (else APSP_EINVAL). One GPU per
+ * handle (world_size 1). Run with apsp_solve; apsp_get_dist as usual;
+ * apsp_info.edges_scanned reports the arcs the last run relaxed.
+ */
+apsp_status apsp_init_johnson(apsp_handle** out, int64_t n, const int64_t* row_ptr,
+                              const int32_t* col_idx, const void* weights, apsp_dtype dtype,
+                              double delta, int64_t batch, const apsp_config* cfg);
+
+/*
  * apsp_solve — run the method the handle was created for: the blocked
- * Floyd–Warshall (apsp_init_from_csr, same as apsp_fw_blocked) or the boundary
- * algorithm (apsp_init_boundary). Blocks until done; APSP_ENEGCYCLE as
- * apsp_fw_blocked.
+ * Floyd–Warshall (apsp_init_from_csr, same as apsp_fw_blocked), the boundary
+ * algorithm (apsp_init_boundary) or Johnson's algorithm (apsp_init_johnson).
+ * Blocks until done; APSP_ENEGCYCLE as apsp_fw_blocked.
  */
 apsp_status apsp_solve(apsp_handle* h);
 
@@ -221,6 +247,7 @@ typedef struct {
                                                   result (or of the next run) */
   int32_t packed16_eligible;                   /* packed16 requested and the input allows it */
   int64_t boundary_nodes;                      /* boundary algorithm: boundary nodes, else 0 */
+  int64_t edges_scanned;                       /* Johnson: arcs relaxed by the last run, else 0 */
 } apsp_info;
 
 #define APSP_ARITH_I32 0   /* VIADDMNMX (int32 DPX), 1 relaxation / instruction */

@@ -32,7 +32,7 @@ APSP_OK, APSP_EINVAL, APSP_ERANGE, APSP_ENOMEM, APSP_ECUDA, APSP_ENCCL, APSP_ENE
 STATUS_NAMES = ["APSP_OK", "APSP_EINVAL", "APSP_ERANGE", "APSP_ENOMEM", "APSP_ECUDA", "APSP_ENCCL",
                 "APSP_ENEGCYCLE", "APSP_ESTATE"]
 APSP_INF_I32 = 0x3FFFFFFF
-APSP_MODE_INCORE, APSP_MODE_OUT_OF_CORE, APSP_MODE_BOUNDARY = 0, 1, 2
+APSP_MODE_INCORE, APSP_MODE_OUT_OF_CORE, APSP_MODE_BOUNDARY, APSP_MODE_JOHNSON = 0, 1, 2, 3
 TILE = 128
 
 
@@ -64,6 +64,7 @@ class apsp_info(ctypes.Structure):
         ("dist_device", ctypes.c_void_p), ("ld", ctypes.c_int64),
         ("arith", ctypes.c_int32), ("packed16_eligible", ctypes.c_int32),
         ("boundary_nodes", ctypes.c_int64),
+        ("edges_scanned", ctypes.c_int64),
     ]
 
 
@@ -86,6 +87,8 @@ _sig = {
     "apsp_fw_blocked": (ctypes.c_int, [_H]),
     "apsp_init_boundary": (ctypes.c_int, [ctypes.POINTER(_H), _I64, _P, _P, _P, ctypes.c_int, _P, _I32,
                                           ctypes.POINTER(apsp_config)]),
+    "apsp_init_johnson": (ctypes.c_int, [ctypes.POINTER(_H), _I64, _P, _P, _P, ctypes.c_int, ctypes.c_double,
+                                         _I64, ctypes.POINTER(apsp_config)]),
     "apsp_solve": (ctypes.c_int, [_H]),
     "apsp_reinit": (ctypes.c_int, [_H]),
     "apsp_fw_rounds": (ctypes.c_int, [_H, _I64, _I64]),
@@ -231,6 +234,25 @@ def apsp_init_boundary(n: int, row_ptr, col_idx, weights, comp, k: int, dtype: i
     return Handle(raw, dtype, n, (cfg,))
 
 
+def apsp_init_johnson(n: int, row_ptr, col_idx, weights, dtype: int | None = None, delta: float = 0.0,
+                      batch: int = 0, cfg: apsp_config | None = None) -> Handle:
+    """Johnson's algorithm with batched Near-Far SSSP (Algorithm 2)."""
+    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
+    w = np.asarray(weights)
+    if dtype is None:
+        dtype = APSP_F32 if w.dtype.kind == "f" else APSP_I32
+    w = np.ascontiguousarray(w, dtype=np.int32 if dtype == APSP_I32 else np.float32)
+    if row_ptr.shape[0] != n + 1:
+        raise ApspError(APSP_EINVAL, "row_ptr must have n+1 entries")
+    if cfg is None:
+        cfg = apsp_config_default()
+    raw = ctypes.c_void_p()
+    _check(_lib.apsp_init_johnson(ctypes.byref(raw), n, _ptr(row_ptr), _ptr(col_idx), _ptr(w), dtype,
+                                  float(delta), int(batch), ctypes.byref(cfg)))
+    return Handle(raw, dtype, n, (cfg,))
+
+
 def apsp_solve(h: Handle) -> None:
     _check(_lib.apsp_solve(h.raw), h.raw)
 
@@ -295,6 +317,13 @@ def solve(g, cfg: apsp_config | None = None, dtype: int | None = None) -> np.nda
     """Full APSP of a ``graphgen.CSR``-like object (n, row_ptr, col, w) -> n x n host array."""
     with apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, dtype=dtype, cfg=cfg) as h:
         apsp_fw_blocked(h)
+        return apsp_get_dist(h)
+
+
+def solve_johnson(g, delta: float = 0.0, batch: int = 0, cfg: apsp_config | None = None) -> np.ndarray:
+    """Full APSP by Johnson's algorithm (batched Near-Far SSSP)."""
+    with apsp_init_johnson(g.n, g.row_ptr, g.col, g.w, delta=delta, batch=batch, cfg=cfg) as h:
+        apsp_solve(h)
         return apsp_get_dist(h)
 
 

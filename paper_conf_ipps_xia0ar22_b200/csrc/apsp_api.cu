@@ -495,15 +495,66 @@ apsp_status apsp_init_boundary(apsp_handle** out, int64_t n, const int64_t* row_
   return APSP_OK;
 }
 
+apsp_status apsp_init_johnson(apsp_handle** out, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                              const void* weights, apsp_dtype dtype, double delta, int64_t batch,
+                              const apsp_config* cfg_in) {
+  if (!out) return fail_global(APSP_EINVAL, "apsp_init_johnson: out is NULL");
+  *out = nullptr;
+  apsp_config cfg;
+  apsp_config_default(&cfg);
+  if (cfg_in) {
+    if (cfg_in->struct_size != 0 && cfg_in->struct_size != (int32_t)sizeof(apsp_config))
+      return fail_global(APSP_EINVAL, "apsp_config.struct_size %d != %d", cfg_in->struct_size,
+                         (int)sizeof(apsp_config));
+    cfg = *cfg_in;
+  }
+  if (n < 1 || n > (int64_t)INT32_MAX) return fail_global(APSP_EINVAL, "bad n");
+  if (!row_ptr) return fail_global(APSP_EINVAL, "row_ptr is NULL");
+  if (dtype != APSP_I32 && dtype != APSP_F32) return fail_global(APSP_EINVAL, "bad dtype");
+  if (cfg.world_size != 1) return fail_global(APSP_EINVAL, "Johnson's algorithm runs on one GPU per handle");
+  if (!(delta >= 0) || !std::isfinite(delta)) return fail_global(APSP_EINVAL, "delta must be finite and >= 0");
+  bool has_neg = false;
+  int64_t maxabs = 0;
+  apsp_status vst = validate_csr(n, row_ptr, col_idx, weights, dtype, &has_neg, &maxabs);
+  if (vst != APSP_OK) return vst;
+
+  Handle* h = new Handle();
+  h->n = n;
+  h->dtype = dtype;
+  h->timing = cfg.timing != 0;
+  h->has_neg = has_neg;
+  h->max_abs_w = maxabs;
+  h->arith = dtype == APSP_F32 ? APSP_ARITH_F32 : APSP_ARITH_I32;
+  h->elem = 4;
+  h->mode = APSP_MODE_JOHNSON;
+  apsp_status st = setup_device(h, cfg);
+  if (!st) st = jn_setup(h, cfg, row_ptr, col_idx, weights, delta, batch);
+  if (st != APSP_OK) {
+    g_last_error = h->err;
+    delete_handle(h);
+    return st;
+  }
+  *out = reinterpret_cast<apsp_handle*>(h);
+  return APSP_OK;
+}
+
 apsp_status apsp_solve(apsp_handle* hh) {
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
-  if (h->mode != APSP_MODE_BOUNDARY) return apsp_fw_blocked(hh);
+  if (h->mode != APSP_MODE_BOUNDARY && h->mode != APSP_MODE_JOHNSON) return apsp_fw_blocked(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
   if (h->fw_done) return h->fail(APSP_ESTATE, "apsp_solve already ran (apsp_reinit first)");
   apsp_status st;
   if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
   memset(&h->stats, 0, sizeof(h->stats));
+  if (h->mode == APSP_MODE_JOHNSON) {
+    if ((st = jn_run(h))) return st;
+    if (h->timing) h->collect_events();
+    h->stats.relax[2] = (double)jn_edges(h);
+    h->fw_done = true;
+    h->canonical = true;
+    return APSP_OK;
+  }
   if ((st = bnd_run(h))) return st;
   return finish_fw(h, true);
 }
@@ -529,7 +580,8 @@ apsp_status apsp_fw_blocked(apsp_handle* hh) {
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
   if (h->fw_done) return h->fail(APSP_ESTATE, "apsp_fw_blocked already ran");
-  if (h->mode == APSP_MODE_BOUNDARY) return h->fail(APSP_ESTATE, "boundary-algorithm handle: use apsp_solve");
+  if (h->mode == APSP_MODE_BOUNDARY || h->mode == APSP_MODE_JOHNSON)
+    return h->fail(APSP_ESTATE, "boundary / Johnson handle: use apsp_solve");
   apsp_status st;
   if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
   memset(&h->stats, 0, sizeof(h->stats));
@@ -557,6 +609,7 @@ apsp_status apsp_reinit(apsp_handle* hh) {
   if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
   if (h->mode == APSP_MODE_OUT_OF_CORE) return ooc_reinit(h);
   if (h->mode == APSP_MODE_BOUNDARY) return bnd_reinit(h);
+  if (h->mode == APSP_MODE_JOHNSON) return jn_reinit(h);
   return run_init(h);
 }
 
@@ -605,6 +658,7 @@ apsp_status apsp_get_info(const apsp_handle* hh, apsp_info* info) {
   info->packed16_eligible = h->mode16 ? 1 : 0;
   if (h->result16) info->dist_device = h->d16;
   info->boundary_nodes = bnd_boundary_nodes(h);
+  info->edges_scanned = jn_edges(h);
   return APSP_OK;
 }
 

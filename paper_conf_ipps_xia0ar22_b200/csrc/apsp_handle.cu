@@ -286,6 +286,7 @@ void delete_handle(Handle* h) {
   if (h->comm) ncclCommDestroy(static_cast<ncclComm_t>(h->comm));
   ooc_free(h);
   bnd_free(h);
+  jn_free(h);
   for (auto& sh : h->shards) {
     cudaFree(sh.d_rp);
     cudaFree(sh.d_col);
@@ -333,6 +334,7 @@ apsp_status finish_fw(Handle* h, bool all_rounds) {
 apsp_status get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out) {
   if (h->mode == APSP_MODE_OUT_OF_CORE) return ooc_get_rows(h, r0, cnt, out, ld_out);
   if (h->mode == APSP_MODE_BOUNDARY) return bnd_get_rows(h, r0, cnt, out, ld_out);
+  if (h->mode == APSP_MODE_JOHNSON) return jn_get_rows(h, r0, cnt, out, ld_out);
   apsp_status st;
   if (h->mode16 && !h->shards[0].D && !h->result16)
     return h->fail(APSP_ESTATE, "no int32 matrix yet");

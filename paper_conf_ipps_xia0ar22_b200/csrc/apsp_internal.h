@@ -69,6 +69,8 @@ struct Handle {
   void* ooc_streams[3] = {nullptr, nullptr, nullptr};
   // boundary algorithm (apsp_boundary.cu)
   void* bnd = nullptr;
+  // Johnson's algorithm, batched Near-Far (apsp_johnson.cu)
+  void* jn = nullptr;
   // single-GPU in-core dataflow kernel (apsp_fw_dataflow.cu)
   bool dataflow = true;     // apsp_config.reserved[4] = 1 selects the launch-per-phase schedule
   long long df_delay = 0;   // reserved[5] (0 = auto)
@@ -120,6 +122,14 @@ apsp_status bnd_run(Handle* h);
 apsp_status bnd_get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out);
 long long bnd_boundary_nodes(const Handle* h);
 void bnd_free(Handle* h);
+// Johnson's algorithm with batched Near-Far SSSP (apsp_johnson.cu)
+apsp_status jn_setup(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, const int32_t* col, const void* w,
+                     double delta, long long batch);
+apsp_status jn_reinit(Handle* h);
+apsp_status jn_run(Handle* h);
+apsp_status jn_get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out);
+long long jn_edges(const Handle* h);
+void jn_free(Handle* h);
 // common device / stream setup of a handle (apsp_handle.cu)
 apsp_status setup_device(Handle* h, const apsp_config& cfg);
 
