@@ -174,6 +174,36 @@ apsp_status apsp_init_johnson(apsp_handle** out, int64_t n, const int64_t* row_p
                               double delta, int64_t batch, const apsp_config* cfg);
 
 /*
+ * apsp_select — choose the method for a graph as the paper does (§IV,
+ * PAPER.md:199-323). Density filter (§IV-C), density = m / n^2:
+ *   > 1 %       blocked FW or Johnson
+ *   < 0.01 %    Johnson or the boundary algorithm (only if a partition comp/k is
+ *               given; the paper computes one with METIS)
+ *   otherwise   Johnson
+ * then the smallest cost-model estimate among the kept methods (§IV-B),
+ * calibrated on this device at call time: blocked FW T0*(n/n0)^3 from a timed
+ * random graph of n0 <= 8192 vertices; Johnson (n_b/k)*T from k = 5
+ * randomly chosen batches actually run; boundary N_op * c_unit
+ * with c_unit = the FW kernels' per-relaxation cost; plus the data
+ * transfer models when the n x n result exceeds device memory.
+ * Arguments as apsp_init_from_csr; comp/k as apsp_init_boundary or NULL/0.
+ * Runs kernels on cfg->device (about 0.1-1 s); the graph is not retained.
+ */
+typedef struct {
+  int32_t method;          /* APSP_MODE_INCORE (blocked FW; out of core when too big),
+                              APSP_MODE_JOHNSON or APSP_MODE_BOUNDARY */
+  int32_t candidates;      /* bit (1 << mode) per method the density filter kept */
+  double density;          /* m / n^2 */
+  double est_seconds[4];   /* estimate per mode index ([0] FW, [2] boundary,
+                              [3] Johnson); -1 = not estimated */
+  int64_t boundary_nodes;  /* boundary nodes of the given partition, else 0 */
+} apsp_selection;
+
+apsp_status apsp_select(int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
+                        const void* weights, apsp_dtype dtype, const int32_t* comp, int32_t k,
+                        const apsp_config* cfg, apsp_selection* out);
+
+/*
  * apsp_solve — run the method the handle was created for: the blocked
  * Floyd–Warshall (apsp_init_from_csr, same as apsp_fw_blocked), the boundary
  * algorithm (apsp_init_boundary) or Johnson's algorithm (apsp_init_johnson).

@@ -72,6 +72,11 @@ APSP_ARITH_I32, APSP_ARITH_S16X2, APSP_ARITH_F32 = 0, 1, 2
 ARITH_NAMES = {0: "i32", 1: "s16x2", 2: "f32"}
 
 
+class apsp_selection(ctypes.Structure):
+    _fields_ = [("method", ctypes.c_int32), ("candidates", ctypes.c_int32), ("density", ctypes.c_double),
+                ("est_seconds", ctypes.c_double * 4), ("boundary_nodes", ctypes.c_int64)]
+
+
 class apsp_phase_stats(ctypes.Structure):
     _fields_ = [("ms", ctypes.c_double * 4), ("launches", ctypes.c_int64 * 4), ("relax", ctypes.c_double * 4)]
 
@@ -89,6 +94,8 @@ _sig = {
                                           ctypes.POINTER(apsp_config)]),
     "apsp_init_johnson": (ctypes.c_int, [ctypes.POINTER(_H), _I64, _P, _P, _P, ctypes.c_int, ctypes.c_double,
                                          _I64, ctypes.POINTER(apsp_config)]),
+    "apsp_select": (ctypes.c_int, [_I64, _P, _P, _P, ctypes.c_int, _P, _I32, ctypes.POINTER(apsp_config),
+                                   ctypes.POINTER(apsp_selection)]),
     "apsp_solve": (ctypes.c_int, [_H]),
     "apsp_reinit": (ctypes.c_int, [_H]),
     "apsp_fw_rounds": (ctypes.c_int, [_H, _I64, _I64]),
@@ -251,6 +258,30 @@ def apsp_init_johnson(n: int, row_ptr, col_idx, weights, dtype: int | None = Non
     _check(_lib.apsp_init_johnson(ctypes.byref(raw), n, _ptr(row_ptr), _ptr(col_idx), _ptr(w), dtype,
                                   float(delta), int(batch), ctypes.byref(cfg)))
     return Handle(raw, dtype, n, (cfg,))
+
+
+def apsp_select(n: int, row_ptr, col_idx, weights, comp=None, k: int = 0, dtype: int | None = None,
+                cfg: apsp_config | None = None) -> apsp_selection:
+    """The paper's method selection (§IV): density filter + device-calibrated cost models."""
+    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
+    w = np.asarray(weights)
+    if dtype is None:
+        dtype = APSP_F32 if w.dtype.kind == "f" else APSP_I32
+    w = np.ascontiguousarray(w, dtype=np.int32 if dtype == APSP_I32 else np.float32)
+    if row_ptr.shape[0] != n + 1:
+        raise ApspError(APSP_EINVAL, "row_ptr must have n+1 entries")
+    cp = None
+    if comp is not None:
+        cp = np.ascontiguousarray(comp, dtype=np.int32)
+        if cp.shape[0] != n:
+            raise ApspError(APSP_EINVAL, "comp must have n entries")
+    if cfg is None:
+        cfg = apsp_config_default()
+    sel = apsp_selection()
+    _check(_lib.apsp_select(n, _ptr(row_ptr), _ptr(col_idx), _ptr(w), dtype,
+                            _ptr(cp) if cp is not None else None, int(k), ctypes.byref(cfg), ctypes.byref(sel)))
+    return sel
 
 
 def apsp_solve(h: Handle) -> None:

@@ -538,6 +538,93 @@ apsp_status apsp_init_johnson(apsp_handle** out, int64_t n, const int64_t* row_p
   return APSP_OK;
 }
 
+apsp_status apsp_select(int64_t n, const int64_t* row_ptr, const int32_t* col_idx, const void* weights,
+                        apsp_dtype dtype, const int32_t* comp, int32_t k, const apsp_config* cfg_in,
+                        apsp_selection* out) {
+  if (!out) return fail_global(APSP_EINVAL, "apsp_select: out is NULL");
+  memset(out, 0, sizeof(*out));
+  for (double& e : out->est_seconds) e = -1.0;
+  apsp_config cfg;
+  apsp_config_default(&cfg);
+  if (cfg_in) {
+    if (cfg_in->struct_size != 0 && cfg_in->struct_size != (int32_t)sizeof(apsp_config))
+      return fail_global(APSP_EINVAL, "apsp_config.struct_size %d != %d", cfg_in->struct_size,
+                         (int)sizeof(apsp_config));
+    cfg = *cfg_in;
+  }
+  if (n < 1 || n > (int64_t)INT32_MAX || !row_ptr) return fail_global(APSP_EINVAL, "bad n / row_ptr");
+  if (dtype != APSP_I32 && dtype != APSP_F32) return fail_global(APSP_EINVAL, "bad dtype");
+  if (comp && k < 1) return fail_global(APSP_EINVAL, "k < 1");
+  bool has_neg = false;
+  int64_t maxabs = 0;
+  apsp_status st = validate_csr(n, row_ptr, col_idx, weights, dtype, &has_neg, &maxabs);
+  if (st) return st;
+  const double dn = (double)n, m = (double)row_ptr[n];
+  out->density = m / (dn * dn);
+  // §IV-C density filter
+  int cand;
+  if (out->density > 0.01) cand = (1 << APSP_MODE_INCORE) | (1 << APSP_MODE_JOHNSON);
+  else if (out->density < 1e-4) cand = (1 << APSP_MODE_JOHNSON) | (1 << APSP_MODE_BOUNDARY);
+  else cand = 1 << APSP_MODE_JOHNSON;
+  if (!comp) cand &= ~(1 << APSP_MODE_BOUNDARY);  // no partition given (the paper uses METIS)
+  if (!cand) cand = 1 << APSP_MODE_JOHNSON;
+  if (dtype == APSP_F32 && has_neg) cand = 1 << APSP_MODE_INCORE;  // Johnson takes fp32 w >= 0 (R19)
+  int64_t nb_nodes = 0;
+  if (comp) {
+    for (int64_t v = 0; v < n; ++v)
+      if (comp[v] < 0 || comp[v] >= k) return fail_global(APSP_EINVAL, "comp[%lld] out of [0, k)", (long long)v);
+    std::vector<char> isb(n, 0);
+    for (int64_t u = 0; u < n; ++u)
+      for (int64_t e = row_ptr[u]; e < row_ptr[u + 1]; ++e)
+        if (comp[col_idx[e]] != comp[u]) isb[u] = isb[col_idx[e]] = 1;
+    for (int64_t v = 0; v < n; ++v) nb_nodes += isb[v];
+    out->boundary_nodes = nb_nodes;
+  }
+  out->candidates = cand;
+  // cost models (§IV-B), calibrated on this device
+  std::string err;
+  int dev = cfg.device;
+  if (dev < 0 && cudaGetDevice(&dev) != cudaSuccess) return fail_global(APSP_ECUDA, "no CUDA device");
+  size_t free_b = 0, total_b = 0;
+  if (cudaSetDevice(dev) != cudaSuccess || cudaMemGetInfo(&free_b, &total_b) != cudaSuccess)
+    return fail_global(APSP_ECUDA, "no CUDA device (the library has no CPU path)");
+  const double budget = cfg.device_budget_bytes > 0 ? (double)cfg.device_budget_bytes : (double)free_b - (1 << 30);
+  const double W = 4.0, mat = dn * dn * W;
+  const bool ooc = mat > budget;
+  double c_unit = 0, TH = 0;
+  const bool need_fw = (cand >> APSP_MODE_INCORE & 1) || (cand >> APSP_MODE_BOUNDARY & 1);
+  if (need_fw && (st = fw_seconds_per_relax(cfg, std::min<int64_t>(8192, std::max<int64_t>(1024, n)), &c_unit, &err)))
+    return fail_global(st, "apsp_select: FW calibration: %s", err.c_str());
+  if (ooc && (st = hostlink_rate(dev, &TH, &err))) return fail_global(st, "apsp_select: host link: %s", err.c_str());
+  if (cand >> APSP_MODE_INCORE & 1) {
+    double t = c_unit * dn * dn * dn;
+    if (ooc) {
+      const double b = 4096, nd = std::ceil(dn / b);
+      t = std::max(t, nd * W * (3 * b * b + dn * dn) / TH);
+    }
+    out->est_seconds[APSP_MODE_INCORE] = t;
+  }
+  if (cand >> APSP_MODE_JOHNSON & 1) {
+    double t = 0;
+    if ((st = johnson_seconds(cfg, n, row_ptr, col_idx, weights, dtype, has_neg, 5, &t, &err)))
+      return fail_global(st, "apsp_select: Johnson sampling: %s", err.c_str());
+    if (ooc) t = std::max(t, W * dn * dn / TH);
+    out->est_seconds[APSP_MODE_JOHNSON] = t;
+  }
+  if (cand >> APSP_MODE_BOUNDARY & 1) {
+    const double kk = (double)k, B = (double)nb_nodes / kk;
+    const double nop = dn * dn * dn / (kk * kk) + std::pow(kk * B, 3) + dn * kk * B * B + dn * dn * B;
+    out->est_seconds[APSP_MODE_BOUNDARY] = nop * c_unit;
+  }
+  out->method = -1;
+  for (int mth : {APSP_MODE_INCORE, APSP_MODE_JOHNSON, APSP_MODE_BOUNDARY})
+    if ((out->candidates >> mth & 1) && out->est_seconds[mth] >= 0 &&
+        (out->method < 0 || out->est_seconds[mth] < out->est_seconds[out->method]))
+      out->method = mth;
+  if (out->method < 0) out->method = APSP_MODE_JOHNSON;
+  return APSP_OK;
+}
+
 apsp_status apsp_solve(apsp_handle* hh) {
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);

@@ -124,12 +124,18 @@ long long bnd_boundary_nodes(const Handle* h);
 void bnd_free(Handle* h);
 // Johnson's algorithm with batched Near-Far SSSP (apsp_johnson.cu)
 apsp_status jn_setup(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, const int32_t* col, const void* w,
-                     double delta, long long batch);
+                     double delta, long long batch, bool sample = false);
+apsp_status jn_sample_seconds(Handle* h, int k, unsigned long long seed, double* seconds);
 apsp_status jn_reinit(Handle* h);
 apsp_status jn_run(Handle* h);
 apsp_status jn_get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out);
 long long jn_edges(const Handle* h);
 void jn_free(Handle* h);
+// method selection (apsp_select.cu)
+apsp_status fw_seconds_per_relax(const apsp_config& cfg, long long n0, double* out, std::string* err);
+apsp_status hostlink_rate(int device, double* out, std::string* err);
+apsp_status johnson_seconds(const apsp_config& cfg, long long n, const int64_t* row_ptr, const int32_t* col,
+                            const void* w, apsp_dtype dtype, bool has_neg, int k, double* out, std::string* err);
 // common device / stream setup of a handle (apsp_handle.cu)
 apsp_status setup_device(Handle* h, const apsp_config& cfg);
 

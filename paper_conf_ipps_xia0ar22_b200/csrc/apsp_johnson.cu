@@ -109,9 +109,10 @@ __device__ __forceinline__ void append(int* q, int* cnt, int v) {
   q[base + g.thread_rank()] = v;
 }
 
-template <typename T, int G>
-__global__ void __launch_bounds__(kJThreads) mssp_kernel(MsspArgs<T> a) {
-  extern __shared__ unsigned jsm[];
+// NT threads per block, G lanes per frontier vertex (power of two <= 32)
+template <typename T, int NT, int G>
+__global__ void __launch_bounds__(NT) mssp_kernel(MsspArgs<T> a) {
+  extern __shared__ __align__(16) unsigned jsm[];
   __shared__ int s_qn, s_qn2, s_fn, s_fn2;
   __shared__ T s_T, s_min;
   const int tid = threadIdx.x;
@@ -124,13 +125,13 @@ __global__ void __launch_bounds__(kJThreads) mssp_kernel(MsspArgs<T> a) {
   int* F2 = F + n;
   const int lane_g = tid % G;
   const int grp = tid / G;
-  constexpr int NG = kJThreads / G;
+  constexpr int NG = NT / G;
   unsigned long long scanned = 0;
 
   for (long long s = a.src_begin + blockIdx.x; s < a.src_end; s += gridDim.x) {
-    T* row = a.out + (s - a.row_base) * a.ld;
-    for (long long v = tid; v < n; v += kJThreads) row[v] = JV<T>::inf();
-    for (long long x = tid; x < 2 * a.nwords; x += kJThreads) nearb[x] = 0u;
+    T* const row = a.out + (s - a.row_base) * a.ld;
+    for (long long v = tid; v < n; v += NT) row[v] = JV<T>::inf();
+    for (long long x = tid; x < 2 * a.nwords; x += NT) nearb[x] = 0u;
     __syncthreads();
     if (tid == 0) {
       row[s] = T(0);
@@ -157,7 +158,7 @@ __global__ void __launch_bounds__(kJThreads) mssp_kernel(MsspArgs<T> a) {
         // Near queue of that bucket ran empty), so Far entries below it are stale
         const T told = s_T;
         T mn = JV<T>::inf();
-        for (int i = tid; i < fn; i += kJThreads) {
+        for (int i = tid; i < fn; i += NT) {
           const int v = F[i];
           clr(farb, v);
           const T d = JV<T>::load(row + v);
@@ -170,7 +171,7 @@ __global__ void __launch_bounds__(kJThreads) mssp_kernel(MsspArgs<T> a) {
         if ((tid & 31) == 0) JV<T>::amin(&s_min, mn);
         __syncthreads();
         const T thr = JV<T>::plus_delta(s_min, a.delta);
-        for (int i = tid; i < fn; i += kJThreads) {
+        for (int i = tid; i < fn; i += NT) {
           const int v = F[i];
           const T d = JV<T>::load(row + v);
           if (d < told) {
@@ -195,7 +196,7 @@ __global__ void __launch_bounds__(kJThreads) mssp_kernel(MsspArgs<T> a) {
       }
       // expand the Near queue; its entries' flags are cleared first so that a
       // vertex improved during this iteration is queued again
-      for (int i = tid; i < qn; i += kJThreads) clr(nearb, Q[i]);
+      for (int i = tid; i < qn; i += NT) clr(nearb, Q[i]);
       if (tid == 0) s_qn2 = 0;
       __syncthreads();
       const T thr = s_T;
@@ -229,7 +230,7 @@ __global__ void __launch_bounds__(kJThreads) mssp_kernel(MsspArgs<T> a) {
     // Johnson epilogue: undo the reweighting, dist(s,t) = dist'(s,t) - p(s) + p(t)
     if (a.pot) {
       const long long ps = a.pot[s];
-      for (long long v = tid; v < n; v += kJThreads) {
+      for (long long v = tid; v < n; v += NT) {
         const T d = row[v];
         if (d < JV<T>::inf()) row[v] = (T)((long long)d - ps + a.pot[v]);
       }
@@ -274,11 +275,12 @@ struct Jn {
   int* work = nullptr;
   unsigned* gbits = nullptr;
   long long nwords = 0;
-  int grid = 0, G = 1, smem_bits = 0;
+  int grid = 0, G = 1, smem_bits = 0, nt = 256;
   size_t smem = 0;
   long long bat = 0;         // sources per batch (Alg. 2's bat)
   double delta = 0;
   bool ooc = false;
+  bool sample = false;       // apsp_select's estimation handle (no result matrix)
   unsigned long long edges_last = 0;
   cudaStream_t d2h = nullptr;
   cudaEvent_t computed[2] = {nullptr, nullptr}, stored[2] = {nullptr, nullptr};
@@ -286,40 +288,50 @@ struct Jn {
 
 Jn* J_(Handle* h) { return static_cast<Jn*>(h->jn); }
 
-template <typename T, int G>
-cudaError_t launch_g(const MsspArgs<T>& a, int grid, size_t smem, cudaStream_t s) {
-  auto k = mssp_kernel<T, G>;
+template <typename T, int NT, int G>
+cudaError_t launch_v(const MsspArgs<T>& a, int grid, size_t smem, cudaStream_t s) {
+  auto k = mssp_kernel<T, NT, G>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
-  k<<<grid, kJThreads, smem, s>>>(a);
+  k<<<grid, NT, smem, s>>>(a);
   return cudaGetLastError();
 }
 
-template <typename T>
-cudaError_t launch_mssp(const MsspArgs<T>& a, int G, int grid, size_t smem, cudaStream_t s) {
+template <typename T, int NT, int G>
+int occ_v(size_t smem) {
+  auto k = mssp_kernel<T, NT, G>;
+  if (cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess) return 0;
+  int nb = 0;
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k, NT, smem) == cudaSuccess ? nb : 0;
+}
+
+// one (NT, G) instantiation: launch it (grid > 0) or report its occupancy (grid == 0)
+template <typename T, int NT>
+int dispatch_g(const MsspArgs<T>* a, int G, int grid, size_t smem, cudaStream_t s, cudaError_t* err) {
+#define JN_CASE(g)                                                   \
+  case g:                                                            \
+    if (grid == 0) return occ_v<T, NT, g>(smem);                     \
+    *err = launch_v<T, NT, g>(*a, grid, smem, s);                    \
+    return 0;
   switch (G) {
-    case 1: return launch_g<T, 1>(a, grid, smem, s);
-    case 2: return launch_g<T, 2>(a, grid, smem, s);
-    case 4: return launch_g<T, 4>(a, grid, smem, s);
-    case 8: return launch_g<T, 8>(a, grid, smem, s);
-    case 16: return launch_g<T, 16>(a, grid, smem, s);
-    default: return launch_g<T, 32>(a, grid, smem, s);
+    JN_CASE(1) JN_CASE(2) JN_CASE(4) JN_CASE(8) JN_CASE(16) default: JN_CASE(32)
   }
+#undef JN_CASE
 }
 
 template <typename T>
-int occupancy(int G, size_t smem) {
-  int nb = 0;
-  cudaError_t e;
-  switch (G) {
-    case 1: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, mssp_kernel<T, 1>, kJThreads, smem); break;
-    case 2: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, mssp_kernel<T, 2>, kJThreads, smem); break;
-    case 4: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, mssp_kernel<T, 4>, kJThreads, smem); break;
-    case 8: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, mssp_kernel<T, 8>, kJThreads, smem); break;
-    case 16: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, mssp_kernel<T, 16>, kJThreads, smem); break;
-    default: e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, mssp_kernel<T, 32>, kJThreads, smem); break;
-  }
-  return e == cudaSuccess ? nb : 0;
+cudaError_t launch_mssp(const MsspArgs<T>& a, int nt, int G, int grid, size_t smem, cudaStream_t s) {
+  cudaError_t e = cudaSuccess;
+  if (nt == 1024) dispatch_g<T, 1024>(&a, G, grid, smem, s, &e);
+  else dispatch_g<T, 256>(&a, G, grid, smem, s, &e);
+  return e;
+}
+
+template <typename T>
+int occupancy(int nt, int G, size_t smem) {
+  cudaError_t e = cudaSuccess;
+  return nt == 1024 ? dispatch_g<T, 1024>(nullptr, G, 0, smem, nullptr, &e)
+                    : dispatch_g<T, 256>(nullptr, G, 0, smem, nullptr, &e);
 }
 
 template <typename T>
@@ -387,7 +399,7 @@ apsp_status run_t(Handle* h) {
   if (!j->ooc) {
     MsspArgs<T> a = make_args<T>(h, 0, n, static_cast<T*>(j->D), 0);
     h->ev_begin(2);
-    if ((st = h->cuda(launch_mssp<T>(a, j->G, j->grid, j->smem, h->stream), "mssp"))) return st;
+    if ((st = h->cuda(launch_mssp<T>(a, j->nt, j->G, j->grid, j->smem, h->stream), "mssp"))) return st;
     h->ev_end(0);
   } else {
     // Algorithm 2: batches of `bat` sources; batch b+1 runs while batch b is copied back
@@ -398,7 +410,7 @@ apsp_status run_t(Handle* h) {
       if ((st = h->cuda(cudaStreamWaitEvent(h->stream, j->stored[sl], 0), "wait"))) return st;
       MsspArgs<T> a = make_args<T>(h, s0, s1, static_cast<T*>(j->buf[sl]), s0);
       h->ev_begin(2);
-      if ((st = h->cuda(launch_mssp<T>(a, j->G, j->grid, j->smem, h->stream), "mssp"))) return st;
+      if ((st = h->cuda(launch_mssp<T>(a, j->nt, j->G, j->grid, j->smem, h->stream), "mssp"))) return st;
       h->ev_end(0);
       if ((st = h->cuda(cudaEventRecord(j->computed[sl], h->stream), "event"))) return st;
       if ((st = h->cuda(cudaStreamWaitEvent(j->d2h, j->computed[sl], 0), "wait"))) return st;
@@ -423,7 +435,7 @@ apsp_status run_t(Handle* h) {
 }  // namespace
 
 apsp_status jn_setup(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, const int32_t* col, const void* w,
-                     double delta, long long batch) {
+                     double delta, long long batch, bool sample) {
   apsp_status st;
   Jn* j = new Jn();
   h->jn = j;
@@ -455,7 +467,10 @@ apsp_status jn_setup(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, 
   const double avg_deg = n > 0 ? (double)m / n : 0.0;
   j->G = 1;
   while (j->G < 32 && j->G < avg_deg) j->G *= 2;
-  // Delta: default = 4 x the mean |weight| (measured sweep)
+  // Delta: default = mean |weight| x 64 / degree^2, clamped to [mean/4, 4 mean]
+  // (measured optimum: 4 x mean on the degree-4 grid of config 2, mean/4 on the
+  // degree-16 ER graph of config 3; larger degrees favour narrower buckets because
+  // every expansion already exposes many arcs)
   if (delta > 0) {
     j->delta = delta;
   } else {
@@ -465,7 +480,9 @@ apsp_status jn_setup(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, 
     } else {
       for (long long e = 0; e < m; ++e) sum += std::fabs((double)static_cast<const float*>(w)[e]);
     }
-    j->delta = std::max(1.0, 4.0 * (m > 0 ? sum / m : 1.0));
+    const double mean = m > 0 ? sum / m : 1.0;
+    const double d = std::max(1.0, avg_deg);
+    j->delta = std::max(1.0, mean * std::min(4.0, std::max(0.25, 64.0 / (d * d))));
     if (h->has_neg) j->delta *= 2;  // reweighted arcs are longer on average
   }
   if (h->dtype == APSP_I32) j->delta = std::floor(std::min(j->delta, (double)(1 << 29)));
@@ -473,13 +490,21 @@ apsp_status jn_setup(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, 
   // flags: two bitmaps per block, in shared memory when they fit
   j->nwords = (n + 31) / 32;
   const size_t bits_bytes = 2 * (size_t)j->nwords * sizeof(unsigned);
+  const size_t row_bytes = (size_t)n * h->elem;
   j->smem_bits = bits_bytes <= 96 * 1024 ? 1 : 0;
-  if (std::getenv("APSP_TEST_JN_GLOBAL_BITS")) j->smem_bits = 0;  // test hook (tests/test_gpu_johnson.py)
-  j->smem = j->smem_bits ? bits_bytes : 0;
   int sms = 148;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device);
-  int per_sm = h->dtype == APSP_I32 ? occupancy<int>(j->G, j->smem) : occupancy<float>(j->G, j->smem);
+  // threads per block: 256 (8 sources per SM in flight: small frontiers, e.g. road
+  // graphs, need many concurrent sources) unless those 8 x 148 rows overflow ~96 MB
+  // of the 126 MB L2 — relaxations are random atomics into the rows — then 1024
+  // (2 per SM); measured on configs 2 and 3
+  j->nt = (long long)sms * 8 * (long long)row_bytes > (96ll << 20) ? 1024 : 256;
+  if (const char* e = std::getenv("APSP_JN_THREADS")) j->nt = std::atoi(e) == 1024 ? 1024 : 256;
+  if (std::getenv("APSP_TEST_JN_GLOBAL_BITS")) j->smem_bits = 0;  // test hook (tests/test_gpu_johnson.py)
+  j->smem = j->smem_bits ? bits_bytes : 0;
+  int per_sm = h->dtype == APSP_I32 ? occupancy<int>(j->nt, j->G, j->smem) : occupancy<float>(j->nt, j->G, j->smem);
   if (per_sm < 1) return h->fail(APSP_ECUDA, "mssp kernel cannot be resident (smem %zu B)", j->smem);
+  if (const char* e = std::getenv("APSP_JN_CTAS_PER_SM")) per_sm = std::max(1, std::min(per_sm, std::atoi(e)));
   j->grid = (int)std::max<long long>(1, std::min<long long>((long long)sms * per_sm, n));
   // per-block queues (4 x n) and global bitmaps
   const size_t work_bytes = (size_t)j->grid * 4 * std::max<long long>(n, 1) * sizeof(int);
@@ -497,7 +522,13 @@ apsp_status jn_setup(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, 
   h->n_pad = n;
   h->ld = n;
   h->rows_per_rank = n;
-  if (!j->ooc) {
+  if (sample) {
+    // selector cost model (apsp_select): room for one batch of `grid` sources only
+    j->sample = true;
+    j->bat = j->grid;
+    if ((st = h->cuda(cudaMalloc(&j->buf[0], (size_t)j->bat * n * h->elem), "cudaMalloc sample"))) return st;
+    h->device_bytes = graph_bytes + (long long)j->bat * n * (long long)h->elem;
+  } else if (!j->ooc) {
     if ((st = h->cuda(cudaMallocAsync(&j->D, std::max<long long>(mat, 4), h->stream), "cudaMalloc dist"))) return st;
     h->device_bytes = graph_bytes + mat;
   } else {
@@ -519,6 +550,43 @@ apsp_status jn_setup(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, 
     }
   }
   return h->cuda(cudaStreamSynchronize(h->stream), "johnson setup sync");
+}
+
+// The paper's Johnson cost model (§IV-B-2): run k randomly chosen
+// batches, T_comp = (n_b / k) * T. One batch = one wave of `grid` sources.
+apsp_status jn_sample_seconds(Handle* h, int k, unsigned long long seed, double* seconds) {
+  Jn* j = J_(h);
+  apsp_status st;
+  if (!j->sample) return h->fail(APSP_ESTATE, "not a sampling handle");
+  const long long n = h->n;
+  if (j->d_w2 && (st = reweight(h))) return st;
+  const long long nb = (n + j->bat - 1) / j->bat;
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  double total_ms = 0;
+  unsigned long long x = seed * 6364136223846793005ull + 1442695040888963407ull;
+  for (int i = 0; i <= k; ++i) {  // i = 0 is a warm-up batch (not counted)
+    x = x * 6364136223846793005ull + 1442695040888963407ull;
+    const long long b = (long long)((x >> 33) % (unsigned long long)nb);
+    const long long s0 = b * j->bat, s1 = std::min(n, s0 + j->bat);
+    cudaEventRecord(e0, h->stream);
+    cudaError_t e = h->dtype == APSP_I32
+        ? launch_mssp<int>(make_args<int>(h, s0, s1, static_cast<int*>(j->buf[0]), s0), j->nt, j->G, j->grid,
+                           j->smem, h->stream)
+        : launch_mssp<float>(make_args<float>(h, s0, s1, static_cast<float*>(j->buf[0]), s0), j->nt, j->G, j->grid,
+                             j->smem, h->stream);
+    if ((st = h->cuda(e, "mssp sample"))) return st;
+    cudaEventRecord(e1, h->stream);
+    if ((st = h->cuda(cudaEventSynchronize(e1), "sample sync"))) return st;
+    float ms = 0;
+    cudaEventElapsedTime(&ms, e0, e1);
+    if (i > 0) total_ms += ms * (double)j->bat / (double)(s1 - s0);  // a ragged last batch counts as a full one
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  *seconds = (double)nb / k * total_ms * 1e-3;
+  return APSP_OK;
 }
 
 apsp_status jn_reinit(Handle* h) {

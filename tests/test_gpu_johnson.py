@@ -147,6 +147,28 @@ def test_johnson_global_bitmaps(lib, monkeypatch):
     assert np.array_equal(got.astype(np.int64), oracle_i32(g))
 
 
+@pytest.mark.parametrize("env", [{"APSP_JN_THREADS": "256"}, {"APSP_JN_THREADS": "1024"},
+                                 {"APSP_JN_CTAS_PER_SM": "1"}, {"APSP_JN_THREADS": "1024", "APSP_JN_CTAS_PER_SM": "1"}])
+def test_johnson_kernel_variants_same_result(lib, monkeypatch, env):
+    """256/1024 threads per block, grid caps: schedule-only choices, identical distances
+    (int32 with negatives, and fp32)."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    g = gg.grid_2d(30, 37, seed=12)
+    rng = np.random.default_rng(5)
+    p = rng.integers(-50, 50, size=g.n)
+    s, t, w = g.arcs()
+    gn = gg.csr_from_arcs(g.n, s, t, (w.astype(np.int64) + p[s] - p[t]).astype(np.int32))
+    got, _ = solve(lib, gn)
+    assert np.array_equal(got.astype(np.int64), oracle_i32(gn))
+    gf = gg.erdos_renyi(600, 40 * 600, seed=6, dtype="f32")
+    got, _ = solve(lib, gf)
+    want, _ = oracle.fw_f64(gf.row_ptr, gf.col, gf.w)
+    fin = np.isfinite(want)
+    assert np.array_equal(np.isfinite(got), fin)
+    assert np.all(np.abs(got[fin] - want[fin]) <= 1e-5 * np.abs(want[fin]))
+
+
 def test_johnson_reinit_and_second_solve(lib):
     g = gg.erdos_renyi(500, 3000, seed=13)
     with lib.apsp_init_johnson(g.n, g.row_ptr, g.col, g.w) as h:

@@ -36,6 +36,8 @@ def main():
     ap.add_argument("--cpu-sources", type=int, default=512)
     ap.add_argument("--fw", action="store_true", help="also time the blocked FW on the same graph")
     ap.add_argument("--ooc", action="store_true", help="force Algorithm 2's batches to pinned host memory")
+    ap.add_argument("--env", nargs="+", default=[""],
+                    help="kernel variants to sweep, e.g. 'APSP_JN_THREADS=512,APSP_JN_SMEM_DIST=0'")
     a = ap.parse_args()
     import torch
     torch.cuda.set_device(0)
@@ -67,18 +69,27 @@ def main():
             return e0.elapsed_time(e1) / a.steps, wall * 1e3, st, info
 
         out = {"workload": wl, "n": n, "m": g.m, "runs": []}
-        for d in a.deltas:
+        variants = [(d, e) for e in a.env for d in a.deltas]
+        for d, env in variants:
+            for k in ("APSP_JN_THREADS", "APSP_JN_SMEM_DIST", "APSP_JN_CTAS_PER_SM"):
+                os.environ.pop(k, None)
+            for kv in filter(None, env.split(",")):
+                k, v = kv.split("=")
+                os.environ[k] = v
             ms, wall_ms, st, info = timed(
                 lambda c: apsp.apsp_init_johnson(n, g.row_ptr, g.col, g.w, delta=d, cfg=c), apsp.apsp_solve)
             # the library synchronises inside apsp_solve, so wall time is the honest one
             t = max(ms, wall_ms)
-            out["runs"].append({"delta": d, "ms": t, "kernel_ms": st.ms[2], "reweight_ms": st.ms[1],
+            out["runs"].append({"delta": d, "env": env, "ms": t, "kernel_ms": st.ms[2], "reweight_ms": st.ms[1],
                                 "d2h_ms": st.ms[3], "edges_scanned": info.edges_scanned,
                                 "edges_per_source": info.edges_scanned / n, "reexpansion": info.edges_scanned / n / g.m,
                                 "arcs_per_s": info.edges_scanned / (t * 1e-3),
                                 "fw_equivalent_n3_per_s": float(n) ** 3 / (t * 1e-3),
                                 "result_bytes": n * n * 4, "host_bytes": info.host_bytes})
+        for k in ("APSP_JN_THREADS", "APSP_JN_SMEM_DIST", "APSP_JN_CTAS_PER_SM"):
+            os.environ.pop(k, None)
         best = min(out["runs"], key=lambda r: r["ms"])
+        out["best"] = {"delta": best["delta"], "env": best["env"]}
         out["best_ms"] = best["ms"]
         if a.fw:
             ms_f, wall_f, _, _ = timed(lambda c: apsp.apsp_init_from_csr(n, g.row_ptr, g.col, g.w, cfg=c),
