@@ -54,6 +54,7 @@ def parse():
                     help="min-plus kernel for A/B: 0 cp.async + mbarrier pipeline (default), "
                          "1 cp.async + CTA barrier per chunk, 2 TMA persistent")
     ap.add_argument("--no-packed16", action="store_true", help="skip the packed-int16 alternative measurement")
+    ap.add_argument("--no-johnson", action="store_true", help="skip the Johnson (Near-Far) alternative measurement")
     ap.add_argument("--packed16", action="store_true",
                     help="packed int16 arithmetic (VIADDMNMX.S16x2) when exact, int32 otherwise")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle sample time")
@@ -376,6 +377,31 @@ def run_ours(args):
                 "note": "apsp_init_from_csr(host CSR, pinned) + apsp_fw_blocked + apsp_get_dist(pinned host) + "
                         "destroy, host wall clock (synchronous C-ABI calls)"}
 
+    def johnson_timed():
+        cfg = apsp.apsp_config_default(device=0, timing=1)
+        cfg.stream = stream.cuda_stream
+        h = apsp.apsp_init_johnson(n, g.row_ptr, g.col, g.w, cfg=cfg)
+        for _ in range(args.warmup):
+            apsp.apsp_reinit(h)
+            apsp.apsp_solve(h)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        t0 = time.perf_counter()
+        e0.record(stream)
+        for _ in range(args.steps):
+            apsp.apsp_reinit(h)
+            apsp.apsp_solve(h)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ms = max(e0.elapsed_time(e1), (time.perf_counter() - t0) * 1e3) / args.steps
+        edges = apsp.apsp_get_info(h).edges_scanned
+        apsp.apsp_destroy(h)
+        return {"ms_per_apsp": ms, "speedup_vs_fw_step": main_run["ms_per_step"] / ms,
+                "arcs_relaxed_per_apsp": edges, "arcs_per_s": edges / (ms * 1e-3),
+                "fw_equivalent_relax_per_s": float(n) ** 3 / (ms * 1e-3),
+                "note": "apsp_init_johnson + apsp_solve (one block per source, Near-Far queues; PAPER.md:66, "
+                        ":72, Alg. 2), same graph, result resident in HBM; bit-exact in tests/test_gpu_johnson.py"}
+
     main_run = device_timed(args.packed16)
     e2e = None if args.no_e2e else end_to_end(args.packed16)
 
@@ -390,6 +416,13 @@ def run_ours(args):
                          "instruction) with the exactness check of DESIGN.md R16; the result is the exact int32 "
                          "APSP (bit-exact in tests/test_gpu_packed16.py); falls back to int32 when distances "
                          "reach 8192 (dtype then reads i32)"}
+
+    # Johnson's algorithm on the same graph (batched Near-Far SSSP): the
+    # paper's method for sparse graphs; a different algorithm (O(n m) work, not n^3), so it is
+    # reported as time per APSP beside the FW step, not as the metric
+    alt_jn = None
+    if world == 1 and not args.no_johnson and not args.force_ooc and not (is_f and bool((g.w < 0).any())):
+        alt_jn = johnson_timed()
 
     # ---------------- CPU oracle baseline (rank 0, N=1 only) ------------------
     cpu = None
@@ -416,6 +449,7 @@ def run_ours(args):
             "roofline": main_run["roofline"],
             "cpu_baseline": cpu,
             "packed16": alt16,
+            "johnson": alt_jn,
             "relax_per_step_rank0": main_run["relax_per_step_rank0"],
             "phase_ms_per_step_rank0": main_run["phase_ms_per_step_rank0"],
         }
