@@ -1,0 +1,48 @@
+#!/usr/bin/env python
+"""A/B of the in-core FW schedules on a seeded ER graph: the persistent dataflow kernel vs the
+launch-per-phase schedule (apsp_config.reserved[4] = 1), int32 or fp32.
+
+    python tools/fw_ab.py --n 32768 --deg 256 --dtype f32 --runs 2
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import graphgen as gg  # noqa: E402
+import paper_conf_ipps_xia0ar22_b200 as apsp  # noqa: E402
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--n", type=int, default=32768)
+    ap.add_argument("--deg", type=int, default=256)
+    ap.add_argument("--dtype", default="f32", choices=["i32", "f32"])
+    ap.add_argument("--runs", type=int, default=2)
+    a = ap.parse_args()
+    g = gg.erdos_renyi(a.n, a.deg * a.n, seed=4, dtype=a.dtype)
+    out = {"n": a.n, "deg": a.deg, "dtype": a.dtype}
+    for name, legacy in (("dataflow", 0), ("per_phase", 1)):
+        cfg = apsp.apsp_config_default(device=0, timing=1)
+        cfg.reserved[4] = legacy
+        with apsp.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=cfg) as h:
+            best = 1e30
+            for r in range(a.runs + 1):
+                apsp.apsp_reinit(h)
+                t0 = time.perf_counter()
+                apsp.apsp_fw_blocked(h)
+                t = time.perf_counter() - t0
+                if r:
+                    best = min(best, t)
+            st = apsp.apsp_get_phase_stats(h)
+        out[name] = {"s": best, "relax_per_s": float(a.n) ** 3 / best,
+                     "phase3_rate": st.relax[2] / (st.ms[2] * 1e-3) if st.ms[2] else None}
+    print(json.dumps(out), flush=True)
+
+
+if __name__ == "__main__":
+    main()

@@ -22,12 +22,16 @@ def main():
     ap.add_argument("--legacy", action="store_true")
     ap.add_argument("--packed16", action="store_true")
     ap.add_argument("--df-delay", type=int, default=0)
+    ap.add_argument("--ooc-block", type=int, default=0, help="> 0: out-of-core path with this band height")
     a = ap.parse_args()
     g = gg.baseline_config(a.workload)
     cfg = apsp.apsp_config_default(device=0)
     cfg.reserved[4] = 1 if a.legacy else 0
     cfg.reserved[5] = a.df_delay
     cfg.packed16 = 1 if a.packed16 else 0
+    if a.ooc_block:
+        cfg.force_out_of_core = 1
+        cfg.ooc_block = a.ooc_block
     with apsp.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=cfg) as h:
         for _ in range(a.runs):
             apsp.apsp_reinit(h)
