@@ -294,7 +294,7 @@ def run_ours(args):
         dpx = pk.get("dpx", {})
         if is_f:
             peak = dpx.get("f32_relax_per_s")
-            peak_src = "measured fp32 FADD+FMNMX min-plus rate (MEASURED_DPX.json)"
+            peak_src = "measured fp32 min-plus rate, FADD2 (broadcast) + FMNMX3 form (MEASURED_DPX.json)"
         elif arith == "s16x2":
             peak = dpx.get("s16x2_relax_per_s")
             peak_src = "measured VIADDMNMX.S16x2 rate, 2 relaxations/instruction (MEASURED_DPX.json)"

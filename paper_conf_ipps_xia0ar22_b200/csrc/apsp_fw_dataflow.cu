@@ -196,23 +196,47 @@ __device__ __forceinline__ Task g3l_task(int nb, int k, long long x) {
   t.i = skip3((int)x, k, k + 1, -1); t.j = k + 1;
   return t;
 }
+// The bulk of a round's phase 3 (an R x W block of tiles) in column bands of
+// BAND tiles: all rows of band 0, then band 1, ... Consecutive tasks share the
+// band's row-panel tiles (BAND x 64 KB, L2-resident) and one column-panel tile
+// per row, so the round's panels never need to fit in L2 at once (at nb = 1024
+// the two panels are 128 MB > the 126 MB L2; row-major order re-read the whole
+// row panel from HBM for every tile row).
+constexpr int BAND = 64;
+__device__ __forceinline__ void banded(long long x, int R, int W, int& r, int& c) {
+  const int nfull = W / BAND;
+  const long long per = (long long)R * BAND;
+  if (x < nfull * per) {
+    const int b = (int)(x / per);
+    const long long y = x - b * per;
+    r = (int)(y / BAND);
+    c = b * BAND + (int)(y % BAND);
+  } else {
+    const long long y = x - nfull * per;
+    const int wl = W - nfull * BAND;
+    r = (int)(y / wl);
+    c = nfull * BAND + (int)(y % wl);
+  }
+}
+
 // G3R(k), k <= nb-2: tiles with i,j not in {k,k+1}; row k+2, column k+2 first
 __device__ __forceinline__ Task g3r_task(int nb, int k, long long x) {
   Task t;
   t.type = T_P3; t.k = k;
+  int r, c;
   if (k + 2 < nb) {
     if (x < nb - 2) { t.i = k + 2; t.j = skip3((int)x, k, k + 1, -1); return t; }
     x -= nb - 2;
     if (x < nb - 3) { t.i = skip3((int)x, k, k + 1, k + 2); t.j = k + 2; return t; }
     x -= nb - 3;
-    const int w = nb - 3;
-    t.i = skip3((int)(x / w), k, k + 1, k + 2);
-    t.j = skip3((int)(x % w), k, k + 1, k + 2);
+    banded(x, nb - 3, nb - 3, r, c);
+    t.i = skip3(r, k, k + 1, k + 2);
+    t.j = skip3(c, k, k + 1, k + 2);
     return t;
   }
-  const int w = nb - 2;
-  t.i = skip3((int)(x / w), k, k + 1, -1);
-  t.j = skip3((int)(x % w), k, k + 1, -1);
+  banded(x, nb - 2, nb - 2, r, c);
+  t.i = skip3(r, k, k + 1, -1);
+  t.j = skip3(c, k, k + 1, -1);
   return t;
 }
 
@@ -244,7 +268,9 @@ __device__ Task decode(long long g, int nb, long long delay) {
     if (g >= last) {                           // tail: G3R(nb-1), all (i,j) != nb-1
       g -= last;
       t.type = T_P3; t.k = nb - 1;
-      t.i = (int)(g / n1); t.j = (int)(g % n1);
+      int r, c;
+      banded(g, (int)n1, (int)n1, r, c);
+      t.i = r; t.j = c;
       return t;
     }
     k = nb - 1;
@@ -582,18 +608,54 @@ __device__ __noinline__ void group_minplus(const GDesc<T>* d, T* stage0, unsigne
     mb_wait(full0 + 8 * s, (G / STAGES) & 1);
     const T* as = stage0 + s * STAGE_ELEMS;  // As[kk][r]
     const T* bs = as + BK * ALD;             // Bs[kk][c]
+    if constexpr (sizeof(T) == 4 && T(0.5) != T(0)) {
+      // fp32: two depth steps per accumulator update, FADD2 (a scalar broadcast
+      // against a column pair) + FMNMX3 = 1 instruction per relaxation instead of
+      // FADD + FMNMX. Every candidate a + b is still one RN add and min is exact,
+      // so the result is bit-identical to the one-step update.
 #pragma unroll
-    for (int kk = 0; kk < BK; ++kk) {
-      const V4 a0 = *reinterpret_cast<const V4*>(as + kk * ALD + ty * 4);
-      const V4 a1 = *reinterpret_cast<const V4*>(as + kk * ALD + 64 + ty * 4);
-      const V4 b0 = *reinterpret_cast<const V4*>(bs + kk * BLD + tx * 4);
-      const V4 b1 = *reinterpret_cast<const V4*>(bs + kk * BLD + 64 + tx * 4);
-      const T av[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
-      const T bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+      for (int kk = 0; kk < BK; kk += 2) {
+        const V4 b00 = *reinterpret_cast<const V4*>(bs + kk * BLD + tx * 4);
+        const V4 b01 = *reinterpret_cast<const V4*>(bs + kk * BLD + 64 + tx * 4);
+        const V4 b10 = *reinterpret_cast<const V4*>(bs + (kk + 1) * BLD + tx * 4);
+        const V4 b11 = *reinterpret_cast<const V4*>(bs + (kk + 1) * BLD + 64 + tx * 4);
+        const float2 p0[4] = {make_float2(b00.x, b00.y), make_float2(b00.z, b00.w), make_float2(b01.x, b01.y),
+                              make_float2(b01.z, b01.w)};
+        const float2 p1[4] = {make_float2(b10.x, b10.y), make_float2(b10.z, b10.w), make_float2(b11.x, b11.y),
+                              make_float2(b11.z, b11.w)};
 #pragma unroll
-      for (int i = 0; i < 8; ++i)
+        for (int h = 0; h < 2; ++h) {
+          const V4 a0 = *reinterpret_cast<const V4*>(as + kk * ALD + 64 * h + ty * 4);
+          const V4 a1 = *reinterpret_cast<const V4*>(as + (kk + 1) * ALD + 64 * h + ty * 4);
+          const float x0[4] = {a0.x, a0.y, a0.z, a0.w};
+          const float x1[4] = {a1.x, a1.y, a1.z, a1.w};
 #pragma unroll
-        for (int j = 0; j < 8; ++j) acc[i][j] = DV<T>::relax(av[i], bv[j], acc[i][j]);
+          for (int i = 0; i < 4; ++i)
+#pragma unroll
+            for (int jp = 0; jp < 4; ++jp) {
+              const float2 s0 = __fadd2_rn(make_float2(x0[i], x0[i]), p0[jp]);
+              const float2 s1 = __fadd2_rn(make_float2(x1[i], x1[i]), p1[jp]);
+              float& c0 = acc[4 * h + i][2 * jp];
+              float& c1 = acc[4 * h + i][2 * jp + 1];
+              c0 = fminf(fminf(c0, s0.x), s1.x);
+              c1 = fminf(fminf(c1, s0.y), s1.y);
+            }
+        }
+      }
+    } else {
+#pragma unroll
+      for (int kk = 0; kk < BK; ++kk) {
+        const V4 a0 = *reinterpret_cast<const V4*>(as + kk * ALD + ty * 4);
+        const V4 a1 = *reinterpret_cast<const V4*>(as + kk * ALD + 64 + ty * 4);
+        const V4 b0 = *reinterpret_cast<const V4*>(bs + kk * BLD + tx * 4);
+        const V4 b1 = *reinterpret_cast<const V4*>(bs + kk * BLD + 64 + tx * 4);
+        const T av[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+        const T bv[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+#pragma unroll
+          for (int j = 0; j < 8; ++j) acc[i][j] = DV<T>::relax(av[i], bv[j], acc[i][j]);
+      }
     }
     __syncwarp();
     if (lane == 0) mb_arrive(empty0 + 8 * s);

@@ -132,7 +132,9 @@ apsp_status setup_device(Handle* h, const apsp_config& cfg) {
     }
   }
   g_minplus_variant = cfg.reserved[3];  // test hook: min-plus kernel variant (apsp_kernels.cuh)
-  h->dataflow = cfg.reserved[4] == 0;   // reserved[4] = 1: launch-per-phase schedule instead of the dataflow kernel
+  // reserved[4]: 0 = auto (the persistent dataflow kernel for int32; the launch-per-phase
+  // schedule for fp32, measured faster there: DESIGN.md §5), 1 = launch-per-phase, 2 = dataflow
+  h->dataflow = cfg.reserved[4] == 2 || (cfg.reserved[4] == 0 && h->dtype == APSP_I32);
   h->df_delay = cfg.reserved[5];
   if (cfg.stream) {
     h->stream = static_cast<cudaStream_t>(cfg.stream);

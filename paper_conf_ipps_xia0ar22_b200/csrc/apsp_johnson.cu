@@ -88,7 +88,6 @@ struct MsspArgs {
   unsigned* gbits;      // per block: 2 bitmaps of nwords (when not in shared memory)
   long long nwords;     // ceil(n / 32)
   int smem_bits;        // 1: bitmaps in dynamic shared memory
-  int qcap;             // queue entries held in shared memory (per queue)
   T delta;
   const long long* pot; // Johnson potentials (negative weights) or nullptr
   unsigned long long* edges;  // arcs scanned (statistics)
@@ -101,45 +100,29 @@ __device__ __forceinline__ bool tas(unsigned* bits, int v) {
 }
 __device__ __forceinline__ void clr(unsigned* bits, int v) { atomicAnd(bits + (v >> 5), ~(1u << (v & 31))); }
 
-// A work queue: its first `cap` entries live in shared memory, the rest spill to a
-// global slice (n entries per queue per block), so the common short frontiers never
-// leave the SM while a frontier of any size still fits.
-struct JQ {
-  int* sm;
-  int* gl;
-  __device__ __forceinline__ int get(int i, int cap) const { return i < cap ? sm[i] : gl[i - cap]; }
-  __device__ __forceinline__ void put(int i, int cap, int v) const {
-    if (i < cap) sm[i] = v;
-    else gl[i - cap] = v;
-  }
-};
-
 // warp-aggregated append of v to q (counter in shared memory)
-__device__ __forceinline__ void append(const JQ& q, int cap, int* cnt, int v) {
+__device__ __forceinline__ void append(int* q, int* cnt, int v) {
   cg::coalesced_group g = cg::coalesced_threads();
   int base = 0;
   if (g.thread_rank() == 0) base = atomicAdd(cnt, (int)g.size());
   base = g.shfl(base, 0);
-  q.put(base + (int)g.thread_rank(), cap, v);
+  q[base + g.thread_rank()] = v;
 }
 
-// NT threads per block, G lanes per frontier vertex (power of two <= 32).
-// Shared memory: [near bitmap | far bitmap] (if smem_bits) then 4 x qcap queue heads.
-// Queue counters are double-buffered by iteration parity, so one Near-Far iteration
-// costs two block barriers (clear flags | expand).
+// NT threads per block, G lanes per frontier vertex (power of two <= 32)
 template <typename T, int NT, int G>
 __global__ void __launch_bounds__(NT) mssp_kernel(MsspArgs<T> a) {
   extern __shared__ __align__(16) unsigned jsm[];
-  __shared__ int s_qc[2], s_fc[2];
+  __shared__ int s_qn, s_qn2, s_fn, s_fn2;
   __shared__ T s_T, s_min;
   const int tid = threadIdx.x;
   const long long n = a.n;
   unsigned* nearb = a.smem_bits ? jsm : a.gbits + (size_t)blockIdx.x * 2 * a.nwords;
   unsigned* farb = nearb + a.nwords;
-  int* qsm = reinterpret_cast<int*>(jsm) + (a.smem_bits ? 2 * a.nwords : 0);
-  const int cap = a.qcap;
-  int* qgl = a.work + (size_t)blockIdx.x * 4 * n;
-  JQ Q{qsm, qgl}, Q2{qsm + cap, qgl + n}, F{qsm + 2 * cap, qgl + 2 * n}, F2{qsm + 3 * cap, qgl + 3 * n};
+  int* Q = a.work + (size_t)blockIdx.x * 4 * n;
+  int* Q2 = Q + n;
+  int* F = Q2 + n;
+  int* F2 = F + n;
   const int lane_g = tid % G;
   const int grp = tid / G;
   constexpr int NG = NT / G;
@@ -152,26 +135,31 @@ __global__ void __launch_bounds__(NT) mssp_kernel(MsspArgs<T> a) {
     __syncthreads();
     if (tid == 0) {
       row[s] = T(0);
-      Q.put(0, cap, (int)s);
-      s_qc[0] = 1;
-      s_fc[0] = 0;
+      Q[0] = (int)s;
+      s_qn = 1;
+      s_fn = 0;
       s_T = a.delta;
     }
     __syncthreads();
-    int qp = 0, fp = 0;  // parity of the live Near / Far counters
     for (;;) {
-      const int qn = s_qc[qp];
+      int qn = s_qn;
       if (qn == 0) {
         // Near queue empty: advance the threshold past the smallest Far distance
         // and split the Far queue ("swap Near Queue and Far Queue ... (i+1)Delta")
-        const int fn = s_fc[fp];
+        const int fn = s_fn;
         if (fn == 0) break;
+        if (tid == 0) {
+          s_min = JV<T>::inf();
+          s_qn2 = 0;
+          s_fn2 = 0;
+        }
+        __syncthreads();
         // every vertex below the old threshold told is settled (weights >= 0 and the
         // Near queue of that bucket ran empty), so Far entries below it are stale
         const T told = s_T;
         T mn = JV<T>::inf();
         for (int i = tid; i < fn; i += NT) {
-          const int v = F.get(i, cap);
+          const int v = F[i];
           clr(farb, v);
           const T d = JV<T>::load(row + v);
           if (d >= told) mn = d < mn ? d : mn;
@@ -180,46 +168,40 @@ __global__ void __launch_bounds__(NT) mssp_kernel(MsspArgs<T> a) {
           const T x = __shfl_xor_sync(0xffffffffu, mn, o);
           mn = x < mn ? x : mn;
         }
-        if (tid == 0) {
-          s_min = JV<T>::inf();
-          s_qc[qp ^ 1] = 0;
-          s_fc[fp ^ 1] = 0;
-        }
-        __syncthreads();
         if ((tid & 31) == 0) JV<T>::amin(&s_min, mn);
         __syncthreads();
         const T thr = JV<T>::plus_delta(s_min, a.delta);
         for (int i = tid; i < fn; i += NT) {
-          const int v = F.get(i, cap);
+          const int v = F[i];
           const T d = JV<T>::load(row + v);
           if (d < told) {
             // stale: improved below the old threshold later and expanded then
           } else if (d < thr) {
-            if (tas(nearb, v)) append(Q, cap, &s_qc[qp ^ 1], v);
+            if (tas(nearb, v)) append(Q, &s_qn2, v);
           } else if (tas(farb, v)) {
-            append(F2, cap, &s_fc[fp ^ 1], v);
+            append(F2, &s_fn2, v);
           }
         }
-        if (tid == 0) s_T = thr;
         __syncthreads();
-        // Q was empty: the split wrote the new Near entries into Q itself
-        qp ^= 1;
-        fp ^= 1;
-        const JQ t = F;
+        if (tid == 0) {
+          s_T = thr;
+          s_qn = s_qn2;
+          s_fn = s_fn2;
+        }
+        int* t = F;
         F = F2;
         F2 = t;
+        __syncthreads();
         continue;
       }
       // expand the Near queue; its entries' flags are cleared first so that a
       // vertex improved during this iteration is queued again
-      for (int i = tid; i < qn; i += NT) clr(nearb, Q.get(i, cap));
-      if (tid == 0) s_qc[qp ^ 1] = 0;
+      for (int i = tid; i < qn; i += NT) clr(nearb, Q[i]);
+      if (tid == 0) s_qn2 = 0;
       __syncthreads();
       const T thr = s_T;
-      int* const qcnt = &s_qc[qp ^ 1];
-      int* const fcnt = &s_fc[fp];
       for (int i = grp; i < qn; i += NG) {
-        const int u = Q.get(i, cap);
+        const int u = Q[i];
         const T du = JV<T>::load(row + u);
         const long long e0 = a.rp[u], e1 = a.rp[u + 1];
         scanned += (unsigned long long)((e1 - e0 + G - 1 - lane_g) / G);
@@ -230,19 +212,20 @@ __global__ void __launch_bounds__(NT) mssp_kernel(MsspArgs<T> a) {
             const T old = JV<T>::amin(row + v, nd);
             if (nd < old) {
               if (nd < thr) {
-                if (tas(nearb, v)) append(Q2, cap, qcnt, v);
+                if (tas(nearb, v)) append(Q2, &s_qn2, v);
               } else if (tas(farb, v)) {
-                append(F, cap, fcnt, v);
+                append(F, &s_fn, v);
               }
             }
           }
         }
       }
       __syncthreads();
-      qp ^= 1;
-      const JQ t = Q;
+      if (tid == 0) s_qn = s_qn2;
+      int* t = Q;
       Q = Q2;
       Q2 = t;
+      __syncthreads();
     }
     // Johnson epilogue: undo the reweighting, dist(s,t) = dist'(s,t) - p(s) + p(t)
     if (a.pot) {
@@ -292,7 +275,7 @@ struct Jn {
   int* work = nullptr;
   unsigned* gbits = nullptr;
   long long nwords = 0;
-  int grid = 0, G = 1, smem_bits = 0, nt = 256, qcap = 0;
+  int grid = 0, G = 1, smem_bits = 0, nt = 256;
   size_t smem = 0;
   long long bat = 0;         // sources per batch (Alg. 2's bat)
   double delta = 0;
@@ -368,7 +351,6 @@ MsspArgs<T> make_args(Handle* h, long long s0, long long s1, T* out, long long r
   a.gbits = j->gbits;
   a.nwords = j->nwords;
   a.smem_bits = j->smem_bits;
-  a.qcap = j->qcap;
   a.delta = (T)j->delta;
   a.pot = j->d_pot;
   a.edges = j->d_edges;
@@ -519,15 +501,7 @@ apsp_status jn_setup(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, 
   j->nt = (long long)sms * 8 * (long long)row_bytes > (96ll << 20) ? 1024 : 256;
   if (const char* e = std::getenv("APSP_JN_THREADS")) j->nt = std::atoi(e) == 1024 ? 1024 : 256;
   if (std::getenv("APSP_TEST_JN_GLOBAL_BITS")) j->smem_bits = 0;  // test hook (tests/test_gpu_johnson.py)
-  // queue heads in shared memory: what is left of ~208 KB per SM after the bitmaps
-  // of the 8 (256-thread) or 2 (1024-thread) resident blocks, <= n entries per queue
-  {
-    const long long per_block = (208ll << 10) / (j->nt == 1024 ? 2 : 8);
-    const long long left = per_block - (j->smem_bits ? (long long)bits_bytes : 0) - 256;
-    j->qcap = (int)std::max<long long>(0, std::min<long long>(n, left / (4 * (long long)sizeof(int))));
-    if (const char* e = std::getenv("APSP_JN_QCAP")) j->qcap = (int)std::min<long long>(n, std::atoll(e));
-  }
-  j->smem = (j->smem_bits ? bits_bytes : 0) + 4 * (size_t)j->qcap * sizeof(int);
+  j->smem = j->smem_bits ? bits_bytes : 0;
   int per_sm = h->dtype == APSP_I32 ? occupancy<int>(j->nt, j->G, j->smem) : occupancy<float>(j->nt, j->G, j->smem);
   if (per_sm < 1) return h->fail(APSP_ECUDA, "mssp kernel cannot be resident (smem %zu B)", j->smem);
   if (const char* e = std::getenv("APSP_JN_CTAS_PER_SM")) per_sm = std::max(1, std::min(per_sm, std::atoi(e)));

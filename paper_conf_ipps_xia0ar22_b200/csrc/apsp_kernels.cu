@@ -80,6 +80,49 @@ constexpr int minplus_smem_bytes() {
   return MP_STAGES * MP_STAGE_ELEMS * (int)sizeof(T);
 }
 
+// Two depth steps kk, kk+1 of the 8x8 register block: acc[i][j] = min(acc[i][j],
+// a[i][u] + b_u[j]) for u = 0, 1 (b_u = row kk+u of the B stage at column tx*4 and
+// 64+tx*4). int32: one VIADDMNMX per relaxation. fp32: FADD2 (scalar a broadcast
+// against a column pair) + FMNMX3 folding both steps = 1 instruction per relaxation
+// instead of FADD + FMNMX; each candidate is still one RN add and min is exact, so
+// the result is bit-identical to the one-step update.
+template <typename T>
+__device__ __forceinline__ void relax_two_steps(T (&acc)[8][8], const T (&a)[8][2], const T* brow0, const T* brow1,
+                                                int tx) {
+  using V4 = typename Vec4<T>::type;
+  if constexpr (sizeof(T) == 4 && T(0.5) != T(0)) {
+    const V4 b00 = *reinterpret_cast<const V4*>(brow0 + tx * 4);
+    const V4 b01 = *reinterpret_cast<const V4*>(brow0 + 64 + tx * 4);
+    const V4 b10 = *reinterpret_cast<const V4*>(brow1 + tx * 4);
+    const V4 b11 = *reinterpret_cast<const V4*>(brow1 + 64 + tx * 4);
+    const float2 p0[4] = {make_float2(b00.x, b00.y), make_float2(b00.z, b00.w), make_float2(b01.x, b01.y),
+                          make_float2(b01.z, b01.w)};
+    const float2 p1[4] = {make_float2(b10.x, b10.y), make_float2(b10.z, b10.w), make_float2(b11.x, b11.y),
+                          make_float2(b11.z, b11.w)};
+#pragma unroll
+    for (int i = 0; i < 8; ++i)
+#pragma unroll
+      for (int jp = 0; jp < 4; ++jp) {
+        const float2 s0 = __fadd2_rn(make_float2(a[i][0], a[i][0]), p0[jp]);
+        const float2 s1 = __fadd2_rn(make_float2(a[i][1], a[i][1]), p1[jp]);
+        acc[i][2 * jp] = fminf(fminf(acc[i][2 * jp], s0.x), s1.x);
+        acc[i][2 * jp + 1] = fminf(fminf(acc[i][2 * jp + 1], s0.y), s1.y);
+      }
+  } else {
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      const T* brow = u ? brow1 : brow0;
+      const V4 b0 = *reinterpret_cast<const V4*>(brow + tx * 4);
+      const V4 b1 = *reinterpret_cast<const V4*>(brow + 64 + tx * 4);
+      const T b[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+#pragma unroll
+        for (int j = 0; j < 8; ++j) acc[i][j] = Val<T>::relax(a[i][u], b[j], acc[i][j]);
+    }
+  }
+}
+
 template <typename T>
 __global__ void __launch_bounds__(MP_NT, 2) minplus_kernel(const __grid_constant__ MinPlusArgs<T> args) {
   using V4 = typename Vec4<T>::type;
@@ -169,17 +212,7 @@ __global__ void __launch_bounds__(MP_NT, 2) minplus_kernel(const __grid_constant
         const T* ap = as + r * MP_ALD + k2 * 2;
         a[i][0] = ap[0]; a[i][1] = ap[1];
       }
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const T* brow = bs + (k2 * 2 + u) * MP_BLD;
-        V4 b0 = *reinterpret_cast<const V4*>(brow + tx * 4);
-        V4 b1 = *reinterpret_cast<const V4*>(brow + 64 + tx * 4);
-        const T b[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
-#pragma unroll
-        for (int i = 0; i < 8; ++i)
-#pragma unroll
-          for (int j = 0; j < 8; ++j) acc[i][j] = Val<T>::relax(a[i][u], b[j], acc[i][j]);
-      }
+      relax_two_steps<T>(acc, a, bs + (k2 * 2) * MP_BLD, bs + (k2 * 2 + 1) * MP_BLD, tx);
     }
   }
   cp_async_wait<0>();
@@ -367,17 +400,7 @@ __device__ __forceinline__ void minplus_mbar_tile(const MinPlusDesc<T>& d, int t
         const T* ap = as + r * MP_ALD + k2 * 2;
         a[i][0] = ap[0]; a[i][1] = ap[1];
       }
-#pragma unroll
-      for (int u = 0; u < 2; ++u) {
-        const T* brow = bs + (k2 * 2 + u) * MP_BLD;
-        V4 b0 = *reinterpret_cast<const V4*>(brow + tx * 4);
-        V4 b1 = *reinterpret_cast<const V4*>(brow + 64 + tx * 4);
-        const T b[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
-#pragma unroll
-        for (int i = 0; i < 8; ++i)
-#pragma unroll
-          for (int j = 0; j < 8; ++j) acc[i][j] = Val<T>::relax(a[i][u], b[j], acc[i][j]);
-      }
+      relax_two_steps<T>(acc, a, bs + (k2 * 2) * MP_BLD, bs + (k2 * 2 + 1) * MP_BLD, tx);
     }
     __syncwarp();
     if (lane == 0) mb_arrive(empty0 + 8 * s);

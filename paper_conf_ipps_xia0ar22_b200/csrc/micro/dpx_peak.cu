@@ -6,6 +6,8 @@
 //   s16x2   : __viaddmin_s16x2     -> SASS VIADDMNMX.S16x2  (2 relax / instr)
 //   f32     : fminf(c, a + b)      -> SASS FADD + FMNMX     (1 relax / 2 instr)
 //   f32x2   : __fadd2_rn + 3-input min -> FADD2 + FMNMX3    (2 relax / 2 instr)
+//   f32b, f32x2b: the same without per-step int->float conversions (the b
+//             operand advances by FADD), f32x2b in the kernels' broadcast form
 // plus the host link (pinned H2D, D2H, both at once), used by the
 // out-of-core roofline. Prints one JSON object on stdout.
 #include <cuda_runtime.h>
@@ -101,6 +103,62 @@ __global__ void k_f32x2(const int* __restrict__ in, int* __restrict__ out, int i
   out[blockIdx.x * blockDim.x + threadIdx.x] = (int)s;
 }
 
+// f32 without per-step int->float conversions: the b operand is a register
+// advanced by one FADD per step (1 extra instruction per CH2 relaxations)
+constexpr int CH2 = 32;
+__global__ void k_f32b(const int* __restrict__ in, int* __restrict__ out, int iters) {
+  float x[CH2], acc[CH2];
+#pragma unroll
+  for (int j = 0; j < CH2; ++j) { x[j] = (float)in[(threadIdx.x + j) & 255]; acc[j] = 1e30f; }
+  float y = (float)in[threadIdx.x & 255];
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      y = __fadd_rn(y, 1.0f);
+#pragma unroll
+      for (int j = 0; j < CH2; ++j) acc[j] = fminf(acc[j], __fadd_rn(x[j], y));
+    }
+  }
+  float s = 0;
+#pragma unroll
+  for (int j = 0; j < CH2; ++j) s += acc[j];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = (int)s;
+}
+
+// FADD2 (scalar broadcast x pair) + FMNMX3, as in the kernels: per step and chain
+// pair, 2 FADD2 + 2 FMNMX3 = 4 relaxations
+__global__ void k_f32x2b(const int* __restrict__ in, int* __restrict__ out, int iters) {
+  float x0[CH2 / 2], x1[CH2 / 2];
+  float acc[CH2];
+#pragma unroll
+  for (int j = 0; j < CH2 / 2; ++j) {
+    x0[j] = (float)in[(threadIdx.x + j) & 255];
+    x1[j] = (float)in[(threadIdx.x + j + 7) & 255];
+  }
+#pragma unroll
+  for (int j = 0; j < CH2; ++j) acc[j] = 1e30f;
+  float2 y0 = make_float2((float)in[threadIdx.x & 255], 3.0f), y1 = make_float2(5.0f, 7.0f);
+  const float2 one = make_float2(1.0f, 1.0f);
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      y0 = __fadd2_rn(y0, one);
+      y1 = __fadd2_rn(y1, one);
+#pragma unroll
+      for (int j = 0; j < CH2 / 2; ++j) {
+        const float2 s0 = __fadd2_rn(make_float2(x0[j], x0[j]), y0);
+        const float2 s1 = __fadd2_rn(make_float2(x1[j], x1[j]), y1);
+        acc[2 * j] = fminf(fminf(acc[2 * j], s0.x), s1.x);
+        acc[2 * j + 1] = fminf(fminf(acc[2 * j + 1], s0.y), s1.y);
+      }
+    }
+  }
+  float s = 0;
+#pragma unroll
+  for (int j = 0; j < CH2; ++j) s += acc[j];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = (int)s;
+}
+
 typedef void (*kfn)(const int*, int*, int);
 
 static double run(kfn f, int blocks, int threads, int iters, const int* in, int* out, double relax_per_op) {
@@ -151,7 +209,8 @@ int main(int argc, char** argv) {
   printf("{\"gpu\": \"%s\", \"sms\": %d, \"cc\": \"%d.%d\"", p.name, p.multiProcessorCount, p.major, p.minor);
   int cfgs[][2] = {{4, 256}, {8, 256}, {16, 128}, {4, 512}};
   struct V { const char* name; kfn f; double rpo; } vs[] = {
-    {"s32", k_s32, 1.0}, {"s16x2", k_s16x2, 2.0}, {"f32", k_f32, 1.0}, {"f32x2", k_f32x2, 2.0}};
+    {"s32", k_s32, 1.0}, {"s16x2", k_s16x2, 2.0}, {"f32", k_f32, 1.0}, {"f32x2", k_f32x2, 2.0},
+    {"f32b", k_f32b, 1.0}, {"f32x2b", k_f32x2b, 1.0}};
   CK(cudaMalloc(&out, (size_t)p.multiProcessorCount * 16 * 512 * sizeof(int)));
   for (auto& v : vs) {
     double best = 0;

@@ -26,7 +26,7 @@ def want_i32(g):
 
 def run(lib, g, delay=0, legacy=False, timing=0):
     c = lib.apsp_config_default(device=0, timing=timing)
-    c.reserved[4] = 1 if legacy else 0
+    c.reserved[4] = 1 if legacy else 2  # 2 = force the dataflow kernel (fp32 default is per-phase)
     c.reserved[5] = delay
     return lib.solve(g, cfg=c)
 
@@ -95,3 +95,15 @@ def test_dataflow_phase_stats(lib):
         n_pad = lib.apsp_get_info(h).n_pad
     assert sum(st.relax[:3]) == float(n_pad) ** 3
     assert st.launches[2] == 1 and st.launches[0] == 0 and st.ms[2] > 0
+
+
+def test_dataflow_banded_phase3_order_partial_band(lib):
+    """nb = 70 tile rows: the round's bulk phase 3 runs in 64-column bands plus a partial
+    band; dataflow == launch-per-phase bit for bit, sampled rows == the oracle's Dijkstra."""
+    g = gg.erdos_renyi(128 * 70 - 3, (128 * 70 - 3) * 4, seed=17)
+    a = run(lib, g)
+    b = run(lib, g, legacy=True)
+    assert np.array_equal(a, b)
+    srcs = np.array([0, 4500, g.n - 1])
+    want = oracle.dijkstra_rows_i64(g.row_ptr, g.col, g.w, srcs)
+    assert np.array_equal(a[srcs].astype(np.int64), np.where(want == oracle.INF_I64, INF32, want))

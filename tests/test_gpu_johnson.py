@@ -148,12 +148,10 @@ def test_johnson_global_bitmaps(lib, monkeypatch):
 
 
 @pytest.mark.parametrize("env", [{"APSP_JN_THREADS": "256"}, {"APSP_JN_THREADS": "1024"},
-                                 {"APSP_JN_CTAS_PER_SM": "1"}, {"APSP_JN_THREADS": "1024", "APSP_JN_CTAS_PER_SM": "1"},
-                                 {"APSP_JN_QCAP": "0"}, {"APSP_JN_QCAP": "5"}, {"APSP_JN_QCAP": "64"}])
+                                 {"APSP_JN_CTAS_PER_SM": "1"}, {"APSP_JN_THREADS": "1024", "APSP_JN_CTAS_PER_SM": "1"}])
 def test_johnson_kernel_variants_same_result(lib, monkeypatch, env):
-    """256/1024 threads per block, grid caps, queue heads of 0/5/64 entries in shared memory
-    (the rest spills to global): schedule-only choices, identical distances (int32 with
-    negatives, and fp32)."""
+    """256/1024 threads per block, grid caps: schedule-only choices, identical distances
+    (int32 with negatives, and fp32)."""
     for k, v in env.items():
         monkeypatch.setenv(k, v)
     g = gg.grid_2d(30, 37, seed=12)

@@ -23,10 +23,13 @@ def main():
     ap.add_argument("--deg", type=int, default=256)
     ap.add_argument("--dtype", default="f32", choices=["i32", "f32"])
     ap.add_argument("--runs", type=int, default=2)
+    ap.add_argument("--modes", nargs="+", default=["dataflow", "per_phase"])
     a = ap.parse_args()
     g = gg.erdos_renyi(a.n, a.deg * a.n, seed=4, dtype=a.dtype)
     out = {"n": a.n, "deg": a.deg, "dtype": a.dtype}
-    for name, legacy in (("dataflow", 0), ("per_phase", 1)):
+    for name, legacy in (("dataflow", 2), ("per_phase", 1)):
+        if name not in a.modes:
+            continue
         cfg = apsp.apsp_config_default(device=0, timing=1)
         cfg.reserved[4] = legacy
         with apsp.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=cfg) as h:
