@@ -168,9 +168,12 @@ apsp_status apsp_init_boundary(apsp_handle** out, int64_t n, const int64_t* row_
  * free memory), otherwise in pinned host memory (cfg->force_out_of_core = 1
  * forces this). Negative int32 weights are reweighted (Johnson: Bellman–Ford
  * potentials); a negative cycle makes apsp_solve return
- * APSP_ENEGCYCLE. fp32 weights must be >= 0 (else APSP_EINVAL). One GPU per
- * handle (world_size 1). Run with apsp_solve; apsp_get_dist as usual;
- * apsp_info.edges_scanned reports the arcs the last run relaxed.
+ * APSP_ENEGCYCLE. fp32 weights must be >= 0 (else APSP_EINVAL). With
+ * cfg->world_size = P > 1 (one handle per GPU / rank, cfg->rank set) rank r
+ * computes the rows of sources [r*ceil(n/P), (r+1)*ceil(n/P)) (apsp_local_rows):
+ * the SSSP instances are independent, so no communicator is used and
+ * nccl_unique_id may be NULL. Run with apsp_solve; apsp_get_dist as usual (own
+ * rows only); apsp_info.edges_scanned reports the arcs the last run relaxed.
  */
 apsp_status apsp_init_johnson(apsp_handle** out, int64_t n, const int64_t* row_ptr,
                               const int32_t* col_idx, const void* weights, apsp_dtype dtype,

@@ -511,7 +511,8 @@ apsp_status apsp_init_johnson(apsp_handle** out, int64_t n, const int64_t* row_p
   if (n < 1 || n > (int64_t)INT32_MAX) return fail_global(APSP_EINVAL, "bad n");
   if (!row_ptr) return fail_global(APSP_EINVAL, "row_ptr is NULL");
   if (dtype != APSP_I32 && dtype != APSP_F32) return fail_global(APSP_EINVAL, "bad dtype");
-  if (cfg.world_size != 1) return fail_global(APSP_EINVAL, "Johnson's algorithm runs on one GPU per handle");
+  if (cfg.world_size < 1 || cfg.rank < 0 || cfg.rank >= cfg.world_size)
+    return fail_global(APSP_EINVAL, "bad world_size/rank");
   if (!(delta >= 0) || !std::isfinite(delta)) return fail_global(APSP_EINVAL, "delta must be finite and >= 0");
   bool has_neg = false;
   int64_t maxabs = 0;
@@ -527,6 +528,8 @@ apsp_status apsp_init_johnson(apsp_handle** out, int64_t n, const int64_t* row_p
   h->arith = dtype == APSP_F32 ? APSP_ARITH_F32 : APSP_ARITH_I32;
   h->elem = 4;
   h->mode = APSP_MODE_JOHNSON;
+  h->world = cfg.world_size;  // sources are split by rank; no communicator is needed
+  h->rank = cfg.rank;
   apsp_status st = setup_device(h, cfg);
   if (!st) st = jn_setup(h, cfg, row_ptr, col_idx, weights, delta, batch);
   if (st != APSP_OK) {
@@ -715,6 +718,13 @@ apsp_status apsp_get_dist(apsp_handle* hh, int64_t row_begin, int64_t row_count,
 apsp_status apsp_local_rows(const apsp_handle* hh, int64_t* row_begin, int64_t* row_count) {
   if (!hh || !row_begin || !row_count) return fail_global(APSP_EINVAL, "NULL argument");
   const Handle* h = reinterpret_cast<const Handle*>(hh);
+  if (h->mode == APSP_MODE_JOHNSON) {
+    long long r0, rc;
+    jn_local_rows(h, &r0, &rc);
+    *row_begin = r0;
+    *row_count = rc;
+    return APSP_OK;
+  }
   if (h->virt || h->world == 1) {
     *row_begin = 0;
     *row_count = h->n;

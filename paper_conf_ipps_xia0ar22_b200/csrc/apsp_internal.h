@@ -130,6 +130,7 @@ apsp_status jn_reinit(Handle* h);
 apsp_status jn_run(Handle* h);
 apsp_status jn_get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out);
 long long jn_edges(const Handle* h);
+void jn_local_rows(const Handle* h, long long* r0, long long* rc);
 void jn_free(Handle* h);
 // method selection (apsp_select.cu)
 apsp_status fw_seconds_per_relax(const apsp_config& cfg, long long n0, double* out, std::string* err);

@@ -280,6 +280,7 @@ struct Jn {
   long long bat = 0;         // sources per batch (Alg. 2's bat)
   double delta = 0;
   bool ooc = false;
+  long long r0 = 0, rc = 0;  // this rank's sources = result rows [r0, r0 + rc)
   bool sample = false;       // apsp_select's estimation handle (no result matrix)
   unsigned long long edges_last = 0;
   cudaStream_t d2h = nullptr;
@@ -397,16 +398,16 @@ apsp_status run_t(Handle* h) {
   if (j->d_w2 && (st = reweight(h))) return st;
   if ((st = h->cuda(cudaMemsetAsync(j->d_edges, 0, sizeof(unsigned long long), h->stream), "memset"))) return st;
   if (!j->ooc) {
-    MsspArgs<T> a = make_args<T>(h, 0, n, static_cast<T*>(j->D), 0);
+    MsspArgs<T> a = make_args<T>(h, j->r0, j->r0 + j->rc, static_cast<T*>(j->D), j->r0);
     h->ev_begin(2);
     if ((st = h->cuda(launch_mssp<T>(a, j->nt, j->G, j->grid, j->smem, h->stream), "mssp"))) return st;
     h->ev_end(0);
   } else {
     // Algorithm 2: batches of `bat` sources; batch b+1 runs while batch b is copied back
-    const long long nb = (n + j->bat - 1) / j->bat;
+    const long long nb = (j->rc + j->bat - 1) / j->bat;
     for (long long b = 0; b < nb; ++b) {
       const int sl = (int)(b & 1);
-      const long long s0 = b * j->bat, s1 = std::min(n, s0 + j->bat);
+      const long long s0 = j->r0 + b * j->bat, s1 = std::min(j->r0 + j->rc, s0 + j->bat);
       if ((st = h->cuda(cudaStreamWaitEvent(h->stream, j->stored[sl], 0), "wait"))) return st;
       MsspArgs<T> a = make_args<T>(h, s0, s1, static_cast<T*>(j->buf[sl]), s0);
       h->ev_begin(2);
@@ -415,7 +416,7 @@ apsp_status run_t(Handle* h) {
       if ((st = h->cuda(cudaEventRecord(j->computed[sl], h->stream), "event"))) return st;
       if ((st = h->cuda(cudaStreamWaitEvent(j->d2h, j->computed[sl], 0), "wait"))) return st;
       h->ev_begin(3, j->d2h);
-      if ((st = h->cuda(cudaMemcpyAsync(static_cast<char*>(j->h_D) + (size_t)s0 * n * sizeof(T), j->buf[sl],
+      if ((st = h->cuda(cudaMemcpyAsync(static_cast<char*>(j->h_D) + (size_t)(s0 - j->r0) * n * sizeof(T), j->buf[sl],
                                         (size_t)(s1 - s0) * n * sizeof(T), cudaMemcpyDeviceToHost, j->d2h),
                         "D2H batch")))
         return st;
@@ -517,7 +518,14 @@ apsp_status jn_setup(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, 
   if ((st = h->cuda(cudaMemGetInfo(&free_b, &total_b), "cudaMemGetInfo"))) return st;
   const long long budget = cfg.device_budget_bytes > 0 ? cfg.device_budget_bytes - graph_bytes
                                                        : (long long)free_b - (1ll << 30);
-  const long long mat = n * n * (long long)h->elem;
+  // sources of this rank (world_size > 1): a contiguous block of result rows; the
+  // SSSP instances are independent, so ranks need no communication at all
+  {
+    const long long per = (n + h->world - 1) / h->world;
+    j->r0 = std::min<long long>(n, (long long)h->rank * per);
+    j->rc = std::min<long long>(n, j->r0 + per) - j->r0;
+  }
+  const long long mat = j->rc * n * (long long)h->elem;
   j->ooc = cfg.force_out_of_core || mat > budget;
   h->n_pad = n;
   h->ld = n;
@@ -535,7 +543,7 @@ apsp_status jn_setup(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, 
     // Alg. 2: bat sources per batch; two batch buffers (compute / copy back)
     const long long row = n * (long long)h->elem;
     long long bat = batch > 0 ? batch : std::max<long long>(1, std::min<long long>(budget / 2, 4ll << 30) / row);
-    bat = std::min(bat, n);
+    bat = std::max<long long>(1, std::min(bat, j->rc));
     j->bat = bat;
     for (int i = 0; i < 2; ++i)
       if ((st = h->cuda(cudaMalloc(&j->buf[i], bat * row), "cudaMalloc batch"))) return st;
@@ -600,6 +608,10 @@ apsp_status jn_run(Handle* h) { return h->dtype == APSP_I32 ? run_t<int>(h) : ru
 apsp_status jn_get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out) {
   Jn* j = J_(h);
   if (!h->fw_done) return h->fail(APSP_ESTATE, "Johnson handle: apsp_solve first");
+  if (r0 < j->r0 || r0 + cnt > j->r0 + j->rc)
+    return h->fail(APSP_EINVAL, "get_dist: rows [%lld, %lld) are not this rank's [%lld, %lld)", r0, r0 + cnt, j->r0,
+                   j->r0 + j->rc);
+  r0 -= j->r0;
   const size_t es = h->elem;
   if (j->ooc) {
     for (long long r = 0; r < cnt; ++r)
@@ -613,6 +625,12 @@ apsp_status jn_get_rows(Handle* h, long long r0, long long cnt, void* out, long 
                     "get rows")))
     return st;
   return h->cuda(cudaStreamSynchronize(h->stream), "get rows sync");
+}
+
+void jn_local_rows(const Handle* h, long long* r0, long long* rc) {
+  const Jn* j = static_cast<const Jn*>(h->jn);
+  *r0 = j ? j->r0 : 0;
+  *rc = j ? j->rc : h->n;
 }
 
 long long jn_edges(const Handle* h) { return h->jn ? (long long)static_cast<const Jn*>(h->jn)->edges_last : 0; }

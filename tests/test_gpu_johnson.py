@@ -206,3 +206,26 @@ def test_johnson_config3_er65536_every_row_certified(lib):
         want = oracle.dijkstra_rows_i64(g.row_ptr, g.col, g.w, srcs)
         for i, s in enumerate(srcs):
             assert np.array_equal(lib.apsp_get_dist(h, int(s), 1)[0].astype(np.int64), want[i])
+
+
+@pytest.mark.parametrize("world,ooc", [(2, 0), (3, 0), (3, 1)])
+def test_johnson_sharded_by_source(lib, world, ooc):
+    """world_size > 1: rank r computes the rows of its block of sources (no communicator:
+    the SSSP instances are independent); the ranks' rows together equal the oracle.
+    All ranks run here as separate handles on one GPU."""
+    g = gg.erdos_renyi(700, 700 * 5, seed=31)
+    want = oracle_i32(g)
+    got = np.full((g.n, g.n), -1, dtype=np.int64)
+    covered = 0
+    for r in range(world):
+        cfg = lib.apsp_config_default(device=0, world_size=world, rank=r, force_out_of_core=ooc)
+        with lib.apsp_init_johnson(g.n, g.row_ptr, g.col, g.w, cfg=cfg, batch=50 if ooc else 0) as h:
+            rb, rc = lib.apsp_local_rows(h)
+            assert rb == r * (-(-g.n // world)) and rc > 0
+            lib.apsp_solve(h)
+            got[rb:rb + rc] = lib.apsp_get_dist(h, rb, rc)
+            covered += rc
+            with pytest.raises(lib.ApspError):
+                lib.apsp_get_dist(h, (rb + rc) % g.n, 1)
+    assert covered == g.n
+    assert np.array_equal(got, want)
