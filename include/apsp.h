@@ -236,12 +236,32 @@ apsp_status apsp_fw_blocked(apsp_handle* h);
 apsp_status apsp_reinit(apsp_handle* h);
 
 /*
- * apsp_fw_rounds — run rounds [k_begin, k_end) only (in-core mode). After
- * rounds 0..K-1, dist[i][j] is the shortest path whose intermediates all lie
- * in {0 .. K*b - 1}, i.e. the plain FW state after K*b outer iterations
- * (PAPER.md:60). Used for per-round parity. Rounds must be run in order.
+ * apsp_fw_rounds — run rounds [k_begin, k_end) only. After rounds 0..K-1,
+ * dist[i][j] is the shortest path whose intermediates all lie in
+ * {0 .. K*b - 1}, i.e. the plain FW state after K*b outer iterations
+ * (PAPER.md:60). Used for per-round parity and checkpointing. Rounds must be
+ * run in order; out of core they run in whole super-rounds (k_begin and k_end
+ * multiples of ooc_block/tile, or k_end = the last round). apsp_fw_blocked
+ * afterwards runs the remaining rounds.
  */
 apsp_status apsp_fw_rounds(apsp_handle* h, int64_t k_begin, int64_t k_end);
+
+/*
+ * apsp_checkpoint / apsp_restore — save and resume a blocked-FW run (in core or
+ * out of core; not packed16, virtual ranks, boundary or Johnson handles). After
+ * rounds 0 .. k-1 the matrix is the FW state "intermediates in {0 .. k*b-1}"
+ * (PAPER.md:60); out of core it is the pinned host bands plus the HBM-resident
+ * bands after a super-round (Algorithm 1). apsp_checkpoint
+ * writes this rank's padded rows and the next round to `path` (a 128-byte
+ * header + rows x n_pad elements); apsp_restore loads such a file into a handle
+ * created by apsp_init_from_csr for the same graph, dtype and placement (n,
+ * n_pad, world/rank, out-of-core band height), after which apsp_fw_rounds or
+ * apsp_fw_blocked continue with the remaining rounds. Synchronous.
+ * Errors: APSP_EINVAL (cannot open / short file / mismatching checkpoint),
+ * APSP_ESTATE (unsupported handle), APSP_ECUDA, APSP_ENOMEM.
+ */
+apsp_status apsp_checkpoint(apsp_handle* h, const char* path);
+apsp_status apsp_restore(apsp_handle* h, const char* path);
 
 /*
  * apsp_get_dist — copy rows [row_begin, row_begin+row_count), columns [0, n),

@@ -96,6 +96,8 @@ _sig = {
                                          _I64, ctypes.POINTER(apsp_config)]),
     "apsp_select": (ctypes.c_int, [_I64, _P, _P, _P, ctypes.c_int, _P, _I32, ctypes.POINTER(apsp_config),
                                    ctypes.POINTER(apsp_selection)]),
+    "apsp_checkpoint": (ctypes.c_int, [_H, ctypes.c_char_p]),
+    "apsp_restore": (ctypes.c_int, [_H, ctypes.c_char_p]),
     "apsp_solve": (ctypes.c_int, [_H]),
     "apsp_reinit": (ctypes.c_int, [_H]),
     "apsp_fw_rounds": (ctypes.c_int, [_H, _I64, _I64]),
@@ -282,6 +284,16 @@ def apsp_select(n: int, row_ptr, col_idx, weights, comp=None, k: int = 0, dtype:
     _check(_lib.apsp_select(n, _ptr(row_ptr), _ptr(col_idx), _ptr(w), dtype,
                             _ptr(cp) if cp is not None else None, int(k), ctypes.byref(cfg), ctypes.byref(sel)))
     return sel
+
+
+def apsp_checkpoint(h: Handle, path: str) -> None:
+    """Save the blocked-FW state (this rank's rows + next round) to path."""
+    _check(_lib.apsp_checkpoint(h.raw, os.fsencode(path)), h.raw)
+
+
+def apsp_restore(h: Handle, path: str) -> None:
+    """Load a checkpoint into a handle made for the same graph / placement."""
+    _check(_lib.apsp_restore(h.raw, os.fsencode(path)), h.raw)
 
 
 def apsp_solve(h: Handle) -> None:

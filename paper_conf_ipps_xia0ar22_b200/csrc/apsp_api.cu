@@ -41,6 +41,8 @@ static apsp_status fail_global(apsp_status st, const char* fmt, ...) {
 
 namespace apsp {
 
+apsp_status global_fail(apsp_status st, const char* msg) { return fail_global(st, "%s", msg); }
+
 apsp_status Handle::fail(apsp_status st, const char* fmt, ...) {
   char buf[512];
   va_list ap;
@@ -653,13 +655,24 @@ apsp_status apsp_fw_rounds(apsp_handle* hh, int64_t k_begin, int64_t k_end) {
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
-  if (h->mode != APSP_MODE_INCORE) return h->fail(APSP_ESTATE, "apsp_fw_rounds: in-core mode only");
+  if (h->mode != APSP_MODE_INCORE && h->mode != APSP_MODE_OUT_OF_CORE)
+    return h->fail(APSP_ESTATE, "apsp_fw_rounds: blocked-FW handles only");
   if (h->mode16) return h->fail(APSP_ESTATE, "apsp_fw_rounds: not available with packed16");
   const long long nb = h->n_pad / h->b;
   if (k_begin != h->next_round || k_end < k_begin || k_end > nb)
     return h->fail(APSP_ESTATE, "rounds must run in order: next is %lld of %lld", h->next_round, nb);
   apsp_status st;
   if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
+  if (h->mode == APSP_MODE_OUT_OF_CORE) {
+    // out of core the unit is a super-round of B/b rounds (Algorithm 1)
+    const long long kb = h->ooc_B / h->b;
+    if (k_begin % kb || (k_end % kb && k_end != nb))
+      return h->fail(APSP_EINVAL, "out of core, rounds run in super-rounds of %lld", kb);
+    memset(&h->stats, 0, sizeof(h->stats));
+    if ((st = run_out_of_core_range(h, k_begin / kb, (k_end + kb - 1) / kb))) return st;
+    h->next_round = k_end;
+    return finish_fw(h, k_end == nb);
+  }
   if ((st = run_incore_rounds(h, k_begin, k_end))) return st;
   h->next_round = k_end;
   return finish_fw(h, k_end == nb);
@@ -675,18 +688,22 @@ apsp_status apsp_fw_blocked(apsp_handle* hh) {
   apsp_status st;
   if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
   memset(&h->stats, 0, sizeof(h->stats));
+  const long long nb = h->n_pad / h->b;
+  // the remaining rounds: all of them, or those after apsp_fw_rounds / apsp_restore
   if (h->mode == APSP_MODE_OUT_OF_CORE) {
-    if ((st = run_out_of_core(h))) return st;
+    const long long kb = h->ooc_B / h->b;
+    if (h->next_round % kb) return h->fail(APSP_ESTATE, "out of core, rounds run in super-rounds of %lld", kb);
+    if ((st = run_out_of_core_range(h, h->next_round / kb, nb / kb))) return st;
+    h->next_round = nb;
     return finish_fw(h, true);
   }
-  const long long nb = h->n_pad / h->b;
-  if (h->next_round != 0) return h->fail(APSP_ESTATE, "apsp_fw_rounds already started");
   if (h->mode16) {
+    if (h->next_round != 0) return h->fail(APSP_ESTATE, "packed16: no partial runs");
     if ((st = run_fw16(h))) return st;
     h->next_round = nb;
     return finish_fw(h, true);
   }
-  if ((st = run_incore_rounds(h, 0, nb))) return st;
+  if ((st = run_incore_rounds(h, h->next_round, nb))) return st;
   h->next_round = nb;
   return finish_fw(h, true);
 }

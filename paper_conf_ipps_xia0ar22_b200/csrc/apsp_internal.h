@@ -110,6 +110,9 @@ bool nccl_unique_id(void* out128);
 apsp_status ooc_setup(Handle* h, const apsp_config& cfg, long long budget, const int64_t* row_ptr,
                       const int32_t* col, const void* w);
 apsp_status run_out_of_core(Handle* h);
+apsp_status run_out_of_core_range(Handle* h, long long K0, long long K1);
+long long ooc_bands(const Handle* h);
+apsp_status ooc_band_copy(Handle* h, long long I, void* buf, bool to_handle);
 apsp_status ooc_get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out);
 void ooc_free(Handle* h);
 apsp_status ooc_reinit(Handle* h);
@@ -137,6 +140,8 @@ apsp_status fw_seconds_per_relax(const apsp_config& cfg, long long n0, double* o
 apsp_status hostlink_rate(int device, double* out, std::string* err);
 apsp_status johnson_seconds(const apsp_config& cfg, long long n, const int64_t* row_ptr, const int32_t* col,
                             const void* w, apsp_dtype dtype, bool has_neg, int k, double* out, std::string* err);
+// checkpoint / resume helpers
+apsp_status global_fail(apsp_status st, const char* msg);
 // common device / stream setup of a handle (apsp_handle.cu)
 apsp_status setup_device(Handle* h, const apsp_config& cfg);
 
