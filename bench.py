@@ -318,7 +318,8 @@ def run_ours(args):
                         traffic = tj["dram_bytes_per_relax"] * p3_relax
             except Exception:
                 pass
-        kname = ("fw_dataflow_kernel: all rounds and phases 1-3 in one persistent launch (%s)" % arith if dataflow
+        kname = ("%s: all rounds and phases 1-3 in one persistent launch (%s)"
+                 % ("fw_dataflow16_kernel" if arith == "s16x2" else "fw_dataflow_kernel", arith) if dataflow
                  else "phase-3 min-plus (%s)" % arith)
         roofline = {"bound": "alu", "kernel": kname, "achieved": achieved / 1e12,
                     "peak": peak / 1e12, "unit": "Trelax/s", "frac": achieved / peak, "traffic": traffic,

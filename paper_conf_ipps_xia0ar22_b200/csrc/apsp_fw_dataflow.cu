@@ -54,6 +54,7 @@
 // task usually starts without waiting; the SIG thread publishes a finished
 // task (fence.release, then the flags) right after the task's last barrier.
 #include "apsp_kernels.cuh"
+#include "apsp_df_common.cuh"
 
 #include <cuda_runtime.h>
 #include <climits>
@@ -93,54 +94,8 @@ template <> struct DV<float> {
   static __device__ __forceinline__ float vmin(float a, float b) { return fminf(a, b); }
 };
 
-__device__ __forceinline__ unsigned saddr(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void cp16(void* smem, const void* gmem) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(saddr(smem)), "l"(gmem));
-}
-__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;\n" ::); }
-__device__ __forceinline__ void cp_wait_all() { asm volatile("cp.async.wait_group 0;\n" ::); }
-__device__ __forceinline__ void mb_init(unsigned bar, unsigned count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count));
-}
-__device__ __forceinline__ void mb_arrive(unsigned bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
-}
-__device__ __forceinline__ void mb_wait(unsigned bar, unsigned parity) {
-  asm volatile(
-      "{\n"
-      ".reg .pred p;\n"
-      "DFW_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-      "@!p bra DFW_%=;\n"
-      "}\n" ::"r"(bar),
-      "r"(parity)
-      : "memory");
-}
-__device__ __forceinline__ void mb_expect_tx(unsigned bar, unsigned bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void bulk_g2s(unsigned dst, const void* src, unsigned bytes, unsigned bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-               "l"(src), "r"(bytes), "r"(bar)
-               : "memory");
-}
-__device__ __forceinline__ void mb_cp_arrive_inc(unsigned bar) {  // counts +1 then -1: no net arrival
-  asm volatile("cp.async.mbarrier.arrive.shared::cta.b64 [%0];" ::"r"(bar) : "memory");
-}
 // named barrier of one 256-thread group (id 0 is __syncthreads)
 __device__ __forceinline__ void gbar(int g) { asm volatile("bar.sync %0, %1;" ::"r"(g + 1), "r"(GNT) : "memory"); }
-
-__device__ __forceinline__ int ld_relaxed(const int* p) {
-  int v;
-  asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void st_relaxed(int* p, int v) {
-  asm volatile("st.relaxed.gpu.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-__device__ __forceinline__ void red_relaxed_add(int* p, int v) {
-  asm volatile("red.relaxed.gpu.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
 
 template <typename T>
 struct DFArgs {
@@ -162,133 +117,6 @@ struct DFArgs {
   unsigned long long* prof;  // optional [CTAs x GROUPS x 8] cycle counters (thread 0 of each group)
 };
 
-enum { T_P1 = 0, T_P2R = 1, T_P2C = 2, T_P3 = 3 };
-struct Task {
-  int type, k, i, j;
-};
-
-// i-th value of [0, nb) without the excluded values s0 < s1 < s2 (-1 = none)
-__device__ __forceinline__ int skip3(int x, int s0, int s1, int s2) {
-  if (s0 >= 0 && x >= s0) ++x;
-  if (s1 >= 0 && x >= s1) ++x;
-  if (s2 >= 0 && x >= s2) ++x;
-  return x;
-}
-
-__device__ __forceinline__ Task p2_task(int nb, int k, long long x) {
-  Task t;
-  t.k = k;
-  if (x < nb - 1) {
-    t.type = T_P2R; t.i = k; t.j = skip3((int)x, k, -1, -1);
-  } else {
-    t.type = T_P2C; t.i = skip3((int)(x - (nb - 1)), k, -1, -1); t.j = k;
-  }
-  return t;
-}
-// G3L(k): (k+1,k+1), row k+1 (j not in {k,k+1}), column k+1 (i not in {k,k+1})
-__device__ __forceinline__ Task g3l_task(int nb, int k, long long x) {
-  Task t;
-  t.type = T_P3; t.k = k;
-  if (x == 0) { t.i = k + 1; t.j = k + 1; return t; }
-  x -= 1;
-  if (x < nb - 2) { t.i = k + 1; t.j = skip3((int)x, k, k + 1, -1); return t; }
-  x -= nb - 2;
-  t.i = skip3((int)x, k, k + 1, -1); t.j = k + 1;
-  return t;
-}
-// The bulk of a round's phase 3 (an R x W block of tiles) in column bands of
-// BAND tiles: all rows of band 0, then band 1, ... Consecutive tasks share the
-// band's row-panel tiles (BAND x 64 KB, L2-resident) and one column-panel tile
-// per row, so the round's panels never need to fit in L2 at once (at nb = 1024
-// the two panels are 128 MB > the 126 MB L2; row-major order re-read the whole
-// row panel from HBM for every tile row).
-constexpr int BAND = 64;
-__device__ __forceinline__ void banded(long long x, int R, int W, int& r, int& c) {
-  const int nfull = W / BAND;
-  const long long per = (long long)R * BAND;
-  if (x < nfull * per) {
-    const int b = (int)(x / per);
-    const long long y = x - b * per;
-    r = (int)(y / BAND);
-    c = b * BAND + (int)(y % BAND);
-  } else {
-    const long long y = x - nfull * per;
-    const int wl = W - nfull * BAND;
-    r = (int)(y / wl);
-    c = nfull * BAND + (int)(y % wl);
-  }
-}
-
-// G3R(k), k <= nb-2: tiles with i,j not in {k,k+1}; row k+2, column k+2 first
-__device__ __forceinline__ Task g3r_task(int nb, int k, long long x) {
-  Task t;
-  t.type = T_P3; t.k = k;
-  int r, c;
-  if (k + 2 < nb) {
-    if (x < nb - 2) { t.i = k + 2; t.j = skip3((int)x, k, k + 1, -1); return t; }
-    x -= nb - 2;
-    if (x < nb - 3) { t.i = skip3((int)x, k, k + 1, k + 2); t.j = k + 2; return t; }
-    x -= nb - 3;
-    banded(x, nb - 3, nb - 3, r, c);
-    t.i = skip3(r, k, k + 1, k + 2);
-    t.j = skip3(c, k, k + 1, k + 2);
-    return t;
-  }
-  banded(x, nb - 2, nb - 2, r, c);
-  t.i = skip3(r, k, k + 1, -1);
-  t.j = skip3(c, k, k + 1, -1);
-  return t;
-}
-
-__device__ Task decode(long long g, int nb, long long delay) {
-  Task t;
-  if (g == 0) { t.type = T_P1; t.k = 0; t.i = t.j = 0; return t; }
-  g -= 1;
-  const long long n1 = nb - 1, n2 = nb - 2;
-  const long long s0 = 4 * n1;  // seg(0) = G2(0) + G3L(0) + P1(1)
-  if (g < s0) {
-    if (g < 2 * n1) return p2_task(nb, 0, g);
-    g -= 2 * n1;
-    if (g == 0) return g3l_task(nb, 0, 0);
-    if (g == 1) { t.type = T_P1; t.k = 1; t.i = t.j = 1; return t; }
-    return g3l_task(nb, 0, g - 1);
-  }
-  g -= s0;
-  int k;
-  long long r3;  // segment k: G3R(k-1) size r3
-  const long long mid = (long long)(nb - 2) * nb * nb;  // segments 1..nb-2 are nb^2 tasks each
-  if (g < mid) {
-    k = 1 + (int)(g / ((long long)nb * nb));
-    g -= (long long)(k - 1) * nb * nb;
-    r3 = n2 * n2;
-
-  } else {
-    g -= mid;
-    const long long last = n2 * n2 + 2 * n1;  // seg(nb-1) = G3R(nb-2) + G2(nb-1)
-    if (g >= last) {                           // tail: G3R(nb-1), all (i,j) != nb-1
-      g -= last;
-      t.type = T_P3; t.k = nb - 1;
-      int r, c;
-      banded(g, (int)n1, (int)n1, r, c);
-      t.i = r; t.j = c;
-      return t;
-    }
-    k = nb - 1;
-    r3 = n2 * n2;
-
-  }
-  const long long d = delay < r3 ? delay : r3;
-  if (g < d) return g3r_task(nb, k - 1, g);
-  g -= d;
-  if (g < 2 * n1) return p2_task(nb, k, g);
-  g -= 2 * n1;
-  if (g < r3 - d) return g3r_task(nb, k - 1, d + g);
-  g -= r3 - d;
-
-  if (g == 0) return g3l_task(nb, k, 0);
-  if (g == 1) { t.type = T_P1; t.k = k + 1; t.i = t.j = k + 1; return t; }
-  return g3l_task(nb, k, g - 1);
-}
 
 // panel copies of round k (parity k % 2), 128x128 tiles with ld 128:
 //   D = A(k,k) closed, D^T, row panel A(k,j), column panel A(i,k) transposed
@@ -309,51 +137,6 @@ __device__ __forceinline__ T* pb_colT(const DFArgs<T>& a, int k, int i) {
   return pb_diag(a, k) + (long long)(2 + a.nb + i) * TILE_ELEMS;
 }
 
-// Dependency test of task t (one thread): up to three flags, read with
-// independent relaxed loads (one round trip), then an acquire fence once met.
-template <typename T>
-__device__ bool deps_met(const DFArgs<T>& a, const Task& t) {
-  const int nb = a.nb, k = t.k, p = k & 1;
-  const int* f0 = a.ver + (long long)t.i * nb + t.j;
-  const int* f1;
-  const int* f2;
-  int v1, v2;
-  const int v0 = k;
-  if (t.type == T_P1) {
-    f1 = a.done2 + (k >= 2 ? k - 2 : 0); v1 = k >= 2 ? 2 * (nb - 1) : INT_MIN;
-    f2 = f1; v2 = v1;
-  } else if (t.type == T_P3) {
-    f1 = a.rowready + p * nb + t.j; v1 = k + 1;
-    f2 = a.colready + p * nb + t.i; v2 = k + 1;
-  } else {
-    f1 = a.diagready + p; v1 = k + 1;
-    f2 = a.done3 + (k >= 2 ? k - 2 : 0); v2 = k >= 2 ? (nb - 1) * (nb - 1) : INT_MIN;
-  }
-  const int x0 = ld_relaxed(f0), x1 = ld_relaxed(f1), x2 = ld_relaxed(f2);
-  if (x0 >= v0 && x1 >= v1 && x2 >= v2) {
-    // acquire: later reads (after the CTA learns of this) see the producers' data.
-    // fence.acquire (an L1 invalidation here) instead of fence.acq_rel, which would
-    // also wait for this thread's own outstanding copies
-    asm volatile("fence.acquire.gpu;" ::: "memory");
-    return true;
-  }
-  return false;
-}
-
-// Publish task t (one thread, after a group barrier that follows every
-// thread's stores of t): one release fence, then the flags.
-template <typename T>
-__device__ void signal_done(const DFArgs<T>& a, const Task& t) {
-  const int nb = a.nb, k = t.k, p = k & 1;
-  asm volatile("fence.release.gpu;" ::: "memory");
-  st_relaxed(a.ver + (long long)t.i * nb + t.j, k + 1);
-  switch (t.type) {
-    case T_P1: st_relaxed(a.diagready + p, k + 1); break;
-    case T_P2R: st_relaxed(a.rowready + p * nb + t.j, k + 1); red_relaxed_add(a.done2 + k, 1); break;
-    case T_P2C: st_relaxed(a.colready + p * nb + t.i, k + 1); red_relaxed_add(a.done2 + k, 1); break;
-    default: red_relaxed_add(a.done3 + k, 1); break;
-  }
-}
 
 // Phase 1 inside a group: in-place FW closure of one 128x128 tile (the same
 // register blocking as phase1_kernel in apsp_kernels.cu); result also to out2.
@@ -449,24 +232,6 @@ struct GDesc {
 };
 
 
-// flags (and the values they must reach) that task t waits for
-template <typename T>
-__device__ __forceinline__ void dep_flags(const DFArgs<T>& a, const Task& t, const int* (&f)[3], int (&v)[3]) {
-  const int nb = a.nb, k = t.k, p = k & 1;
-  f[0] = a.ver + (long long)t.i * nb + t.j;
-  v[0] = k;
-  if (t.type == T_P1) {
-    f[1] = a.done2 + (k >= 2 ? k - 2 : 0); v[1] = k >= 2 ? 2 * (nb - 1) : INT_MIN;
-    f[2] = f[1]; v[2] = v[1];
-  } else if (t.type == T_P3) {
-    f[1] = a.rowready + p * nb + t.j; v[1] = k + 1;
-    f[2] = a.colready + p * nb + t.i; v[2] = k + 1;
-  } else {
-    f[1] = a.diagready + p; v[1] = k + 1;
-    f[2] = a.done3 + (k >= 2 ? k - 2 : 0); v[2] = k >= 2 ? (nb - 1) * (nb - 1) : INT_MIN;
-  }
-}
-
 // A group's task slot (shared memory, double-buffered by iteration parity):
 // the task index, its decoded form, the operands of a min-plus task and
 // whether its dependencies were already seen met. Thread 0 fills the slot of
@@ -504,8 +269,13 @@ __device__ void fill_desc(const DFArgs<T>& a, const Task& tk, GDesc<T>& d) {
 // parity = (chunk / 3) & 1); the task uses chunks c0 .. c0+3.
 // The SCH thread also prepares the slot of the next task `nxt` during chunk 1:
 // decoded, operands filled, dependencies checked once.
+#ifdef DF_INLINE
+#define DF_MP_INLINE __forceinline__
+#else
+#define DF_MP_INLINE __noinline__
+#endif
 template <typename T>
-__device__ __noinline__ void group_minplus(const GDesc<T>* d, T* stage0, unsigned full0, unsigned empty0, unsigned c0,
+__device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigned full0, unsigned empty0, unsigned c0,
                                            int gtid, int g, const DFArgs<T>* args, long long nxt,
                                            Slot<T>* ns) {
   using V4 = typename DV<T>::V4;

@@ -228,13 +228,38 @@ static apsp_status init_placement(Handle* h, const apsp_config& cfg, const int64
   return h->cuda(cudaStreamSynchronize(h->stream), "init sync");
 }
 
+// The packed int16 closure as one persistent dataflow launch, timed as one
+// event of class 2 carrying all n_pad^3 relaxations (as run_dataflow in apsp_api.cu).
+static apsp_status run_dataflow16(Handle* h) {
+  const int nb = (int)(h->n_pad / h->b);
+  apsp_status st;
+  if (!h->df_work) {
+    if ((st = h->cuda(cudaMallocAsync(&h->df_work, fw_dataflow16_work_bytes(nb), h->stream), "cudaMalloc dataflow16")))
+      return st;
+    h->device_bytes += fw_dataflow16_work_bytes(nb);
+  }
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const long long delay = h->df_delay > 0 ? h->df_delay : 4ll * fw_dataflow16_ctas_per_sm() * sms;
+  h->ev_begin(2);
+  if ((st = h->cuda(launch_fw_dataflow16(h->d16, h->ld, nb, h->df_work, delay, h->stream), "fw_dataflow16")))
+    return st;
+  h->ev_end((double)h->n_pad * h->n_pad * h->n_pad);
+  return APSP_OK;
+}
+
 // Packed int16 closure (VIADDMNMX.S16x2) with exactness check; int32 redo if the
 // largest finite distance reaches 8192 (R16).
 apsp_status run_fw16(Handle* h) {
   apsp_status st;
   const long long nb = h->n_pad / h->b;
   if (!h->fell_back16) {
-    if ((st = fw_closure<short>(h, h->d16, h->ld, h->n_pad, 0, nb, h->stream))) return st;
+    if (h->dataflow) {  // default: every round in one persistent launch (apsp_fw_dataflow16.cu)
+      if ((st = run_dataflow16(h))) return st;
+    } else if ((st = fw_closure<short>(h, h->d16, h->ld, h->n_pad, 0, nb, h->stream))) {
+      return st;
+    }
     int mx = 0;
     if ((st = h->cuda(launch_max_finite16(h->d16, h->ld, h->n_pad, h->n_pad, h->d_max16, h->stream), "max16")))
       return st;

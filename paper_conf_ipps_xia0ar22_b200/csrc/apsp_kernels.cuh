@@ -118,4 +118,11 @@ long long fw_dataflow_pbuf_bytes(int nb, size_t elem);
 long long fw_dataflow_flag_bytes(int nb);
 long long fw_dataflow_work_bytes(int nb, size_t elem);
 
+// The packed int16 closure (R16) as one persistent dataflow launch
+// (apsp_fw_dataflow16.cu); `work` holds fw_dataflow16_work_bytes(nb) bytes.
+cudaError_t launch_fw_dataflow16(short* D, long long ld, int nb, void* work, long long delay, cudaStream_t s,
+                                 unsigned long long* prof = nullptr);
+long long fw_dataflow16_work_bytes(int nb);
+int fw_dataflow16_ctas_per_sm();
+
 }  // namespace apsp

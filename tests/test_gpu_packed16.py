@@ -1,6 +1,7 @@
 """Packed int16 path (apsp_config.packed16 = 1; VIADDMNMX.S16x2, two relaxations per DPX
 instruction): bit-exact against the int32 oracle, with the exactness check and the int32
-redo exercised (reading R16)."""
+redo exercised (reading R16). Both schedules: the persistent dataflow kernel
+(fw_dataflow16_kernel, the default) and the launch-per-phase kernels (reserved[4] = 1)."""
 import numpy as np
 import pytest
 
@@ -17,8 +18,10 @@ def want_i32(g):
     return np.where(d == oracle.INF_I64, INF32, d)
 
 
-def run16(lib, g):
+def run16(lib, g, legacy=False, delay=0):
     c = lib.apsp_config_default(device=0, packed16=1, timing=1)
+    c.reserved[4] = 1 if legacy else 0
+    c.reserved[5] = delay
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
         eligible = lib.apsp_get_info(h).packed16_eligible
         lib.apsp_fw_blocked(h)
@@ -28,14 +31,15 @@ def run16(lib, g):
     return d, part, eligible, arith
 
 
+@pytest.mark.parametrize("legacy", [False, True], ids=["dataflow", "per_phase"])
 @pytest.mark.parametrize("n", [1, 2, 5, 127, 128, 129, 300, 640, 1000])
-def test_packed16_bit_exact(lib, n):
+def test_packed16_bit_exact(lib, n, legacy):
     gens = [gg.erdos_renyi(n, 4 * n, seed=n), gg.erdos_renyi(n, 3 * n, seed=n + 1, undirected=True)]
     if n >= 16:
         gens.append(gg.grid_2d(max(1, n // 16), 16, seed=n))
         gens.append(gg.disjoint_union(gg.erdos_renyi(n // 2, 2 * n, seed=3), gg.directed_ring(n - n // 2, 7)))
     for g in gens:
-        d, part, eligible, arith = run16(lib, g)
+        d, part, eligible, arith = run16(lib, g, legacy)
         w = want_i32(g)
         assert eligible == 1
         assert np.array_equal(d.astype(np.int64), w)
@@ -102,3 +106,28 @@ def test_packed16_config1(lib):
     d, _, eligible, arith = run16(lib, g)
     assert eligible == 1 and arith == lib.APSP_ARITH_S16X2
     assert np.array_equal(d.astype(np.int64), want_i32(g))
+
+
+@pytest.mark.parametrize("delay", [1, 7, 1000000])
+def test_packed16_dataflow_queue_delays(lib, delay):
+    """Panel tasks right behind the diagonal (1), a few phase-3 tiles ahead (7), or after the
+    whole previous phase 3 (huge): every order is dependency-safe and gives the same result."""
+    g = gg.erdos_renyi(1280, 1280 * 6, seed=11)
+    d, _, _, arith = run16(lib, g, delay=delay)
+    assert arith == lib.APSP_ARITH_S16X2
+    assert np.array_equal(d.astype(np.int64), want_i32(g))
+
+
+def test_packed16_dataflow_matches_per_phase_grid(lib):
+    """A relabelled grid (long unique shortest paths cross every tile boundary) at n = 2560
+    (20 rounds): dataflow and launch-per-phase schedules agree bit for bit, and a sample of rows
+    equals the oracle's Dijkstra."""
+    g = gg.grid_2d(40, 64, seed=12, hi=60)  # max distance < 8192: stays in int16
+    a, _, _, arith_a = run16(lib, g)
+    b, _, _, arith_b = run16(lib, g, legacy=True)
+    assert arith_a == arith_b == lib.APSP_ARITH_S16X2
+    assert np.array_equal(a, b)
+    rows = np.arange(0, g.n, 97)
+    want = oracle.dijkstra_rows_i64(g.row_ptr, g.col, g.w, rows)
+    want = np.where(want == oracle.INF_I64, INF32, want)
+    assert np.array_equal(a[rows].astype(np.int64), want)

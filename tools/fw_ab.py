@@ -24,13 +24,14 @@ def main():
     ap.add_argument("--dtype", default="f32", choices=["i32", "f32"])
     ap.add_argument("--runs", type=int, default=2)
     ap.add_argument("--modes", nargs="+", default=["dataflow", "per_phase"])
+    ap.add_argument("--packed16", action="store_true", help="int32 input solved on the packed int16 path")
     a = ap.parse_args()
     g = gg.erdos_renyi(a.n, a.deg * a.n, seed=4, dtype=a.dtype)
-    out = {"n": a.n, "deg": a.deg, "dtype": a.dtype}
+    out = {"n": a.n, "deg": a.deg, "dtype": a.dtype, "packed16": a.packed16}
     for name, legacy in (("dataflow", 2), ("per_phase", 1)):
         if name not in a.modes:
             continue
-        cfg = apsp.apsp_config_default(device=0, timing=1)
+        cfg = apsp.apsp_config_default(device=0, timing=1, packed16=int(a.packed16))
         cfg.reserved[4] = legacy
         with apsp.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=cfg) as h:
             best = 1e30
@@ -42,8 +43,9 @@ def main():
                 if r:
                     best = min(best, t)
             st = apsp.apsp_get_phase_stats(h)
+            arith = apsp.ARITH_NAMES[apsp.apsp_get_info(h).arith]
         out[name] = {"s": best, "relax_per_s": float(a.n) ** 3 / best,
-                     "phase3_rate": st.relax[2] / (st.ms[2] * 1e-3) if st.ms[2] else None}
+                     "phase3_rate": st.relax[2] / (st.ms[2] * 1e-3) if st.ms[2] else None, "arith": arith}
     print(json.dumps(out), flush=True)
 
 
