@@ -274,6 +274,43 @@ apsp_status apsp_restore(apsp_handle* h, const char* path);
 apsp_status apsp_get_dist(apsp_handle* h, int64_t row_begin, int64_t row_count, void* out,
                           int64_t ld_out);
 
+/*
+ * Asynchronous variants for serving loops (several graphs in flight: the D2H of
+ * one result overlaps the closure of the next graph on another handle).
+ *
+ * apsp_fw_blocked_async — enqueue the whole blocked Floyd–Warshall
+ *   on the handle's stream and return without waiting. In-core, not packed16:
+ *   otherwise it runs synchronously like apsp_fw_blocked (same statuses). The
+ *   negative-cycle status is delivered by apsp_synchronize.
+ * apsp_get_dist_async — enqueue the D2H of rows [row_begin, row_begin+row_count)
+ *   (same arguments and row rules as apsp_get_dist) behind the closure on the
+ *   handle's stream; `out` must stay valid until apsp_synchronize returns and
+ *   should be pinned (pageable memory makes the copy synchronous). Out-of-core,
+ *   packed16, boundary and Johnson handles copy synchronously.
+ * apsp_synchronize — wait for everything enqueued on the handle; returns
+ *   APSP_ENEGCYCLE if the asynchronous closure found a negative cycle (the
+ *   distances, including those already copied, are then unspecified),
+ *   APSP_ECUDA on a device error, APSP_OK otherwise. Every other call on a
+ *   handle with pending asynchronous work synchronizes it first (and returns
+ *   its error, if any).
+ */
+apsp_status apsp_fw_blocked_async(apsp_handle* h);
+/*
+ * apsp_load_csr — put the next graph (same n and dtype, any arc count) into an
+ *   existing in-core handle (not out of core / virtual ranks: APSP_ESTATE; a
+ *   packed16 handle solves it in int16 if its weights qualify, else in int32) instead
+ *   of creating a new one: validated and range-checked as in apsp_init_from_csr
+ *   (same errors), copied to the handle's device CSR arrays (grown if needed)
+ *   before return — the caller may reuse its arrays — and the CSR -> dense init
+ *    enqueued on the handle's stream. Then apsp_fw_blocked[_async].
+ *   With world_size > 1 every rank passes the whole CSR (each uploads its rows).
+ */
+apsp_status apsp_load_csr(apsp_handle* h, const int64_t* row_ptr, const int32_t* col_idx,
+                          const void* weights);
+apsp_status apsp_get_dist_async(apsp_handle* h, int64_t row_begin, int64_t row_count, void* out,
+                                int64_t ld_out);
+apsp_status apsp_synchronize(apsp_handle* h);
+
 /* Rows [*row_begin, *row_begin + *row_count) of dist held by this rank. */
 apsp_status apsp_local_rows(const apsp_handle* h, int64_t* row_begin, int64_t* row_count);
 

@@ -102,6 +102,10 @@ _sig = {
     "apsp_reinit": (ctypes.c_int, [_H]),
     "apsp_fw_rounds": (ctypes.c_int, [_H, _I64, _I64]),
     "apsp_get_dist": (ctypes.c_int, [_H, _I64, _I64, _P, _I64]),
+    "apsp_fw_blocked_async": (ctypes.c_int, [_H]),
+    "apsp_get_dist_async": (ctypes.c_int, [_H, _I64, _I64, _P, _I64]),
+    "apsp_synchronize": (ctypes.c_int, [_H]),
+    "apsp_load_csr": (ctypes.c_int, [_H, _P, _P, _P]),
     "apsp_local_rows": (ctypes.c_int, [_H, ctypes.POINTER(_I64), ctypes.POINTER(_I64)]),
     "apsp_partition": (ctypes.c_int, [_I64, _I32, _I32, _I32, ctypes.POINTER(_I64), ctypes.POINTER(_I64),
                                       ctypes.POINTER(_I64)]),
@@ -322,6 +326,32 @@ def apsp_get_dist(h: Handle, row_begin: int = 0, row_count: int | None = None, o
 def apsp_get_dist_ptr(h: Handle, row_begin: int, row_count: int, out_ptr: int, ld_out: int) -> None:
     """Raw-pointer form (e.g. a pinned torch tensor's data_ptr())."""
     _check(_lib.apsp_get_dist(h.raw, row_begin, row_count, ctypes.c_void_p(out_ptr), ld_out), h.raw)
+
+
+def apsp_fw_blocked_async(h: Handle) -> None:
+    """Enqueue the closure and return (in core); the status comes from apsp_synchronize."""
+    _check(_lib.apsp_fw_blocked_async(h.raw), h.raw)
+
+
+def apsp_get_dist_async(h: Handle, row_begin: int, row_count: int, out_ptr: int, ld_out: int) -> None:
+    """Enqueue the D2H of rows into caller memory (pinned: e.g. a pinned tensor's data_ptr()),
+    valid after apsp_synchronize."""
+    _check(_lib.apsp_get_dist_async(h.raw, row_begin, row_count, ctypes.c_void_p(out_ptr), ld_out), h.raw)
+
+
+def apsp_load_csr(h: Handle, row_ptr, col_idx, weights) -> None:
+    """Next graph (same n and dtype) into an in-core handle; the init is enqueued. Arrays are
+    numpy (converted like apsp_init_from_csr; pinned arrays copy fastest)."""
+    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
+    w = np.ascontiguousarray(weights, dtype=np.float32 if h.dtype == APSP_F32 else np.int32)
+    if row_ptr.shape[0] != h.n + 1:
+        raise ValueError("row_ptr must have n+1 entries")
+    _check(_lib.apsp_load_csr(h.raw, _ptr(row_ptr), _ptr(col_idx), _ptr(w)), h.raw)
+
+
+def apsp_synchronize(h: Handle) -> None:
+    _check(_lib.apsp_synchronize(h.raw), h.raw)
 
 
 def apsp_local_rows(h: Handle):

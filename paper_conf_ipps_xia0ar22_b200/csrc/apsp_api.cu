@@ -635,6 +635,7 @@ apsp_status apsp_solve(apsp_handle* hh) {
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->mode != APSP_MODE_BOUNDARY && h->mode != APSP_MODE_JOHNSON) return apsp_fw_blocked(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  if (apsp_status pst = settle(h)) return pst;  // pending asynchronous work first
   if (h->fw_done) return h->fail(APSP_ESTATE, "apsp_solve already ran (apsp_reinit first)");
   apsp_status st;
   if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
@@ -655,6 +656,7 @@ apsp_status apsp_fw_rounds(apsp_handle* hh, int64_t k_begin, int64_t k_end) {
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  if (apsp_status pst = settle(h)) return pst;  // pending asynchronous work first
   if (h->mode != APSP_MODE_INCORE && h->mode != APSP_MODE_OUT_OF_CORE)
     return h->fail(APSP_ESTATE, "apsp_fw_rounds: blocked-FW handles only");
   if (h->mode16) return h->fail(APSP_ESTATE, "apsp_fw_rounds: not available with packed16");
@@ -682,6 +684,7 @@ apsp_status apsp_fw_blocked(apsp_handle* hh) {
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  if (apsp_status pst = settle(h)) return pst;  // pending asynchronous work first
   if (h->fw_done) return h->fail(APSP_ESTATE, "apsp_fw_blocked already ran");
   if (h->mode == APSP_MODE_BOUNDARY || h->mode == APSP_MODE_JOHNSON)
     return h->fail(APSP_ESTATE, "boundary / Johnson handle: use apsp_solve");
@@ -708,10 +711,73 @@ apsp_status apsp_fw_blocked(apsp_handle* hh) {
   return finish_fw(h, true);
 }
 
+apsp_status apsp_fw_blocked_async(apsp_handle* hh) {
+  if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
+  Handle* h = reinterpret_cast<Handle*>(hh);
+  if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  if (apsp_status pst = settle(h)) return pst;
+  if (h->mode != APSP_MODE_INCORE || h->mode16) return apsp_fw_blocked(hh);  // synchronous placements
+  if (h->fw_done) return h->fail(APSP_ESTATE, "apsp_fw_blocked already ran");
+  apsp_status st;
+  if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
+  memset(&h->stats, 0, sizeof(h->stats));
+  const long long nb = h->n_pad / h->b;
+  if ((st = run_incore_rounds(h, h->next_round, nb))) return st;
+  h->next_round = nb;
+  return finish_fw_async(h);
+}
+
+apsp_status apsp_get_dist_async(apsp_handle* hh, int64_t row_begin, int64_t row_count, void* out, int64_t ld_out) {
+  if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
+  Handle* h = reinterpret_cast<Handle*>(hh);
+  if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  if (row_count < 0 || row_begin < 0 || row_begin + row_count > h->n || ld_out < h->n || (row_count > 0 && !out))
+    return h->fail(APSP_EINVAL, "get_dist: bad row range / ld_out / out");
+  if (row_count == 0) return APSP_OK;
+  apsp_status st;
+  if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
+  if (h->mode != APSP_MODE_INCORE || h->result16) {  // synchronous placements: settle first
+    if ((st = settle(h))) return st;
+    return get_rows(h, row_begin, row_count, out, ld_out);
+  }
+  return get_rows_async(h, row_begin, row_count, out, ld_out);
+}
+
+apsp_status apsp_load_csr(apsp_handle* hh, const int64_t* row_ptr, const int32_t* col_idx, const void* weights) {
+  if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
+  Handle* h = reinterpret_cast<Handle*>(hh);
+  if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  if (apsp_status pst = settle(h)) return pst;
+  if (h->mode != APSP_MODE_INCORE || h->virt)
+    return h->fail(APSP_ESTATE, "apsp_load_csr: in-core handles without virtual ranks only");
+  if (!row_ptr) return h->fail(APSP_EINVAL, "row_ptr is NULL");
+  bool has_neg = false;
+  int64_t maxabs = 0;
+  if (apsp_status vst = validate_csr(h->n, row_ptr, col_idx, weights, h->dtype, &has_neg, &maxabs)) {
+    h->err = g_last_error;
+    return vst;
+  }
+  apsp_status st;
+  if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
+  h->has_neg = has_neg;
+  h->max_abs_w = maxabs;
+  // packed16 handle (R16): int16 again if this graph is eligible, else straight to int32
+  if (h->mode16) h->fell_back16 = has_neg || maxabs > 8191;
+  return load_csr(h, row_ptr, col_idx, weights);
+}
+
+apsp_status apsp_synchronize(apsp_handle* hh) {
+  if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
+  Handle* h = reinterpret_cast<Handle*>(hh);
+  if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  return settle(h);
+}
+
 apsp_status apsp_reinit(apsp_handle* hh) {
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  if (apsp_status pst = settle(h)) return pst;  // pending asynchronous work first
   apsp_status st;
   if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
   if (h->mode == APSP_MODE_OUT_OF_CORE) return ooc_reinit(h);
@@ -724,6 +790,7 @@ apsp_status apsp_get_dist(apsp_handle* hh, int64_t row_begin, int64_t row_count,
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  if (apsp_status pst = settle(h)) return pst;  // pending asynchronous work first
   if (row_count < 0 || row_begin < 0 || row_begin + row_count > h->n || ld_out < h->n || (row_count > 0 && !out))
     return h->fail(APSP_EINVAL, "get_dist: bad row range / ld_out / out");
   if (row_count == 0) return APSP_OK;

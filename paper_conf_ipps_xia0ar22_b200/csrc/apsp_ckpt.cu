@@ -55,6 +55,7 @@ void fill_header(const Handle* h, CkptHeader* hd) {
 
 apsp_status check_handle(Handle* h) {
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
+  if (apsp_status pst = settle(h)) return pst;  // pending asynchronous work first
   if (h->mode != APSP_MODE_INCORE && h->mode != APSP_MODE_OUT_OF_CORE)
     return h->fail(APSP_ESTATE, "checkpoint: blocked-FW handles only");
   if (h->mode16) return h->fail(APSP_ESTATE, "checkpoint: not available with packed16");

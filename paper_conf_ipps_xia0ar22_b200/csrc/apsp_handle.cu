@@ -44,6 +44,7 @@ static apsp_status upload_csr(Handle* h, const int64_t* row_ptr, const int32_t* 
     if (me > 0) {
       if ((st = h->cuda(cudaMalloc(&sh.d_col, me * sizeof(int)), "cudaMalloc csr"))) return st;
       if ((st = h->cuda(cudaMalloc(&sh.d_w, me * sizeof(T)), "cudaMalloc csr"))) return st;
+      sh.cap_arcs = me;
       if ((st = h->cuda(cudaMemcpyAsync(sh.d_col, col + e0, me * sizeof(int), cudaMemcpyHostToDevice, h->stream),
                         "H2D col")))
         return st;
@@ -54,6 +55,48 @@ static apsp_status upload_csr(Handle* h, const int64_t* row_ptr, const int32_t* 
     }
   }
   return APSP_OK;
+}
+
+// A new graph with the same n and dtype into an in-core handle (serving loops):
+// the CSR slices are copied into the handle's device arrays (grown only if the
+// arc count exceeds their capacity; the copy completes before return, so the
+// caller may reuse its arrays) and the CSR -> dense init is enqueued.
+apsp_status load_csr(Handle* h, const int64_t* row_ptr, const int32_t* col, const void* w) {
+  apsp_status st;
+  const size_t we = sizeof(int32_t);  // int32 and fp32 weights
+  for (auto& sh : h->shards) {
+    const long long real = sh.real_rows;
+    if (real <= 0) continue;
+    const long long e0 = row_ptr[sh.row_begin];
+    const long long me = row_ptr[sh.row_begin + real] - e0;
+    sh.e0 = e0;
+    if (me > sh.cap_arcs) {
+      cudaFree(sh.d_col);
+      cudaFree(sh.d_w);
+      sh.d_col = nullptr;
+      sh.d_w = nullptr;
+      if ((st = h->cuda(cudaMalloc(&sh.d_col, me * sizeof(int)), "cudaMalloc csr"))) return st;
+      if ((st = h->cuda(cudaMalloc(&sh.d_w, me * we), "cudaMalloc csr"))) return st;
+      h->device_bytes += (me - sh.cap_arcs) * (sizeof(int) + we);
+      sh.cap_arcs = me;
+    }
+    if ((st = h->cuda(cudaMemcpyAsync(sh.d_rp, row_ptr + sh.row_begin, (real + 1) * sizeof(long long),
+                                      cudaMemcpyHostToDevice, h->stream), "H2D row_ptr")))
+      return st;
+    if (me > 0) {
+      if ((st = h->cuda(cudaMemcpyAsync(sh.d_col, col + e0, me * sizeof(int), cudaMemcpyHostToDevice, h->stream),
+                        "H2D col")))
+        return st;
+      if ((st = h->cuda(cudaMemcpyAsync(sh.d_w, static_cast<const char*>(w) + e0 * we, me * we,
+                                        cudaMemcpyHostToDevice, h->stream), "H2D w")))
+        return st;
+    }
+  }
+  // the host arrays are read before return (the stream was idle: settled by the caller)
+  if ((st = h->cuda(cudaStreamSynchronize(h->stream), "H2D csr sync"))) return st;
+  h->fw_done = false;
+  h->next_round = 0;
+  return run_init(h);
 }
 
 // a1: CSR -> dense for every local shard, from the device CSR.
@@ -328,6 +371,7 @@ void delete_handle(Handle* h) {
     if (e) cudaEventDestroy(e);
   cudaFree(h->d_widen);
   cudaFree(h->d_flag);
+  if (h->h_flag) cudaFreeHost(h->h_flag);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
   if (h->side) {
     cudaStreamSynchronize(h->side);
@@ -338,6 +382,70 @@ void delete_handle(Handle* h) {
   for (auto& e : h->ev_sh)
     if (e) cudaEventDestroy(e);
   delete h;
+}
+
+apsp_status settle(Handle* h) {
+  if (!h->pending) return APSP_OK;
+  const bool fw = h->pending_fw;
+  h->pending = h->pending_fw = false;
+  apsp_status st;
+  if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
+  if ((st = h->cuda(cudaStreamSynchronize(h->stream), "async sync"))) return st;
+  if (h->copy_stream && (st = h->cuda(cudaStreamSynchronize(h->copy_stream), "async sync"))) return st;
+  if (fw) {
+    if (h->timing) h->collect_events();
+    if (*h->h_flag) return h->fail(APSP_ENEGCYCLE, "negative cycle detected: distances are unspecified");
+  }
+  return APSP_OK;
+}
+
+// The end of an asynchronous closure: the flag's D2H is enqueued, settle() reads it.
+apsp_status finish_fw_async(Handle* h) {
+  apsp_status st;
+  if (h->use_comm) {
+    ncclResult_t r = ncclAllReduce(h->d_flag, h->d_flag, 1, ncclInt32, ncclMax, static_cast<ncclComm_t>(h->comm),
+                                   h->stream);
+    if (r != ncclSuccess) return h->fail(APSP_ENCCL, "ncclAllReduce(flag): %s", ncclGetErrorString(r));
+  }
+  if (!h->h_flag && (st = h->cuda(cudaHostAlloc(&h->h_flag, sizeof(int), cudaHostAllocDefault), "cudaHostAlloc flag")))
+    return st;
+  if ((st = h->cuda(cudaMemcpyAsync(h->h_flag, h->d_flag, sizeof(int), cudaMemcpyDeviceToHost, h->stream),
+                    "D2H flag")))
+    return st;
+  h->canonical = false;
+  h->fw_done = true;
+  h->pending = h->pending_fw = true;
+  return APSP_OK;
+}
+
+// Enqueue the D2H of rows [r0, r0+cnt) on the handle's stream (in core, not
+// packed16); other placements copy synchronously through get_rows.
+apsp_status get_rows_async(Handle* h, long long r0, long long cnt, void* out, long long ld_out) {
+  if (h->mode != APSP_MODE_INCORE || h->result16) return get_rows(h, r0, cnt, out, ld_out);
+  if (h->mode16 && !h->shards[0].D) return h->fail(APSP_ESTATE, "no int32 matrix yet");
+  apsp_status st;
+  const char* base;
+  if (h->world > 1 && !h->virt) {
+    const long long rb = h->shards[0].row_begin;
+    if (r0 < rb || r0 + cnt > rb + h->rows_per_rank)
+      return h->fail(APSP_EINVAL, "rows [%lld, %lld) are not local to rank %d", r0, r0 + cnt, h->rank);
+    base = static_cast<const char*>(h->shards[0].D) + (size_t)(r0 - rb) * h->ld * h->elem;
+  } else {
+    base = static_cast<const char*>(h->d_base) + (size_t)r0 * h->ld * h->elem;
+  }
+  if (h->dtype == APSP_I32 && h->has_neg && !h->canonical) {
+    for (auto& sh : h->shards)
+      if ((st = h->cuda(launch_canonicalize_i32(static_cast<int*>(sh.D), h->ld, h->rows_per_rank, h->n_pad, h->stream),
+                        "canonicalize")))
+        return st;
+    h->canonical = true;
+  }
+  if ((st = h->cuda(cudaMemcpy2DAsync(out, (size_t)ld_out * h->elem, base, (size_t)h->ld * h->elem,
+                                      (size_t)h->n * h->elem, (size_t)cnt, cudaMemcpyDeviceToHost, h->stream),
+                    "D2H dist")))
+    return st;
+  h->pending = true;
+  return APSP_OK;
 }
 
 apsp_status finish_fw(Handle* h, bool all_rounds) {
@@ -400,26 +508,9 @@ apsp_status get_rows(Handle* h, long long r0, long long cnt, void* out, long lon
     }
     return h->cuda(cudaStreamSynchronize(h->copy_stream), "get_dist sync");
   }
-  const char* base;
-  if (h->world > 1 && !h->virt) {
-    const long long rb = h->shards[0].row_begin;
-    if (r0 < rb || r0 + cnt > rb + h->rows_per_rank)
-      return h->fail(APSP_EINVAL, "rows [%lld, %lld) are not local to rank %d", r0, r0 + cnt, h->rank);
-    base = static_cast<const char*>(h->shards[0].D) + (size_t)(r0 - rb) * h->ld * h->elem;
-  } else {
-    base = static_cast<const char*>(h->d_base) + (size_t)r0 * h->ld * h->elem;
-  }
-  if (h->dtype == APSP_I32 && h->has_neg && !h->canonical) {
-    for (auto& sh : h->shards)
-      if ((st = h->cuda(launch_canonicalize_i32(static_cast<int*>(sh.D), h->ld, h->rows_per_rank, h->n_pad, h->stream),
-                        "canonicalize")))
-        return st;
-    h->canonical = true;
-  }
-  if ((st = h->cuda(cudaMemcpy2DAsync(out, (size_t)ld_out * h->elem, base, (size_t)h->ld * h->elem,
-                                      (size_t)h->n * h->elem, (size_t)cnt, cudaMemcpyDeviceToHost, h->stream),
-                    "D2H dist")))
-    return st;
+  const bool was_pending = h->pending;
+  if ((st = get_rows_async(h, r0, cnt, out, ld_out))) return st;
+  h->pending = was_pending;
   return h->cuda(cudaStreamSynchronize(h->stream), "get_dist sync");
 }
 

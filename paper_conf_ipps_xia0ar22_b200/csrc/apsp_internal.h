@@ -19,6 +19,7 @@ struct Shard {
   int* d_col = nullptr;
   void* d_w = nullptr;
   long long real_rows = 0, e0 = 0;
+  long long cap_arcs = 0;    // arcs d_col / d_w can hold (apsp_load_csr reuses them)
 };
 
 struct TimedEvent {
@@ -79,6 +80,9 @@ struct Handle {
   long long device_bytes = 0, host_bytes = 0;
   long long next_round = 0;
   bool fw_done = false, canonical = false, poisoned = false;
+  bool pending = false;     // asynchronous work enqueued (apsp_*_async); settle() waits for it
+  bool pending_fw = false;  // ... including a closure whose negative-cycle flag is still unread
+  int* h_flag = nullptr;    // pinned host copy of d_flag for the asynchronous closure
   bool timing = false;
   std::vector<TimedEvent> events;
   apsp_phase_stats stats{};
@@ -103,6 +107,12 @@ apsp_status run_init(Handle* h);
 apsp_status run_fw16(Handle* h);  // packed int16 closure, verify, int32 fallback
 apsp_status run_incore_rounds(Handle* h, long long k0, long long k1);
 apsp_status finish_fw(Handle* h, bool all_rounds);
+// wait for pending asynchronous work (apsp_fw_blocked_async / apsp_get_dist_async)
+apsp_status settle(Handle* h);
+// apsp_load_csr: a new CSR (same n, dtype) into an in-core handle, init enqueued
+apsp_status load_csr(Handle* h, const int64_t* row_ptr, const int32_t* col, const void* w);
+apsp_status finish_fw_async(Handle* h);
+apsp_status get_rows_async(Handle* h, long long r0, long long cnt, void* out, long long ld_out);
 apsp_status get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out);
 bool nccl_unique_id(void* out128);
 
