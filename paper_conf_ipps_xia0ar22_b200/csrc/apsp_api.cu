@@ -403,6 +403,7 @@ static apsp_status validate_csr(int64_t n, const int64_t* row_ptr, const int32_t
 
 apsp_status apsp_init_from_csr(apsp_handle** out, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
                                const void* weights, apsp_dtype dtype, const apsp_config* cfg_in) {
+  NvtxRange nvtx_("apsp_init_from_csr");
   if (!out) return fail_global(APSP_EINVAL, "apsp_init_from_csr: out is NULL");
   *out = nullptr;
   apsp_config cfg;
@@ -455,6 +456,7 @@ apsp_status apsp_init_from_csr(apsp_handle** out, int64_t n, const int64_t* row_
 apsp_status apsp_init_boundary(apsp_handle** out, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
                                const void* weights, apsp_dtype dtype, const int32_t* comp, int32_t k,
                                const apsp_config* cfg_in) {
+  NvtxRange nvtx_("apsp_init_boundary");
   if (!out) return fail_global(APSP_EINVAL, "apsp_init_boundary: out is NULL");
   *out = nullptr;
   apsp_config cfg;
@@ -500,6 +502,7 @@ apsp_status apsp_init_boundary(apsp_handle** out, int64_t n, const int64_t* row_
 apsp_status apsp_init_johnson(apsp_handle** out, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
                               const void* weights, apsp_dtype dtype, double delta, int64_t batch,
                               const apsp_config* cfg_in) {
+  NvtxRange nvtx_("apsp_init_johnson");
   if (!out) return fail_global(APSP_EINVAL, "apsp_init_johnson: out is NULL");
   *out = nullptr;
   apsp_config cfg;
@@ -546,6 +549,7 @@ apsp_status apsp_init_johnson(apsp_handle** out, int64_t n, const int64_t* row_p
 apsp_status apsp_select(int64_t n, const int64_t* row_ptr, const int32_t* col_idx, const void* weights,
                         apsp_dtype dtype, const int32_t* comp, int32_t k, const apsp_config* cfg_in,
                         apsp_selection* out) {
+  NvtxRange nvtx_("apsp_select");
   if (!out) return fail_global(APSP_EINVAL, "apsp_select: out is NULL");
   memset(out, 0, sizeof(*out));
   for (double& e : out->est_seconds) e = -1.0;
@@ -631,6 +635,7 @@ apsp_status apsp_select(int64_t n, const int64_t* row_ptr, const int32_t* col_id
 }
 
 apsp_status apsp_solve(apsp_handle* hh) {
+  NvtxRange nvtx_("apsp_solve");
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->mode != APSP_MODE_BOUNDARY && h->mode != APSP_MODE_JOHNSON) return apsp_fw_blocked(hh);
@@ -653,6 +658,7 @@ apsp_status apsp_solve(apsp_handle* hh) {
 }
 
 apsp_status apsp_fw_rounds(apsp_handle* hh, int64_t k_begin, int64_t k_end) {
+  NvtxRange nvtx_("apsp_fw_rounds");
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
@@ -681,6 +687,7 @@ apsp_status apsp_fw_rounds(apsp_handle* hh, int64_t k_begin, int64_t k_end) {
 }
 
 apsp_status apsp_fw_blocked(apsp_handle* hh) {
+  NvtxRange nvtx_("apsp_fw_blocked");
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
@@ -712,6 +719,7 @@ apsp_status apsp_fw_blocked(apsp_handle* hh) {
 }
 
 apsp_status apsp_fw_blocked_async(apsp_handle* hh) {
+  NvtxRange nvtx_("apsp_fw_blocked_async");
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
@@ -728,6 +736,7 @@ apsp_status apsp_fw_blocked_async(apsp_handle* hh) {
 }
 
 apsp_status apsp_get_dist_async(apsp_handle* hh, int64_t row_begin, int64_t row_count, void* out, int64_t ld_out) {
+  NvtxRange nvtx_("apsp_get_dist_async");
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
@@ -744,6 +753,7 @@ apsp_status apsp_get_dist_async(apsp_handle* hh, int64_t row_begin, int64_t row_
 }
 
 apsp_status apsp_load_csr(apsp_handle* hh, const int64_t* row_ptr, const int32_t* col_idx, const void* weights) {
+  NvtxRange nvtx_("apsp_load_csr");
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
@@ -767,6 +777,7 @@ apsp_status apsp_load_csr(apsp_handle* hh, const int64_t* row_ptr, const int32_t
 }
 
 apsp_status apsp_synchronize(apsp_handle* hh) {
+  NvtxRange nvtx_("apsp_synchronize");
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
@@ -774,6 +785,7 @@ apsp_status apsp_synchronize(apsp_handle* hh) {
 }
 
 apsp_status apsp_reinit(apsp_handle* hh) {
+  NvtxRange nvtx_("apsp_reinit");
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
@@ -787,6 +799,7 @@ apsp_status apsp_reinit(apsp_handle* hh) {
 }
 
 apsp_status apsp_get_dist(apsp_handle* hh, int64_t row_begin, int64_t row_count, void* out, int64_t ld_out) {
+  NvtxRange nvtx_("apsp_get_dist");
   if (!hh) return fail_global(APSP_EINVAL, "NULL handle");
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");

@@ -459,6 +459,13 @@ apsp_status finish_fw(Handle* h, bool all_rounds) {
   if ((st = h->cuda(cudaMemcpyAsync(&flag, h->d_flag, sizeof(int), cudaMemcpyDeviceToHost, h->stream), "D2H flag")))
     return st;
   if ((st = h->cuda(cudaStreamSynchronize(h->stream), "fw sync"))) return st;
+  if (h->use_comm) {  // a peer's failure surfaces here instead of as a later hang
+    ncclResult_t ar = ncclSuccess;
+    if (ncclCommGetAsyncError(static_cast<ncclComm_t>(h->comm), &ar) != ncclSuccess || ar != ncclSuccess) {
+      h->poisoned = true;
+      return h->fail(APSP_ENCCL, "NCCL asynchronous error: %s", ncclGetErrorString(ar));
+    }
+  }
   if (h->timing) h->collect_events();
   h->canonical = false;
   if (all_rounds) h->fw_done = true;

@@ -4,10 +4,21 @@
 #include "apsp_kernels.cuh"
 
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 #include <string>
 #include <vector>
 
 namespace apsp {
+
+// NVTX range for the duration of a scope (C-ABI entry points, out-of-core
+// super-rounds): shows up in Nsight timelines and `ncu --nvtx` filters; a
+// no-op when no tool is attached (NVTX3 is header-only).
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+  NvtxRange(const NvtxRange&) = delete;
+  NvtxRange& operator=(const NvtxRange&) = delete;
+};
 
 // A block of rows of the (padded) distance matrix resident on the device.
 struct Shard {

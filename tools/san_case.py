@@ -37,37 +37,49 @@ def same(a, b, what):
 
 def main():
     n = int(os.environ.get("SAN_N", "300"))
+    only = os.environ.get("SAN_CASES", "")  # comma-separated case names; empty = all
+    want = lambda c: not only or c in only.split(",")  # noqa: E731
     g = gg.erdos_renyi(n, 5 * n, seed=1)
-    same(run(g), run(g, r4=1), "int32 dataflow vs per-phase")
     gf = gg.erdos_renyi(n, 5 * n, seed=2, dtype="f32")
-    same(run(gf, r4=2), run(gf, r4=1), "fp32 dataflow vs per-phase")
-    same(run(g, packed16=1), run(g, packed16=1, r4=1), "packed16 dataflow vs per-phase")
-    same(run(g, packed16=1), run(g), "packed16 vs int32")
     gb = gg.erdos_renyi(512, 2500, seed=3)
-    same(run(gb, force_out_of_core=1, ooc_block=256), run(gb), "out of core vs in core")
-    same(run(gb, world_size=2, virtual_ranks=1), run(gb), "2 virtual ranks vs 1 GPU")
     p = np.random.default_rng(4).integers(0, 30, n)
     s, t, w = g.arcs()
     gn = gg.csr_from_arcs(n, s, t, (w + p[s] - p[t]).astype(np.int32))
-    same(run(gn), run(gn, r4=1), "negative weights (canonicalize)")
-    with apsp.apsp_init_johnson(n, g.row_ptr, g.col, g.w) as h:
-        apsp.apsp_solve(h)
-        dj = apsp.apsp_get_dist(h)
-    same(dj, run(g), "Johnson vs blocked FW")
-    gg2 = gg.grid_2d(16, 16, seed=5, permute=False)
-    comp, k = gg.grid_block_partition(gg2, 2, 2)
-    with apsp.apsp_init_boundary(gg2.n, gg2.row_ptr, gg2.col, gg2.w, comp, k) as h:
-        apsp.apsp_solve(h)
-        db = apsp.apsp_get_dist(h)
-    same(db, run(gg2), "boundary vs blocked FW")
-    import torch
-    out = torch.empty((n, n), dtype=torch.int32, pin_memory=True)
-    with apsp.apsp_init_from_csr(n, g.row_ptr, g.col, g.w) as h:
-        apsp.apsp_load_csr(h, gn.row_ptr, gn.col, gn.w)
-        apsp.apsp_fw_blocked_async(h)
-        apsp.apsp_get_dist_async(h, 0, n, out.data_ptr(), n)
-        apsp.apsp_synchronize(h)
-    same(out.numpy(), run(gn), "load_csr + async vs blocking")
+    if want("dataflow"):
+        same(run(g), run(g, r4=1), "int32 dataflow vs per-phase")
+        same(run(gf, r4=2), run(gf, r4=1), "fp32 dataflow vs per-phase")
+        same(run(g, packed16=1), run(g, packed16=1, r4=1), "packed16 dataflow vs per-phase")
+    if want("barrier"):  # per-phase kernels with CTA barriers only (reserved[3] = 1: no mbarriers)
+        same(run(g, r3=1, r4=1), run(g, r4=1), "int32 per-phase, CTA-barrier pipeline")
+        same(run(gf, r3=1, r4=1), run(gf, r4=1), "fp32 per-phase, CTA-barrier pipeline")
+        same(run(g, packed16=1, r4=1), run(g), "packed16 per-phase vs int32")
+        same(run(gn, r3=1, r4=1), run(gn, r4=1), "negative weights, CTA-barrier pipeline")
+    if want("ooc"):
+        same(run(gb, force_out_of_core=1, ooc_block=256, r3=1), run(gb, r4=1), "out of core vs in core")
+        same(run(gb, world_size=2, virtual_ranks=1, r3=1), run(gb, r4=1), "2 virtual ranks vs 1 GPU")
+    if want("neg"):
+        same(run(gn), run(gn, r4=1), "negative weights (canonicalize)")
+    if want("johnson"):
+        with apsp.apsp_init_johnson(n, g.row_ptr, g.col, g.w) as h:
+            apsp.apsp_solve(h)
+            dj = apsp.apsp_get_dist(h)
+        same(dj, run(g, r4=1), "Johnson vs blocked FW")
+    if want("boundary"):
+        gg2 = gg.grid_2d(16, 16, seed=5, permute=False)
+        comp, k = gg.grid_block_partition(gg2, 2, 2)
+        with apsp.apsp_init_boundary(gg2.n, gg2.row_ptr, gg2.col, gg2.w, comp, k) as h:
+            apsp.apsp_solve(h)
+            db = apsp.apsp_get_dist(h)
+        same(db, run(gg2, r4=1), "boundary vs blocked FW")
+    if want("async"):
+        import torch
+        out = torch.empty((n, n), dtype=torch.int32, pin_memory=True)
+        with apsp.apsp_init_from_csr(n, g.row_ptr, g.col, g.w) as h:
+            apsp.apsp_load_csr(h, gn.row_ptr, gn.col, gn.w)
+            apsp.apsp_fw_blocked_async(h)
+            apsp.apsp_get_dist_async(h, 0, n, out.data_ptr(), n)
+            apsp.apsp_synchronize(h)
+        same(out.numpy(), run(gn, r4=1), "load_csr + async vs blocking")
     print("san_case done", flush=True)
 
 
