@@ -23,10 +23,14 @@ def main():
     ap.add_argument("--packed16", action="store_true")
     ap.add_argument("--df-delay", type=int, default=0)
     ap.add_argument("--ooc-block", type=int, default=0, help="> 0: out-of-core path with this band height")
+    ap.add_argument("--er", type=int, default=0, help="> 0: seeded ER graph with this n instead of --workload")
+    ap.add_argument("--deg", type=int, default=16)
+    ap.add_argument("--dtype", default="i32", choices=["i32", "f32"])
+    ap.add_argument("--dataflow", action="store_true", help="force the dataflow kernel (fp32 default is per-phase)")
     a = ap.parse_args()
-    g = gg.baseline_config(a.workload)
+    g = gg.erdos_renyi(a.er, a.deg * a.er, seed=4, dtype=a.dtype) if a.er else gg.baseline_config(a.workload)
     cfg = apsp.apsp_config_default(device=0)
-    cfg.reserved[4] = 1 if a.legacy else 0
+    cfg.reserved[4] = 1 if a.legacy else (2 if a.dataflow else 0)
     cfg.reserved[5] = a.df_delay
     cfg.packed16 = 1 if a.packed16 else 0
     if a.ooc_block:

@@ -50,27 +50,27 @@ def main():
         same(run(gf, r4=2), run(gf, r4=1), "fp32 dataflow vs per-phase")
         same(run(g, packed16=1), run(g, packed16=1, r4=1), "packed16 dataflow vs per-phase")
     if want("barrier"):  # per-phase kernels with CTA barriers only (reserved[3] = 1: no mbarriers)
-        same(run(g, r3=1, r4=1), run(g, r4=1), "int32 per-phase, CTA-barrier pipeline")
-        same(run(gf, r3=1, r4=1), run(gf, r4=1), "fp32 per-phase, CTA-barrier pipeline")
-        same(run(g, packed16=1, r4=1), run(g), "packed16 per-phase vs int32")
-        same(run(gn, r3=1, r4=1), run(gn, r4=1), "negative weights, CTA-barrier pipeline")
+        same(run(g, r3=1, r4=1), run(g, r3=1, r4=1, packed16=1), "int32 vs packed16, per-phase CTA-barrier kernels")
+        same(run(gf, r3=1, r4=1), run(gf, r3=1, r4=1, world_size=2, virtual_ranks=1), "fp32 per-phase, 1 vs 2 virtual ranks")
+        same(run(g, packed16=1, r4=1), run(g, r3=1, r4=1), "packed16 per-phase vs int32")
+        same(run(gn, r3=1, r4=1), run(gn, r3=1, r4=1, world_size=2, virtual_ranks=1), "negative weights, 1 vs 2 virtual ranks")
     if want("ooc"):
-        same(run(gb, force_out_of_core=1, ooc_block=256, r3=1), run(gb, r4=1), "out of core vs in core")
-        same(run(gb, world_size=2, virtual_ranks=1, r3=1), run(gb, r4=1), "2 virtual ranks vs 1 GPU")
+        same(run(gb, force_out_of_core=1, ooc_block=256, r3=1), run(gb, r3=1, r4=1), "out of core vs in core")
+        same(run(gb, world_size=2, virtual_ranks=1, r3=1), run(gb, r3=1, r4=1), "2 virtual ranks vs 1 GPU")
     if want("neg"):
         same(run(gn), run(gn, r4=1), "negative weights (canonicalize)")
     if want("johnson"):
         with apsp.apsp_init_johnson(n, g.row_ptr, g.col, g.w) as h:
             apsp.apsp_solve(h)
             dj = apsp.apsp_get_dist(h)
-        same(dj, run(g, r4=1), "Johnson vs blocked FW")
+        same(dj, run(g, r3=1, r4=1), "Johnson vs blocked FW")
     if want("boundary"):
         gg2 = gg.grid_2d(16, 16, seed=5, permute=False)
         comp, k = gg.grid_block_partition(gg2, 2, 2)
         with apsp.apsp_init_boundary(gg2.n, gg2.row_ptr, gg2.col, gg2.w, comp, k) as h:
             apsp.apsp_solve(h)
             db = apsp.apsp_get_dist(h)
-        same(db, run(gg2, r4=1), "boundary vs blocked FW")
+        same(db, run(gg2, r3=1, r4=1), "boundary vs blocked FW")
     if want("async"):
         import torch
         out = torch.empty((n, n), dtype=torch.int32, pin_memory=True)
