@@ -47,6 +47,9 @@ def parse():
     ap.add_argument("--ooc-block", type=int, default=0, help="out-of-core band height B (0 = auto)")
     ap.add_argument("--stream-all", action="store_true", help="out-of-core: keep no band resident")
     ap.add_argument("--no-lookahead", action="store_true", help="in-core: no phase-3 split / overlap")
+    ap.add_argument("--sharded-dataflow", action="store_true",
+                    help="N > 1: the sharded dataflow kernel (owner stores the pivot panels into every GPU's "
+                         "panel buffer over NVLink) instead of the launch-per-phase schedule with NCCL broadcasts")
     ap.add_argument("--legacy", action="store_true",
                     help="single GPU: launch-per-phase schedule instead of the persistent dataflow kernel")
     ap.add_argument("--df-delay", type=int, default=0, help="dataflow kernel queue delay (0 = auto)")
@@ -235,6 +238,8 @@ def run_ours(args):
         cfg.reserved[3] = args.minplus_variant
         if args.legacy:
             cfg.reserved[4] = 1
+        if args.sharded_dataflow:
+            cfg.reserved[4] = 2
         cfg.reserved[5] = args.df_delay
         if packed16:
             cfg.packed16 = 1
@@ -321,6 +326,9 @@ def run_ours(args):
         kname = ("%s: all rounds and phases 1-3 in one persistent launch (%s)"
                  % ("fw_dataflow16_kernel" if arith == "s16x2" else "fw_dataflow_kernel", arith) if dataflow
                  else "phase-3 min-plus (%s)" % arith)
+        if dataflow and world > 1:
+            kname = ("fw_dataflow_kernel<sharded>: this rank's tile rows, all rounds in one persistent launch, "
+                     "pivot panels stored into every GPU by their owner (%s)" % arith)
         roofline = {"bound": "alu", "kernel": kname, "achieved": achieved / 1e12,
                     "peak": peak / 1e12, "unit": "Trelax/s", "frac": achieved / peak, "traffic": traffic,
                     "traffic_unit": "bytes per launch (DRAM read+write)",

@@ -15,6 +15,7 @@
 #include "apsp_internal.h"
 
 #include <cstdlib>
+#include <nccl.h>
 #include "apsp_sched.cuh"
 
 #include <cstdio>
@@ -303,9 +304,153 @@ static apsp_status run_dataflow(Handle* h) {
   return APSP_OK;
 }
 
+// All rounds over a 1-D block-row shard in one persistent launch per GPU
+// (launch_fw_dataflow_sharded): the owner of each round stores the pivot panels
+// into every rank's panel buffer itself (peer stores over NVLink between GPUs,
+// plain stores between virtual ranks), so no collective runs between rounds.
+// NCCL ranks exchange CUDA IPC handles of their work buffers once (ncclAllGather)
+// and pass a barrier after zeroing their flags, before any peer may store into them.
+template <typename T>
+static apsp_status run_dataflow_sharded(Handle* h) {
+  const int nb = (int)(h->n_pad / h->b), P = h->world, nl = nb / P;
+  const long long wb = fw_dataflow_work_bytes(nb, nl, sizeof(T));
+  const long long pbb = fw_dataflow_pbuf_bytes(nb, nl, sizeof(T)), fbb = fw_dataflow_flag_bytes(nb, nl);
+  apsp_status st;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const long long delay = h->df_delay > 0 ? h->df_delay : 8ll * sms / (h->virt ? P : 1);
+  std::vector<DFShard> ranks;
+  if (h->virt) {
+    if (h->sh_work.empty()) {
+      for (int r = 0; r < P; ++r) {
+        void* w = nullptr;
+        if ((st = h->cuda(cudaMallocAsync(&w, wb, h->stream), "cudaMalloc dataflow shard"))) return st;
+        h->sh_work.push_back(w);
+        h->device_bytes += wb;
+      }
+    }
+    for (int r = 0; r < P; ++r) {
+      DFShard d;
+      memset(&d, 0, sizeof(d));
+      d.rank = r;
+      d.D = h->shards[r].D;
+      d.work = h->sh_work[r];
+      for (int e = 0; e < P; ++e) d.peer_work[e] = h->sh_work[e];
+      ranks.push_back(d);
+      if ((st = h->cuda(cudaMemsetAsync(static_cast<char*>(h->sh_work[r]) + pbb, 0, fbb, h->stream), "memset flags")))
+        return st;
+    }
+  } else {
+    // (work buffer and peer mappings: prepare_sharded_peers, called by run_incore_rounds)
+    DFShard d;
+    memset(&d, 0, sizeof(d));
+    d.rank = h->rank;
+    d.D = h->shards[0].D;
+    d.work = h->sh_work[0];
+    for (int e = 0; e < P; ++e) d.peer_work[e] = h->sh_peer[e];
+    ranks.push_back(d);
+    if ((st = h->cuda(cudaMemsetAsync(static_cast<char*>(h->sh_work[0]) + pbb, 0, fbb, h->stream), "memset flags")))
+      return st;
+    if (P > 1) {  // every rank's flags are zero before any rank's kernel may store into them
+      ncclResult_t r = ncclAllReduce(h->d_flag, h->d_flag, 1, ncclInt32, ncclMax, static_cast<ncclComm_t>(h->comm),
+                                     h->stream);
+      if (r != ncclSuccess) return h->fail(APSP_ENCCL, "ncclAllReduce(barrier): %s", ncclGetErrorString(r));
+    }
+  }
+  h->ev_begin(2);
+  if ((st = h->cuda(launch_fw_dataflow_sharded<T>(ranks.data(), (int)ranks.size(), P, nb, h->ld, h->d_flag, delay,
+                                                  h->stream),
+                    "fw_dataflow_sharded")))
+    return st;
+  h->ev_end((double)h->n_pad * h->n_pad * h->n_pad / (h->virt ? 1 : P));
+  return APSP_OK;
+}
+
+// NCCL ranks: this rank's shard work buffer (plain cudaMalloc, exportable through CUDA
+// IPC) and every peer's, mapped once per handle: the 64-B IPC handles are all-gathered
+// over the communicator, then every rank reports whether it could open all of them
+// (all-reduce min). If any rank could not (no P2P path between the GPUs), every rank
+// keeps the launch-per-phase schedule with NCCL broadcasts (h->sh_disabled).
+template <typename T>
+static apsp_status prepare_sharded_peers(Handle* h) {
+  if (h->sh_ipc_open || h->sh_disabled) return APSP_OK;
+  const int nb = (int)(h->n_pad / h->b), P = h->world, nl = nb / P;
+  const long long wb = fw_dataflow_work_bytes(nb, nl, sizeof(T));
+  apsp_status st;
+  if (h->sh_work.empty()) {
+    void* w = nullptr;
+    if ((st = h->cuda(cudaMalloc(&w, wb), "cudaMalloc dataflow shard"))) return st;
+    h->sh_work.push_back(w);
+    h->device_bytes += wb;
+  }
+  h->sh_peer[h->rank] = h->sh_work[0];
+  if (P == 1) {
+    h->sh_ipc_open = true;
+    return APSP_OK;
+  }
+  struct Msg {
+    cudaIpcMemHandle_t hd;
+    int ok;
+    int pad[15];
+  };
+  Msg mine;
+  memset(&mine, 0, sizeof(mine));
+  mine.ok = cudaIpcGetMemHandle(&mine.hd, h->sh_work[0]) == cudaSuccess;
+  cudaGetLastError();
+  char* dbuf = nullptr;
+  if ((st = h->cuda(cudaMalloc(&dbuf, (size_t)(P + 1) * sizeof(Msg)), "cudaMalloc ipc"))) return st;
+  std::vector<Msg> all(P);
+  ncclComm_t comm = static_cast<ncclComm_t>(h->comm);
+  Msg* dmsg = reinterpret_cast<Msg*>(dbuf);
+  int* dok = reinterpret_cast<int*>(dbuf + (size_t)P * sizeof(Msg));
+  cudaError_t ce = cudaMemcpyAsync(dmsg + h->rank, &mine, sizeof(mine), cudaMemcpyHostToDevice, h->stream);
+  ncclResult_t r = ncclSuccess;
+  if (ce == cudaSuccess) r = ncclAllGather(dmsg + h->rank, dmsg, sizeof(Msg), ncclUint8, comm, h->stream);
+  if (ce == cudaSuccess && r == ncclSuccess)
+    ce = cudaMemcpyAsync(all.data(), dmsg, (size_t)P * sizeof(Msg), cudaMemcpyDeviceToHost, h->stream);
+  if (ce == cudaSuccess) ce = cudaStreamSynchronize(h->stream);
+  int ok = 1;
+  if (ce == cudaSuccess && r == ncclSuccess) {
+    for (int e = 0; e < P; ++e) ok &= all[e].ok;
+    for (int e = 0; e < P && ok; ++e) {
+      if (e == h->rank) continue;
+      if (cudaIpcOpenMemHandle(&h->sh_peer[e], all[e].hd, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+        cudaGetLastError();
+        h->sh_peer[e] = nullptr;
+        ok = 0;
+      }
+    }
+    ce = cudaMemcpyAsync(dok, &ok, sizeof(int), cudaMemcpyHostToDevice, h->stream);
+    if (ce == cudaSuccess) r = ncclAllReduce(dok, dok, 1, ncclInt32, ncclMin, comm, h->stream);
+    if (ce == cudaSuccess && r == ncclSuccess) ce = cudaMemcpyAsync(&ok, dok, sizeof(int), cudaMemcpyDeviceToHost, h->stream);
+    if (ce == cudaSuccess) ce = cudaStreamSynchronize(h->stream);
+  }
+  cudaFree(dbuf);
+  if (r != ncclSuccess) return h->fail(APSP_ENCCL, "IPC handle exchange: %s", ncclGetErrorString(r));
+  if ((st = h->cuda(ce, "IPC handle exchange"))) return st;
+  if (!ok) {
+    for (int e = 0; e < P; ++e)
+      if (e != h->rank && h->sh_peer[e]) cudaIpcCloseMemHandle(h->sh_peer[e]);
+    for (auto& p : h->sh_peer) p = nullptr;
+    h->sh_disabled = true;
+    return APSP_OK;
+  }
+  h->sh_ipc_open = true;
+  return APSP_OK;
+}
+
 apsp_status run_incore_rounds(Handle* h, long long k0, long long k1) {
   if (h->world == 1 && !h->use_comm && !h->virt && h->dataflow && k0 == 0 && k1 == h->n_pad / h->b)
     return h->dtype == APSP_I32 ? run_dataflow<int>(h) : run_dataflow<float>(h);
+  if ((h->virt || h->use_comm) && h->dataflow && h->world <= 8 && k0 == 0 && k1 == h->n_pad / h->b) {
+    apsp_status st;
+    if (!h->virt &&
+        (st = h->dtype == APSP_I32 ? prepare_sharded_peers<int>(h) : prepare_sharded_peers<float>(h)))
+      return st;
+    if (!h->sh_disabled)
+      return h->dtype == APSP_I32 ? run_dataflow_sharded<int>(h) : run_dataflow_sharded<float>(h);
+  }
   if (h->world == 1 && !h->use_comm) {  // single GPU: the whole closure, with lookahead
     return h->dtype == APSP_I32
                ? fw_closure<int>(h, static_cast<int*>(h->shards[0].D), h->ld, h->n_pad, k0, k1, h->stream)

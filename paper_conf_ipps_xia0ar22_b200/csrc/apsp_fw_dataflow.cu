@@ -59,6 +59,8 @@
 #include <cuda_runtime.h>
 #include <climits>
 #include <cstdint>
+#include <cstring>
+#include <vector>
 
 namespace apsp {
 namespace {
@@ -97,32 +99,42 @@ template <> struct DV<float> {
 // named barrier of one 256-thread group (id 0 is __syncthreads)
 __device__ __forceinline__ void gbar(int g) { asm volatile("bar.sync %0, %1;" ::"r"(g + 1), "r"(GNT) : "memory"); }
 
+constexpr int kMaxRanks = 8;  // one node
+
 template <typename T>
 struct DFArgs {
-  T* D;            // n_pad x n_pad, row-major, ld
+  T* D;            // this rank's rows (all n_pad rows on one GPU), row-major, ld
   long long ld;
-  int nb;
-  T* pbuf;         // 2 x (2nb+1) tiles of 128x128: [p][0] diagonal, [p][1+j] row panel, [p][1+nb+i] column panel
-  int* ver;        // nb*nb
+  int nb;          // tile rows / columns of the whole matrix
+  T* pbuf;         // 2 parities x (2 + nb + nl) tiles of 128x128: [0] diagonal, [1] its transpose,
+                   // [2 + j] row panel, [2 + nb + il] column panel of local tile row il (transposed)
+  int* ver;        // [nl][nb] rounds applied to each local tile
   int* diagready;  // [2]
   int* rowready;   // [2][nb]
-  int* colready;   // [2][nb]
+  int* colready;   // [2][nl]
   int* done2;      // [nb]
   int* done3;      // [nb]
   unsigned long long* counter;
   int* negflag;
-  long long total;   // nb^3 tasks
+  long long total;   // tasks in this rank's queue (nb^3 on one GPU)
   long long delay;   // G3R tasks placed before G2 in a segment
   long long stagger; // clock cycles group 1 waits before its first task
   unsigned long long* prof;  // optional [CTAs x GROUPS x 8] cycle counters (thread 0 of each group)
+  // 1-D block-row shard over P ranks (sharded kernel only; P = 1, q = 0, nl = nb otherwise):
+  // rank q owns tile rows [q*nl, (q+1)*nl); the owner of round k writes the closed diagonal
+  // block and the row panel straight into every rank's pbuf (peer stores over NVLink) and
+  // raises their flags; owners read every rank's done2/done3 before reusing a parity.
+  int P, q, nl;
+  const long long* segstart;  // [nb + 1] queue position of segment k (k = nb: the last round's phase 3)
+  T* peer_pbuf[kMaxRanks];    // pbuf of every rank (peer_pbuf[q] == pbuf)
+  int* peer_base[kMaxRanks];  // flag block of every rank (== its counter address)
 };
-
 
 // panel copies of round k (parity k % 2), 128x128 tiles with ld 128:
 //   D = A(k,k) closed, D^T, row panel A(k,j), column panel A(i,k) transposed
 template <typename T>
 __device__ __forceinline__ T* pb_diag(const DFArgs<T>& a, int k) {
-  return a.pbuf + (long long)(k & 1) * (2 * a.nb + 2) * TILE_ELEMS;
+  return a.pbuf + (long long)(k & 1) * (2 + a.nb + a.nl) * TILE_ELEMS;
 }
 template <typename T>
 __device__ __forceinline__ T* pb_diagT(const DFArgs<T>& a, int k) {
@@ -133,16 +145,187 @@ __device__ __forceinline__ T* pb_row(const DFArgs<T>& a, int k, int j) {
   return pb_diag(a, k) + (long long)(2 + j) * TILE_ELEMS;
 }
 template <typename T>
-__device__ __forceinline__ T* pb_colT(const DFArgs<T>& a, int k, int i) {
-  return pb_diag(a, k) + (long long)(2 + a.nb + i) * TILE_ELEMS;
+__device__ __forceinline__ T* pb_colT(const DFArgs<T>& a, int k, int i) {  // i: global tile row (local to q)
+  return pb_diag(a, k) + (long long)(2 + a.nb + (i - a.q * a.nl)) * TILE_ELEMS;
+}
+// the same address in rank r's flag block / pbuf
+template <typename T>
+__device__ __forceinline__ int* peer_flag(const DFArgs<T>& a, int r, const int* local) {
+  return a.peer_base[r] + (local - reinterpret_cast<const int*>(a.counter));
+}
+template <typename T>
+__device__ __forceinline__ T* peer_pb(const DFArgs<T>& a, int r, const T* local) {
+  return a.peer_pbuf[r] + (local - a.pbuf);
 }
 
+// ---- sharded queue (rank q of P): segments as in decode() (apsp_df_common.cuh), restricted to
+// the local tile rows; segment starts come from the host (fw_dataflow_sharded_segments).
+//   pre        P1(0) if q owns row 0
+//   seg(k)     [G3R(k-1)[0:d], G2(k), G3R(k-1)[d:], G3Lx(k)]   (k >= 1 parts exist only if defined)
+//   tail       round nb-1's phase 3
+//   G2(k)      owner: P2R(k, j != k); every rank: P2C(k, local i != k)
+//   G3Lx(k)    owner of k+1: (k+1,k+1), P1(k+1), row k+1 (j not in {k,k+1}), local column k+1;
+//              others: local column k+1 (i != k)
+//   G3R(k)     local rows not in {k,k+1} x columns not in {k,k+1}, banded
+// Every cross-rank dependency points to an earlier segment or, inside segment k, from G3Lx(k)
+// to G2(k): with the same part order on every rank no cycle exists.
+__device__ __forceinline__ int loc_of(int k, int q, int nl) { return (k / nl) == q ? k - q * nl : -1; }
+__device__ __forceinline__ int lrow(int x, int e0, int e1) {  // x-th local row skipping local e0, e1 (-1 none)
+  const int s0 = (e0 >= 0 && e1 >= 0) ? min(e0, e1) : (e0 >= 0 ? e0 : e1);
+  const int s1 = (e0 >= 0 && e1 >= 0) ? max(e0, e1) : -1;
+  return skip3(x, s0, s1, -1);
+}
+__device__ __forceinline__ long long g3r_size_sh(int nb, int nl, int q, int k) {
+  const int l0 = loc_of(k, q, nl) >= 0, l1 = loc_of(k + 1, q, nl) >= 0;
+  return (long long)(nl - l0 - l1) * (nb - 2);
+}
+__device__ __forceinline__ long long g2_size_sh(int nb, int nl, int q, int k) {
+  const int l0 = loc_of(k, q, nl) >= 0;
+  return (long long)l0 * (nb - 1) + (nl - l0);
+}
+__device__ Task decode_sh(long long g, int nb, int nl, int q, long long delay, const long long* segstart) {
+  Task t;
+  const int base = q * nl;
+  if (g < segstart[0]) { t.type = T_P1; t.k = 0; t.i = t.j = 0; return t; }
+  int lo = 0, hi = nb;  // largest k with segstart[k] <= g
+  while (lo < hi) {
+    const int mid = (lo + hi + 1) >> 1;
+    if (segstart[mid] <= g) lo = mid; else hi = mid - 1;
+  }
+  const int k = lo;
+  long long x = g - segstart[k];
+  t.type = T_P3;
+  if (k == nb) {  // tail: round nb-1, local rows != nb-1 x columns != nb-1
+    const int kl = loc_of(nb - 1, q, nl);
+    int r, c;
+    banded(x, nl - (kl >= 0), nb - 1, r, c);
+    t.k = nb - 1; t.i = base + lrow(r, kl, -1); t.j = c;
+    return t;
+  }
+  auto g3r = [&](int kk, long long y) {  // G3R(kk)
+    const int l0 = loc_of(kk, q, nl), l1 = loc_of(kk + 1, q, nl);
+    int r, c;
+    banded(y, nl - (l0 >= 0) - (l1 >= 0), nb - 2, r, c);
+    Task u;
+    u.type = T_P3; u.k = kk; u.i = base + lrow(r, l0, l1); u.j = skip3(c, kk, kk + 1, -1);
+    return u;
+  };
+  long long r3 = 0, d = 0;
+  if (k >= 1) {
+    r3 = g3r_size_sh(nb, nl, q, k - 1);
+    d = delay < r3 ? delay : r3;
+    if (x < d) return g3r(k - 1, x);
+    x -= d;
+  }
+  const long long n2 = g2_size_sh(nb, nl, q, k);
+  if (x < n2) {
+    const int l0 = loc_of(k, q, nl);
+    t.k = k;
+    if (l0 >= 0) {
+      if (x < nb - 1) { t.type = T_P2R; t.i = k; t.j = skip3((int)x, k, -1, -1); return t; }
+      x -= nb - 1;
+    }
+    t.type = T_P2C; t.i = base + lrow((int)x, l0, -1); t.j = k;
+    return t;
+  }
+  x -= n2;
+  if (k >= 1) {
+    if (x < r3 - d) return g3r(k - 1, d + x);
+    x -= r3 - d;
+  }
+  // G3Lx(k), k <= nb-2
+  const int l0 = loc_of(k, q, nl), l1 = loc_of(k + 1, q, nl);
+  t.k = k;
+  if (l1 >= 0) {
+    if (x == 0) { t.i = k + 1; t.j = k + 1; return t; }
+    if (x == 1) { t.type = T_P1; t.k = k + 1; t.i = t.j = k + 1; return t; }
+    x -= 2;
+    if (x < nb - 2) { t.i = k + 1; t.j = skip3((int)x, k, k + 1, -1); return t; }
+    x -= nb - 2;
+    t.i = base + lrow((int)x, l0, l1); t.j = k + 1;
+    return t;
+  }
+  t.i = base + lrow((int)x, l0, -1); t.j = k + 1;
+  return t;
+}
+
+// completed P2 / P3 tasks rank r runs in round k
+__device__ __forceinline__ int cnt2_sh(int nb, int nl, int r, int k) {
+  const int l0 = (k / nl) == r;
+  return l0 * (nb - 1) + (nl - l0);
+}
+__device__ __forceinline__ int cnt3_sh(int nb, int nl, int r, int k) {
+  const int l0 = (k / nl) == r;
+  return (nl - l0) * (nb - 1);
+}
+
+// Dependencies of task t on rank q (one thread). Local flags, some of them written by the
+// owner of the round over NVLink (diagready, rowready), plus for the owner's P1 / P2R the
+// done counters of round k-2 on every rank (parity reuse of the panels it broadcasts).
+template <typename T>
+__device__ bool deps_met_sh(const DFArgs<T>& a, const Task& t) {
+  const int nb = a.nb, nl = a.nl, k = t.k, p = k & 1;
+  if (ld_relaxed_sys(a.ver + (long long)(t.i - a.q * nl) * nb + t.j) < k) return false;
+  if (t.type == T_P3) {
+    if (ld_relaxed_sys(a.rowready + p * nb + t.j) < k + 1) return false;
+    if (ld_relaxed_sys(a.colready + p * nl + (t.i - a.q * nl)) < k + 1) return false;
+  } else if (t.type == T_P2C) {
+    if (ld_relaxed_sys(a.diagready + p) < k + 1) return false;
+    if (k >= 2 && ld_relaxed_sys(a.done3 + k - 2) < cnt3_sh(nb, nl, a.q, k - 2)) return false;
+  } else {
+    if (t.type == T_P2R && ld_relaxed_sys(a.diagready + p) < k + 1) return false;
+    if (k >= 2) {
+      for (int r = 0; r < a.P; ++r) {
+        const int* f = t.type == T_P1 ? a.done2 + k - 2 : a.done3 + k - 2;
+        const int need = t.type == T_P1 ? cnt2_sh(nb, nl, r, k - 2) : cnt3_sh(nb, nl, r, k - 2);
+        if (ld_relaxed_sys(peer_flag(a, r, f)) < need) return false;
+      }
+    }
+  }
+  asm volatile("fence.acq_rel.sys;" ::: "memory");
+  return true;
+}
+
+// Publish task t on rank q (one thread, after the group barrier that follows its stores,
+// including the peer stores of P1 / P2R): a system-scope fence, then the flags.
+template <typename T>
+__device__ void signal_done_sh(const DFArgs<T>& a, const Task& t) {
+  const int nb = a.nb, nl = a.nl, k = t.k, p = k & 1;
+  asm volatile("fence.acq_rel.sys;" ::: "memory");
+  st_relaxed_sys(a.ver + (long long)(t.i - a.q * nl) * nb + t.j, k + 1);
+  switch (t.type) {
+    case T_P1:
+      for (int r = 0; r < a.P; ++r) st_relaxed_sys(peer_flag(a, r, a.diagready + p), k + 1);
+      break;
+    case T_P2R:
+      for (int r = 0; r < a.P; ++r) st_relaxed_sys(peer_flag(a, r, a.rowready + p * nb + t.j), k + 1);
+      red_relaxed_sys_add(a.done2 + k, 1);
+      break;
+    case T_P2C:
+      st_relaxed_sys(a.colready + p * nl + (t.i - a.q * nl), k + 1);
+      red_relaxed_sys_add(a.done2 + k, 1);
+      break;
+    default: red_relaxed_sys_add(a.done3 + k, 1); break;
+  }
+}
+
+template <bool SH, typename T>
+__device__ __forceinline__ Task decode_any(const DFArgs<T>& a, long long g) {
+  if constexpr (SH) return decode_sh(g, a.nb, a.nl, a.q, a.delay, a.segstart);
+  else return decode(g, a.nb, a.delay);
+}
+template <bool SH, typename T>
+__device__ __forceinline__ bool deps_any(const DFArgs<T>& a, const Task& t) {
+  if constexpr (SH) return deps_met_sh(a, t);
+  else return deps_met(a, t);
+}
 
 // Phase 1 inside a group: in-place FW closure of one 128x128 tile (the same
 // register blocking as phase1_kernel in apsp_kernels.cu); result also to out2.
+// Sharded kernel: `peers` (npeer entries) also receive D at the same offset (peer stores).
 template <typename T>
 __device__ __noinline__ void group_phase1(T* tile, long long ld, T* out2, T* out2t, int* negflag, T* scratch, int g,
-                                         int gtid) {
+                                         int gtid, T* const* peers = nullptr, int npeer = 0) {
   using V4 = typename DV<T>::V4;
   T* rowbuf = scratch;            // [2][128]
   T* colbuf = scratch + 2 * 128;  // [2][128]
@@ -205,6 +388,10 @@ __device__ __noinline__ void group_phase1(T* tile, long long ld, T* out2, T* out
     *reinterpret_cast<V4*>(tile + r * ld + 64 + tx * 4) = v1;
     *reinterpret_cast<V4*>(out2 + r * BN + tx * 4) = v0;
     *reinterpret_cast<V4*>(out2 + r * BN + 64 + tx * 4) = v1;
+    for (int e = 0; e < npeer; ++e) {
+      *reinterpret_cast<V4*>(peers[e] + r * BN + tx * 4) = v0;
+      *reinterpret_cast<V4*>(peers[e] + r * BN + 64 + tx * 4) = v1;
+    }
   }
 #pragma unroll
   for (int j = 0; j < 8; ++j) {  // D^T: column c of the block = 4 + 4 consecutive rows
@@ -229,6 +416,7 @@ struct GDesc {
   int lda, ldb, ldc;
   int a_rows, c2t;
   int bulk;  // 1: A and B chunks are contiguous 16 KB blocks (panel copies): one thread copies them
+  int bcast; // sharded P2R: Cout2 also goes to every other rank's pbuf (same offset)
 };
 
 
@@ -247,11 +435,12 @@ struct Slot {
 template <typename T>
 __device__ void fill_desc(const DFArgs<T>& a, const Task& tk, GDesc<T>& d) {
   const int k = tk.k;
-  T* const tile = a.D + (long long)tk.i * BM * a.ld + (long long)tk.j * BN;
+  T* const tile = a.D + (long long)(tk.i - a.q * a.nl) * BM * a.ld + (long long)tk.j * BN;
   d.Cin = tile; d.Cout = tile; d.ldc = (int)a.ld;
-  d.a_rows = 0; d.c2t = 0; d.bulk = 0;
+  d.a_rows = 0; d.c2t = 0; d.bulk = 0; d.bcast = 0;
   if (tk.type == T_P2R) {         // A(k,j) = D (x) A(k,j)
     d.A = pb_diagT(a, k); d.lda = BM; d.B = tile; d.ldb = (int)a.ld; d.Cout2 = pb_row(a, k, tk.j);
+    d.bcast = a.P > 1;
   } else if (tk.type == T_P2C) {  // A(i,k) = A(i,k) (x) D; the copy goes to the transposed column panel
     d.A = tile; d.lda = (int)a.ld; d.a_rows = 1; d.B = pb_diag(a, k); d.ldb = BN;
     d.Cout2 = pb_colT(a, k, tk.i); d.c2t = 1;
@@ -274,7 +463,7 @@ __device__ void fill_desc(const DFArgs<T>& a, const Task& tk, GDesc<T>& d) {
 #else
 #define DF_MP_INLINE __noinline__
 #endif
-template <typename T>
+template <bool SH, typename T>
 __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigned full0, unsigned empty0, unsigned c0,
                                            int gtid, int g, const DFArgs<T>* args, long long nxt,
                                            Slot<T>* ns) {
@@ -369,10 +558,10 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
     if (c == 1 && gtid == SCH) {  // the next task's slot
       ns->t = nxt;
       if (nxt < args->total) {
-        const Task tn = decode(nxt, args->nb, args->delay);
+        const Task tn = decode_any<SH>(*args, nxt);
         ns->tk = tn;
         if (tn.type != T_P1) fill_desc(*args, tn, ns->d);
-        ns->ready = deps_met(*args, tn) ? 1 : 0;
+        ns->ready = deps_any<SH>(*args, tn) ? 1 : 0;
       }
     }
     mb_wait(full0 + 8 * s, (G / STAGES) & 1);
@@ -460,6 +649,16 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
       if (Cout2 && !d->c2t) {
         *reinterpret_cast<V4*>(Cout2 + r * BN + tx * 4) = v0;
         *reinterpret_cast<V4*>(Cout2 + r * BN + 64 + tx * 4) = v1;
+        if constexpr (SH) {
+          if (d->bcast) {  // the row panel tile into every other rank's pbuf (NVLink peer stores)
+            for (int e = 0; e < args->P; ++e) {
+              if (e == args->q) continue;
+              T* const o = peer_pb(*args, e, Cout2);
+              *reinterpret_cast<V4*>(o + r * BN + tx * 4) = v0;
+              *reinterpret_cast<V4*>(o + r * BN + 64 + tx * 4) = v1;
+            }
+          }
+        }
       }
     }
     if (Cout2 && d->c2t) {  // transposed copy: column c of the block = 4 + 4 consecutive rows
@@ -476,11 +675,20 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
   }
 }
 
+// Launch parameters: one argument block per rank run by this launch (nv > 1 only for
+// virtual ranks, i.e. several shards on one GPU in one launch: CTA b serves rank b % nv).
 template <typename T>
-__global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(const __grid_constant__ DFArgs<T> a) {
+struct DFLaunch {
+  DFArgs<T> r[kMaxRanks];
+  int nv;
+};
+
+template <bool SH, typename T>
+__global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(const __grid_constant__ DFLaunch<T> L) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ __align__(8) unsigned long long bars[GROUPS][2 * STAGES];
   __shared__ Slot<T> slots[GROUPS][2];
+  const DFArgs<T>& a = L.r[SH ? blockIdx.x % L.nv : 0];
   const int g = threadIdx.x / GNT, gtid = threadIdx.x % GNT;
   T* const stage0 = reinterpret_cast<T*>(smem_raw) + g * STAGES * STAGE_ELEMS;
   const unsigned full0 = saddr(&bars[g][0]), empty0 = full0 + 8 * STAGES;
@@ -492,7 +700,7 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (gtid == SCH) {
-    if ((GROUPS > 1 ? g > 0 : blockIdx.x >= gridDim.x / 2) && a.stagger > 0) {  // half the groups start later
+    if (!SH && (GROUPS > 1 ? g > 0 : blockIdx.x >= gridDim.x / 2) && a.stagger > 0) {  // half the groups start later
       const long long t0 = clock64();
       while (clock64() - t0 < a.stagger) __nanosleep(256);
     }
@@ -500,7 +708,7 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
     s0.t = (long long)atomicAdd(a.counter, 1ull);
     s0.ready = 0;
     if (s0.t < a.total) {
-      s0.tk = decode(s0.t, a.nb, a.delay);
+      s0.tk = decode_any<SH>(a, s0.t);
       if (s0.tk.type != T_P1) fill_desc(a, s0.tk, s0.d);
     }
   }
@@ -515,8 +723,14 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
     if (t >= a.total) break;
     const Task tk = S.tk;
     if (!S.ready) {  // uniform: the slot was published by the last barrier
-      if (gtid == SCH && !deps_met(a, tk)) {
-        while (!deps_met(a, tk)) __nanosleep(64);
+      if (gtid == SCH && !deps_any<SH>(a, tk)) {
+        const long long w0 = clock64();
+        while (!deps_any<SH>(a, tk)) {
+          __nanosleep(64);
+          // sharded: a peer that never delivers (a dead rank) must not hang the GPU: after
+          // ~30 s of waiting the kernel traps (the launch fails, the handle reports APSP_ECUDA)
+          if (SH && clock64() - w0 > 60000000000ll) __trap();
+        }
         pr[5]++;
       }
       gbar(g);
@@ -526,18 +740,26 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
     const long long tc1 = clock64();
     pr[0] += tc1 - tc0;
     if (tk.type == T_P1) {
-      T* const tile = a.D + (long long)tk.i * BM * a.ld + (long long)tk.j * BN;
-      group_phase1<T>(tile, a.ld, pb_diag(a, tk.k), pb_diagT(a, tk.k), a.negflag, stage0, g, gtid);
+      T* const tile = a.D + (long long)(tk.i - a.q * a.nl) * BM * a.ld + (long long)tk.j * BN;
+      if constexpr (SH) {  // D also into every other rank's pbuf
+        T* peers[kMaxRanks];
+        int np = 0;
+        for (int e = 0; e < a.P; ++e)
+          if (e != a.q) peers[np++] = peer_pb(a, e, pb_diag(a, tk.k));
+        group_phase1<T>(tile, a.ld, pb_diag(a, tk.k), pb_diagT(a, tk.k), a.negflag, stage0, g, gtid, peers, np);
+      } else {
+        group_phase1<T>(tile, a.ld, pb_diag(a, tk.k), pb_diagT(a, tk.k), a.negflag, stage0, g, gtid);
+      }
       if (gtid == SCH) {
         N->t = nxt;
         if (nxt < a.total) {
-          N->tk = decode(nxt, a.nb, a.delay);
+          N->tk = decode_any<SH>(a, nxt);
           N->ready = 0;
           if (N->tk.type != T_P1) fill_desc(a, N->tk, N->d);
         }
       }
     } else {
-      group_minplus<T>(&S.d, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N);
+      group_minplus<SH, T>(&S.d, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N);
       chunk += BM / BK;
     }
     const long long tc2 = clock64();
@@ -547,7 +769,10 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
     gbar(g);  // every thread's stores of this task are issued; the next slot is published
     // published right away by the SIG thread (its warp absorbs the fence; measured
     // better than deferring it under the next task's first loads)
-    if (gtid == SIG) signal_done(a, tk);
+    if (gtid == SIG) {
+      if constexpr (SH) signal_done_sh(a, tk);
+      else signal_done(a, tk);
+    }
     tc0 = clock64();
     pr[2] += tc0 - tc2;
   }
@@ -559,48 +784,133 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
 
 }  // namespace
 
+// Work-buffer layout of one rank: pbuf (2 parities x (2 + nb + nl) tiles), then the
+// flag block, then (sharded) the nb + 1 segment starts.
+template <typename T>
+static void df_layout(DFArgs<T>& a, void* work, int nb, int nl) {
+  a.nb = nb;
+  a.nl = nl;
+  a.pbuf = static_cast<T*>(work);
+  char* const fb = static_cast<char*>(work) + fw_dataflow_pbuf_bytes(nb, nl, sizeof(T));
+  int* f = reinterpret_cast<int*>(fb);
+  a.counter = reinterpret_cast<unsigned long long*>(f); f += 2;  // first: 8-byte aligned
+  a.ver = f; f += (long long)nl * nb;
+  a.diagready = f; f += 2;
+  a.rowready = f; f += 2 * nb;
+  a.colready = f; f += 2 * nl;
+  a.done2 = f; f += nb;
+  a.done3 = f; f += nb;
+  a.segstart = reinterpret_cast<const long long*>(fb + fw_dataflow_flag_bytes(nb, nl));
+}
+
 template <typename T>
 cudaError_t launch_fw_dataflow(T* D, long long ld, int nb, void* work, int* negflag, long long delay,
                                long long stagger, cudaStream_t s, unsigned long long* prof) {
   if (nb <= 0) return cudaSuccess;
   const int smem = GROUPS * STAGES * STAGE_ELEMS * (int)sizeof(T);
-  cudaError_t e = cudaFuncSetAttribute(fw_dataflow_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaError_t e = cudaFuncSetAttribute(fw_dataflow_kernel<false, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return e;
   int dev = 0, sms = 0;
   if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
   if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
-  DFArgs<T> a;
-  a.D = D; a.ld = ld; a.nb = nb;
-  a.pbuf = static_cast<T*>(work);
-  int* f = reinterpret_cast<int*>(static_cast<char*>(work) + fw_dataflow_pbuf_bytes(nb, sizeof(T)));
-  a.counter = reinterpret_cast<unsigned long long*>(f); f += 2;  // first: 8-byte aligned
-  a.ver = f; f += (long long)nb * nb;
-  a.diagready = f; f += 2;
-  a.rowready = f; f += 2 * nb;
-  a.colready = f; f += 2 * nb;
-  a.done2 = f; f += nb;
-  a.done3 = f; f += nb;
+  DFLaunch<T> L;
+  memset(&L, 0, sizeof(L));
+  L.nv = 1;
+  DFArgs<T>& a = L.r[0];
+  df_layout(a, work, nb, nb);
+  a.D = D; a.ld = ld;
   a.negflag = negflag;
   a.total = (long long)nb * nb * nb;
   a.delay = delay;
   a.stagger = stagger;
   a.prof = prof;
-  e = cudaMemsetAsync(a.counter, 0, fw_dataflow_flag_bytes(nb), s);
+  a.P = 1; a.q = 0;
+  a.peer_pbuf[0] = a.pbuf;
+  a.peer_base[0] = reinterpret_cast<int*>(a.counter);
+  e = cudaMemsetAsync(a.counter, 0, fw_dataflow_flag_bytes(nb, nb), s);
   if (e != cudaSuccess) return e;
   long long grid = (long long)sms * CTAS_PER_SM;
   if (grid > a.total) grid = a.total;
-  fw_dataflow_kernel<T><<<(unsigned)grid, GNT * GROUPS, smem, s>>>(a);
+  fw_dataflow_kernel<false, T><<<(unsigned)grid, GNT * GROUPS, smem, s>>>(L);
   return cudaGetLastError();
 }
 
-long long fw_dataflow_pbuf_bytes(int nb, size_t elem) {
-  return 2ll * (2 * nb + 2) * TILE_ELEMS * (long long)elem;  // (kept a multiple of 8 bytes)
-}
-long long fw_dataflow_flag_bytes(int nb) { return ((long long)nb * nb + 6ll * nb + 4) * 4; }
-long long fw_dataflow_work_bytes(int nb, size_t elem) {
-  return fw_dataflow_pbuf_bytes(nb, elem) + fw_dataflow_flag_bytes(nb);
+// Queue of rank q (segment starts and length): the host mirror of decode_sh.
+long long fw_dataflow_sharded_segments(int nb, int nl, int q, long long* segstart) {
+  auto loc = [&](int k) { return (k / nl) == q ? 1 : 0; };
+  long long pos = loc(0);
+  for (int k = 0; k < nb; ++k) {
+    segstart[k] = pos;
+    long long sz = (long long)loc(k) * (nb - 1) + (nl - loc(k));          // G2(k)
+    if (k >= 1) sz += (long long)(nl - loc(k - 1) - loc(k)) * (nb - 2);    // G3R(k-1)
+    if (k <= nb - 2)                                                         // G3Lx(k)
+      sz += loc(k + 1) ? 2 + (nb - 2) + (nl - 1 - loc(k)) : (nl - loc(k));
+    pos += sz;
+  }
+  segstart[nb] = pos;
+  return pos + (long long)(nl - loc(nb - 1)) * (nb - 1);  // + the last round's phase 3
 }
 
+template <typename T>
+cudaError_t launch_fw_dataflow_sharded(const DFShard* ranks, int nv, int P, int nb, long long ld, int* negflag,
+                                       long long delay, cudaStream_t s) {
+  if (nb <= 0 || nv < 1 || nv > kMaxRanks || P < 1 || P > kMaxRanks || nb % P) return cudaErrorInvalidValue;
+  const int nl = nb / P;
+  const int smem = GROUPS * STAGES * STAGE_ELEMS * (int)sizeof(T);
+  cudaError_t e = cudaFuncSetAttribute(fw_dataflow_kernel<true, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return e;
+  int dev = 0, sms = 0;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+  if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
+  DFLaunch<T> L;
+  memset(&L, 0, sizeof(L));
+  L.nv = nv;
+  std::vector<long long> seg((size_t)nb + 1);
+  for (int v = 0; v < nv; ++v) {
+    DFArgs<T>& a = L.r[v];
+    const DFShard& sh = ranks[v];
+    df_layout(a, sh.work, nb, nl);
+    a.D = static_cast<T*>(sh.D); a.ld = ld;
+    a.negflag = negflag;
+    a.P = P; a.q = sh.rank;
+    a.total = fw_dataflow_sharded_segments(nb, nl, sh.rank, seg.data());
+    a.delay = delay;
+    a.stagger = 0;
+    a.prof = nullptr;
+    for (int r = 0; r < P; ++r) {
+      a.peer_pbuf[r] = static_cast<T*>(sh.peer_work[r]);
+      a.peer_base[r] = reinterpret_cast<int*>(static_cast<char*>(sh.peer_work[r]) +
+                                              fw_dataflow_pbuf_bytes(nb, nl, sizeof(T)));
+    }
+    // blocking copy: `seg` is reused for the next rank (a few KB)
+    if ((e = cudaMemcpyAsync(const_cast<long long*>(a.segstart), seg.data(), seg.size() * sizeof(long long),
+                             cudaMemcpyHostToDevice, s)) != cudaSuccess)
+      return e;
+    if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return e;
+  }
+  long long grid = (long long)sms * CTAS_PER_SM;
+  grid -= grid % nv;
+  fw_dataflow_kernel<true, T><<<(unsigned)grid, GNT * GROUPS, smem, s>>>(L);
+  return cudaGetLastError();
+}
+
+long long fw_dataflow_pbuf_bytes(int nb, int nl, size_t elem) {
+  return 2ll * (2 + nb + nl) * TILE_ELEMS * (long long)elem;  // (kept a multiple of 8 bytes)
+}
+long long fw_dataflow_flag_bytes(int nb, int nl) {  // rounded to 16 B: the segment starts (int64) follow
+  return ((((long long)nl * nb + 4ll * nb + 2ll * nl + 4) * 4 + 15) / 16) * 16;
+}
+long long fw_dataflow_work_bytes(int nb, int nl, size_t elem) {
+  return fw_dataflow_pbuf_bytes(nb, nl, elem) + fw_dataflow_flag_bytes(nb, nl) + 8ll * (nb + 1);
+}
+long long fw_dataflow_pbuf_bytes(int nb, size_t elem) { return fw_dataflow_pbuf_bytes(nb, nb, elem); }
+long long fw_dataflow_flag_bytes(int nb) { return fw_dataflow_flag_bytes(nb, nb); }
+long long fw_dataflow_work_bytes(int nb, size_t elem) { return fw_dataflow_work_bytes(nb, nb, elem); }
+
+template cudaError_t launch_fw_dataflow_sharded<int>(const DFShard*, int, int, int, long long, int*, long long,
+                                                     cudaStream_t);
+template cudaError_t launch_fw_dataflow_sharded<float>(const DFShard*, int, int, int, long long, int*, long long,
+                                                       cudaStream_t);
 template cudaError_t launch_fw_dataflow<int>(int*, long long, int, void*, int*, long long, long long, cudaStream_t,
                                              unsigned long long*);
 template cudaError_t launch_fw_dataflow<float>(float*, long long, int, void*, int*, long long, long long,

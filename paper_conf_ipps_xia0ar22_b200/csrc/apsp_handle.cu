@@ -177,7 +177,11 @@ apsp_status setup_device(Handle* h, const apsp_config& cfg) {
   g_minplus_variant = cfg.reserved[3];  // test hook: min-plus kernel variant (apsp_kernels.cuh)
   // reserved[4]: 0 = auto (the persistent dataflow kernel for int32; the launch-per-phase
   // schedule for fp32, measured faster there: DESIGN.md §5), 1 = launch-per-phase, 2 = dataflow
-  h->dataflow = cfg.reserved[4] == 2 || (cfg.reserved[4] == 0 && h->dtype == APSP_I32);
+  // Sharded placements (world > 1, virtual ranks, NCCL at world 1) default to the
+  // launch-per-phase schedule with NCCL broadcasts; reserved[4] = 2 selects the sharded
+  // dataflow kernel (peer stores of the pivot panels).
+  const bool sharded = h->world > 1 || cfg.reserved[2] == 1;
+  h->dataflow = cfg.reserved[4] == 2 || (cfg.reserved[4] == 0 && h->dtype == APSP_I32 && !sharded);
   h->df_delay = cfg.reserved[5];
   if (cfg.stream) {
     h->stream = static_cast<cudaStream_t>(cfg.stream);
@@ -345,6 +349,8 @@ void delete_handle(Handle* h) {
     if (h->d16) cudaFreeAsync(h->d16, h->stream);
     if (h->panel) cudaFreeAsync(h->panel, h->stream);
     if (h->df_work) cudaFreeAsync(h->df_work, h->stream);
+    if (h->virt)
+      for (void* w : h->sh_work) cudaFreeAsync(w, h->stream);
     h->d_base = h->panel = h->df_work = nullptr;
     h->d16 = nullptr;
     cudaStreamSynchronize(h->stream);
@@ -352,6 +358,11 @@ void delete_handle(Handle* h) {
   for (auto& te : h->events) {
     cudaEventDestroy(te.a);
     cudaEventDestroy(te.b);
+  }
+  if (!h->virt) {  // NCCL-rank shard buffer and the peers' buffers opened through CUDA IPC
+    for (int e = 0; e < 8; ++e)
+      if (h->sh_peer[e] && e != h->rank) cudaIpcCloseMemHandle(h->sh_peer[e]);
+    for (void* w : h->sh_work) cudaFree(w);
   }
   if (h->comm) ncclCommDestroy(static_cast<ncclComm_t>(h->comm));
   ooc_free(h);

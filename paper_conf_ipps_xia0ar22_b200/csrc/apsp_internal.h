@@ -87,6 +87,11 @@ struct Handle {
   bool dataflow = true;     // apsp_config.reserved[4] = 1 selects the launch-per-phase schedule
   long long df_delay = 0;   // reserved[5] (0 = auto)
   void* df_work = nullptr;
+  // sharded dataflow kernel (multi-GPU / virtual ranks): per-rank work buffers
+  std::vector<void*> sh_work;          // virtual ranks: one per shard (pool); NCCL ranks: this rank's (cudaMalloc, IPC)
+  void* sh_peer[8] = {};               // NCCL ranks: every rank's work buffer opened through CUDA IPC
+  bool sh_ipc_open = false;
+  bool sh_disabled = false;            // peer mapping failed on some rank: launch-per-phase + NCCL broadcasts
   // bookkeeping
   long long device_bytes = 0, host_bytes = 0;
   long long next_round = 0;

@@ -117,6 +117,27 @@ cudaError_t launch_fw_dataflow(T* D, long long ld, int nb, void* work, int* negf
 long long fw_dataflow_pbuf_bytes(int nb, size_t elem);
 long long fw_dataflow_flag_bytes(int nb);
 long long fw_dataflow_work_bytes(int nb, size_t elem);
+long long fw_dataflow_pbuf_bytes(int nb, int nl, size_t elem);
+long long fw_dataflow_flag_bytes(int nb, int nl);
+
+// The same kernel over a 1-D block-row shard (rank q of P owns tile rows
+// [q*nl, (q+1)*nl), nl = nb/P): the owner of round k stores the closed diagonal
+// block and the row panel straight into every rank's panel buffer (peer stores:
+// NVLink for other GPUs, plain stores for virtual ranks on one GPU) and raises
+// their flags, so no collective runs between rounds. `work` of each rank holds
+// fw_dataflow_work_bytes(nb, nl, elem) bytes at the same layout on every rank;
+// peer_work[r] is rank r's `work` as seen from this process. One launch runs the
+// nv ranks listed (nv = P: virtual ranks on one GPU; nv = 1: this process's rank).
+struct DFShard {
+  int rank;
+  void* D;                 // this rank's rows (rows_per_rank x ld)
+  void* work;              // == peer_work[rank]
+  void* peer_work[8];
+};
+long long fw_dataflow_work_bytes(int nb, int nl, size_t elem);
+template <typename T>
+cudaError_t launch_fw_dataflow_sharded(const DFShard* ranks, int nv, int P, int nb, long long ld, int* negflag,
+                                       long long delay, cudaStream_t s);
 
 // The packed int16 closure (R16) as one persistent dataflow launch
 // (apsp_fw_dataflow16.cu); `work` holds fw_dataflow16_work_bytes(nb) bytes.

@@ -245,6 +245,7 @@ def test_virtual_ranks_without_lookahead(lib, world):
     for g in [gg.grid_2d(20, 33, seed=world + 7), gg.erdos_renyi(1100, 4000, seed=world + 7)]:
         c = cfg(lib, world_size=world, virtual_ranks=1)
         c.reserved[1] = 1
+        c.reserved[4] = 1  # launch-per-phase sharded schedule (the dataflow kernel ignores reserved[1])
         assert_i32_equal(lib.solve(g, cfg=c), oracle_i32(g)[0])
 
 
@@ -254,18 +255,22 @@ def test_virtual_ranks_f32(lib):
     assert_f32_close(got, oracle.fw_f64(g.row_ptr, g.col, g.w)[0])
 
 
-def test_nccl_path_single_rank(lib):
-    """reserved[2] = 1: the sharded schedule with a real 1-rank NCCL communicator
-    (ncclBroadcast of the pivot band every round, ncclAllReduce of the status flag)."""
+@pytest.mark.parametrize("sched", [2, 0], ids=["sharded_dataflow", "per_phase_bcast"])
+def test_nccl_path_single_rank(lib, sched):
+    """reserved[2] = 1: the sharded schedules with a real 1-rank NCCL communicator: the
+    sharded dataflow kernel (reserved[4] = 2; barrier + status all-reduce through NCCL) or the
+    launch-per-phase schedule (default: ncclBroadcast of the pivot band every round)."""
     for g in [gg.grid_2d(17, 31, seed=1), gg.erdos_renyi(700, 2800, seed=2)]:
         c = cfg(lib)
         c.reserved[2] = 1
+        c.reserved[4] = sched
         got = lib.solve(g, cfg=c)
         want, _ = oracle_i32(g)
         assert_i32_equal(got, want)
     g = gg.with_arcs(gg.erdos_renyi(300, 900, seed=3), [10, 290], [290, 10], [-100, 20])
     c = cfg(lib)
     c.reserved[2] = 1
+    c.reserved[4] = sched
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
         with pytest.raises(lib.NegativeCycleError):
             lib.apsp_fw_blocked(h)
