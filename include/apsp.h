@@ -314,6 +314,16 @@ apsp_status apsp_get_dist_async(apsp_handle* h, int64_t row_begin, int64_t row_c
                                 int64_t ld_out);
 apsp_status apsp_synchronize(apsp_handle* h);
 
+/*
+ * apsp_debug_queue — diagnostics for tests: the persistent dataflow kernel's task queue,
+ * computed on the host by the same decoder the kernel runs. P = 0: the single-GPU queue;
+ * P >= 1: rank q's queue of the sharded kernel (nb % P == 0). Writes up to `cap` tasks as
+ * (type, k, i, j) int32 quadruples (type 0 = phase 1 of round k, 1 = row-panel tile (k, j),
+ * 2 = column-panel tile (i, k), 3 = phase-3 tile (i, j); i, j global tile indices) and
+ * returns the queue length (-1 on bad arguments). No device is touched.
+ */
+int64_t apsp_debug_queue(int32_t nb, int32_t P, int32_t q, int64_t delay, int32_t* out, int64_t cap);
+
 /* Rows [*row_begin, *row_begin + *row_count) of dist held by this rank. */
 apsp_status apsp_local_rows(const apsp_handle* h, int64_t* row_begin, int64_t* row_count);
 

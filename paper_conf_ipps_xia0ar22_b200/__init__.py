@@ -106,6 +106,7 @@ _sig = {
     "apsp_get_dist_async": (ctypes.c_int, [_H, _I64, _I64, _P, _I64]),
     "apsp_synchronize": (ctypes.c_int, [_H]),
     "apsp_load_csr": (ctypes.c_int, [_H, _P, _P, _P]),
+    "apsp_debug_queue": (ctypes.c_int64, [_I32, _I32, _I32, _I64, _P, _I64]),
     "apsp_local_rows": (ctypes.c_int, [_H, ctypes.POINTER(_I64), ctypes.POINTER(_I64)]),
     "apsp_partition": (ctypes.c_int, [_I64, _I32, _I32, _I32, ctypes.POINTER(_I64), ctypes.POINTER(_I64),
                                       ctypes.POINTER(_I64)]),
@@ -348,6 +349,16 @@ def apsp_load_csr(h: Handle, row_ptr, col_idx, weights) -> None:
     if row_ptr.shape[0] != h.n + 1:
         raise ValueError("row_ptr must have n+1 entries")
     _check(_lib.apsp_load_csr(h.raw, _ptr(row_ptr), _ptr(col_idx), _ptr(w)), h.raw)
+
+
+def apsp_debug_queue(nb: int, P: int, q: int, delay: int) -> np.ndarray:
+    """The dataflow kernel's task queue (host decoder): (total, 4) int32 rows (type, k, i, j)."""
+    total = _lib.apsp_debug_queue(nb, P, q, delay, None, 0)
+    if total < 0:
+        raise ValueError("bad queue arguments")
+    out = np.zeros((max(total, 1), 4), dtype=np.int32)
+    _lib.apsp_debug_queue(nb, P, q, delay, _ptr(out), total)
+    return out[:total]
 
 
 def apsp_synchronize(h: Handle) -> None:

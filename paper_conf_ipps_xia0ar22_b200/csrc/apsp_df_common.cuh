@@ -76,14 +76,14 @@ struct Task {
 };
 
 // i-th value of [0, nb) without the excluded values s0 < s1 < s2 (-1 = none)
-__device__ __forceinline__ int skip3(int x, int s0, int s1, int s2) {
+__host__ __device__ __forceinline__ int skip3(int x, int s0, int s1, int s2) {
   if (s0 >= 0 && x >= s0) ++x;
   if (s1 >= 0 && x >= s1) ++x;
   if (s2 >= 0 && x >= s2) ++x;
   return x;
 }
 
-__device__ __forceinline__ Task p2_task(int nb, int k, long long x) {
+__host__ __device__ __forceinline__ Task p2_task(int nb, int k, long long x) {
   Task t;
   t.k = k;
   if (x < nb - 1) {
@@ -94,7 +94,7 @@ __device__ __forceinline__ Task p2_task(int nb, int k, long long x) {
   return t;
 }
 // G3L(k): (k+1,k+1), row k+1 (j not in {k,k+1}), column k+1 (i not in {k,k+1})
-__device__ __forceinline__ Task g3l_task(int nb, int k, long long x) {
+__host__ __device__ __forceinline__ Task g3l_task(int nb, int k, long long x) {
   Task t;
   t.type = T_P3; t.k = k;
   if (x == 0) { t.i = k + 1; t.j = k + 1; return t; }
@@ -111,7 +111,7 @@ __device__ __forceinline__ Task g3l_task(int nb, int k, long long x) {
 // the two panels are 128 MB > the 126 MB L2; row-major order re-read the whole
 // row panel from HBM for every tile row).
 constexpr int BAND = 64;
-__device__ __forceinline__ void banded(long long x, int R, int W, int& r, int& c) {
+__host__ __device__ __forceinline__ void banded(long long x, int R, int W, int& r, int& c) {
   const int nfull = W / BAND;
   const long long per = (long long)R * BAND;
   if (x < nfull * per) {
@@ -128,7 +128,7 @@ __device__ __forceinline__ void banded(long long x, int R, int W, int& r, int& c
 }
 
 // G3R(k), k <= nb-2: tiles with i,j not in {k,k+1}; row k+2, column k+2 first
-__device__ __forceinline__ Task g3r_task(int nb, int k, long long x) {
+__host__ __device__ __forceinline__ Task g3r_task(int nb, int k, long long x) {
   Task t;
   t.type = T_P3; t.k = k;
   int r, c;
@@ -148,7 +148,7 @@ __device__ __forceinline__ Task g3r_task(int nb, int k, long long x) {
   return t;
 }
 
-__device__ Task decode(long long g, int nb, long long delay) {
+__host__ __device__ Task decode(long long g, int nb, long long delay) {
   Task t;
   if (g == 0) { t.type = T_P1; t.k = 0; t.i = t.j = 0; return t; }
   g -= 1;

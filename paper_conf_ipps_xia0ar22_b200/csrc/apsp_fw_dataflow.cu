@@ -169,21 +169,21 @@ __device__ __forceinline__ T* peer_pb(const DFArgs<T>& a, int r, const T* local)
 //   G3R(k)     local rows not in {k,k+1} x columns not in {k,k+1}, banded
 // Every cross-rank dependency points to an earlier segment or, inside segment k, from G3Lx(k)
 // to G2(k): with the same part order on every rank no cycle exists.
-__device__ __forceinline__ int loc_of(int k, int q, int nl) { return (k / nl) == q ? k - q * nl : -1; }
-__device__ __forceinline__ int lrow(int x, int e0, int e1) {  // x-th local row skipping local e0, e1 (-1 none)
-  const int s0 = (e0 >= 0 && e1 >= 0) ? min(e0, e1) : (e0 >= 0 ? e0 : e1);
-  const int s1 = (e0 >= 0 && e1 >= 0) ? max(e0, e1) : -1;
+__host__ __device__ __forceinline__ int loc_of(int k, int q, int nl) { return (k / nl) == q ? k - q * nl : -1; }
+__host__ __device__ __forceinline__ int lrow(int x, int e0, int e1) {  // x-th local row skipping local e0, e1 (-1 none)
+  const int s0 = (e0 >= 0 && e1 >= 0) ? (e0 < e1 ? e0 : e1) : (e0 >= 0 ? e0 : e1);
+  const int s1 = (e0 >= 0 && e1 >= 0) ? (e0 < e1 ? e1 : e0) : -1;
   return skip3(x, s0, s1, -1);
 }
-__device__ __forceinline__ long long g3r_size_sh(int nb, int nl, int q, int k) {
+__host__ __device__ __forceinline__ long long g3r_size_sh(int nb, int nl, int q, int k) {
   const int l0 = loc_of(k, q, nl) >= 0, l1 = loc_of(k + 1, q, nl) >= 0;
   return (long long)(nl - l0 - l1) * (nb - 2);
 }
-__device__ __forceinline__ long long g2_size_sh(int nb, int nl, int q, int k) {
+__host__ __device__ __forceinline__ long long g2_size_sh(int nb, int nl, int q, int k) {
   const int l0 = loc_of(k, q, nl) >= 0;
   return (long long)l0 * (nb - 1) + (nl - l0);
 }
-__device__ Task decode_sh(long long g, int nb, int nl, int q, long long delay, const long long* segstart) {
+__host__ __device__ Task decode_sh(long long g, int nb, int nl, int q, long long delay, const long long* segstart) {
   Task t;
   const int base = q * nl;
   if (g < segstart[0]) { t.type = T_P1; t.k = 0; t.i = t.j = 0; return t; }
@@ -906,6 +906,25 @@ long long fw_dataflow_work_bytes(int nb, int nl, size_t elem) {
 long long fw_dataflow_pbuf_bytes(int nb, size_t elem) { return fw_dataflow_pbuf_bytes(nb, nb, elem); }
 long long fw_dataflow_flag_bytes(int nb) { return fw_dataflow_flag_bytes(nb, nb); }
 long long fw_dataflow_work_bytes(int nb, size_t elem) { return fw_dataflow_work_bytes(nb, nb, elem); }
+
+}  // namespace apsp
+
+// Test hook (declared in include/apsp.h): the task queue the dataflow kernel decodes, on the
+// host. P = 0: the single-GPU queue (decode); P >= 1: rank q's sharded queue (decode_sh).
+extern "C" int64_t apsp_debug_queue(int32_t nb, int32_t P, int32_t q, int64_t delay, int32_t* out, int64_t cap) {
+  using namespace apsp;
+  if (nb <= 0 || P < 0 || (P > 0 && (nb % P || q < 0 || q >= P))) return -1;
+  const int nl = P > 0 ? nb / P : nb;
+  std::vector<long long> seg((size_t)nb + 1);
+  const long long total = P > 0 ? fw_dataflow_sharded_segments(nb, nl, q, seg.data()) : (long long)nb * nb * nb;
+  for (long long g = 0; g < total && g < cap; ++g) {
+    const Task t = P > 0 ? decode_sh(g, nb, nl, q, delay, seg.data()) : decode(g, nb, delay);
+    out[4 * g] = t.type; out[4 * g + 1] = t.k; out[4 * g + 2] = t.i; out[4 * g + 3] = t.j;
+  }
+  return total;
+}
+
+namespace apsp {
 
 template cudaError_t launch_fw_dataflow_sharded<int>(const DFShard*, int, int, int, long long, int*, long long,
                                                      cudaStream_t);

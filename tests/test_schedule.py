@@ -1,0 +1,131 @@
+"""Host-side checks of the dataflow kernels' task queues (apsp_debug_queue: the decoder the
+kernels run, evaluated on the host; no GPU): every task of the blocked FW (PAPER.md:62 steps
+1-3, Alg. 1 l.3/7/11/17) appears exactly once, on the rank that owns its tile row, and the
+queues cannot deadlock — a simulation that runs every rank's queue strictly in order with ONE
+worker per rank (the most constrained schedule) completes, with dependencies exactly those
+the kernels wait for (per-tile versions, diagonal / panel readiness, panel-parity reuse).
+This covers configurations the single test GPU cannot run (P real GPUs)."""
+import itertools
+
+import numpy as np
+import pytest
+
+P1, P2R, P2C, P3 = 0, 1, 2, 3
+
+
+def expected_tasks(nb):
+    for k in range(nb):
+        yield (P1, k, k, k)
+        for j in range(nb):
+            if j != k:
+                yield (P2R, k, k, j)
+                yield (P2C, k, j, k)
+        for i, j in itertools.product(range(nb), range(nb)):
+            if i != k and j != k:
+                yield (P3, k, i, j)
+
+
+def simulate(nb, queues):
+    """queues[r]: array (total, 4) of rank r (P = len(queues); P = 1 single GPU). One worker
+    per rank, strictly in queue order; returns True iff every queue drains."""
+    P = len(queues)
+    nl = nb // P
+    owner = lambda row: row // nl  # noqa: E731
+    ver = np.zeros((nb, nb), dtype=np.int64)  # rounds applied per tile
+    p1_done = set()
+    p2r_done = set()
+    p2c_done = set()
+    done2 = np.zeros((P, nb), dtype=np.int64)
+    done3 = np.zeros((P, nb), dtype=np.int64)
+
+    def cnt2(r, k):
+        l0 = owner(k) == r
+        return l0 * (nb - 1) + (nl - l0)
+
+    def cnt3(r, k):
+        return (nl - (owner(k) == r)) * (nb - 1)
+
+    def ready(r, t):
+        typ, k, i, j = (int(x) for x in t)
+        if ver[i, j] < k:
+            return False
+        if typ == P3:
+            return (k, j) in p2r_done and (k, i) in p2c_done
+        if typ == P2C:
+            return k in p1_done and (k < 2 or done3[r, k - 2] >= cnt3(r, k - 2))
+        if typ == P2R:
+            return k in p1_done and (k < 2 or all(done3[x, k - 2] >= cnt3(x, k - 2) for x in range(P)))
+        return k < 2 or all(done2[x, k - 2] >= cnt2(x, k - 2) for x in range(P))
+
+    pos = [0] * P
+    total = sum(len(q) for q in queues)
+    ndone = 0
+    while ndone < total:
+        progressed = False
+        for r in range(P):
+            while pos[r] < len(queues[r]) and ready(r, queues[r][pos[r]]):
+                typ, k, i, j = (int(x) for x in queues[r][pos[r]])
+                ver[i, j] = k + 1
+                if typ == P1:
+                    p1_done.add(k)
+                elif typ == P2R:
+                    p2r_done.add((k, j))
+                    done2[r, k] += 1
+                elif typ == P2C:
+                    p2c_done.add((k, i))
+                    done2[r, k] += 1
+                else:
+                    done3[r, k] += 1
+                pos[r] += 1
+                ndone += 1
+                progressed = True
+        if not progressed:
+            return False
+    return True
+
+
+@pytest.mark.parametrize("nb,delay", [(1, 8), (2, 8), (3, 1), (5, 3), (9, 1184), (16, 40), (40, 1)])
+def test_single_gpu_queue_complete_and_deadlock_free(lib, nb, delay):
+    q = lib.apsp_debug_queue(nb, 0, 0, delay)
+    assert len(q) == nb ** 3
+    assert sorted(map(tuple, q.tolist())) == sorted(expected_tasks(nb))
+    assert simulate(nb, [q])
+
+
+@pytest.mark.parametrize("nb,P,delay", [(1, 1, 8), (2, 2, 8), (3, 3, 1), (4, 2, 5), (8, 4, 2), (8, 8, 1),
+                                        (12, 3, 37), (16, 8, 4), (24, 4, 1000), (32, 8, 64)])
+def test_sharded_queues_complete_and_deadlock_free(lib, nb, P, delay):
+    nl = nb // P
+    queues = [lib.apsp_debug_queue(nb, P, q, delay) for q in range(P)]
+    allt = []
+    for r, qu in enumerate(queues):
+        for typ, k, i, j in qu.tolist():
+            assert i // nl == r, "task on a row the rank does not own"  # P1 / P2R rows = k, owned
+            allt.append((typ, k, i, j))
+    assert sorted(allt) == sorted(expected_tasks(nb))
+    assert simulate(nb, queues)
+
+
+def test_sharded_queue_with_one_rank_matches_single_gpu_tasks(lib):
+    nb = 10
+    a = lib.apsp_debug_queue(nb, 1, 0, 5)
+    b = lib.apsp_debug_queue(nb, 0, 0, 5)
+    assert sorted(map(tuple, a.tolist())) == sorted(map(tuple, b.tolist()))
+
+
+def test_simulator_detects_a_deadlocking_order(lib):
+    """Pin of the checker itself: swapping a round's phase-1 task behind that round's
+    phase-3 tasks cannot complete."""
+    nb = 4
+    q = lib.apsp_debug_queue(nb, 0, 0, 8).tolist()
+    k1 = next(x for x, t in enumerate(q) if t[0] == P1 and t[1] == 1)
+    moved = q.pop(k1)
+    q.append(moved)
+    assert not simulate(nb, [np.array(q)])
+
+
+def test_bad_arguments(lib):
+    with pytest.raises(ValueError):
+        lib.apsp_debug_queue(10, 3, 0, 1)  # nb % P != 0
+    with pytest.raises(ValueError):
+        lib.apsp_debug_queue(8, 4, 4, 1)   # q >= P
