@@ -219,11 +219,12 @@ def run_ours(args):
     is_f = g.w.dtype.kind == "f"
     stream = torch.cuda.current_stream()
 
-    uid = None
-    if world > 1:
+    def fresh_uid():
+        """A new ncclUniqueId for every handle (a communicator per handle; an id serves one
+        ncclCommInitRank): rank 0 draws it, every rank receives it (collective, SPMD order)."""
         obj = [apsp.apsp_nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
-        uid = obj[0]
+        return obj[0]
 
     def make_cfg(timing, packed16):
         cfg = apsp.apsp_config_default(device=local, world_size=world, rank=rank, timing=timing)
@@ -243,8 +244,8 @@ def run_ours(args):
         cfg.reserved[5] = args.df_delay
         if packed16:
             cfg.packed16 = 1
-        if uid is not None:
-            cfg._uid_buf = ctypes.create_string_buffer(uid, 128)
+        if world > 1:
+            cfg._uid_buf = ctypes.create_string_buffer(fresh_uid(), 128)
             cfg.nccl_unique_id = ctypes.cast(cfg._uid_buf, ctypes.c_void_p)
         return cfg
 
