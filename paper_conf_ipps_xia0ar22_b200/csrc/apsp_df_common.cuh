@@ -110,7 +110,10 @@ __host__ __device__ __forceinline__ Task g3l_task(int nb, int k, long long x) {
 // per row, so the round's panels never need to fit in L2 at once (at nb = 1024
 // the two panels are 128 MB > the 126 MB L2; row-major order re-read the whole
 // row panel from HBM for every tile row).
-constexpr int BAND = 64;
+#ifndef DF_BAND
+#define DF_BAND 64
+#endif
+constexpr int BAND = DF_BAND;
 __host__ __device__ __forceinline__ void banded(long long x, int R, int W, int& r, int& c) {
   const int nfull = W / BAND;
   const long long per = (long long)R * BAND;
