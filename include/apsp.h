@@ -98,8 +98,8 @@ typedef struct {
   int32_t reserved[6];          /* test hooks: [0] out-of-core streams every band,
                                    [1] no lookahead, [2] NCCL at world 1,
                                    [3] min-plus kernel variant, [4] in-core schedule
-                                   (0 auto: single GPU dataflow kernel for int32,
-                                   launch-per-phase for fp32 and for every sharded
+                                   (0 auto: single GPU dataflow kernel,
+                                   launch-per-phase for every sharded
                                    placement; 1 launch-per-phase; 2 dataflow: on
                                    sharded placements the sharded dataflow kernel with
                                    peer stores of the pivot panels), [5] dataflow queue

@@ -430,6 +430,7 @@ struct Slot {
   Task tk;
   GDesc<T> d;
   int ready;
+  int pref;  // fp32: chunk 0 already issued by the previous task (during its last chunk)
 };
 
 template <typename T>
@@ -469,9 +470,17 @@ __device__ void fill_desc(const DFArgs<T>& a, const Task& tk, GDesc<T>& d) {
 template <bool SH, typename T>
 __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigned full0, unsigned empty0, unsigned c0,
                                            int gtid, int g, const DFArgs<T>* args, long long nxt,
-                                           Slot<T>* ns) {
+                                           Slot<T>* ns, int pref) {
   using V4 = typename DV<T>::V4;
   constexpr int NK = BM / BK;  // 4 chunks of depth 32
+  // fp32: fold the top half of C before the last chunk and issue the next phase-3 task's
+  // chunk 0 into the freed stage (measured +1.2 % for fp32, -1.7 % for int32, so int32 keeps
+  // the C fetch into both free stages during the last chunk and the fold at the end)
+#ifdef DF_XPREF_ALL
+  constexpr bool kXpref = true;
+#else
+  constexpr bool kXpref = sizeof(T) == 4 && T(0.5) != T(0);
+#endif
   const int lane = gtid & 31;
   const int tx = gtid & 15, ty = gtid >> 4;
   // Chunk c of A and B into stage `stage`, completing one phase of full[stage]
@@ -529,7 +538,7 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
     gbar(g);
     if (gtid == 0) mb_arrive(full0 + 8 * stage);
   };
-  load_chunk((int)(c0 % STAGES), 0, -1);  // (the previous task ended with a barrier)
+  if (!pref) load_chunk((int)(c0 % STAGES), 0, -1);  // (the previous task ended with a barrier)
   load_chunk((int)((c0 + 1) % STAGES), 1, -1);
 
   T acc[8][8];
@@ -543,7 +552,7 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
   for (int c = 0; c < NK; ++c) {
     const unsigned G = c0 + c;
     const int s = (int)(G % STAGES);
-    if (c == NK - 1) {
+    if (!kXpref && c == NK - 1) {
       // C goes to the stages of chunks c0+1 and c0+2 once every warp released them
       mb_wait(empty0 + 8 * s_lo, ((c0 + 1) / STAGES) & 1);
       mb_wait(empty0 + 8 * s_hi, ((c0 + 2) / STAGES) & 1);
@@ -558,6 +567,22 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
       for (int q = 0; q < 8; ++q) cp16(cs_hi + cd + q * 8 * CLD, cg + (64 + q * 8) * ldc);
       cp_commit();
     }
+    // fp32 (kXpref): C rows 0-63 go to stage s_lo as soon as chunk c0+1 released it (start of chunk c0+2),
+    // rows 64-127 to s_hi at the start of the last chunk. The top half is folded into the
+    // accumulators right before the last chunk (min is order-free), which frees s_lo for the
+    // NEXT task's chunk 0 (stage of chunk c0+4): thread 0 issues it then, if that task is a
+    // phase-3 task whose dependencies were seen met, so its latency hides under this chunk.
+    if (kXpref && c >= NK - 2) {
+      const int sC = c == NK - 2 ? s_lo : s_hi;
+      mb_wait(empty0 + 8 * sC, ((c0 + (c == NK - 2 ? 1 : 2)) / STAGES) & 1);
+      const int ldc = d->ldc;
+      const T* cg = d->Cin + ((gtid >> 5) + (c == NK - 2 ? 0 : 64)) * (long long)ldc + (gtid & 31) * 4;
+      const int cd = (gtid >> 5) * CLD + (gtid & 31) * 4;
+      T* const cs = stage0 + sC * STAGE_ELEMS;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) cp16(cs + cd + q * 8 * CLD, cg + q * 8 * ldc);
+      cp_commit();
+    }
     if (c == 1 && gtid == SCH) {  // the next task's slot
       ns->t = nxt;
       if (nxt < args->total) {
@@ -565,6 +590,35 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
         ns->tk = tn;
         if (tn.type != T_P1) fill_desc(*args, tn, ns->d);
         ns->ready = deps_any<SH>(*args, tn) ? 1 : 0;
+      }
+    }
+    if (kXpref && c == NK - 1) {
+      asm volatile("cp.async.wait_group 1;\n" ::: "memory");  // this thread's C-top copies
+      gbar(g);
+      const T* const cs_lo = stage0 + s_lo * STAGE_ELEMS;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const T* crow = cs_lo + (ty * 4 + i) * CLD;
+        const V4 x0 = *reinterpret_cast<const V4*>(crow + tx * 4);
+        const V4 x1 = *reinterpret_cast<const V4*>(crow + 64 + tx * 4);
+        acc[i][0] = DV<T>::vmin(acc[i][0], x0.x); acc[i][1] = DV<T>::vmin(acc[i][1], x0.y);
+        acc[i][2] = DV<T>::vmin(acc[i][2], x0.z); acc[i][3] = DV<T>::vmin(acc[i][3], x0.w);
+        acc[i][4] = DV<T>::vmin(acc[i][4], x1.x); acc[i][5] = DV<T>::vmin(acc[i][5], x1.y);
+        acc[i][6] = DV<T>::vmin(acc[i][6], x1.z); acc[i][7] = DV<T>::vmin(acc[i][7], x1.w);
+      }
+      gbar(g);  // s_lo read by every thread: free for the next task's chunk 0
+      if (gtid == 0) {
+        int pf = 0;
+        if (ns->t < args->total && ns->ready && ns->tk.type == T_P3 && ns->d.bulk) {
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          const unsigned bytes = BK * BM * (unsigned)sizeof(T);
+          T* const dst = stage0 + s_lo * STAGE_ELEMS;
+          mb_expect_tx(full0 + 8 * s_lo, 2 * bytes);
+          bulk_g2s(saddr(dst), ns->d.A, bytes, full0 + 8 * s_lo);
+          bulk_g2s(saddr(dst + BK * ALD), ns->d.B, bytes, full0 + 8 * s_lo);
+          pf = 1;
+        }
+        ns->pref = pf;
       }
     }
     mb_wait(full0 + 8 * s, (G / STAGES) & 1);
@@ -637,13 +691,15 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
       const int r = (i < 4) ? (ty * 4 + i) : (64 + ty * 4 + i - 4);
-      const T* crow = (i < 4 ? cs_lo : cs_hi) + (ty * 4 + (i & 3)) * CLD;
-      const V4 x0 = *reinterpret_cast<const V4*>(crow + tx * 4);
-      const V4 x1 = *reinterpret_cast<const V4*>(crow + 64 + tx * 4);
-      acc[i][0] = DV<T>::vmin(acc[i][0], x0.x); acc[i][1] = DV<T>::vmin(acc[i][1], x0.y);
-      acc[i][2] = DV<T>::vmin(acc[i][2], x0.z); acc[i][3] = DV<T>::vmin(acc[i][3], x0.w);
-      acc[i][4] = DV<T>::vmin(acc[i][4], x1.x); acc[i][5] = DV<T>::vmin(acc[i][5], x1.y);
-      acc[i][6] = DV<T>::vmin(acc[i][6], x1.z); acc[i][7] = DV<T>::vmin(acc[i][7], x1.w);
+      if (!kXpref || i >= 4) {  // (kXpref: the top half was folded before the last chunk)
+        const T* crow = (i < 4 ? cs_lo : cs_hi) + (ty * 4 + (i & 3)) * CLD;
+        const V4 x0 = *reinterpret_cast<const V4*>(crow + tx * 4);
+        const V4 x1 = *reinterpret_cast<const V4*>(crow + 64 + tx * 4);
+        acc[i][0] = DV<T>::vmin(acc[i][0], x0.x); acc[i][1] = DV<T>::vmin(acc[i][1], x0.y);
+        acc[i][2] = DV<T>::vmin(acc[i][2], x0.z); acc[i][3] = DV<T>::vmin(acc[i][3], x0.w);
+        acc[i][4] = DV<T>::vmin(acc[i][4], x1.x); acc[i][5] = DV<T>::vmin(acc[i][5], x1.y);
+        acc[i][6] = DV<T>::vmin(acc[i][6], x1.z); acc[i][7] = DV<T>::vmin(acc[i][7], x1.w);
+      }
       V4 v0, v1;
       v0.x = acc[i][0]; v0.y = acc[i][1]; v0.z = acc[i][2]; v0.w = acc[i][3];
       v1.x = acc[i][4]; v1.y = acc[i][5]; v1.z = acc[i][6]; v1.w = acc[i][7];
@@ -710,6 +766,8 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
     Slot<T>& s0 = slots[g][0];
     s0.t = (long long)atomicAdd(a.counter, 1ull);
     s0.ready = 0;
+    s0.pref = 0;
+    slots[g][1].pref = 0;
     if (s0.t < a.total) {
       s0.tk = decode_any<SH>(a, s0.t);
       if (s0.tk.type != T_P1) fill_desc(a, s0.tk, s0.d);
@@ -755,6 +813,7 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
       }
       if (gtid == SCH) {
         N->t = nxt;
+        N->pref = 0;
         if (nxt < a.total) {
           N->tk = decode_any<SH>(a, nxt);
           N->ready = 0;
@@ -762,7 +821,7 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
         }
       }
     } else {
-      group_minplus<SH, T>(&S.d, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N);
+      group_minplus<SH, T>(&S.d, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N, S.pref);
       chunk += BM / BK;
     }
     const long long tc2 = clock64();

@@ -181,7 +181,7 @@ apsp_status setup_device(Handle* h, const apsp_config& cfg) {
   // launch-per-phase schedule with NCCL broadcasts; reserved[4] = 2 selects the sharded
   // dataflow kernel (peer stores of the pivot panels).
   const bool sharded = h->world > 1 || cfg.reserved[2] == 1;
-  h->dataflow = cfg.reserved[4] == 2 || (cfg.reserved[4] == 0 && h->dtype == APSP_I32 && !sharded);
+  h->dataflow = cfg.reserved[4] == 2 || (cfg.reserved[4] == 0 && !sharded);
   h->df_delay = cfg.reserved[5];
   if (cfg.stream) {
     h->stream = static_cast<cudaStream_t>(cfg.stream);

@@ -26,7 +26,7 @@ def want_i32(g):
 
 def run(lib, g, delay=0, legacy=False, timing=0):
     c = lib.apsp_config_default(device=0, timing=timing)
-    c.reserved[4] = 1 if legacy else 2  # 2 = force the dataflow kernel (fp32 default is per-phase)
+    c.reserved[4] = 1 if legacy else 2  # 2 = the dataflow kernel (the single-GPU default for both dtypes)
     c.reserved[5] = delay
     return lib.solve(g, cfg=c)
 

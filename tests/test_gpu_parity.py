@@ -194,20 +194,26 @@ def test_get_dist_row_ranges(lib):
 
 # ---------------------------------------------------------------- fp32 -----
 
+@pytest.mark.parametrize("sched", [0, 1], ids=["dataflow", "per_phase"])
 @pytest.mark.parametrize("n", [7, 128, 300, 515])
-def test_fw_f32_integer_weights_bit_exact(lib, n):
+def test_fw_f32_integer_weights_bit_exact(lib, n, sched):
     g = gg.erdos_renyi(n, 5 * n, seed=n, dtype="f32int")
-    got = lib.solve(g, cfg=cfg(lib))
+    c = cfg(lib)
+    c.reserved[4] = sched
+    got = lib.solve(g, cfg=c)
     gi = gg.csr_from_arcs(g.n, *g.arcs()[:2], g.w.astype(np.int32))
     want, _ = oracle.fw_i64(gi.row_ptr, gi.col, gi.w)
     fin = want != oracle.INF_I64
     assert np.array_equal(got[fin].astype(np.int64), want[fin]) and np.all(np.isinf(got[~fin]))
 
 
+@pytest.mark.parametrize("sched", [0, 1], ids=["dataflow", "per_phase"])
 @pytest.mark.parametrize("n", [100, 256, 700])
-def test_fw_f32_real_weights(lib, n):
+def test_fw_f32_real_weights(lib, n, sched):
     g = gg.erdos_renyi(n, 8 * n, seed=n + 1, dtype="f32")
-    got = lib.solve(g, cfg=cfg(lib))
+    c = cfg(lib)
+    c.reserved[4] = sched
+    got = lib.solve(g, cfg=c)
     want, _ = oracle.fw_f64(g.row_ptr, g.col, g.w)
     assert_f32_close(got, want)
 
