@@ -402,6 +402,10 @@ def run_ours(args):
             tb = time.perf_counter()
             apsp.apsp_load_csr(hs[b], rp, cl, ww)  # this step's input, host -> device
             tc = time.perf_counter()
+            if world > 1:
+                # one communicator per handle: keep at most one of them with NCCL work in flight
+                # (concurrent collectives on two communicators can deadlock across ranks)
+                apsp.apsp_synchronize(hs[1 - b])
             apsp.apsp_fw_blocked_async(hs[b])
             if rc > 0:
                 apsp.apsp_get_dist_async(hs[b], rb, rc, host_out[b].data_ptr(), n)
