@@ -4,7 +4,7 @@ multi-core CPU APSP comparator (BGL-Plus = parallel Dijkstra per s
 here the oracle's OpenMP Dijkstra rows, timed on a sample of sources and extrapolated,
 the paper's own sampling method).
 
-    python tools/boundary_bench.py [--workload cfg2_grid16384] [--blocks 4 8] [--steps 5]
+    python tests/perf/boundary_bench.py [--workload cfg2_grid16384] [--blocks 4 8] [--steps 5]
 
 Prints one JSON line. The boundary algorithm does far fewer than n^3 relaxations, so its
 rate is reported as time (and as n^3/time "FW-equivalent" for comparison only).
@@ -17,7 +17,7 @@ import time
 
 import numpy as np
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROOT = os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 sys.path.insert(0, ROOT)
 
 import graphgen as gg  # noqa: E402

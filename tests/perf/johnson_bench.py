@@ -4,7 +4,7 @@ FW on the same graph, plus the paper-style multi-core CPU APSP comparator (PAPER
 parallel Dijkstra per source; here the oracle's OpenMP Dijkstra rows on a sample of sources,
 extrapolated — the paper's own sampling method).
 
-    python tools/johnson_bench.py [--workload cfg2_grid16384] [--deltas 0 100 400] [--steps 3]
+    python tests/perf/johnson_bench.py [--workload cfg2_grid16384] [--deltas 0 100 400] [--steps 3]
 
 Prints one JSON line per workload. Johnson does O(n * m * re-expansions) work instead of n^3,
 so its rate is reported as arcs relaxed per second (and n^3/time "FW-equivalent", for
@@ -19,7 +19,7 @@ import time
 
 import numpy as np
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROOT = os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 sys.path.insert(0, ROOT)
 
 import graphgen as gg  # noqa: E402

@@ -6,7 +6,7 @@ pinned host memory. Prints one JSON object: wall/device times, relax/s, per-phas
 time, host-link traffic, and a bit-exact check of sampled rows against the CPU oracle's
 Dijkstra (PAPER.md:66).
 
-    python tools/ooc_scale.py [--workload cfg5_grid262144] [--rows 16] [--block 0] [--certify]
+    python tests/perf/ooc_scale.py [--workload cfg5_grid262144] [--rows 16] [--block 0] [--certify]
 
 --certify additionally reads EVERY row back through apsp_get_dist (in chunks, the next
 chunk's copy overlapping the current chunk's check) and checks it with the oracle's
@@ -21,7 +21,7 @@ import time
 
 import numpy as np
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROOT = os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 sys.path.insert(0, ROOT)
 
 import graphgen as gg  # noqa: E402
