@@ -282,7 +282,7 @@ __device__ bool deps_met_sh(const DFArgs<T>& a, const Task& t) {
       }
     }
   }
-  asm volatile("fence.acq_rel.sys;" ::: "memory");
+  asm volatile("fence.acquire.sys;" ::: "memory");  // (an acquire: no wait for this thread's own stores)
   return true;
 }
 
@@ -291,7 +291,7 @@ __device__ bool deps_met_sh(const DFArgs<T>& a, const Task& t) {
 template <typename T>
 __device__ void signal_done_sh(const DFArgs<T>& a, const Task& t) {
   const int nb = a.nb, nl = a.nl, k = t.k, p = k & 1;
-  asm volatile("fence.acq_rel.sys;" ::: "memory");
+  asm volatile("fence.release.sys;" ::: "memory");
   st_relaxed_sys(a.ver + (long long)(t.i - a.q * nl) * nb + t.j, k + 1);
   switch (t.type) {
     case T_P1:
@@ -311,7 +311,14 @@ __device__ void signal_done_sh(const DFArgs<T>& a, const Task& t) {
 
 template <bool SH, typename T>
 __device__ __forceinline__ Task decode_any(const DFArgs<T>& a, long long g) {
-  if constexpr (SH) return decode_sh(g, a.nb, a.nl, a.q, a.delay, a.segstart);
+  // sharded: the segment starts are binary-searched in a shared-memory copy (the kernel
+  // fills it after its stages): from global memory the ~log2(nb) dependent loads went to
+  // L2 every time (each dependency check's acquire fence invalidates L1) and delayed the
+  // decoding warp, and with it its CTA, by thousands of cycles per task
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  if constexpr (SH)
+    return decode_sh(g, a.nb, a.nl, a.q, a.delay,
+                     reinterpret_cast<const long long*>(smem_raw + GROUPS * STAGES * STAGE_ELEMS * sizeof(T)));
   else return decode(g, a.nb, a.delay);
 }
 template <bool SH, typename T>
@@ -751,6 +758,11 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
   const int g = threadIdx.x / GNT, gtid = threadIdx.x % GNT;
   T* const stage0 = reinterpret_cast<T*>(smem_raw) + g * STAGES * STAGE_ELEMS;
   const unsigned full0 = saddr(&bars[g][0]), empty0 = full0 + 8 * STAGES;
+  if constexpr (SH) {  // segment starts -> shared memory (decode_any), before the first decode
+    long long* const seg = reinterpret_cast<long long*>(smem_raw + GROUPS * STAGES * STAGE_ELEMS * sizeof(T));
+    for (int x = threadIdx.x; x <= a.nb; x += blockDim.x) seg[x] = a.segstart[x];
+    __syncthreads();
+  }
   if (gtid == 0) {
     for (int s = 0; s < STAGES; ++s) {
       mb_init(full0 + 8 * s, 1);  // one arrival per chunk (+ transaction bytes of bulk copies)
@@ -918,7 +930,7 @@ cudaError_t launch_fw_dataflow_sharded(const DFShard* ranks, int nv, int P, int 
                                        long long delay, cudaStream_t s) {
   if (nb <= 0 || nv < 1 || nv > kMaxRanks || P < 1 || P > kMaxRanks || nb % P) return cudaErrorInvalidValue;
   const int nl = nb / P;
-  const int smem = GROUPS * STAGES * STAGE_ELEMS * (int)sizeof(T);
+  const int smem = GROUPS * STAGES * STAGE_ELEMS * (int)sizeof(T) + 8 * (nb + 1);  // + segment starts
   cudaError_t e = cudaFuncSetAttribute(fw_dataflow_kernel<true, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return e;
   int dev = 0, sms = 0;
@@ -950,8 +962,16 @@ cudaError_t launch_fw_dataflow_sharded(const DFShard* ranks, int nv, int P, int 
       return e;
     if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return e;
   }
-  long long grid = (long long)sms * CTAS_PER_SM;
+  // a persistent grid must be fully resident (tasks wait on each other): CTAs per SM as the
+  // occupancy calculator allows with this launch's shared memory (the segment starts grow it)
+  int occ = 0;
+  if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fw_dataflow_kernel<true, T>, GNT * GROUPS, smem)) !=
+      cudaSuccess)
+    return e;
+  if (occ < 1) return cudaErrorInvalidConfiguration;
+  long long grid = (long long)sms * (occ < CTAS_PER_SM ? occ : CTAS_PER_SM);
   grid -= grid % nv;
+  if (grid < nv) return cudaErrorInvalidConfiguration;
   fw_dataflow_kernel<true, T><<<(unsigned)grid, GNT * GROUPS, smem, s>>>(L);
   return cudaGetLastError();
 }

@@ -1,0 +1,4 @@
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
+timeout 900 python tools/vr_bench.py --n 16384 --worlds 1 2 4 --delays 0 1 16 64 256 2>&1 | tail -1
+timeout 900 python tools/vr_bench.py --n 32768 --worlds 1 2 --delays 0 16 2>&1 | tail -1

@@ -42,6 +42,7 @@ def main():
     ap.add_argument("--n", type=int, default=16384)
     ap.add_argument("--worlds", type=int, nargs="+", default=[1, 2, 4, 8])
     ap.add_argument("--runs", type=int, default=2)
+    ap.add_argument("--delays", type=int, nargs="+", default=[0], help="queue delays (reserved[5]; 0 = auto)")
     a = ap.parse_args()
     g = gg.erdos_renyi(a.n, 8 * a.n, seed=4)
     out = {"n": a.n}
@@ -50,10 +51,11 @@ def main():
             t = timed(g, a.runs)
             out["single_gpu_dataflow"] = {"s": t, "relax_per_s": a.n ** 3 / t}
             continue
-        t = timed(g, a.runs, world_size=w, virtual_ranks=1, r4=2)
         tp = timed(g, a.runs, world_size=w, virtual_ranks=1, r4=1)
-        out["virtual_%d" % w] = {"sharded_dataflow_s": t, "relax_per_s": a.n ** 3 / t,
-                                 "per_phase_bcast_s": tp, "per_phase_relax_per_s": a.n ** 3 / tp}
+        out["virtual_%d" % w] = {"per_phase_bcast_s": tp, "per_phase_relax_per_s": a.n ** 3 / tp}
+        for d in a.delays:
+            t = timed(g, a.runs, world_size=w, virtual_ranks=1, r4=2, r5=d)
+            out["virtual_%d" % w]["sharded_dataflow_delay_%d" % d] = {"s": t, "relax_per_s": a.n ** 3 / t}
     print(json.dumps(out), flush=True)
 
 
