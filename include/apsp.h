@@ -282,14 +282,16 @@ apsp_status apsp_get_dist(apsp_handle* h, int64_t row_begin, int64_t row_count, 
  * one result overlaps the closure of the next graph on another handle).
  *
  * apsp_fw_blocked_async — enqueue the whole blocked Floyd–Warshall
- *   on the handle's stream and return without waiting. In-core, not packed16:
- *   otherwise it runs synchronously like apsp_fw_blocked (same statuses). The
- *   negative-cycle status is delivered by apsp_synchronize.
+ *   on the handle's stream and return without waiting (in core; out of core it
+ *   runs synchronously like apsp_fw_blocked, same statuses). The negative-cycle
+ *   status is delivered by apsp_synchronize; with packed16 the int16 exactness
+ *   check too (if it fails, apsp_synchronize redoes the closure in int32 and
+ *   replays the copies already enqueued, so `out` buffers end exact).
  * apsp_get_dist_async — enqueue the D2H of rows [row_begin, row_begin+row_count)
  *   (same arguments and row rules as apsp_get_dist) behind the closure on the
  *   handle's stream; `out` must stay valid until apsp_synchronize returns and
  *   should be pinned (pageable memory makes the copy synchronous). Out-of-core,
- *   packed16, boundary and Johnson handles copy synchronously.
+ *   boundary and Johnson handles copy synchronously.
  * apsp_synchronize — wait for everything enqueued on the handle; returns
  *   APSP_ENEGCYCLE if the asynchronous closure found a negative cycle (the
  *   distances, including those already copied, are then unspecified),

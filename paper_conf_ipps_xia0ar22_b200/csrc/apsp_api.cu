@@ -869,13 +869,18 @@ apsp_status apsp_fw_blocked_async(apsp_handle* hh) {
   Handle* h = reinterpret_cast<Handle*>(hh);
   if (h->poisoned) return h->fail(APSP_ESTATE, "handle poisoned by an earlier CUDA/NCCL error");
   if (apsp_status pst = settle(h)) return pst;
-  if (h->mode != APSP_MODE_INCORE || h->mode16) return apsp_fw_blocked(hh);  // synchronous placements
+  if (h->mode != APSP_MODE_INCORE) return apsp_fw_blocked(hh);  // synchronous placements
   if (h->fw_done) return h->fail(APSP_ESTATE, "apsp_fw_blocked already ran");
   apsp_status st;
   if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
   memset(&h->stats, 0, sizeof(h->stats));
   const long long nb = h->n_pad / h->b;
-  if ((st = run_incore_rounds(h, h->next_round, nb))) return st;
+  if (h->mode16) {  // packed16: the exactness check is read by apsp_synchronize
+    if (h->next_round != 0) return h->fail(APSP_ESTATE, "packed16: no partial runs");
+    if ((st = enqueue_fw16(h))) return st;
+  } else if ((st = run_incore_rounds(h, h->next_round, nb))) {
+    return st;
+  }
   h->next_round = nb;
   return finish_fw_async(h);
 }
@@ -890,11 +895,11 @@ apsp_status apsp_get_dist_async(apsp_handle* hh, int64_t row_begin, int64_t row_
   if (row_count == 0) return APSP_OK;
   apsp_status st;
   if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
-  if (h->mode != APSP_MODE_INCORE || h->result16) {  // synchronous placements: settle first
+  if (h->mode != APSP_MODE_INCORE) {  // synchronous placements: settle first
     if ((st = settle(h))) return st;
     return get_rows(h, row_begin, row_count, out, ld_out);
   }
-  return get_rows_async(h, row_begin, row_count, out, ld_out);
+  return get_rows_async(h, row_begin, row_count, out, ld_out);  // (packed16 int16 result: widened on the device)
 }
 
 apsp_status apsp_load_csr(apsp_handle* hh, const int64_t* row_ptr, const int32_t* col_idx, const void* weights) {

@@ -298,28 +298,56 @@ static apsp_status run_dataflow16(Handle* h) {
 
 // Packed int16 closure (VIADDMNMX.S16x2) with exactness check; int32 redo if the
 // largest finite distance reaches 8192 (R16).
-apsp_status run_fw16(Handle* h) {
+static apsp_status run_fw16_int32(Handle* h);
+
+// Enqueue the int16 closure and its exactness check (the max finite entry to pinned
+// h_max16); the result is provisionally int16 (result16) until check_fw16 reads it.
+// A graph already known to need int32 (fell_back16) is enqueued in int32 directly.
+apsp_status enqueue_fw16(Handle* h) {
   apsp_status st;
   const long long nb = h->n_pad / h->b;
-  if (!h->fell_back16) {
-    if (h->dataflow) {  // default: every round in one persistent launch (apsp_fw_dataflow16.cu)
-      if ((st = run_dataflow16(h))) return st;
-    } else if ((st = fw_closure<short>(h, h->d16, h->ld, h->n_pad, 0, nb, h->stream))) {
-      return st;
-    }
-    int mx = 0;
-    if ((st = h->cuda(launch_max_finite16(h->d16, h->ld, h->n_pad, h->n_pad, h->d_max16, h->stream), "max16")))
-      return st;
-    if ((st = h->cuda(cudaMemcpyAsync(&mx, h->d_max16, sizeof(int), cudaMemcpyDeviceToHost, h->stream), "D2H max")))
-      return st;
-    if ((st = h->cuda(cudaStreamSynchronize(h->stream), "fw16 sync"))) return st;
-    if (mx < 8192) {
-      h->result16 = true;
-      h->arith = APSP_ARITH_S16X2;
-      return APSP_OK;
-    }
-    h->fell_back16 = true;  // distances too long for int16: redo (and from now on run) in int32
+  if (h->fell_back16) return run_fw16_int32(h);
+  if (h->dataflow) {  // default: every round in one persistent launch (apsp_fw_dataflow16.cu)
+    if ((st = run_dataflow16(h))) return st;
+  } else if ((st = fw_closure<short>(h, h->d16, h->ld, h->n_pad, 0, nb, h->stream))) {
+    return st;
   }
+  if (!h->h_max16 && (st = h->cuda(cudaHostAlloc(&h->h_max16, sizeof(int), cudaHostAllocDefault), "cudaHostAlloc")))
+    return st;
+  if ((st = h->cuda(launch_max_finite16(h->d16, h->ld, h->n_pad, h->n_pad, h->d_max16, h->stream), "max16")))
+    return st;
+  if ((st = h->cuda(cudaMemcpyAsync(h->h_max16, h->d_max16, sizeof(int), cudaMemcpyDeviceToHost, h->stream),
+                    "D2H max")))
+    return st;
+  h->result16 = true;
+  h->arith = APSP_ARITH_S16X2;
+  h->pending16 = true;
+  return APSP_OK;
+}
+
+// After the stream is synchronized: keep the int16 result if it is provably exact, else
+// redo in int32 (and from now on run this graph in int32), synchronously.
+static apsp_status check_fw16(Handle* h) {
+  if (!h->pending16) return APSP_OK;
+  h->pending16 = false;
+  if (*h->h_max16 < 8192) return APSP_OK;
+  h->fell_back16 = true;  // distances too long for int16
+  h->result16 = false;
+  apsp_status st;
+  if ((st = run_fw16_int32(h))) return st;
+  return h->cuda(cudaStreamSynchronize(h->stream), "fw16 int32 redo");
+}
+
+apsp_status run_fw16(Handle* h) {
+  apsp_status st;
+  if ((st = enqueue_fw16(h))) return st;
+  if ((st = h->cuda(cudaStreamSynchronize(h->stream), "fw16 sync"))) return st;
+  return check_fw16(h);
+}
+
+static apsp_status run_fw16_int32(Handle* h) {
+  apsp_status st;
+  const long long nb = h->n_pad / h->b;
   Shard& sh = h->shards[0];
   if (!sh.D) {
     const long long mat_bytes = h->n_pad * h->ld * 4;
@@ -383,6 +411,7 @@ void delete_handle(Handle* h) {
   cudaFree(h->d_widen);
   cudaFree(h->d_flag);
   if (h->h_flag) cudaFreeHost(h->h_flag);
+  if (h->h_max16) cudaFreeHost(h->h_max16);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
   if (h->side) {
     cudaStreamSynchronize(h->side);
@@ -403,6 +432,16 @@ apsp_status settle(Handle* h) {
   if ((st = h->cuda(cudaSetDevice(h->device), "cudaSetDevice"))) return st;
   if ((st = h->cuda(cudaStreamSynchronize(h->stream), "async sync"))) return st;
   if (h->copy_stream && (st = h->cuda(cudaStreamSynchronize(h->copy_stream), "async sync"))) return st;
+  if (h->pending16) {
+    const bool redo = *h->h_max16 >= 8192;
+    std::vector<Handle::CopyReq> reqs;
+    reqs.swap(h->pending_copies);
+    if ((st = check_fw16(h))) return st;
+    if (redo)  // the copies enqueued from the provisional int16 result: again from the int32 redo
+      for (const auto& q : reqs)
+        if ((st = get_rows(h, q.r0, q.cnt, q.out, q.ld))) return st;
+  }
+  h->pending_copies.clear();
   if (fw) {
     if (h->timing) h->collect_events();
     if (*h->h_flag) return h->fail(APSP_ENEGCYCLE, "negative cycle detected: distances are unspecified");
@@ -432,7 +471,7 @@ apsp_status finish_fw_async(Handle* h) {
 // Enqueue the D2H of rows [r0, r0+cnt) on the handle's stream (in core, not
 // packed16); other placements copy synchronously through get_rows.
 apsp_status get_rows_async(Handle* h, long long r0, long long cnt, void* out, long long ld_out) {
-  if (h->mode != APSP_MODE_INCORE || h->result16) return get_rows(h, r0, cnt, out, ld_out);
+  if (h->mode != APSP_MODE_INCORE || h->result16) return get_rows(h, r0, cnt, out, ld_out);  // (int16: async while pending16)
   if (h->mode16 && !h->shards[0].D) return h->fail(APSP_ESTATE, "no int32 matrix yet");
   apsp_status st;
   const char* base;
@@ -523,6 +562,11 @@ apsp_status get_rows(Handle* h, long long r0, long long cnt, void* out, long lon
                         "D2H dist")))
         return st;
       if ((st = h->cuda(cudaEventRecord(h->copy_ev[2 + b], h->copy_stream), "event"))) return st;
+    }
+    if (h->pending16) {  // asynchronous: settle() waits (and replays if the int16 result is rejected)
+      h->pending_copies.push_back({r0, cnt, out, ld_out});
+      h->pending = true;
+      return APSP_OK;
     }
     return h->cuda(cudaStreamSynchronize(h->copy_stream), "get_dist sync");
   }

@@ -99,6 +99,16 @@ struct Handle {
   bool pending = false;     // asynchronous work enqueued (apsp_*_async); settle() waits for it
   bool pending_fw = false;  // ... including a closure whose negative-cycle flag is still unread
   int* h_flag = nullptr;    // pinned host copy of d_flag for the asynchronous closure
+  // packed16 asynchronous closure: the exactness check (max finite entry < 8192) is read
+  // by settle(); copies enqueued meanwhile are replayed from the int32 redo if it fails
+  int* h_max16 = nullptr;   // pinned
+  bool pending16 = false;
+  struct CopyReq {
+    long long r0, cnt;
+    void* out;
+    long long ld;
+  };
+  std::vector<CopyReq> pending_copies;
   bool timing = false;
   std::vector<TimedEvent> events;
   apsp_phase_stats stats{};
@@ -121,6 +131,7 @@ apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_pt
 void delete_handle(Handle* h);
 apsp_status run_init(Handle* h);
 apsp_status run_fw16(Handle* h);  // packed int16 closure, verify, int32 fallback
+apsp_status enqueue_fw16(Handle* h);  // the same without waiting: settle() checks (h->pending16)
 apsp_status run_incore_rounds(Handle* h, long long k0, long long k1);
 apsp_status finish_fw(Handle* h, bool all_rounds);
 // wait for pending asynchronous work (apsp_fw_blocked_async / apsp_get_dist_async)

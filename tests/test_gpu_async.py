@@ -216,3 +216,44 @@ def test_load_csr_packed16_eligibility(lib):
             lib.apsp_fw_blocked(h)
             assert lib.apsp_get_info(h).arith == arith
             check(g, lib.apsp_get_dist(h))
+
+
+def test_async_packed16_exact_and_replayed_fallback(lib):
+    """packed16 asynchronously: the int16 exactness check (R16) is read by
+    apsp_synchronize. An eligible graph keeps the int16 result; a graph whose distances
+    reach 8192 is redone in int32 there and the copies already enqueued from the provisional
+    int16 result are replayed, so the caller's buffer always holds the exact int32 APSP."""
+    c = lib.apsp_config_default(device=0, packed16=1)
+    g1 = gg.erdos_renyi(700, 4200, seed=51)
+    g2 = gg.weighted_path(np.full(299, 100))  # far ends 29900 apart
+    for g, arith in ((g1, lib.APSP_ARITH_S16X2), (g2, lib.APSP_ARITH_I32)):
+        out = pinned(g.n, False)
+        part = pinned(g.n, False)
+        with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
+            lib.apsp_fw_blocked_async(h)
+            lib.apsp_get_dist_async(h, 0, g.n, out.data_ptr(), out.shape[1])
+            lib.apsp_get_dist_async(h, g.n // 3, g.n // 2, part.data_ptr(), part.shape[1])
+            lib.apsp_synchronize(h)
+            assert lib.apsp_get_info(h).arith == arith
+        w, _ = want(g)
+        assert np.array_equal(out.numpy()[:g.n, :g.n].astype(np.int64), w)
+        assert np.array_equal(part.numpy()[:g.n // 2, :g.n].astype(np.int64), w[g.n // 3:g.n // 3 + g.n // 2])
+
+
+def test_async_packed16_serving_loop(lib):
+    """load_csr + async on one packed16 handle across eligible and ineligible graphs."""
+    n = 600
+    c = lib.apsp_config_default(device=0, packed16=1)
+    ga = gg.erdos_renyi(n, 3000, seed=61)
+    s, t, w = ga.arcs()
+    w2 = w.copy()
+    w2[0] = 9000  # weight above the int16 bound: this graph runs in int32
+    gb = gg.csr_from_arcs(n, s, t, w2)
+    out = pinned(n, False)
+    with lib.apsp_init_from_csr(n, ga.row_ptr, ga.col, ga.w, cfg=c) as h:
+        for g in (ga, gb, ga):
+            lib.apsp_load_csr(h, g.row_ptr, g.col, g.w)
+            lib.apsp_fw_blocked_async(h)
+            lib.apsp_get_dist_async(h, 0, n, out.data_ptr(), out.shape[1])
+            lib.apsp_synchronize(h)
+            check(g, out.numpy()[:n, :n])
