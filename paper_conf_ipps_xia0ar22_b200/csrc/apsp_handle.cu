@@ -412,6 +412,7 @@ void delete_handle(Handle* h) {
   cudaFree(h->d_flag);
   if (h->h_flag) cudaFreeHost(h->h_flag);
   if (h->h_max16) cudaFreeHost(h->h_max16);
+  cudaFree(h->d_widen_async);
   if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
   if (h->side) {
     cudaStreamSynchronize(h->side);
@@ -546,6 +547,34 @@ apsp_status get_rows(Handle* h, long long r0, long long cnt, void* out, long lon
       for (auto& e : h->copy_ev)
         if ((st = h->cuda(cudaEventCreateWithFlags(&e, cudaEventDisableTiming), "event"))) return st;
     }
+    if (h->pending16) {
+      // asynchronous copy: the whole request is widened in ONE kernel right behind the
+      // closure (in submission order it precedes the next graph's persistent kernel, which
+      // would otherwise hold every SM while later staging blocks wait), then one D2H on the
+      // copy stream overlaps whatever runs next. settle() waits (and replays if the int16
+      // result is rejected).
+      const long long need = cnt * ldw;
+      if (h->widen_async_elems < need) {
+        cudaFree(h->d_widen_async);
+        h->d_widen_async = nullptr;
+        if ((st = h->cuda(cudaMalloc(&h->d_widen_async, need * 4), "cudaMalloc widen"))) return st;
+        h->widen_async_elems = need;
+      }
+      if ((st = h->cuda(cudaStreamWaitEvent(h->stream, h->copy_ev[2], 0), "wait"))) return st;  // previous async D2H
+      if ((st = h->cuda(launch_widen16(h->d16 + r0 * h->ld, h->ld, h->d_widen_async, ldw, cnt, h->n, h->stream),
+                        "widen16")))
+        return st;
+      if ((st = h->cuda(cudaEventRecord(h->copy_ev[0], h->stream), "event"))) return st;
+      if ((st = h->cuda(cudaStreamWaitEvent(h->copy_stream, h->copy_ev[0], 0), "wait"))) return st;
+      if ((st = h->cuda(cudaMemcpy2DAsync(out, (size_t)ld_out * 4, h->d_widen_async, (size_t)ldw * 4,
+                                          (size_t)h->n * 4, (size_t)cnt, cudaMemcpyDeviceToHost, h->copy_stream),
+                        "D2H dist")))
+        return st;
+      if ((st = h->cuda(cudaEventRecord(h->copy_ev[2], h->copy_stream), "event"))) return st;
+      h->pending_copies.push_back({r0, cnt, out, ld_out});
+      h->pending = true;
+      return APSP_OK;
+    }
     int b = 0;
     for (long long r = r0; r < r0 + cnt; r += blk, b ^= 1) {
       const long long rr = std::min(blk, r0 + cnt - r);
@@ -562,11 +591,6 @@ apsp_status get_rows(Handle* h, long long r0, long long cnt, void* out, long lon
                         "D2H dist")))
         return st;
       if ((st = h->cuda(cudaEventRecord(h->copy_ev[2 + b], h->copy_stream), "event"))) return st;
-    }
-    if (h->pending16) {  // asynchronous: settle() waits (and replays if the int16 result is rejected)
-      h->pending_copies.push_back({r0, cnt, out, ld_out});
-      h->pending = true;
-      return APSP_OK;
     }
     return h->cuda(cudaStreamSynchronize(h->copy_stream), "get_dist sync");
   }

@@ -102,6 +102,8 @@ struct Handle {
   // packed16 asynchronous closure: the exactness check (max finite entry < 8192) is read
   // by settle(); copies enqueued meanwhile are replayed from the int32 redo if it fails
   int* h_max16 = nullptr;   // pinned
+  int* d_widen_async = nullptr;      // one staging block for a whole asynchronous int16 -> int32 copy
+  long long widen_async_elems = 0;
   bool pending16 = false;
   struct CopyReq {
     long long r0, cnt;
