@@ -14,8 +14,9 @@ import pytest
 import graphgen as gg
 import oracle
 
+import golden_io
+
 INF = oracle.INF_I64
-GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
 
 
 # ----------------------------------------------------------- brute force --
@@ -141,23 +142,38 @@ def test_disjoint_union_is_block_diagonal():
 
 def test_textbook_worked_example():
     """CLRS 3e Fig. 25.4 (Floyd–Warshall on a 5-vertex graph with negative arcs)."""
-    path = os.path.join(GOLDEN, "clrs_fig25_4.txt")
-    arcs, expect = [], []
-    with open(path) as f:
-        section = None
-        for line in f:
-            line = line.split("#")[0].strip()
-            if not line:
-                continue
-            if line in ("arcs:", "dist:"):
-                section = line
-                continue
-            vals = [int(x) for x in line.split()]
-            (arcs if section == "arcs:" else expect).append(vals)
-    g = csr_of(5, [(u - 1, v - 1, w) for u, v, w in arcs])
+    arcs, _, expect = golden_io.load("clrs_fig25_4.txt", base=1)
+    g = csr_of(5, arcs)
     d, neg = oracle.fw_i64(g.row_ptr, g.col, g.w)
     assert not neg
     assert d.tolist() == expect
+
+
+def test_textbook_bellman_ford_example():
+    """CLRS 3e Fig. 24.4 (negative arcs): FW row s and Bellman–Ford from s both
+    equal the figure's final d[v]."""
+    arcs, s, (expect,) = golden_io.load("clrs_fig24_4.txt")
+    g = csr_of(5, arcs)
+    d, neg = oracle.fw_i64(g.row_ptr, g.col, g.w)
+    assert not neg
+    assert d[s].tolist() == expect
+    row, neg = oracle.bellman_ford_row_i64(g.row_ptr, g.col, g.w, s)
+    assert not neg
+    assert row.tolist() == expect
+
+
+def test_textbook_dijkstra_example():
+    """CLRS 3e Fig. 24.6: FW row s, Dijkstra from s and Bellman–Ford from s all
+    equal the figure's final d[v]."""
+    arcs, s, (expect,) = golden_io.load("clrs_fig24_6.txt")
+    g = csr_of(5, arcs)
+    d, neg = oracle.fw_i64(g.row_ptr, g.col, g.w)
+    assert not neg
+    assert d[s].tolist() == expect
+    assert oracle.dijkstra_rows_i64(g.row_ptr, g.col, g.w, [s])[0].tolist() == expect
+    assert oracle.bellman_ford_row_i64(g.row_ptr, g.col, g.w, s)[0].tolist() == expect
+    df, _ = oracle.fw_f64(g.row_ptr, g.col, g.w.astype(np.float32))
+    assert df[s].tolist() == [float(x) for x in expect]
 
 
 # -------------------------------------------------------------- brute force
