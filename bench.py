@@ -542,6 +542,9 @@ def run_ours(args):
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         r, cores, sample = cpu_oracle_sample(g, args.cpu_seconds)
+        sample += ("; the run's first iterations skip rows whose D[i][k] is still infinite, so this is an "
+                   "upper bound of the whole-run rate (the reference arm, --impl reference, times a whole run "
+                   "when n <= %d)" % FULL_RUN_MAX_N)
         cpu = {"value": r, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample}
 
     if rank == 0:
