@@ -205,16 +205,28 @@ class Handle:
         return np.int32 if self.dtype == APSP_I32 else np.float32
 
 
-def apsp_init_from_csr(n: int, row_ptr, col_idx, weights, dtype: int | None = None,
-                       cfg: apsp_config | None = None) -> Handle:
+def _csr_args(n: int, row_ptr, col_idx, weights, dtype: int | None):
+    """Marshal a CSR graph for the C ABI: contiguous int64 row_ptr[n+1], int32 col_idx and
+    int32/float32 weights with at least row_ptr[n] entries each (the C side reads exactly
+    row_ptr[n] arcs, so shorter arrays are refused here with APSP_EINVAL)."""
     row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
     col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
     w = np.asarray(weights)
     if dtype is None:
         dtype = APSP_F32 if w.dtype.kind == "f" else APSP_I32
     w = np.ascontiguousarray(w, dtype=np.int32 if dtype == APSP_I32 else np.float32)
-    if row_ptr.shape[0] != n + 1:
+    if row_ptr.ndim != 1 or row_ptr.shape[0] != n + 1:
         raise ApspError(APSP_EINVAL, "row_ptr must have n+1 entries")
+    m = int(row_ptr[-1]) if n >= 0 else 0
+    if m < 0 or col_idx.shape[0] < m or w.shape[0] < m:
+        raise ApspError(APSP_EINVAL, "col_idx and weights need row_ptr[n] = %d entries (got %d, %d)"
+                        % (m, col_idx.shape[0], w.shape[0]))
+    return row_ptr, col_idx, w, dtype
+
+
+def apsp_init_from_csr(n: int, row_ptr, col_idx, weights, dtype: int | None = None,
+                       cfg: apsp_config | None = None) -> Handle:
+    row_ptr, col_idx, w, dtype = _csr_args(n, row_ptr, col_idx, weights, dtype)
     if cfg is None:
         cfg = apsp_config_default()
     raw = ctypes.c_void_p()
@@ -231,15 +243,10 @@ def apsp_fw_blocked(h: Handle) -> None:
 def apsp_init_boundary(n: int, row_ptr, col_idx, weights, comp, k: int, dtype: int | None = None,
                        cfg: apsp_config | None = None) -> Handle:
     """Boundary algorithm with the caller's partition comp[v] in [0, k)."""
-    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
-    col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
+    row_ptr, col_idx, w, dtype = _csr_args(n, row_ptr, col_idx, weights, dtype)
     comp = np.ascontiguousarray(comp, dtype=np.int32)
-    w = np.asarray(weights)
-    if dtype is None:
-        dtype = APSP_F32 if w.dtype.kind == "f" else APSP_I32
-    w = np.ascontiguousarray(w, dtype=np.int32 if dtype == APSP_I32 else np.float32)
-    if row_ptr.shape[0] != n + 1 or comp.shape[0] != n:
-        raise ApspError(APSP_EINVAL, "row_ptr must have n+1 entries and comp n")
+    if comp.shape[0] != n:
+        raise ApspError(APSP_EINVAL, "comp must have n entries")
     if cfg is None:
         cfg = apsp_config_default()
     raw = ctypes.c_void_p()
@@ -251,14 +258,7 @@ def apsp_init_boundary(n: int, row_ptr, col_idx, weights, comp, k: int, dtype: i
 def apsp_init_johnson(n: int, row_ptr, col_idx, weights, dtype: int | None = None, delta: float = 0.0,
                       batch: int = 0, cfg: apsp_config | None = None) -> Handle:
     """Johnson's algorithm with batched Near-Far SSSP (Algorithm 2)."""
-    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
-    col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
-    w = np.asarray(weights)
-    if dtype is None:
-        dtype = APSP_F32 if w.dtype.kind == "f" else APSP_I32
-    w = np.ascontiguousarray(w, dtype=np.int32 if dtype == APSP_I32 else np.float32)
-    if row_ptr.shape[0] != n + 1:
-        raise ApspError(APSP_EINVAL, "row_ptr must have n+1 entries")
+    row_ptr, col_idx, w, dtype = _csr_args(n, row_ptr, col_idx, weights, dtype)
     if cfg is None:
         cfg = apsp_config_default()
     raw = ctypes.c_void_p()
@@ -270,14 +270,7 @@ def apsp_init_johnson(n: int, row_ptr, col_idx, weights, dtype: int | None = Non
 def apsp_select(n: int, row_ptr, col_idx, weights, comp=None, k: int = 0, dtype: int | None = None,
                 cfg: apsp_config | None = None) -> apsp_selection:
     """The paper's method selection (§IV): density filter + device-calibrated cost models."""
-    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
-    col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
-    w = np.asarray(weights)
-    if dtype is None:
-        dtype = APSP_F32 if w.dtype.kind == "f" else APSP_I32
-    w = np.ascontiguousarray(w, dtype=np.int32 if dtype == APSP_I32 else np.float32)
-    if row_ptr.shape[0] != n + 1:
-        raise ApspError(APSP_EINVAL, "row_ptr must have n+1 entries")
+    row_ptr, col_idx, w, dtype = _csr_args(n, row_ptr, col_idx, weights, dtype)
     cp = None
     if comp is not None:
         cp = np.ascontiguousarray(comp, dtype=np.int32)
@@ -343,11 +336,7 @@ def apsp_get_dist_async(h: Handle, row_begin: int, row_count: int, out_ptr: int,
 def apsp_load_csr(h: Handle, row_ptr, col_idx, weights) -> None:
     """Next graph (same n and dtype) into an in-core handle; the init is enqueued. Arrays are
     numpy (converted like apsp_init_from_csr; pinned arrays copy fastest)."""
-    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
-    col_idx = np.ascontiguousarray(col_idx, dtype=np.int32)
-    w = np.ascontiguousarray(weights, dtype=np.float32 if h.dtype == APSP_F32 else np.int32)
-    if row_ptr.shape[0] != h.n + 1:
-        raise ValueError("row_ptr must have n+1 entries")
+    row_ptr, col_idx, w, _ = _csr_args(h.n, row_ptr, col_idx, weights, h.dtype)
     _check(_lib.apsp_load_csr(h.raw, _ptr(row_ptr), _ptr(col_idx), _ptr(w)), h.raw)
 
 

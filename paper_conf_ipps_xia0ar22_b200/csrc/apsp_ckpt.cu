@@ -29,7 +29,10 @@ struct CkptHeader {
   int32_t world, rank;
   int64_t row_begin;    // first padded row stored
   int64_t next_round;   // rounds 0 .. next_round-1 applied
-  int32_t has_neg, pad0;
+  int32_t has_neg;      // negative arc weights present (affects canonicalisation)
+  int32_t neg_cycle;    // this rank's negative-cycle flag (d_flag) after rounds 0 .. next_round-1:
+                        // phase 1 flags a cycle only in the round of its largest vertex (R6),
+                        // so a resumed run must inherit it
   int64_t reserved[6];
 };
 static_assert(sizeof(CkptHeader) == 128, "checkpoint header is 128 bytes");
@@ -51,6 +54,7 @@ void fill_header(const Handle* h, CkptHeader* hd) {
   hd->row_begin = h->mode == APSP_MODE_OUT_OF_CORE ? 0 : h->shards[0].row_begin;
   hd->next_round = h->next_round;
   hd->has_neg = h->has_neg ? 1 : 0;
+  hd->neg_cycle = 0;
 }
 
 apsp_status check_handle(Handle* h) {
@@ -123,6 +127,12 @@ apsp_status apsp_checkpoint(apsp_handle* hh, const char* path) {
   if (!f) return h->fail(APSP_EINVAL, "apsp_checkpoint: cannot open %s", path);
   CkptHeader hd;
   fill_header(h, &hd);
+  int flag = 0;
+  if ((st = h->cuda(cudaMemcpy(&flag, h->d_flag, sizeof(int), cudaMemcpyDeviceToHost), "D2H flag"))) {
+    fclose(f);
+    return st;
+  }
+  hd.neg_cycle = flag ? 1 : 0;
   if (fwrite(&hd, sizeof(hd), 1, f) != 1) st = h->fail(APSP_EINVAL, "checkpoint: write failed");
   if (!st) st = h->mode == APSP_MODE_OUT_OF_CORE ? ooc_io(h, f, true) : incore_io(h, f, true);
   if (fclose(f) != 0 && !st) st = h->fail(APSP_EINVAL, "checkpoint: close failed");
@@ -152,6 +162,8 @@ apsp_status apsp_restore(apsp_handle* hh, const char* path) {
   st = h->mode == APSP_MODE_OUT_OF_CORE ? ooc_io(h, f, false) : incore_io(h, f, false);
   fclose(f);
   if (st) return st;
+  const int flag = hd.neg_cycle ? 1 : 0;
+  if ((st = h->cuda(cudaMemcpy(h->d_flag, &flag, sizeof(int), cudaMemcpyHostToDevice), "H2D flag"))) return st;
   h->next_round = hd.next_round;
   h->fw_done = hd.next_round == h->n_pad / h->b;
   h->canonical = false;

@@ -502,6 +502,10 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
     if (bulk) {
       if (gtid == 0) {
         if (wait_G >= 0) mb_wait(empty0 + 8 * stage, ((unsigned)wait_G / STAGES) & 1);
+        // generic-proxy -> async-proxy ordering: the stage was last read by generic loads
+        // (shared::cta), and the panel copies were written by other CTAs (or peer GPUs) with
+        // generic stores that this CTA acquired before the task started (global; once per task)
+        if (c == 0) asm volatile("fence.proxy.async.global;" ::: "memory");
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         const unsigned bytes = BK * BM * (unsigned)sizeof(T);
         mb_expect_tx(full0 + 8 * stage, 2 * bytes);
@@ -617,6 +621,7 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
       if (gtid == 0) {
         int pf = 0;
         if (ns->t < args->total && ns->ready && ns->tk.type == T_P3 && ns->d.bulk) {
+          asm volatile("fence.proxy.async.global;" ::: "memory");  // acquired panel copies (see load_chunk)
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           const unsigned bytes = BK * BM * (unsigned)sizeof(T);
           T* const dst = stage0 + s_lo * STAGE_ELEMS;

@@ -199,6 +199,9 @@ __device__ __forceinline__ void group_minplus16(const GDesc16* d, unsigned char*
     if (bulk) {
       if (gtid == 0) {
         if (wait_G >= 0) mb_wait(empty0 + 8 * stage, ((unsigned)wait_G / STAGES) & 1);
+        // generic -> async proxy: stage (shared::cta) and, once per task, the panel copies other
+        // CTAs wrote with generic stores and this CTA acquired before the task (global)
+        if (c == 0) asm volatile("fence.proxy.async.global;" ::: "memory");
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         mb_expect_tx(full0 + 8 * stage, A_WORDS * 4 + B_HALVES * 2);
         bulk_g2s(saddr(sa), static_cast<const unsigned*>(d->A) + (long long)c * A_WORDS, A_WORDS * 4,

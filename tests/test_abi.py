@@ -112,3 +112,21 @@ def test_binding_constants_match_header(lib):
     for name, val in consts.items():
         if name.startswith("APSP_") and not name.endswith("_H"):
             assert getattr(lib, name) == val, name
+
+
+@pytest.mark.parametrize("short", ["col", "w"])
+def test_binding_refuses_short_csr_arrays(lib, short):
+    """The C side reads exactly row_ptr[n] arcs; the binding refuses shorter col_idx / weights
+    (APSP_EINVAL) before any pointer crosses the boundary."""
+    g = gg.erdos_renyi(50, 200, seed=3)
+    col = g.col[:-1] if short == "col" else g.col
+    w = g.w[:-1] if short == "w" else g.w
+    comp = np.zeros(g.n, np.int32)
+    calls = [lambda: lib.apsp_init_from_csr(g.n, g.row_ptr, col, w),
+             lambda: lib.apsp_init_johnson(g.n, g.row_ptr, col, w),
+             lambda: lib.apsp_init_boundary(g.n, g.row_ptr, col, w, comp, 1),
+             lambda: lib.apsp_select(g.n, g.row_ptr, col, w)]
+    for call in calls:
+        with pytest.raises(lib.ApspError) as e:
+            call()
+        assert e.value.status == lib.APSP_EINVAL and "row_ptr[n]" in str(e.value)

@@ -28,3 +28,40 @@ def test_reference_arm_json_line():
     assert d["e2e"]["value"] == d["value"] and d["e2e"]["h2d_bytes_per_step"] == 0
     with open(os.path.join(ROOT, "BASELINE.json")) as f:
         assert d["metric"] == json.load(f)["metric"]
+
+
+def test_self_launch_two_ranks_rendezvous():
+    """`bench.py --gpus 2` without torchrun re-executes itself under torch.distributed.run (127.0.0.1,
+    a free port); both ranks reach the process-group rendezvous (gloo here, NCCL on the GPU box)."""
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK",
+                                                             "MASTER_ADDR", "MASTER_PORT")}
+    p = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--rendezvous-only"],
+                       capture_output=True, text=True, timeout=300, cwd=ROOT, env=env)
+    assert p.returncode == 0, p.stderr[-2000:]
+    got = sorted(json.loads(l)["rank"] for l in p.stdout.splitlines() if l.strip().startswith("{"))
+    assert got == [0, 1]
+
+
+def test_default_workload_is_the_metric_config():
+    """BASELINE.json quotes the metric 'at 1/2/4/8 B200' on configs[2] (n=65536): every N uses it."""
+    sys.path.insert(0, ROOT)
+    import bench
+    import graphgen as gg
+    for n_gpus in (1, 2, 4, 8):
+        assert bench.default_workload(n_gpus) == "cfg3_er65536"
+    with open(os.path.join(ROOT, "BASELINE.json")) as f:
+        assert "n=65536" in json.load(f)["configs"][2]
+
+
+def test_oracle_steady_rate_counts_full_iterations():
+    """The steady-state CPU sample does every relaxation of every outer iteration (no INF skip):
+    its rate on a sparse graph is below the whole-run rate of the same oracle, never above it by
+    the early-iteration skip (the r1 cpu_baseline bias)."""
+    sys.path.insert(0, ROOT)
+    import bench
+    import graphgen as gg
+    g = gg.erdos_renyi(1536, 1536 * 2, seed=11)  # sparse: many rows skipped early in a real run
+    whole, _, _ = bench.oracle_whole_run(g, 2)
+    steady, cores, sample, rates, _ = bench.oracle_steady_rate(g, warm_s=0.2, step_s=0.3, steps=2)
+    assert cores >= 1 and len(rates) == 2 and "steady-state" in sample
+    assert steady <= whole * 1.3

@@ -123,3 +123,37 @@ def test_restore_rejects_mismatch(lib, tmp_path):
             lib.apsp_restore(h, str(junk))
         with pytest.raises(lib.ApspError):
             lib.apsp_restore(h, str(tmp_path / "missing.ckpt"))
+
+
+@pytest.mark.parametrize("ooc", [False, True])
+def test_checkpoint_carries_negative_cycle_flag(lib, tmp_path, ooc):
+    """A cycle inside tile 0 is flagged by phase 1 of round 0 only (R6: the round of its
+    largest vertex); later rounds never look again. A run checkpointed after round 1 and
+    resumed in a fresh handle must still report the cycle (the flag is saved)."""
+    g0 = gg.erdos_renyi(400, 2400, seed=47)
+    s, t, w = g0.arcs()
+    s = np.concatenate([s, [3, 5]])
+    t = np.concatenate([t, [5, 3]])
+    w = np.concatenate([w, [-5, 2]]).astype(np.int32)
+    g = gg.csr_from_arcs(g0.n, s, t, w)
+    _, neg = oracle.fw_i64(g.row_ptr, g.col, g.w)
+    assert neg
+    path = str(tmp_path / "neg.ckpt")
+
+    def cfg():
+        c = lib.apsp_config_default(device=0)
+        if ooc:
+            c.force_out_of_core = 1
+            c.ooc_block = 128
+        return c
+
+    with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=cfg()) as h:
+        try:
+            lib.apsp_fw_rounds(h, 0, 2)
+        except lib.NegativeCycleError:
+            pass
+        lib.apsp_checkpoint(h, path)
+    with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=cfg()) as h:
+        lib.apsp_restore(h, path)
+        with pytest.raises(lib.NegativeCycleError):
+            lib.apsp_fw_blocked(h)
