@@ -327,15 +327,15 @@ def run_ours(args):
             cfg.force_out_of_core = 1
             cfg.ooc_block = args.ooc_block
             if args.stream_all:
-                cfg.reserved[0] = 1
+                cfg.ooc_stream_all = 1
         if args.no_lookahead:
-            cfg.reserved[1] = 1
-        cfg.reserved[3] = args.minplus_variant
+            cfg.no_lookahead = 1
+        cfg.minplus_variant = args.minplus_variant
         if args.legacy:
-            cfg.reserved[4] = 1
+            cfg.schedule = 1
         if args.sharded_dataflow:
-            cfg.reserved[4] = 2
-        cfg.reserved[5] = args.df_delay
+            cfg.schedule = 2
+        cfg.dataflow_delay = args.df_delay
         if packed16:
             cfg.packed16 = 1
         if world > 1:
@@ -361,7 +361,13 @@ def run_ours(args):
         CUDA events on the library's stream, max over ranks; roofline of phase 3."""
         steps = args.steps if steps is None else steps
         warmup = args.warmup if warmup is None else warmup
-        h = apsp.apsp_init_from_csr(n, g.row_ptr, g.col, g.w, cfg=make_cfg(1, packed16))
+        cfg = make_cfg(1, packed16)
+        dist_buf = None
+        if not args.force_ooc:  # torch owns the distance matrix (apsp_config.dist_device)
+            need = apsp.apsp_dist_device_bytes(n, world)
+            dist_buf = torch.empty(need // 4, dtype=torch.int32, device="cuda")
+            cfg.dist_device, cfg.dist_device_bytes = dist_buf.data_ptr(), need
+        h = apsp.apsp_init_from_csr(n, g.row_ptr, g.col, g.w, cfg=cfg)
         info = apsp.apsp_get_info(h)
         for _ in range(warmup):
             apsp.apsp_reinit(h)
@@ -389,6 +395,7 @@ def run_ours(args):
         value = float(n) ** 3 / (ms_step * 1e-3)
         arith = apsp.ARITH_NAMES[apsp.apsp_get_info(h).arith]
         apsp.apsp_destroy(h)
+        del dist_buf
         # roofline of the dominant kernel: phase-3 min-plus launches
         p3_ms = st_acc[0][2] / max(1, st_acc[1][2])
         p3_relax = st_acc[2][2] / max(1, st_acc[1][2])
@@ -611,7 +618,8 @@ def run_ours(args):
                        else "single GPU",
                        "l2": "inputs larger than L2 (dist = %.2f GB per step >> 126 MB L2); no flush" %
                              (float(main_run["n_pad"]) ** 2 * (2 if main_run["arith"] == "s16x2" else 4) / 1e9),
-                       "step": "apsp_reinit (CSR->dense, CSR resident in HBM) + apsp_fw_blocked"},
+                       "step": "apsp_reinit (CSR->dense, CSR resident in HBM) + apsp_fw_blocked",
+                       "dist_memory": "torch-allocated device tensor passed as apsp_config.dist_device"},
             "clocks": main_run["clocks"],
             "e2e": e2e,
             "gpu_launches": main_run["launches_per_step"] * args.steps,

@@ -66,6 +66,15 @@ typedef enum {
 #define APSP_MODE_BOUNDARY 2
 #define APSP_MODE_JOHNSON 3
 
+/* apsp_config.schedule: how the in-core blocked FW is scheduled. */
+#define APSP_SCHED_AUTO 0       /* single GPU: the persistent dataflow kernel (all rounds and
+                                   phases in one launch); sharded placements: launch-per-phase
+                                   rounds with NCCL pivot-band broadcasts */
+#define APSP_SCHED_PER_PHASE 1  /* one launch per phase and round (phase 1, phase 2, phase 3) */
+#define APSP_SCHED_DATAFLOW 2   /* the dataflow kernel; on sharded placements its sharded form,
+                                   whose round owners store the pivot panels into every rank's
+                                   panel buffer over NVLink (peer stores) */
+
 typedef struct {
   int32_t struct_size;          /* = sizeof(apsp_config) (ABI versioning); 0 = defaults */
   int32_t device;               /* CUDA ordinal; -1 = current device */
@@ -80,6 +89,19 @@ typedef struct {
   int32_t tile;                 /* round depth b (tile edge); 0 = auto (128). Must be 128
                                    in this build (the kernels' tile edge) */
   void* stream;                 /* cudaStream_t to enqueue on; NULL = library stream */
+  void* dist_device;            /* optional CALLER-OWNED device buffer (e.g. a torch tensor's
+                                   data_ptr on cfg.device) that holds this process's rows of
+                                   dist: row-major, ld = n_pad elements (apsp_dist_device_bytes
+                                   gives the size; 256-byte aligned). The library never frees
+                                   it; it must outlive the handle and not be touched while the
+                                   handle's work is in flight. In-core blocked FW only
+                                   (apsp_init_from_csr); APSP_EINVAL if it is too small, with
+                                   force_out_of_core, or for boundary / Johnson handles. The
+                                   matrix then does not count against device_budget_bytes (the
+                                   handle never goes out of core). With packed16 the int16
+                                   working matrix occupies the first half of the buffer.
+                                   NULL = the library allocates */
+  int64_t dist_device_bytes;    /* size of dist_device in bytes (>= apsp_dist_device_bytes) */
   int64_t device_budget_bytes;  /* 0 = use free device memory; smaller forces the
                                    out-of-core path (tests) */
   int32_t ooc_block;            /* out-of-core super-block (band height) B; 0 = auto;
@@ -95,15 +117,21 @@ typedef struct {
                                    the output is always the exact int32 APSP. Single-GPU
                                    in-core only; ignored elsewhere. apsp_info.arith
                                    reports which arithmetic produced the result */
-  int32_t reserved[6];          /* test hooks: [0] out-of-core streams every band,
-                                   [1] no lookahead, [2] NCCL at world 1,
-                                   [3] min-plus kernel variant, [4] in-core schedule
-                                   (0 auto: single GPU dataflow kernel,
-                                   launch-per-phase for every sharded
-                                   placement; 1 launch-per-phase; 2 dataflow: on
-                                   sharded placements the sharded dataflow kernel with
-                                   peer stores of the pivot panels), [5] dataflow queue
-                                   delay; otherwise 0 */
+  int32_t schedule;             /* APSP_SCHED_* (0 = auto) */
+  int32_t no_lookahead;         /* launch-per-phase schedule: 1 = no lookahead (phases 1-2
+                                   of round k+1 are not overlapped with round k's phase 3) */
+  int32_t ooc_stream_all;       /* out of core: 1 = keep no band resident in HBM (every
+                                   band streamed from pinned host memory each super-round,
+                                   the paper's setting) */
+  int32_t force_nccl;           /* 1 = run the sharded schedule with a real 1-rank NCCL
+                                   communicator at world_size 1 (exercises the broadcast /
+                                   all-reduce path on one GPU) */
+  int32_t minplus_variant;      /* launch-per-phase min-plus kernel: 0 = cp.async + mbarrier
+                                   pipeline (default), 1 = cp.async + CTA barrier per chunk,
+                                   2 = TMA persistent (an A/B experiment, measured slower) */
+  int32_t dataflow_delay;       /* dataflow kernel queue delay (phase-3 tasks of round k-1
+                                   queued before round k's panels); 0 = auto */
+  int32_t reserved[4];          /* must be 0 (APSP_EINVAL otherwise) */
 } apsp_config;
 
 /* Fill *cfg with defaults (struct_size set, device -1, world 1, rank 0). */
@@ -339,6 +367,15 @@ apsp_status apsp_local_rows(const apsp_handle* h, int64_t* row_begin, int64_t* r
 apsp_status apsp_partition(int64_t n, int32_t tile, int32_t world_size, int32_t rank,
                            int64_t* n_pad, int64_t* row_begin, int64_t* row_count);
 
+/*
+ * apsp_dist_device_bytes — bytes a caller-owned apsp_config.dist_device buffer needs for
+ * apsp_init_from_csr(n, ..., dtype, cfg) (host-only arithmetic, no device needed):
+ * (n_pad / world_size) * n_pad * 4 per rank (int32 and fp32 elements; n_pad from
+ * apsp_partition), times world_size with virtual_ranks (all shards in one buffer).
+ */
+apsp_status apsp_dist_device_bytes(int64_t n, int32_t tile, int32_t world_size, int32_t virtual_ranks,
+                                   int64_t* bytes);
+
 typedef struct {
   int64_t n, n_pad;
   int32_t tile, dtype, world_size, rank, mode; /* mode: APSP_MODE_* */
@@ -360,7 +397,8 @@ typedef struct {
 
 #define APSP_ARITH_I32 0   /* VIADDMNMX (int32 DPX), 1 relaxation / instruction */
 #define APSP_ARITH_S16X2 1 /* VIADDMNMX.S16x2, 2 relaxations / instruction, verified exact */
-#define APSP_ARITH_F32 2   /* FADD + FMNMX */
+#define APSP_ARITH_F32 2   /* fp32: FADD2 (one A value against a column pair) + FMNMX3
+                              (two depth steps folded into one accumulator update) */
 
 apsp_status apsp_get_info(const apsp_handle* h, apsp_info* info);
 

@@ -34,6 +34,7 @@ STATUS_NAMES = ["APSP_OK", "APSP_EINVAL", "APSP_ERANGE", "APSP_ENOMEM", "APSP_EC
 APSP_INF_I32 = 0x3FFFFFFF
 APSP_MODE_INCORE, APSP_MODE_OUT_OF_CORE, APSP_MODE_BOUNDARY, APSP_MODE_JOHNSON = 0, 1, 2, 3
 TILE = 128
+APSP_SCHED_AUTO, APSP_SCHED_PER_PHASE, APSP_SCHED_DATAFLOW = 0, 1, 2
 
 
 class apsp_config(ctypes.Structure):
@@ -46,12 +47,20 @@ class apsp_config(ctypes.Structure):
         ("virtual_ranks", ctypes.c_int32),
         ("tile", ctypes.c_int32),
         ("stream", ctypes.c_void_p),
+        ("dist_device", ctypes.c_void_p),
+        ("dist_device_bytes", ctypes.c_int64),
         ("device_budget_bytes", ctypes.c_int64),
         ("ooc_block", ctypes.c_int32),
         ("timing", ctypes.c_int32),
         ("force_out_of_core", ctypes.c_int32),
         ("packed16", ctypes.c_int32),
-        ("reserved", ctypes.c_int32 * 6),
+        ("schedule", ctypes.c_int32),
+        ("no_lookahead", ctypes.c_int32),
+        ("ooc_stream_all", ctypes.c_int32),
+        ("force_nccl", ctypes.c_int32),
+        ("minplus_variant", ctypes.c_int32),
+        ("dataflow_delay", ctypes.c_int32),
+        ("reserved", ctypes.c_int32 * 4),
     ]
 
 
@@ -110,6 +119,7 @@ _sig = {
     "apsp_local_rows": (ctypes.c_int, [_H, ctypes.POINTER(_I64), ctypes.POINTER(_I64)]),
     "apsp_partition": (ctypes.c_int, [_I64, _I32, _I32, _I32, ctypes.POINTER(_I64), ctypes.POINTER(_I64),
                                       ctypes.POINTER(_I64)]),
+    "apsp_dist_device_bytes": (ctypes.c_int, [_I64, _I32, _I32, _I32, ctypes.POINTER(_I64)]),
     "apsp_get_info": (ctypes.c_int, [_H, ctypes.POINTER(apsp_info)]),
     "apsp_get_phase_stats": (ctypes.c_int, [_H, ctypes.POINTER(apsp_phase_stats)]),
     "apsp_nccl_unique_id": (ctypes.c_int, [_P]),
@@ -172,6 +182,13 @@ def apsp_partition(n: int, world_size: int, rank: int, tile: int = 0):
     np_, rb, rc = _I64(), _I64(), _I64()
     _check(_lib.apsp_partition(n, tile, world_size, rank, ctypes.byref(np_), ctypes.byref(rb), ctypes.byref(rc)))
     return np_.value, rb.value, rc.value
+
+
+def apsp_dist_device_bytes(n: int, world_size: int = 1, virtual_ranks: int = 0, tile: int = 0) -> int:
+    """Bytes a caller-owned apsp_config.dist_device buffer needs (host arithmetic)."""
+    b = _I64()
+    _check(_lib.apsp_dist_device_bytes(n, tile, world_size, virtual_ranks, ctypes.byref(b)))
+    return b.value
 
 
 class Handle:

@@ -506,6 +506,16 @@ apsp_status apsp_partition(int64_t n, int32_t tile, int32_t world_size, int32_t 
   return APSP_OK;
 }
 
+apsp_status apsp_dist_device_bytes(int64_t n, int32_t tile, int32_t world_size, int32_t virtual_ranks,
+                                   int64_t* bytes) {
+  if (!bytes) return fail_global(APSP_EINVAL, "apsp_dist_device_bytes: NULL");
+  int64_t np = 0, rb = 0, rc = 0;
+  if (apsp_status st = apsp_partition(n, tile, world_size, 0, &np, &rb, &rc)) return st;
+  const int64_t per_rank = (np / world_size) * np * (int64_t)sizeof(int32_t);
+  *bytes = (virtual_ranks && world_size > 1) ? per_rank * world_size : per_rank;
+  return APSP_OK;
+}
+
 apsp_status apsp_nccl_unique_id(void* out128) {
   if (!out128) return fail_global(APSP_EINVAL, "apsp_nccl_unique_id: NULL");
   return nccl_unique_id(out128) ? APSP_OK : fail_global(APSP_ENCCL, "ncclGetUniqueId failed");
@@ -546,19 +556,37 @@ static apsp_status validate_csr(int64_t n, const int64_t* row_ptr, const int32_t
   return APSP_OK;
 }
 
+// Copy the caller's config (NULL = defaults) and check the fields every entry point shares.
+static apsp_status load_config(const apsp_config* cfg_in, apsp_config* cfg) {
+  apsp_config_default(cfg);
+  if (!cfg_in) return APSP_OK;
+  if (cfg_in->struct_size != 0 && cfg_in->struct_size != (int32_t)sizeof(apsp_config))
+    return fail_global(APSP_EINVAL, "apsp_config.struct_size %d != %d", cfg_in->struct_size, (int)sizeof(apsp_config));
+  *cfg = *cfg_in;
+  for (int32_t r : cfg->reserved)
+    if (r != 0) return fail_global(APSP_EINVAL, "apsp_config.reserved must be 0");
+  if (cfg->schedule < APSP_SCHED_AUTO || cfg->schedule > APSP_SCHED_DATAFLOW)
+    return fail_global(APSP_EINVAL, "apsp_config.schedule %d is not an APSP_SCHED_* value", cfg->schedule);
+  if (cfg->minplus_variant < 0 || cfg->minplus_variant > 2)
+    return fail_global(APSP_EINVAL, "apsp_config.minplus_variant must be 0, 1 or 2");
+  if (cfg->dataflow_delay < 0) return fail_global(APSP_EINVAL, "apsp_config.dataflow_delay < 0");
+  if (cfg->dist_device_bytes < 0) return fail_global(APSP_EINVAL, "apsp_config.dist_device_bytes < 0");
+  return APSP_OK;
+}
+
+// Handles other than the in-core blocked FW cannot take a caller-owned matrix.
+static apsp_status no_dist_device(const apsp_config& cfg, const char* what) {
+  if (cfg.dist_device) return fail_global(APSP_EINVAL, "%s: apsp_config.dist_device is for apsp_init_from_csr only", what);
+  return APSP_OK;
+}
+
 apsp_status apsp_init_from_csr(apsp_handle** out, int64_t n, const int64_t* row_ptr, const int32_t* col_idx,
                                const void* weights, apsp_dtype dtype, const apsp_config* cfg_in) {
   NvtxRange nvtx_("apsp_init_from_csr");
   if (!out) return fail_global(APSP_EINVAL, "apsp_init_from_csr: out is NULL");
   *out = nullptr;
   apsp_config cfg;
-  apsp_config_default(&cfg);
-  if (cfg_in) {
-    if (cfg_in->struct_size != 0 && cfg_in->struct_size != (int32_t)sizeof(apsp_config))
-      return fail_global(APSP_EINVAL, "apsp_config.struct_size %d != %d", cfg_in->struct_size,
-                         (int)sizeof(apsp_config));
-    cfg = *cfg_in;
-  }
+  if (apsp_status cst = load_config(cfg_in, &cfg)) return cst;
   if (n < 0) return fail_global(APSP_EINVAL, "n < 0");
   if (n > (int64_t)INT32_MAX) return fail_global(APSP_EINVAL, "n exceeds int32 vertex ids");
   if (!row_ptr) return fail_global(APSP_EINVAL, "row_ptr is NULL");
@@ -569,6 +597,17 @@ apsp_status apsp_init_from_csr(apsp_handle** out, int64_t n, const int64_t* row_
     return fail_global(APSP_EINVAL, "bad world_size/rank");
   if (cfg.world_size > 1 && !cfg.virtual_ranks && !cfg.nccl_unique_id)
     return fail_global(APSP_EINVAL, "world_size > 1 needs nccl_unique_id (or virtual_ranks)");
+  if (cfg.dist_device) {
+    int64_t need = 0;
+    if (apsp_dist_device_bytes(n, cfg.tile, cfg.world_size, cfg.virtual_ranks, &need) != APSP_OK)
+      return fail_global(APSP_EINVAL, "apsp_dist_device_bytes failed");
+    if (cfg.dist_device_bytes < need)
+      return fail_global(APSP_EINVAL, "apsp_config.dist_device_bytes %lld < %lld needed", (long long)cfg.dist_device_bytes,
+                         (long long)need);
+    if (reinterpret_cast<uintptr_t>(cfg.dist_device) % 256 != 0)
+      return fail_global(APSP_EINVAL, "apsp_config.dist_device must be 256-byte aligned");
+    if (cfg.force_out_of_core) return fail_global(APSP_EINVAL, "dist_device and force_out_of_core exclude each other");
+  }
 
   bool has_neg = false;
   int64_t maxabs = 0;
@@ -605,18 +644,13 @@ apsp_status apsp_init_boundary(apsp_handle** out, int64_t n, const int64_t* row_
   if (!out) return fail_global(APSP_EINVAL, "apsp_init_boundary: out is NULL");
   *out = nullptr;
   apsp_config cfg;
-  apsp_config_default(&cfg);
-  if (cfg_in) {
-    if (cfg_in->struct_size != 0 && cfg_in->struct_size != (int32_t)sizeof(apsp_config))
-      return fail_global(APSP_EINVAL, "apsp_config.struct_size %d != %d", cfg_in->struct_size,
-                         (int)sizeof(apsp_config));
-    cfg = *cfg_in;
-  }
+  if (apsp_status cst = load_config(cfg_in, &cfg)) return cst;
   if (n < 1 || n > (int64_t)INT32_MAX) return fail_global(APSP_EINVAL, "bad n");
   if (!row_ptr || !comp) return fail_global(APSP_EINVAL, "row_ptr / comp is NULL");
   if (dtype != APSP_I32 && dtype != APSP_F32) return fail_global(APSP_EINVAL, "bad dtype");
   if (k < 1) return fail_global(APSP_EINVAL, "k < 1");
   if (cfg.world_size != 1) return fail_global(APSP_EINVAL, "the boundary algorithm runs on one GPU");
+  if (apsp_status dst = no_dist_device(cfg, "apsp_init_boundary")) return dst;
   for (int64_t v = 0; v < n; ++v)
     if (comp[v] < 0 || comp[v] >= k) return fail_global(APSP_EINVAL, "comp[%lld] out of [0, k)", (long long)v);
   bool has_neg = false;
@@ -634,7 +668,7 @@ apsp_status apsp_init_boundary(apsp_handle** out, int64_t n, const int64_t* row_
   h->elem = 4;
   h->mode = APSP_MODE_BOUNDARY;
   apsp_status st = setup_device(h, cfg);
-  if (!st) st = bnd_setup(h, row_ptr, col_idx, weights, comp, k);
+  if (!st) st = bnd_setup(h, cfg, row_ptr, col_idx, weights, comp, k);
   if (st != APSP_OK) {
     g_last_error = h->err;
     delete_handle(h);
@@ -651,19 +685,14 @@ apsp_status apsp_init_johnson(apsp_handle** out, int64_t n, const int64_t* row_p
   if (!out) return fail_global(APSP_EINVAL, "apsp_init_johnson: out is NULL");
   *out = nullptr;
   apsp_config cfg;
-  apsp_config_default(&cfg);
-  if (cfg_in) {
-    if (cfg_in->struct_size != 0 && cfg_in->struct_size != (int32_t)sizeof(apsp_config))
-      return fail_global(APSP_EINVAL, "apsp_config.struct_size %d != %d", cfg_in->struct_size,
-                         (int)sizeof(apsp_config));
-    cfg = *cfg_in;
-  }
+  if (apsp_status cst = load_config(cfg_in, &cfg)) return cst;
   if (n < 1 || n > (int64_t)INT32_MAX) return fail_global(APSP_EINVAL, "bad n");
   if (!row_ptr) return fail_global(APSP_EINVAL, "row_ptr is NULL");
   if (dtype != APSP_I32 && dtype != APSP_F32) return fail_global(APSP_EINVAL, "bad dtype");
   if (cfg.world_size < 1 || cfg.rank < 0 || cfg.rank >= cfg.world_size)
     return fail_global(APSP_EINVAL, "bad world_size/rank");
   if (!(delta >= 0) || !std::isfinite(delta)) return fail_global(APSP_EINVAL, "delta must be finite and >= 0");
+  if (apsp_status dst = no_dist_device(cfg, "apsp_init_johnson")) return dst;
   bool has_neg = false;
   int64_t maxabs = 0;
   apsp_status vst = validate_csr(n, row_ptr, col_idx, weights, dtype, &has_neg, &maxabs);
@@ -699,13 +728,7 @@ apsp_status apsp_select(int64_t n, const int64_t* row_ptr, const int32_t* col_id
   memset(out, 0, sizeof(*out));
   for (double& e : out->est_seconds) e = -1.0;
   apsp_config cfg;
-  apsp_config_default(&cfg);
-  if (cfg_in) {
-    if (cfg_in->struct_size != 0 && cfg_in->struct_size != (int32_t)sizeof(apsp_config))
-      return fail_global(APSP_EINVAL, "apsp_config.struct_size %d != %d", cfg_in->struct_size,
-                         (int)sizeof(apsp_config));
-    cfg = *cfg_in;
-  }
+  if (apsp_status cst = load_config(cfg_in, &cfg)) return cst;
   if (n < 1 || n > (int64_t)INT32_MAX || !row_ptr) return fail_global(APSP_EINVAL, "bad n / row_ptr");
   if (dtype != APSP_I32 && dtype != APSP_F32) return fail_global(APSP_EINVAL, "bad dtype");
   if (comp && k < 1) return fail_global(APSP_EINVAL, "k < 1");
@@ -992,7 +1015,8 @@ apsp_status apsp_get_info(const apsp_handle* hh, apsp_info* info) {
   info->world_size = h->world;
   info->rank = h->rank;
   info->mode = h->mode;
-  info->ooc_block = h->mode == APSP_MODE_OUT_OF_CORE ? (int32_t)h->ooc_B : 0;
+  info->ooc_block = h->mode == APSP_MODE_OUT_OF_CORE ? (int32_t)h->ooc_B
+                   : h->mode == APSP_MODE_BOUNDARY ? (int32_t)bnd_ooc_rows(h) : 0;
   info->rounds = h->n_pad / h->b;
   info->device_bytes = h->device_bytes;
   info->host_bytes = h->host_bytes;

@@ -174,22 +174,21 @@ apsp_status setup_device(Handle* h, const apsp_config& cfg) {
       cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
     }
   }
-  g_minplus_variant = cfg.reserved[3];  // test hook: min-plus kernel variant (apsp_kernels.cuh)
-  // reserved[4]: 0 = auto (the persistent dataflow kernel for int32; the launch-per-phase
-  // schedule for fp32, measured faster there: DESIGN.md §5), 1 = launch-per-phase, 2 = dataflow
-  // Sharded placements (world > 1, virtual ranks, NCCL at world 1) default to the
-  // launch-per-phase schedule with NCCL broadcasts; reserved[4] = 2 selects the sharded
-  // dataflow kernel (peer stores of the pivot panels).
-  const bool sharded = h->world > 1 || cfg.reserved[2] == 1;
-  h->dataflow = cfg.reserved[4] == 2 || (cfg.reserved[4] == 0 && !sharded);
-  h->df_delay = cfg.reserved[5];
+  g_minplus_variant = cfg.minplus_variant;  // launch-per-phase min-plus kernel (apsp_kernels.cuh)
+  // schedule: APSP_SCHED_AUTO = the persistent dataflow kernel on one GPU (int32 and fp32);
+  // sharded placements (world > 1, virtual ranks, NCCL at world 1) default to the
+  // launch-per-phase schedule with NCCL broadcasts; APSP_SCHED_DATAFLOW selects the sharded
+  // dataflow kernel there (peer stores of the pivot panels).
+  const bool sharded = h->world > 1 || cfg.force_nccl == 1;
+  h->dataflow = cfg.schedule == APSP_SCHED_DATAFLOW || (cfg.schedule == APSP_SCHED_AUTO && !sharded);
+  h->df_delay = cfg.dataflow_delay;
   if (cfg.stream) {
     h->stream = static_cast<cudaStream_t>(cfg.stream);
   } else {
     if ((st = h->cuda(cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking), "cudaStreamCreate"))) return st;
     h->own_stream = true;
   }
-  if (!cfg.reserved[1]) {  // reserved[1] = 1 disables the lookahead (tests / A-B timing)
+  if (!cfg.no_lookahead) {  // the launch-per-phase lookahead's side stream (off: tests / A-B timing)
     int lo = 0, hi = 0;
     cudaDeviceGetStreamPriorityRange(&lo, &hi);
     if ((st = h->cuda(cudaStreamCreateWithPriority(&h->side, cudaStreamNonBlocking, hi), "side stream"))) return st;
@@ -206,9 +205,9 @@ static apsp_status init_placement(Handle* h, const apsp_config& cfg, const int64
   apsp_status st;
   const int nshards = h->virt ? h->world : 1;
   const long long mat_bytes = (long long)nshards * h->rows_per_rank * h->ld * (long long)h->elem;
-  // reserved[2] = 1: run the sharded schedule with a 1-rank NCCL communicator even
-  // at world_size 1, so a single GPU exercises the broadcast / all-reduce path
-  h->use_comm = (h->world > 1 && !h->virt) || (h->world == 1 && cfg.reserved[2] == 1);
+  // force_nccl: run the sharded schedule with a 1-rank NCCL communicator even at
+  // world_size 1, so a single GPU exercises the broadcast / all-reduce path
+  h->use_comm = (h->world > 1 && !h->virt) || (h->world == 1 && cfg.force_nccl == 1);
   // two pivot-band panels (double-buffered by round parity)
   const long long panel_bytes =
       (h->world > 1 || h->use_comm) ? 2 * (long long)h->b * h->ld * (long long)h->elem : 0;
@@ -216,7 +215,10 @@ static apsp_status init_placement(Handle* h, const apsp_config& cfg, const int64
   if ((st = h->cuda(cudaMemGetInfo(&free_b, &total_b), "cudaMemGetInfo"))) return st;
   long long budget = cfg.device_budget_bytes > 0 ? cfg.device_budget_bytes
                                                  : (long long)free_b - (1ll << 30);  // keep 1 GiB headroom
-  const bool need_ooc = cfg.force_out_of_core || (mat_bytes + panel_bytes > budget);
+  // a caller-owned matrix (cfg.dist_device, checked against mat_bytes by apsp_init_from_csr)
+  // keeps the handle in core; only the library's own buffers count against the budget
+  const bool need_ooc =
+      cfg.force_out_of_core || ((cfg.dist_device ? 0 : mat_bytes) + panel_bytes > budget);
   if (need_ooc) {
     if (h->world > 1) return h->fail(APSP_ENOMEM, "matrix shard (%lld B) exceeds the device budget (%lld B); "
                                      "out-of-core x multi-GPU is not supported", mat_bytes, budget);
@@ -226,13 +228,18 @@ static apsp_status init_placement(Handle* h, const apsp_config& cfg, const int64
 
   // packed int16 (R16): single GPU, in core, int32 weights in [0, 8191]
   h->mode16 = cfg.packed16 == 1 && h->dtype == APSP_I32 && !h->has_neg && h->max_abs_w <= 8191 &&
-              h->world == 1 && !h->virt && cfg.reserved[2] != 1;
+              h->world == 1 && !h->virt && cfg.force_nccl != 1;
   if (h->mode16) {
     const long long b16 = h->n_pad * h->n_pad * 2;
-    if ((st = h->cuda(cudaMallocAsync(reinterpret_cast<void**>(&h->d16), b16, h->stream), "cudaMalloc dist16")))
+    if (cfg.dist_device) {  // int16 working matrix in the first half; the int32 redo reuses the whole buffer
+      h->dist_external = true;
+      h->d16 = static_cast<short*>(cfg.dist_device);
+    } else if ((st = h->cuda(cudaMallocAsync(reinterpret_cast<void**>(&h->d16), b16, h->stream),
+                             "cudaMalloc dist16"))) {
       return st;
+    }
     if ((st = h->cuda(cudaMalloc(&h->d_max16, sizeof(int)), "cudaMalloc"))) return st;
-    h->device_bytes = b16;
+    h->device_bytes = h->dist_external ? 0 : b16;
     Shard sh;  // the int32 matrix is allocated only if the int16 result must be redone
     h->shards.push_back(sh);
     if ((st = upload_csr<int>(h, row_ptr, col, w))) return st;
@@ -240,8 +247,13 @@ static apsp_status init_placement(Handle* h, const apsp_config& cfg, const int64
     return h->cuda(cudaStreamSynchronize(h->stream), "init sync");
   }
 
-  if ((st = h->cuda(cudaMallocAsync(&h->d_base, mat_bytes, h->stream), "cudaMalloc dist"))) return st;
-  h->device_bytes = mat_bytes;
+  if (cfg.dist_device) {
+    h->dist_external = true;
+    h->d_base = cfg.dist_device;
+  } else {
+    if ((st = h->cuda(cudaMallocAsync(&h->d_base, mat_bytes, h->stream), "cudaMalloc dist"))) return st;
+    h->device_bytes = mat_bytes;
+  }
   if (panel_bytes) {
     if ((st = h->cuda(cudaMallocAsync(&h->panel, panel_bytes, h->stream), "cudaMalloc panel"))) return st;
     h->device_bytes += panel_bytes;
@@ -351,9 +363,13 @@ static apsp_status run_fw16_int32(Handle* h) {
   Shard& sh = h->shards[0];
   if (!sh.D) {
     const long long mat_bytes = h->n_pad * h->ld * 4;
-    if ((st = h->cuda(cudaMallocAsync(&h->d_base, mat_bytes, h->stream), "cudaMalloc dist (int32 fallback)")))
-      return st;
-    h->device_bytes += mat_bytes;
+    if (h->dist_external) {  // the caller's buffer (it held the int16 working matrix)
+      h->d_base = h->d16;
+    } else {
+      if ((st = h->cuda(cudaMallocAsync(&h->d_base, mat_bytes, h->stream), "cudaMalloc dist (int32 fallback)")))
+        return st;
+      h->device_bytes += mat_bytes;
+    }
     sh.D = h->d_base;
   }
   if ((st = h->cuda(launch_init_rows<int>(static_cast<int*>(sh.D), h->ld, h->n_pad, 0, h->n_pad, h->n, sh.d_rp,
@@ -373,8 +389,10 @@ void delete_handle(Handle* h) {
   if (h->stream) {
     // large buffers come from the device's stream-ordered pool (cudaMallocAsync); the
     // pool keeps them for the next handle instead of returning them to the driver
-    if (h->d_base) cudaFreeAsync(h->d_base, h->stream);
-    if (h->d16) cudaFreeAsync(h->d16, h->stream);
+    if (!h->dist_external) {  // a caller-owned apsp_config.dist_device is never freed here
+      if (h->d_base) cudaFreeAsync(h->d_base, h->stream);
+      if (h->d16) cudaFreeAsync(h->d16, h->stream);
+    }
     if (h->panel) cudaFreeAsync(h->panel, h->stream);
     if (h->df_work) cudaFreeAsync(h->df_work, h->stream);
     if (h->virt)

@@ -70,6 +70,7 @@ struct Handle {
   cudaEvent_t ev_la[2] = {nullptr, nullptr};
   std::vector<Shard> shards;
   void* d_base = nullptr;   // allocation behind the shards (in-core)
+  bool dist_external = false;  // d_base / d16 is the caller's apsp_config.dist_device (not freed)
   void* panel = nullptr;    // b x ld pivot band received from the owner
   int* d_flag = nullptr;    // negative-cycle flag (device)
   void* comm = nullptr;     // ncclComm_t
@@ -84,8 +85,8 @@ struct Handle {
   // Johnson's algorithm, batched Near-Far (apsp_johnson.cu)
   void* jn = nullptr;
   // single-GPU in-core dataflow kernel (apsp_fw_dataflow.cu)
-  bool dataflow = true;     // apsp_config.reserved[4] = 1 selects the launch-per-phase schedule
-  long long df_delay = 0;   // reserved[5] (0 = auto)
+  bool dataflow = true;     // apsp_config.schedule (APSP_SCHED_PER_PHASE: launch per phase)
+  long long df_delay = 0;   // apsp_config.dataflow_delay (0 = auto)
   void* df_work = nullptr;
   // sharded dataflow kernel (multi-GPU / virtual ranks): per-rank work buffers
   std::vector<void*> sh_work;          // virtual ranks: one per shard (pool); NCCL ranks: this rank's (cudaMalloc, IPC)
@@ -157,8 +158,9 @@ void ooc_free(Handle* h);
 apsp_status ooc_reinit(Handle* h);
 
 // boundary algorithm (apsp_boundary.cu)
-apsp_status bnd_setup(Handle* h, const int64_t* row_ptr, const int32_t* col, const void* w, const int32_t* comp,
-                      int k);
+apsp_status bnd_setup(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, const int32_t* col, const void* w,
+                      const int32_t* comp, int k);
+long long bnd_ooc_rows(const Handle* h);  // out of core: rows per output buffer, else 0
 apsp_status bnd_reinit(Handle* h);
 apsp_status bnd_run(Handle* h);
 apsp_status bnd_get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out);

@@ -96,7 +96,7 @@ cudaError_t launch_widen16(const short* S, long long lds, int* D, long long ldd,
 cudaError_t configure_kernels16();
 
 // The TMA + mbarrier persistent variant of launch_minplus (apsp_minplus_tma.cu).
-// g_minplus_variant (set from apsp_config.reserved[3]): 0 = cp.async +
+// g_minplus_variant (set from apsp_config.minplus_variant): 0 = cp.async +
 // mbarrier pipeline (default), 1 = cp.async + one CTA barrier per chunk,
 // 2 = TMA persistent kernel (measured slower in round 1: its persistent grid
 // also blocks the lookahead phases 1+2).

@@ -48,6 +48,8 @@ apsp_status fw_seconds_per_relax(const apsp_config& cfg, long long n0, double* o
   c.device_budget_bytes = 0;
   c.packed16 = 0;
   c.timing = 0;
+  c.dist_device = nullptr;  // the calibration graph gets its own matrix
+  c.dist_device_bytes = 0;
   apsp_handle* h = nullptr;
   apsp_status st = apsp_init_from_csr(&h, n0, rp.data(), col.data(), w.data(), APSP_I32, &c);
   if (st) {

@@ -130,3 +130,52 @@ def test_binding_refuses_short_csr_arrays(lib, short):
         with pytest.raises(lib.ApspError) as e:
             call()
         assert e.value.status == lib.APSP_EINVAL and "row_ptr[n]" in str(e.value)
+
+
+def test_config_named_fields_and_reserved(lib):
+    """The schedule / test switches are named apsp_config fields; reserved[] must stay zero
+    (checked before any device work, so APSP_EINVAL even without a GPU)."""
+    names = [f[0] for f in lib.apsp_config._fields_]
+    for f in ("dist_device", "dist_device_bytes", "schedule", "no_lookahead", "ooc_stream_all", "force_nccl",
+              "minplus_variant", "dataflow_delay", "reserved"):
+        assert f in names, f
+    hdr = open(os.path.join(ROOT, "include", "apsp.h")).read()
+    body = hdr[hdr.index("typedef struct {\n  int32_t struct_size;"):hdr.index("} apsp_config;")]
+    body = re.sub(r"/\*.*?\*/", "", body, flags=re.S)
+    assert re.findall(r"\b(\w+)(?:\[\d+\])?;", body) == names  # same order as the C struct
+    assert (lib.APSP_SCHED_AUTO, lib.APSP_SCHED_PER_PHASE, lib.APSP_SCHED_DATAFLOW) == (0, 1, 2)
+    g = gg.erdos_renyi(20, 60, seed=1)
+    for field, val in (("reserved", 1), ("schedule", 7), ("minplus_variant", 3), ("dataflow_delay", -1)):
+        cfg = lib.apsp_config_default()
+        if field == "reserved":
+            cfg.reserved[2] = val
+        else:
+            setattr(cfg, field, val)
+        with pytest.raises(lib.ApspError) as e:
+            lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=cfg)
+        assert e.value.status == lib.APSP_EINVAL, field
+
+
+@pytest.mark.parametrize("n,world,virt", [(1, 1, 0), (300, 1, 0), (16384, 1, 0), (1000, 2, 0), (1000, 4, 1),
+                                          (65536, 8, 0)])
+def test_dist_device_bytes(lib, n, world, virt):
+    n_pad, _, _ = lib.apsp_partition(n, world, 0)
+    want = (n_pad // world) * n_pad * 4 * (world if virt else 1)
+    assert lib.apsp_dist_device_bytes(n, world, virt) == want
+
+
+def test_dist_device_too_small_or_misaligned_is_refused(lib):
+    g = gg.erdos_renyi(300, 900, seed=2)
+    need = lib.apsp_dist_device_bytes(g.n)
+    for ptr, nbytes in ((1 << 20, need - 4), ((1 << 20) + 64, need)):  # never dereferenced: refused first
+        cfg = lib.apsp_config_default(dist_device=ptr, dist_device_bytes=nbytes)
+        with pytest.raises(lib.ApspError) as e:
+            lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=cfg)
+        assert e.value.status == lib.APSP_EINVAL
+    cfg = lib.apsp_config_default(dist_device=1 << 20, dist_device_bytes=need)
+    comp = np.zeros(g.n, np.int32)
+    for call in (lambda: lib.apsp_init_johnson(g.n, g.row_ptr, g.col, g.w, cfg=cfg),
+                 lambda: lib.apsp_init_boundary(g.n, g.row_ptr, g.col, g.w, comp, 1, cfg=cfg)):
+        with pytest.raises(lib.ApspError) as e:
+            call()
+        assert e.value.status == lib.APSP_EINVAL

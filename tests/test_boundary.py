@@ -189,3 +189,91 @@ def test_boundary_gpu_config2_size(lib):
             assert np.array_equal(lib.apsp_get_dist(h, int(s), 1)[0].astype(np.int64), want[i])
         blk = lib.apsp_get_dist(h, 100, 300)
         assert np.array_equal(blk[:, srcs].T.astype(np.int64), want[:, 100:400])
+
+
+# --------------------------------------------------- out of core (Alg. 3 l.20)
+
+
+def bnd_cfg(lib, budget=0, force=1):
+    return lib.apsp_config_default(device=0, timing=1, force_out_of_core=force, device_budget_bytes=budget)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("shape,blocks", [((20, 30), (2, 3)), ((40, 40), (4, 4)), ((33, 17), (3, 1)),
+                                          ((64, 48), (8, 6))])
+def test_boundary_out_of_core_forced(lib, shape, blocks):
+    """Every block row streams through the two device buffers into pinned host memory
+    (force_out_of_core), then apsp_get_dist gathers from the host matrix: bit-exact."""
+    g = gg.grid_2d(*shape, seed=shape[1])
+    comp, k = gg.grid_block_partition(g, *blocks)
+    with lib.apsp_init_boundary(g.n, g.row_ptr, g.col, g.w, comp, k, cfg=bnd_cfg(lib)) as h:
+        info = lib.apsp_get_info(h)
+        assert info.mode == lib.APSP_MODE_BOUNDARY and info.ooc_block > 0 and info.host_bytes > 0
+        lib.apsp_solve(h)
+        got = lib.apsp_get_dist(h)
+        st = lib.apsp_get_phase_stats(h)
+        assert st.launches[3] > 0  # the D2H transfers are inside the solve (P:531)
+        lib.apsp_reinit(h)
+        lib.apsp_solve(h)
+        assert np.array_equal(lib.apsp_get_dist(h, 3, 50), got[3:53])
+    assert np.array_equal(got.astype(np.int64), oracle_i32(g))
+
+
+@pytest.mark.gpu
+def test_boundary_out_of_core_budget_many_groups_and_residency(lib):
+    """A device budget (L of P:186) small enough that each buffer holds one or two block rows
+    (N_row), so many groups alternate between the two buffers / streams; a larger budget keeps
+    the last block rows resident in HBM (R21) while the rest stream: both bit-exact."""
+    g = gg.grid_2d(96, 64, seed=9)  # n = 6144
+    comp, k = gg.grid_block_partition(g, 6, 4)  # 24 components of 256 vertices
+    want = oracle_i32(g)
+    seen = set()
+    for budget in (40 << 20, 64 << 20, 120 << 20):
+        with lib.apsp_init_boundary(g.n, g.row_ptr, g.col, g.w, comp, k, cfg=bnd_cfg(lib, budget, 0)) as h:
+            info = lib.apsp_get_info(h)
+            assert info.ooc_block > 0, "the result (%d B) must not fit %d B" % (info.n_pad ** 2 * 4, budget)
+            seen.add((info.host_bytes < info.n_pad ** 2 * 4, info.ooc_block))
+            lib.apsp_solve(h)
+            assert np.array_equal(lib.apsp_get_dist(h).astype(np.int64), want), budget
+    assert any(part for part, _ in seen), "no budget left block rows resident"
+
+
+@pytest.mark.gpu
+def test_boundary_out_of_core_disjoint_negative_f32(lib):
+    # components without boundary nodes (their rows / columns stay +inf but for dist2)
+    g2 = gg.disjoint_union(gg.grid_2d(10, 20, seed=1), gg.erdos_renyi(150, 600, seed=2))
+    comp2 = np.r_[np.zeros(200), np.ones(150)].astype(np.int32)
+    with lib.apsp_init_boundary(g2.n, g2.row_ptr, g2.col, g2.w, comp2, 2, cfg=bnd_cfg(lib)) as h:
+        lib.apsp_solve(h)
+        assert np.array_equal(lib.apsp_get_dist(h).astype(np.int64), oracle_i32(g2))
+    g = gg.grid_2d(24, 24, seed=7)
+    p = np.random.default_rng(3).integers(-300, 300, size=g.n)
+    s, t, w = g.arcs()
+    gn = gg.csr_from_arcs(g.n, s, t, (w.astype(np.int64) + p[s] - p[t]).astype(np.int32))
+    gn.meta = g.meta
+    comp, k = gg.grid_block_partition(gn, 3, 3)
+    with lib.apsp_init_boundary(gn.n, gn.row_ptr, gn.col, gn.w, comp, k, cfg=bnd_cfg(lib)) as h:
+        lib.apsp_solve(h)
+        assert np.array_equal(lib.apsp_get_dist(h).astype(np.int64), oracle_i32(gn))
+    gf = gg.grid_2d(25, 30, seed=2, dtype="f32")
+    comp, k = gg.grid_block_partition(gf, 2, 3)
+    with lib.apsp_init_boundary(gf.n, gf.row_ptr, gf.col, gf.w, comp, k, cfg=bnd_cfg(lib)) as h:
+        lib.apsp_solve(h)
+        got = lib.apsp_get_dist(h)
+    want, _ = oracle.fw_f64(gf.row_ptr, gf.col, gf.w)
+    assert np.all(np.abs(got - want) <= 1e-5 * np.abs(want))
+
+
+@pytest.mark.gpu
+def test_boundary_out_of_core_config2_certified(lib):
+    """Config 2's grid, k = sqrt(n)/4 = 32 components, forced out of core with a
+    budget: EVERY row proven by the oracle's optimality certificate."""
+    g = gg.baseline_config("cfg2_grid16384")
+    comp, k = gg.grid_block_partition(g, 4, 8)
+    with lib.apsp_init_boundary(g.n, g.row_ptr, g.col, g.w, comp, k, cfg=bnd_cfg(lib, 600 << 20, 0)) as h:
+        info = lib.apsp_get_info(h)
+        assert info.ooc_block > 0 and info.host_bytes > 0
+        lib.apsp_solve(h)
+        for r0 in range(0, g.n, 4096):
+            rows = lib.apsp_get_dist(h, r0, 4096)
+            assert oracle.certify_rows_i32(g.row_ptr, g.col, g.w, r0, rows, INF32) == (0, -1), r0

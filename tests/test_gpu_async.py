@@ -130,7 +130,7 @@ def test_async_other_placements(lib, placement):
     elif placement == "packed16":
         c.packed16 = 1
     else:
-        c.reserved[4] = 1
+        c.schedule = 1
     out = pinned(640, False)
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
         lib.apsp_fw_blocked_async(h)

@@ -44,7 +44,7 @@ def test_checkpoint_resume_out_of_core(lib, tmp_path):
 
     def cfg():
         c = lib.apsp_config_default(device=0, force_out_of_core=1, ooc_block=256)
-        c.reserved[0] = 1
+        c.ooc_stream_all = 1
         return c
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=cfg()) as h:
         assert lib.apsp_get_info(h).mode == lib.APSP_MODE_OUT_OF_CORE

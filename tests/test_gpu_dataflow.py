@@ -1,11 +1,11 @@
 """The persistent dataflow kernel (csrc/apsp_fw_dataflow.cu): every round and phase of the
 blocked FW in one launch, tasks ordered by a global queue and synchronised
 by per-tile flags. It is the default single-GPU in-core path, so every test in
-test_gpu_parity.py that does not set reserved[4] already runs it; this file stresses the
+test_gpu_parity.py that does not set schedule already runs it; this file stresses the
 parts specific to it: the queue order at every tile count (segment boundaries, nb = 1, 2,
-3), the queue delay of the panel tasks (reserved[5]: 1 = panels right behind the
+3), the queue delay of the panel tasks (dataflow_delay: 1 = panels right behind the
 diagonal, huge = panels after the whole previous phase 3), deep round overlap on small
-matrices, and agreement with the launch-per-phase schedule (reserved[4] = 1).
+matrices, and agreement with the launch-per-phase schedule (schedule = APSP_SCHED_PER_PHASE).
 """
 import numpy as np
 import pytest
@@ -26,8 +26,8 @@ def want_i32(g):
 
 def run(lib, g, delay=0, legacy=False, timing=0):
     c = lib.apsp_config_default(device=0, timing=timing)
-    c.reserved[4] = 1 if legacy else 2  # 2 = the dataflow kernel (the single-GPU default for both dtypes)
-    c.reserved[5] = delay
+    c.schedule = 1 if legacy else 2  # 2 = the dataflow kernel (the single-GPU default for both dtypes)
+    c.dataflow_delay = delay
     return lib.solve(g, cfg=c)
 
 

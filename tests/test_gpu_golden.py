@@ -35,7 +35,7 @@ def check(got, src, dist):
 def test_golden_fw_i32(lib, name, schedule):
     g, src, dist = load(name)
     c = lib.apsp_config_default(device=0)
-    c.reserved[4] = schedule
+    c.schedule = schedule
     check(lib.solve(g, cfg=c).astype(np.int64), src, dist)
 
 
@@ -51,7 +51,7 @@ def test_golden_fw_f32(lib, name):
 def test_golden_packed16(lib, legacy):
     g, src, dist = load("clrs_fig24_6.txt")  # non-negative weights: int16-eligible
     c = lib.apsp_config_default(device=0, packed16=1)
-    c.reserved[4] = legacy
+    c.schedule = legacy
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
         assert lib.apsp_get_info(h).packed16_eligible
         lib.apsp_fw_blocked(h)

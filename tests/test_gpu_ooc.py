@@ -16,7 +16,7 @@ def ooc_cfg(lib, block, budget_mb=0, stream_all=True):
     if budget_mb:
         c.device_budget_bytes = int(budget_mb * 2 ** 20)
     if stream_all:
-        c.reserved[0] = 1
+        c.ooc_stream_all = 1
     return c
 
 

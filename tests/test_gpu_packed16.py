@@ -1,7 +1,7 @@
 """Packed int16 path (apsp_config.packed16 = 1; VIADDMNMX.S16x2, two relaxations per DPX
 instruction): bit-exact against the int32 oracle, with the exactness check and the int32
 redo exercised (reading R16). Both schedules: the persistent dataflow kernel
-(fw_dataflow16_kernel, the default) and the launch-per-phase kernels (reserved[4] = 1)."""
+(fw_dataflow16_kernel, the default) and the launch-per-phase kernels (schedule = APSP_SCHED_PER_PHASE)."""
 import numpy as np
 import pytest
 
@@ -20,8 +20,8 @@ def want_i32(g):
 
 def run16(lib, g, legacy=False, delay=0):
     c = lib.apsp_config_default(device=0, packed16=1, timing=1)
-    c.reserved[4] = 1 if legacy else 0
-    c.reserved[5] = delay
+    c.schedule = 1 if legacy else 0
+    c.dataflow_delay = delay
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
         eligible = lib.apsp_get_info(h).packed16_eligible
         lib.apsp_fw_blocked(h)

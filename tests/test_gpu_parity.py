@@ -85,29 +85,29 @@ def test_fw_int32_bit_exact(lib, n):
 @pytest.mark.parametrize("variant", [1, 2])
 @pytest.mark.parametrize("n", [129, 640, 1000])
 def test_fw_minplus_variants(lib, n, variant):
-    """reserved[3] selects the min-plus kernel: 1 = cp.async + one CTA barrier per chunk,
+    """minplus_variant selects the min-plus kernel: 1 = cp.async + one CTA barrier per chunk,
     2 = TMA + mbarrier persistent (0, the cp.async + mbarrier pipeline, is the default)."""
     for name, g in graphs_for(n, seed=n + 3):
         c = cfg(lib)
-        c.reserved[3] = variant
-        c.reserved[4] = 1  # launch-per-phase schedule (the min-plus launches take the variant)
+        c.minplus_variant = variant
+        c.schedule = 1  # launch-per-phase schedule (the min-plus launches take the variant)
         got = lib.solve(g, cfg=c)
         want, _ = oracle_i32(g)
         assert_i32_equal(got, want)
     gf = gg.erdos_renyi(n, 6 * n, seed=n, dtype="f32")
     c = cfg(lib)
-    c.reserved[3] = variant
-    c.reserved[4] = 1
+    c.minplus_variant = variant
+    c.schedule = 1
     assert_f32_close(lib.solve(gf, cfg=c), oracle.fw_f64(gf.row_ptr, gf.col, gf.w)[0])
 
 
 @pytest.mark.parametrize("n", [384, 640, 1000])
 def test_fw_without_lookahead(lib, n):
-    """reserved[1] = 1 runs phases 1-3 strictly in order on one stream (no split phase 3)."""
+    """no_lookahead = 1 runs phases 1-3 strictly in order on one stream (no split phase 3)."""
     for name, g in graphs_for(n, seed=n + 7):
         c = cfg(lib)
-        c.reserved[1] = 1
-        c.reserved[4] = 1
+        c.no_lookahead = 1
+        c.schedule = 1
         got = lib.solve(g, cfg=c)
         want, _ = oracle_i32(g)
         assert_i32_equal(got, want)
@@ -199,7 +199,7 @@ def test_get_dist_row_ranges(lib):
 def test_fw_f32_integer_weights_bit_exact(lib, n, sched):
     g = gg.erdos_renyi(n, 5 * n, seed=n, dtype="f32int")
     c = cfg(lib)
-    c.reserved[4] = sched
+    c.schedule = sched
     got = lib.solve(g, cfg=c)
     gi = gg.csr_from_arcs(g.n, *g.arcs()[:2], g.w.astype(np.int32))
     want, _ = oracle.fw_i64(gi.row_ptr, gi.col, gi.w)
@@ -212,7 +212,7 @@ def test_fw_f32_integer_weights_bit_exact(lib, n, sched):
 def test_fw_f32_real_weights(lib, n, sched):
     g = gg.erdos_renyi(n, 8 * n, seed=n + 1, dtype="f32")
     c = cfg(lib)
-    c.reserved[4] = sched
+    c.schedule = sched
     got = lib.solve(g, cfg=c)
     want, _ = oracle.fw_f64(g.row_ptr, g.col, g.w)
     assert_f32_close(got, want)
@@ -247,11 +247,11 @@ def test_virtual_ranks_match_oracle(lib, world):
 
 @pytest.mark.parametrize("world", [2, 4])
 def test_virtual_ranks_without_lookahead(lib, world):
-    """reserved[1] = 1: the sharded schedule round by round on one stream (no pivot lookahead)."""
+    """no_lookahead = 1: the sharded schedule round by round on one stream (no pivot lookahead)."""
     for g in [gg.grid_2d(20, 33, seed=world + 7), gg.erdos_renyi(1100, 4000, seed=world + 7)]:
         c = cfg(lib, world_size=world, virtual_ranks=1)
-        c.reserved[1] = 1
-        c.reserved[4] = 1  # launch-per-phase sharded schedule (the dataflow kernel ignores reserved[1])
+        c.no_lookahead = 1
+        c.schedule = 1  # launch-per-phase sharded schedule (the dataflow kernel ignores no_lookahead)
         assert_i32_equal(lib.solve(g, cfg=c), oracle_i32(g)[0])
 
 
@@ -263,20 +263,20 @@ def test_virtual_ranks_f32(lib):
 
 @pytest.mark.parametrize("sched", [2, 0], ids=["sharded_dataflow", "per_phase_bcast"])
 def test_nccl_path_single_rank(lib, sched):
-    """reserved[2] = 1: the sharded schedules with a real 1-rank NCCL communicator: the
-    sharded dataflow kernel (reserved[4] = 2; barrier + status all-reduce through NCCL) or the
+    """force_nccl = 1: the sharded schedules with a real 1-rank NCCL communicator: the
+    sharded dataflow kernel (schedule = APSP_SCHED_DATAFLOW; barrier + status all-reduce through NCCL) or the
     launch-per-phase schedule (default: ncclBroadcast of the pivot band every round)."""
     for g in [gg.grid_2d(17, 31, seed=1), gg.erdos_renyi(700, 2800, seed=2)]:
         c = cfg(lib)
-        c.reserved[2] = 1
-        c.reserved[4] = sched
+        c.force_nccl = 1
+        c.schedule = sched
         got = lib.solve(g, cfg=c)
         want, _ = oracle_i32(g)
         assert_i32_equal(got, want)
     g = gg.with_arcs(gg.erdos_renyi(300, 900, seed=3), [10, 290], [290, 10], [-100, 20])
     c = cfg(lib)
-    c.reserved[2] = 1
-    c.reserved[4] = sched
+    c.force_nccl = 1
+    c.schedule = sched
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
         with pytest.raises(lib.NegativeCycleError):
             lib.apsp_fw_blocked(h)
@@ -294,7 +294,7 @@ def test_virtual_ranks_negative_cycle(lib):
 def test_phase_stats_count_all_relaxations(lib):
     g = gg.erdos_renyi(1000, 5000, seed=1)
     c = cfg(lib, timing=1)
-    c.reserved[4] = 1  # launch-per-phase schedule
+    c.schedule = 1  # launch-per-phase schedule
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
         lib.apsp_fw_blocked(h)
         st = lib.apsp_get_phase_stats(h)

@@ -4,7 +4,7 @@ straight into every rank's panel buffer and raises their flags (peer stores; no 
 between rounds). Run here as P virtual ranks in ONE launch on one GPU (CTA b serves rank
 b % P), which exercises the same queue decoding, flag protocol and peer stores as P GPUs;
 bit-exact against the oracle and against the launch-per-phase sharded schedule. Selected
-with apsp_config.reserved[4] = 2 (sharded placements default to the launch-per-phase
+with apsp_config.schedule = 2 (sharded placements default to the launch-per-phase
 schedule with NCCL broadcasts)."""
 import numpy as np
 import pytest
@@ -24,8 +24,8 @@ def want_i32(g):
 
 def solve(lib, g, world, sched=2, delay=0, **kw):
     c = lib.apsp_config_default(device=0, world_size=world, virtual_ranks=1, **kw)
-    c.reserved[4] = sched
-    c.reserved[5] = delay
+    c.schedule = sched
+    c.dataflow_delay = delay
     return lib.solve(g, cfg=c)
 
 
@@ -59,7 +59,7 @@ def test_sharded_dataflow_equals_per_phase_and_repeats(lib):
     b = solve(lib, g, 4, sched=1)
     assert np.array_equal(a, b)
     c = lib.apsp_config_default(device=0, world_size=4, virtual_ranks=1)
-    c.reserved[4] = 2
+    c.schedule = 2
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
         for _ in range(3):  # flags are zeroed per run; the shard buffers are reused
             lib.apsp_reinit(h)
@@ -82,7 +82,7 @@ def test_sharded_dataflow_negative_cycle(lib, where):
     u, v = {"first_rank": (3, 40), "rank_boundary": (255, 256), "last_rank": (1000, 1020)}[where]
     g = gg.with_arcs(gg.erdos_renyi(n, 4 * n, seed=6), [u, v], [v, u], [-250, 100])
     c = lib.apsp_config_default(device=0, world_size=4, virtual_ranks=1)
-    c.reserved[4] = 2
+    c.schedule = 2
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
         with pytest.raises(lib.NegativeCycleError):
             lib.apsp_fw_blocked(h)

@@ -424,3 +424,20 @@ def test_certificate_disconnected_and_rejects_zero_weights():
     z = csr_of(3, [(0, 1, 0), (1, 2, 4)])
     with pytest.raises(ValueError):
         oracle.certify_rows_i32(z.row_ptr, z.col, z.w, 0, np.zeros((3, 3), np.int32), INF32)
+
+
+def test_duplicates_and_self_loops_f64():
+    """R2/R3 for the fp64 oracle (init_f64 + fw_f64): duplicate arcs keep the minimum weight, a
+    positive self-loop leaves the diagonal at 0, a negative one is a negative cycle; values the
+    worked-out closure below fixes by hand."""
+    g = csr_of(3, [(0, 1, 9.5), (0, 1, 4.25), (0, 1, 7.0), (1, 1, 5.0), (1, 2, 2.5), (2, 2, 0.5)], np.float32)
+    d0 = oracle.init_f64(g.row_ptr, g.col, g.w)
+    assert d0.tolist() == [[0.0, 4.25, np.inf], [np.inf, 0.0, 2.5], [np.inf, np.inf, 0.0]]
+    d, neg = oracle.fw_f64(g.row_ptr, g.col, g.w)
+    assert not neg
+    assert d.tolist() == [[0.0, 4.25, 6.75], [np.inf, 0.0, 2.5], [np.inf, np.inf, 0.0]]
+    g = csr_of(2, [(0, 1, 1.0), (1, 1, -0.5)], np.float32)
+    d0 = oracle.init_f64(g.row_ptr, g.col, g.w)
+    assert d0[1, 1] == -0.5  # min(0, w) on the diagonal
+    _, neg = oracle.fw_f64(g.row_ptr, g.col, g.w)
+    assert neg

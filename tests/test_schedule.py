@@ -84,7 +84,9 @@ def simulate(nb, queues):
     return True
 
 
-@pytest.mark.parametrize("nb,delay", [(1, 8), (2, 8), (3, 1), (5, 3), (9, 1184), (16, 40), (40, 1)])
+# nb >= 67 takes phase 3's multi-band branch (64-column bands, apsp_df_common.cuh); nb = 130 is a ragged two-band + remainder case
+@pytest.mark.parametrize("nb,delay", [(1, 8), (2, 8), (3, 1), (5, 3), (9, 1184), (16, 40), (40, 1), (70, 1184),
+                                      (130, 592)])
 def test_single_gpu_queue_complete_and_deadlock_free(lib, nb, delay):
     q = lib.apsp_debug_queue(nb, 0, 0, delay)
     assert len(q) == nb ** 3
@@ -93,7 +95,8 @@ def test_single_gpu_queue_complete_and_deadlock_free(lib, nb, delay):
 
 
 @pytest.mark.parametrize("nb,P,delay", [(1, 1, 8), (2, 2, 8), (3, 3, 1), (4, 2, 5), (8, 4, 2), (8, 8, 1),
-                                        (12, 3, 37), (16, 8, 4), (24, 4, 1000), (32, 8, 64)])
+                                        (12, 3, 37), (16, 8, 4), (24, 4, 1000), (32, 8, 64), (70, 2, 1184),
+                                        (128, 8, 1184), (130, 2, 64)])
 def test_sharded_queues_complete_and_deadlock_free(lib, nb, P, delay):
     nl = nb // P
     queues = [lib.apsp_debug_queue(nb, P, q, delay) for q in range(P)]

@@ -1,6 +1,6 @@
 #!/usr/bin/env python
 """A/B of the in-core FW schedules on a seeded ER graph: the persistent dataflow kernel vs the
-launch-per-phase schedule (apsp_config.reserved[4] = 1), int32 or fp32.
+launch-per-phase schedule (apsp_config.schedule = 1), int32 or fp32.
 
     python tools/fw_ab.py --n 32768 --deg 256 --dtype f32 --runs 2
 """
@@ -32,7 +32,7 @@ def main():
         if name not in a.modes:
             continue
         cfg = apsp.apsp_config_default(device=0, timing=1, packed16=int(a.packed16))
-        cfg.reserved[4] = legacy
+        cfg.schedule = legacy
         with apsp.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=cfg) as h:
             best = 1e30
             for r in range(a.runs + 1):

@@ -30,8 +30,8 @@ def main():
     a = ap.parse_args()
     g = gg.erdos_renyi(a.er, a.deg * a.er, seed=4, dtype=a.dtype) if a.er else gg.baseline_config(a.workload)
     cfg = apsp.apsp_config_default(device=0)
-    cfg.reserved[4] = 1 if a.legacy else (2 if a.dataflow else 0)
-    cfg.reserved[5] = a.df_delay
+    cfg.schedule = 1 if a.legacy else (2 if a.dataflow else 0)
+    cfg.dataflow_delay = a.df_delay
     cfg.packed16 = 1 if a.packed16 else 0
     if a.ooc_block:
         cfg.force_out_of_core = 1

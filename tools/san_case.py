@@ -21,10 +21,7 @@ import paper_conf_ipps_xia0ar22_b200 as apsp  # noqa: E402
 def run(g, **kw):
     c = apsp.apsp_config_default(device=0)
     for k, v in kw.items():
-        if k.startswith("r"):
-            c.reserved[int(k[1:])] = v
-        else:
-            setattr(c, k, v)
+        setattr(c, k, v)
     with apsp.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
         apsp.apsp_fw_blocked(h)
         return apsp.apsp_get_dist(h)
@@ -46,31 +43,31 @@ def main():
     s, t, w = g.arcs()
     gn = gg.csr_from_arcs(n, s, t, (w + p[s] - p[t]).astype(np.int32))
     if want("dataflow"):
-        same(run(g), run(g, r4=1), "int32 dataflow vs per-phase")
-        same(run(gf, r4=2), run(gf, r4=1), "fp32 dataflow vs per-phase")
-        same(run(g, packed16=1), run(g, packed16=1, r4=1), "packed16 dataflow vs per-phase")
-    if want("barrier"):  # per-phase kernels with CTA barriers only (reserved[3] = 1: no mbarriers)
-        same(run(g, r3=1, r4=1), run(g, r3=1, r4=1, packed16=1), "int32 vs packed16, per-phase CTA-barrier kernels")
-        same(run(gf, r3=1, r4=1), run(gf, r3=1, r4=1, world_size=2, virtual_ranks=1), "fp32 per-phase, 1 vs 2 virtual ranks")
-        same(run(g, packed16=1, r4=1), run(g, r3=1, r4=1), "packed16 per-phase vs int32")
-        same(run(gn, r3=1, r4=1), run(gn, r3=1, r4=1, world_size=2, virtual_ranks=1), "negative weights, 1 vs 2 virtual ranks")
+        same(run(g), run(g, schedule=1), "int32 dataflow vs per-phase")
+        same(run(gf, schedule=2), run(gf, schedule=1), "fp32 dataflow vs per-phase")
+        same(run(g, packed16=1), run(g, packed16=1, schedule=1), "packed16 dataflow vs per-phase")
+    if want("barrier"):  # per-phase kernels with CTA barriers only (minplus_variant = 1: no mbarriers)
+        same(run(g, minplus_variant=1, schedule=1), run(g, minplus_variant=1, schedule=1, packed16=1), "int32 vs packed16, per-phase CTA-barrier kernels")
+        same(run(gf, minplus_variant=1, schedule=1), run(gf, minplus_variant=1, schedule=1, world_size=2, virtual_ranks=1), "fp32 per-phase, 1 vs 2 virtual ranks")
+        same(run(g, packed16=1, schedule=1), run(g, minplus_variant=1, schedule=1), "packed16 per-phase vs int32")
+        same(run(gn, minplus_variant=1, schedule=1), run(gn, minplus_variant=1, schedule=1, world_size=2, virtual_ranks=1), "negative weights, 1 vs 2 virtual ranks")
     if want("ooc"):
-        same(run(gb, force_out_of_core=1, ooc_block=256, r3=1), run(gb, r3=1, r4=1), "out of core vs in core")
-        same(run(gb, world_size=2, virtual_ranks=1, r3=1), run(gb, r3=1, r4=1), "2 virtual ranks vs 1 GPU")
+        same(run(gb, force_out_of_core=1, ooc_block=256, minplus_variant=1), run(gb, minplus_variant=1, schedule=1), "out of core vs in core")
+        same(run(gb, world_size=2, virtual_ranks=1, minplus_variant=1), run(gb, minplus_variant=1, schedule=1), "2 virtual ranks vs 1 GPU")
     if want("neg"):
-        same(run(gn), run(gn, r4=1), "negative weights (canonicalize)")
+        same(run(gn), run(gn, schedule=1), "negative weights (canonicalize)")
     if want("johnson"):
         with apsp.apsp_init_johnson(n, g.row_ptr, g.col, g.w) as h:
             apsp.apsp_solve(h)
             dj = apsp.apsp_get_dist(h)
-        same(dj, run(g, r3=1, r4=1), "Johnson vs blocked FW")
+        same(dj, run(g, minplus_variant=1, schedule=1), "Johnson vs blocked FW")
     if want("boundary"):
         gg2 = gg.grid_2d(16, 16, seed=5, permute=False)
         comp, k = gg.grid_block_partition(gg2, 2, 2)
         with apsp.apsp_init_boundary(gg2.n, gg2.row_ptr, gg2.col, gg2.w, comp, k) as h:
             apsp.apsp_solve(h)
             db = apsp.apsp_get_dist(h)
-        same(db, run(gg2, r3=1, r4=1), "boundary vs blocked FW")
+        same(db, run(gg2, minplus_variant=1, schedule=1), "boundary vs blocked FW")
     if want("async"):
         import torch
         out = torch.empty((n, n), dtype=torch.int32, pin_memory=True)
@@ -79,7 +76,7 @@ def main():
             apsp.apsp_fw_blocked_async(h)
             apsp.apsp_get_dist_async(h, 0, n, out.data_ptr(), n)
             apsp.apsp_synchronize(h)
-        same(out.numpy(), run(gn, r4=1), "load_csr + async vs blocking")
+        same(out.numpy(), run(gn, schedule=1), "load_csr + async vs blocking")
     print("san_case done", flush=True)
 
 

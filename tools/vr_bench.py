@@ -22,10 +22,7 @@ import paper_conf_ipps_xia0ar22_b200 as apsp  # noqa: E402
 def timed(g, runs, **kw):
     c = apsp.apsp_config_default(device=0)
     for k, v in kw.items():
-        if k.startswith("r") and k[1:].isdigit():
-            c.reserved[int(k[1:])] = v
-        else:
-            setattr(c, k, v)
+        setattr(c, k, v)
     with apsp.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
         best = 1e30
         for r in range(runs + 1):
@@ -42,7 +39,7 @@ def main():
     ap.add_argument("--n", type=int, default=16384)
     ap.add_argument("--worlds", type=int, nargs="+", default=[1, 2, 4, 8])
     ap.add_argument("--runs", type=int, default=2)
-    ap.add_argument("--delays", type=int, nargs="+", default=[0], help="queue delays (reserved[5]; 0 = auto)")
+    ap.add_argument("--delays", type=int, nargs="+", default=[0], help="queue delays (dataflow_delay; 0 = auto)")
     a = ap.parse_args()
     g = gg.erdos_renyi(a.n, 8 * a.n, seed=4)
     out = {"n": a.n}
@@ -51,10 +48,10 @@ def main():
             t = timed(g, a.runs)
             out["single_gpu_dataflow"] = {"s": t, "relax_per_s": a.n ** 3 / t}
             continue
-        tp = timed(g, a.runs, world_size=w, virtual_ranks=1, r4=1)
+        tp = timed(g, a.runs, world_size=w, virtual_ranks=1, schedule=1)
         out["virtual_%d" % w] = {"per_phase_bcast_s": tp, "per_phase_relax_per_s": a.n ** 3 / tp}
         for d in a.delays:
-            t = timed(g, a.runs, world_size=w, virtual_ranks=1, r4=2, r5=d)
+            t = timed(g, a.runs, world_size=w, virtual_ranks=1, schedule=2, dataflow_delay=d)
             out["virtual_%d" % w]["sharded_dataflow_delay_%d" % d] = {"s": t, "relax_per_s": a.n ** 3 / t}
     print(json.dumps(out), flush=True)
 
