@@ -68,12 +68,17 @@ typedef enum {
 
 /* apsp_config.schedule: how the in-core blocked FW is scheduled. */
 #define APSP_SCHED_AUTO 0       /* single GPU: the persistent dataflow kernel (all rounds and
-                                   phases in one launch); sharded placements: launch-per-phase
+                                   phases in one launch; 64x64 tiles for n_pad <= 2048, 128x128
+                                   above); sharded placements: launch-per-phase
                                    rounds with NCCL pivot-band broadcasts */
 #define APSP_SCHED_PER_PHASE 1  /* one launch per phase and round (phase 1, phase 2, phase 3) */
 #define APSP_SCHED_DATAFLOW 2   /* the dataflow kernel; on sharded placements its sharded form,
                                    whose round owners store the pivot panels into every rank's
                                    panel buffer over NVLink (peer stores) */
+#define APSP_SCHED_SMALL 3      /* single GPU: the dataflow schedule with 64x64 tiles (b = 64),
+                                   built for small n, where the 128-tile rounds' critical path
+                                   (phase 1 -> panel tile -> next diagonal tile) dominates; AUTO
+                                   selects it for n_pad <= 2048. Sharded placements: as DATAFLOW */
 
 typedef struct {
   int32_t struct_size;          /* = sizeof(apsp_config) (ABI versioning); 0 = defaults */
@@ -173,10 +178,18 @@ apsp_status apsp_init_from_csr(apsp_handle** out, int64_t n, const int64_t* row_
  *   k         number of components, >= 1
  * A vertex with an arc to another component is a boundary node. Work
  * is O(k s^3 + NB^3 + n * NB * s) for components of size s and NB boundary
- * nodes instead of n^3. Single GPU, in core (the n x n result must fit in
- * device memory). Run with apsp_solve; apsp_get_dist as usual.
+ * nodes instead of n^3. Single GPU. When the n x n result does not fit the
+ * device budget (cfg->device_budget_bytes, else free memory) or
+ * cfg->force_out_of_core = 1, the out-of-core form of Algorithm 3 runs: the
+ * diagonal blocks (S_dia) and the boundary matrix (S_bound) stay in HBM, the
+ * remaining memory S_rem holds two buffers of N_row whole block rows that two
+ * streams fill and copy to a pinned host matrix alternately (Alg. 3
+ * l.20); block rows that still fit stay resident in HBM (R21; none
+ * when forced or with cfg->ooc_stream_all). The transfers are part of
+ * apsp_solve. Run with apsp_solve; apsp_get_dist as usual.
  * Errors: as apsp_init_from_csr; APSP_EINVAL for a bad comp / k; APSP_ENOMEM
- * when the result does not fit.
+ * when not even S_dia + S_bound + two one-block-row buffers fit, or pinned
+ * host memory for the streamed rows cannot be allocated.
  */
 apsp_status apsp_init_boundary(apsp_handle** out, int64_t n, const int64_t* row_ptr,
                                const int32_t* col_idx, const void* weights, apsp_dtype dtype,

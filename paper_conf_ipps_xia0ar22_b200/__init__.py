@@ -34,7 +34,7 @@ STATUS_NAMES = ["APSP_OK", "APSP_EINVAL", "APSP_ERANGE", "APSP_ENOMEM", "APSP_EC
 APSP_INF_I32 = 0x3FFFFFFF
 APSP_MODE_INCORE, APSP_MODE_OUT_OF_CORE, APSP_MODE_BOUNDARY, APSP_MODE_JOHNSON = 0, 1, 2, 3
 TILE = 128
-APSP_SCHED_AUTO, APSP_SCHED_PER_PHASE, APSP_SCHED_DATAFLOW = 0, 1, 2
+APSP_SCHED_AUTO, APSP_SCHED_PER_PHASE, APSP_SCHED_DATAFLOW, APSP_SCHED_SMALL = 0, 1, 2, 3
 
 
 class apsp_config(ctypes.Structure):

@@ -261,8 +261,31 @@ static apsp_status sharded_lookahead(Handle* h) {
 // All rounds of a single-GPU in-core closure in one persistent dataflow launch
 // (apsp_fw_dataflow.cu). The phases are not separable in time, so the launch
 // is timed as one event of class 2 carrying all n_pad^3 relaxations.
+// Small n (apsp_fw_small.cu): the same schedule with 64x64 tiles, all rounds in one launch.
+template <typename T>
+static apsp_status run_small(Handle* h) {
+  const int nb = (int)(h->n_pad / 64);
+  apsp_status st;
+  const long long wb = fw_small_work_bytes(nb, sizeof(T));
+  if (!h->df_work) {
+    if ((st = h->cuda(cudaMallocAsync(&h->df_work, wb, h->stream), "cudaMalloc dataflow (small)"))) return st;
+    h->device_bytes += wb;
+  }
+  int ctas = 1;
+  if (const char* e = getenv("APSP_SMALL_CTAS")) ctas = atoi(e);  // tuning experiments only
+  const long long delay = h->df_delay > 0 ? h->df_delay : 0;
+  h->ev_begin(2);
+  if ((st = h->cuda(launch_fw_small<T>(static_cast<T*>(h->shards[0].D), h->ld, nb, h->df_work, h->d_flag, delay, ctas,
+                                       h->stream),
+                    "fw_small")))
+    return st;
+  h->ev_end((double)h->n_pad * h->n_pad * h->n_pad);
+  return APSP_OK;
+}
+
 template <typename T>
 static apsp_status run_dataflow(Handle* h) {
+  if (h->small) return run_small<T>(h);
   const int nb = (int)(h->n_pad / h->b);
   apsp_status st;
   if (!h->df_work) {
@@ -565,7 +588,7 @@ static apsp_status load_config(const apsp_config* cfg_in, apsp_config* cfg) {
   *cfg = *cfg_in;
   for (int32_t r : cfg->reserved)
     if (r != 0) return fail_global(APSP_EINVAL, "apsp_config.reserved must be 0");
-  if (cfg->schedule < APSP_SCHED_AUTO || cfg->schedule > APSP_SCHED_DATAFLOW)
+  if (cfg->schedule < APSP_SCHED_AUTO || cfg->schedule > APSP_SCHED_SMALL)
     return fail_global(APSP_EINVAL, "apsp_config.schedule %d is not an APSP_SCHED_* value", cfg->schedule);
   if (cfg->minplus_variant < 0 || cfg->minplus_variant > 2)
     return fail_global(APSP_EINVAL, "apsp_config.minplus_variant must be 0, 1 or 2");

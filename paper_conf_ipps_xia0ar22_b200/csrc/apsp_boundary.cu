@@ -203,6 +203,10 @@ apsp_status plan_placement(Handle* h, const apsp_config& cfg, long long fixed) {
   const long long cap_rows = std::max<long long>(1, (1ll << 30) / (n_pad * W));
   long long buf_rows = std::min<long long>(cap_rows, S_rem / 4 / per_row);
   if (buf_rows < b->s_max) buf_rows = std::min<long long>(std::max(cap_rows, b->s_max), S_rem / 2 / per_row);
+  // forced (force_out_of_core / ooc_stream_all): the paper's setting, every block row streams,
+  // in at least ~4 groups so the two buffers alternate even on small graphs
+  const bool stream_all = cfg.force_out_of_core || cfg.ooc_stream_all;
+  if (stream_all) buf_rows = std::max(b->s_max, std::min(buf_rows, n_pad / 4));
   if (buf_rows < b->s_max)
     return h->fail(APSP_ENOMEM, "boundary out of core: S_rem = %lld B leaves %lld rows per buffer < N_max = %lld",
                    S_rem, buf_rows, b->s_max);
@@ -210,7 +214,7 @@ apsp_status plan_placement(Handle* h, const apsp_config& cfg, long long fixed) {
   // groups share one tmp of buf_rows rows)
   long long left = S_rem - 2 * buf_rows * per_row - buf_rows * NB * W;
   int c_res = b->k;
-  while (c_res > 0 && left >= b->s_pad[c_res - 1] * n_pad * W) {
+  while (!stream_all && c_res > 0 && left >= b->s_pad[c_res - 1] * n_pad * W) {
     left -= b->s_pad[c_res - 1] * n_pad * W;
     --c_res;
   }

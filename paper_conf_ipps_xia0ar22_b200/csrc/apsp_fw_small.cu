@@ -1,0 +1,316 @@
+// apsp_fw_small.cu — the whole single-GPU blocked Floyd–Warshall (PAPER.md:62,
+// every round and phase) for SMALL n as one persistent dataflow launch with
+// 64 x 64 tiles (b = 64).
+//
+// Why a second kernel: at small n (config 1, n = 1024) the 128-tile dataflow
+// kernel is latency bound. Each round's critical path is three dependent
+// 128^3 tasks, phase 1 (k) -> panel tiles (k, k+1) / (k+1, k) -> phase-3 tile
+// (k+1, k+1) -> phase 1 (k+1), each ~2.1M relaxations on ONE SM (>= 17 us at
+// 64 DPX lanes/clk), while only 49 of 296 CTAs have phase-3 work per round
+// (8 rounds: 0.77 ms = 0.075 of the DPX peak). With b = 64 a
+// task is 262K relaxations (2.1 us on one SM), so the chain per round shrinks
+// ~8x while the rounds double (16 at n = 1024), and a round has 16^2 = 256
+// tasks for the 148 SMs instead of 64. The blocked FW is the same for any b
+// (R7 pads n to a multiple of 128, hence of 64).
+//
+// Structure (the schedule of apsp_fw_dataflow.cu, shared through
+// apsp_df_common.cuh: the same dependency-ordered queue decode(g, nb, delay),
+// the same per-tile flags deps_met / signal_done and double-buffered panel
+// copies), with a simpler engine sized for latency:
+//   * one CTA of 256 threads per task (one CTA per SM by default), thread
+//     (tx, ty) owns rows 4ty..4ty+3 x columns 4tx..4tx+3 of the 64x64 tile;
+//   * the task's whole depth (64) is staged at once: A^T as As[kk][r] and B as
+//     Bs[kk][c] (16 KB each, cp.async from the L2-resident panel copies; the
+//     column-panel task transposes its own tile through registers); per depth
+//     step 2 LDS.128 feed 16 relaxations (VIADDMNMX for int32);
+//   * C is loaded into the accumulators first (min is exact, any order) and
+//     stored once (out of place per tile, so phase 2, where an operand aliases
+//     C, is exact);
+//   * phase 1: the tile in registers, 64 steps, each publishing row / column kk
+//     through a double-buffered shared copy (one barrier per step), the R6
+//     negative-cycle check at the start of every step;
+//   * thread 0 dequeues and decodes the NEXT task and reads its flags while the
+//     CTA computes the current one.
+#include "apsp_kernels.cuh"
+#include "apsp_df_common.cuh"
+
+#include <cuda_runtime.h>
+#include <cstdint>
+#include <cstring>
+
+namespace apsp {
+namespace {
+
+constexpr int SB = 64;          // tile edge (round depth b)
+constexpr int SNT = 256;        // threads per CTA (one task at a time)
+constexpr int STE = SB * SB;    // elements per tile
+
+template <typename T> struct SV;
+template <> struct SV<int> {
+  using V4 = int4;
+  static __device__ __forceinline__ int relax(int a, int b, int c) { return __viaddmin_s32(a, b, c); }
+};
+template <> struct SV<float> {
+  using V4 = float4;
+  static __device__ __forceinline__ float relax(float a, float b, float c) { return fminf(c, __fadd_rn(a, b)); }
+};
+
+template <typename T>
+struct SmArgs {
+  T* D;            // n_pad x n_pad, row-major, ld
+  long long ld;
+  int nb;          // n_pad / 64
+  T* pbuf;         // 2 parities x (2 + 2 nb) tiles of 64x64: diag, diag^T, row panel [nb], column panel^T [nb]
+  int* ver;        // [nb][nb]
+  int* diagready;  // [2]
+  int* rowready;   // [2][nb]
+  int* colready;   // [2][nb]
+  int* done2;      // [nb]
+  int* done3;      // [nb]
+  unsigned long long* counter;
+  int* negflag;
+  long long total;  // nb^3 tasks
+  long long delay;
+};
+
+template <typename T>
+__device__ __forceinline__ T* sp_diag(const SmArgs<T>& a, int k) {
+  return a.pbuf + (long long)(k & 1) * (2 + 2 * a.nb) * STE;
+}
+template <typename T>
+__device__ __forceinline__ T* sp_diagT(const SmArgs<T>& a, int k) { return sp_diag(a, k) + STE; }
+template <typename T>
+__device__ __forceinline__ T* sp_row(const SmArgs<T>& a, int k, int j) { return sp_diag(a, k) + (2ll + j) * STE; }
+template <typename T>
+__device__ __forceinline__ T* sp_colT(const SmArgs<T>& a, int k, int i) {
+  return sp_diag(a, k) + (2ll + a.nb + i) * STE;
+}
+
+struct SmSlot {
+  long long t;
+  Task tk;
+  int ready;
+};
+
+// Phase 1: in-place FW closure of the 64x64 tile (P:60 restricted to the block); also writes
+// the closed block D and D^T to the round's panel copy.
+template <typename T>
+__device__ __forceinline__ void small_phase1(const SmArgs<T>& a, const Task& tk, T* rowbuf, T* colbuf) {
+  using V4 = typename SV<T>::V4;
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  T* const tile = a.D + (long long)tk.i * SB * a.ld + (long long)tk.j * SB;
+  T acc[4][4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const V4 v = __ldcg(reinterpret_cast<const V4*>(tile + (long long)(ty * 4 + i) * a.ld + tx * 4));
+    acc[i][0] = v.x; acc[i][1] = v.y; acc[i][2] = v.z; acc[i][3] = v.w;
+  }
+  bool neg = false;
+  for (int q = 0; q < 16; ++q) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int kk = q * 4 + u, p = u & 1;
+      if (ty == q) {  // row kk
+        V4 x;
+        x.x = acc[u][0]; x.y = acc[u][1]; x.z = acc[u][2]; x.w = acc[u][3];
+        *reinterpret_cast<V4*>(&rowbuf[p * SB + tx * 4]) = x;
+      }
+      if (tx == q) {  // column kk
+        V4 y;
+        y.x = acc[0][u]; y.y = acc[1][u]; y.z = acc[2][u]; y.w = acc[3][u];
+        *reinterpret_cast<V4*>(&colbuf[p * SB + ty * 4]) = y;
+      }
+      __syncthreads();
+      if (tid == 0 && rowbuf[p * SB + kk] < T(0)) neg = true;  // R6: D[kk][kk] < 0 -> negative cycle
+      const V4 av = *reinterpret_cast<const V4*>(&colbuf[p * SB + ty * 4]);
+      const V4 bv = *reinterpret_cast<const V4*>(&rowbuf[p * SB + tx * 4]);
+      const T A4[4] = {av.x, av.y, av.z, av.w}, B4[4] = {bv.x, bv.y, bv.z, bv.w};
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = SV<T>::relax(A4[i], B4[j], acc[i][j]);
+    }
+  }
+  if (neg) *a.negflag = 1;
+  T* const d = sp_diag(a, tk.k);
+  T* const dt = sp_diagT(a, tk.k);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    V4 v;
+    v.x = acc[i][0]; v.y = acc[i][1]; v.z = acc[i][2]; v.w = acc[i][3];
+    *reinterpret_cast<V4*>(tile + (long long)(ty * 4 + i) * a.ld + tx * 4) = v;
+    *reinterpret_cast<V4*>(d + (ty * 4 + i) * SB + tx * 4) = v;
+  }
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    V4 w;
+    w.x = acc[0][j]; w.y = acc[1][j]; w.z = acc[2][j]; w.w = acc[3][j];
+    *reinterpret_cast<V4*>(dt + (tx * 4 + j) * SB + ty * 4) = w;
+  }
+}
+
+// Phase 2 / phase 3 task: C = min(C, A (x) B) with the depth-64 operands of round k.
+//   P2R(k; k,j): A = D (panel copy D^T), B = A(k,j) itself; result also -> row panel copy
+//   P2C(k; i,k): A = A(i,k) itself (transposed on load), B = D; result also -> column panel^T
+//   P3(k; i,j):  A = column panel^T (i), B = row panel (j)
+template <typename T>
+__device__ __forceinline__ void small_minplus(const SmArgs<T>& a, const Task& tk, T* As, T* Bs) {
+  using V4 = typename SV<T>::V4;
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  T* const C = a.D + (long long)tk.i * SB * a.ld + (long long)tk.j * SB;
+  // operands -> shared memory: 64 rows of 256 B each, 16 B per cp.async, 4 per thread per operand
+  const T* Bsrc;
+  long long ldb;
+  if (tk.type == T_P2R) { Bsrc = C; ldb = a.ld; }
+  else if (tk.type == T_P2C) { Bsrc = sp_diag(a, tk.k); ldb = SB; }
+  else { Bsrc = sp_row(a, tk.k, tk.j); ldb = SB; }
+#pragma unroll
+  for (int e = 0; e < 4; ++e) {
+    const int x = tid + e * SNT;  // 0..1023: row x/16, 16-byte column x%16
+    const int r = x >> 4, c4 = (x & 15) * 4;
+    cp16(Bs + r * SB + c4, Bsrc + r * ldb + c4);
+  }
+  if (tk.type == T_P2C) {  // A(i,k) rows r, depth kk -> As[kk][r]
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const int x = tid + e * SNT;
+      const int r = x >> 4, c4 = (x & 15) * 4;
+      const V4 v = __ldcg(reinterpret_cast<const V4*>(C + (long long)r * a.ld + c4));
+      As[(c4 + 0) * SB + r] = v.x; As[(c4 + 1) * SB + r] = v.y;
+      As[(c4 + 2) * SB + r] = v.z; As[(c4 + 3) * SB + r] = v.w;
+    }
+  } else {
+    const T* Asrc = tk.type == T_P2R ? sp_diagT(a, tk.k) : sp_colT(a, tk.k, tk.i);
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const int x = tid + e * SNT;
+      cp16(As + x * 4, Asrc + x * 4);
+    }
+  }
+  cp_commit();
+  T acc[4][4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const V4 v = __ldcg(reinterpret_cast<const V4*>(C + (long long)(ty * 4 + i) * a.ld + tx * 4));
+    acc[i][0] = v.x; acc[i][1] = v.y; acc[i][2] = v.z; acc[i][3] = v.w;
+  }
+  cp_wait_all();
+  __syncthreads();
+#pragma unroll 8
+  for (int kk = 0; kk < SB; ++kk) {
+    const V4 av = *reinterpret_cast<const V4*>(&As[kk * SB + ty * 4]);
+    const V4 bv = *reinterpret_cast<const V4*>(&Bs[kk * SB + tx * 4]);
+    const T A4[4] = {av.x, av.y, av.z, av.w}, B4[4] = {bv.x, bv.y, bv.z, bv.w};
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j) acc[i][j] = SV<T>::relax(A4[i], B4[j], acc[i][j]);
+  }
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    V4 v;
+    v.x = acc[i][0]; v.y = acc[i][1]; v.z = acc[i][2]; v.w = acc[i][3];
+    *reinterpret_cast<V4*>(C + (long long)(ty * 4 + i) * a.ld + tx * 4) = v;
+    if (tk.type == T_P2R) *reinterpret_cast<V4*>(sp_row(a, tk.k, tk.j) + (ty * 4 + i) * SB + tx * 4) = v;
+  }
+  if (tk.type == T_P2C) {
+    T* const ct = sp_colT(a, tk.k, tk.i);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      V4 w;
+      w.x = acc[0][j]; w.y = acc[1][j]; w.z = acc[2][j]; w.w = acc[3][j];
+      *reinterpret_cast<V4*>(ct + (tx * 4 + j) * SB + ty * 4) = w;
+    }
+  }
+}
+
+// thread 0: the next task (dequeue + decode); its flags are checked by the caller
+template <typename T>
+__device__ __forceinline__ void small_fetch(const SmArgs<T>& a, SmSlot& s) {
+  s.t = (long long)atomicAdd(a.counter, 1ull);
+  s.ready = 0;
+  if (s.t < a.total) s.tk = decode(s.t, a.nb, a.delay);
+}
+
+template <typename T>
+__global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ SmArgs<T> a) {
+  __shared__ __align__(16) T As[STE];
+  __shared__ __align__(16) T Bs[STE];
+  __shared__ __align__(16) T rowbuf[2 * SB];
+  __shared__ __align__(16) T colbuf[2 * SB];
+  __shared__ SmSlot slot[2];
+  const int tid = threadIdx.x;
+  if (tid == 0) small_fetch(a, slot[0]);
+  __syncthreads();
+  for (int it = 0;; ++it) {
+    SmSlot& S = slot[it & 1];
+    SmSlot& N = slot[(it + 1) & 1];
+    if (S.t >= a.total) break;
+    const Task tk = S.tk;
+    if (tid == 0) {
+      if (!S.ready)
+        while (!deps_met(a, tk)) __nanosleep(32);
+      small_fetch(a, N);  // the next task, decoded while this one runs
+    }
+    __syncthreads();  // dependencies met (acquired by thread 0); N published
+    if (tk.type == T_P1) small_phase1(a, tk, rowbuf, colbuf);
+    else small_minplus(a, tk, As, Bs);
+    __syncthreads();  // every thread's stores of this task are issued; As / Bs free again
+    if (tid == 0) {
+      signal_done(a, tk);
+      // the next task's flags, once: if met, it starts without another wait
+      if (N.t < a.total && deps_met(a, N.tk)) N.ready = 1;
+    }
+  }
+}
+
+}  // namespace
+
+long long fw_small_work_bytes(int nb, size_t elem) {
+  const long long pb = 2ll * (2 + 2 * nb) * STE * (long long)elem;
+  const long long flags = ((2 + (long long)nb * nb + 2 + 4ll * nb + 2ll * nb) * 4 + 15) / 16 * 16;
+  return pb + flags;
+}
+
+template <typename T>
+cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag, long long delay, int ctas_per_sm,
+                            cudaStream_t s) {
+  if (nb <= 0) return cudaSuccess;
+  int dev = 0, sms = 0;
+  cudaError_t e;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+  if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess) return e;
+  SmArgs<T> a;
+  memset(&a, 0, sizeof(a));
+  a.D = D;
+  a.ld = ld;
+  a.nb = nb;
+  a.pbuf = static_cast<T*>(work);
+  int* f = reinterpret_cast<int*>(static_cast<char*>(work) + 2ll * (2 + 2 * nb) * STE * (long long)sizeof(T));
+  a.counter = reinterpret_cast<unsigned long long*>(f); f += 2;
+  a.ver = f; f += (long long)nb * nb;
+  a.diagready = f; f += 2;
+  a.rowready = f; f += 2 * nb;
+  a.colready = f; f += 2 * nb;
+  a.done2 = f; f += nb;
+  a.done3 = f; f += nb;
+  a.negflag = negflag;
+  a.total = (long long)nb * nb * nb;
+  a.delay = delay;
+  const long long flag_bytes = fw_small_work_bytes(nb, sizeof(T)) - 2ll * (2 + 2 * nb) * STE * (long long)sizeof(T);
+  if ((e = cudaMemsetAsync(a.counter, 0, flag_bytes, s)) != cudaSuccess) return e;
+  // persistent grid: every CTA must be resident (tasks wait on each other)
+  int occ = 0;
+  if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fw_small_kernel<T>, SNT, 0)) != cudaSuccess) return e;
+  if (occ < 1) return cudaErrorInvalidConfiguration;
+  const int per_sm = ctas_per_sm < 1 ? 1 : (ctas_per_sm > occ ? occ : ctas_per_sm);
+  long long grid = (long long)sms * per_sm;
+  if (grid > a.total) grid = a.total;
+  fw_small_kernel<T><<<(unsigned)grid, SNT, 0, s>>>(a);
+  return cudaGetLastError();
+}
+
+template cudaError_t launch_fw_small<int>(int*, long long, int, void*, int*, long long, int, cudaStream_t);
+template cudaError_t launch_fw_small<float>(float*, long long, int, void*, int*, long long, int, cudaStream_t);
+
+}  // namespace apsp

@@ -143,6 +143,11 @@ apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_pt
   h->n_pad = np;
   h->rows_per_rank = np / h->world;
   h->ld = np;
+  // small n on one GPU: the 64-tile dataflow kernel (its per-round critical path is ~8x
+  // shorter; measured crossover in DESIGN.md §5); APSP_SCHED_SMALL forces it at any n
+  const bool one_gpu = h->world == 1 && !h->virt && cfg.force_nccl != 1;
+  h->small = h->dataflow && one_gpu &&
+             (cfg.schedule == APSP_SCHED_SMALL || (cfg.schedule == APSP_SCHED_AUTO && np <= kSmallAutoMaxN));
 
   // ---- in-core or out-of-core? ---------------------------------------------
   return init_placement(h, cfg, row_ptr, col, w);
@@ -180,7 +185,8 @@ apsp_status setup_device(Handle* h, const apsp_config& cfg) {
   // launch-per-phase schedule with NCCL broadcasts; APSP_SCHED_DATAFLOW selects the sharded
   // dataflow kernel there (peer stores of the pivot panels).
   const bool sharded = h->world > 1 || cfg.force_nccl == 1;
-  h->dataflow = cfg.schedule == APSP_SCHED_DATAFLOW || (cfg.schedule == APSP_SCHED_AUTO && !sharded);
+  h->dataflow = cfg.schedule == APSP_SCHED_DATAFLOW || cfg.schedule == APSP_SCHED_SMALL ||
+                (cfg.schedule == APSP_SCHED_AUTO && !sharded);
   h->df_delay = cfg.dataflow_delay;
   if (cfg.stream) {
     h->stream = static_cast<cudaStream_t>(cfg.stream);

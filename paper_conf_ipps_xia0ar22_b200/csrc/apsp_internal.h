@@ -10,6 +10,9 @@
 
 namespace apsp {
 
+// n_pad up to which APSP_SCHED_AUTO picks the 64-tile small-n kernel (apsp_fw_small.cu)
+constexpr long long kSmallAutoMaxN = 2048;
+
 // NVTX range for the duration of a scope (C-ABI entry points, out-of-core
 // super-rounds): shows up in Nsight timelines and `ncu --nvtx` filters; a
 // no-op when no tool is attached (NVTX3 is header-only).
@@ -86,6 +89,7 @@ struct Handle {
   void* jn = nullptr;
   // single-GPU in-core dataflow kernel (apsp_fw_dataflow.cu)
   bool dataflow = true;     // apsp_config.schedule (APSP_SCHED_PER_PHASE: launch per phase)
+  bool small = false;       // dataflow with 64x64 tiles (apsp_fw_small.cu): small n, APSP_SCHED_SMALL
   long long df_delay = 0;   // apsp_config.dataflow_delay (0 = auto)
   void* df_work = nullptr;
   // sharded dataflow kernel (multi-GPU / virtual ranks): per-rank work buffers

@@ -139,6 +139,14 @@ template <typename T>
 cudaError_t launch_fw_dataflow_sharded(const DFShard* ranks, int nv, int P, int nb, long long ld, int* negflag,
                                        long long delay, cudaStream_t s);
 
+// The whole single-GPU blocked FW for small n with 64x64 tiles (apsp_fw_small.cu): the
+// dataflow schedule above at b = 64 (nb = n_pad / 64 rounds), one 256-thread CTA per task.
+// `work` holds fw_small_work_bytes(nb, elem) bytes (panel copies + flags, zeroed here).
+template <typename T>
+cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag, long long delay, int ctas_per_sm,
+                            cudaStream_t s);
+long long fw_small_work_bytes(int nb, size_t elem);
+
 // The packed int16 closure (R16) as one persistent dataflow launch
 // (apsp_fw_dataflow16.cu); `work` holds fw_dataflow16_work_bytes(nb) bytes.
 cudaError_t launch_fw_dataflow16(short* D, long long ld, int nb, void* work, long long delay, cudaStream_t s,

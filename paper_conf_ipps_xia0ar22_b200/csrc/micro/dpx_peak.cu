@@ -8,6 +8,11 @@
 //   f32x2   : __fadd2_rn + 3-input min -> FADD2 + FMNMX3    (2 relax / 2 instr)
 //   f32b, f32x2b: the same without per-step int->float conversions (the b
 //             operand advances by FADD), f32x2b in the kernels' broadcast form
+//   s32imad3: two adds on the FMA pipe (IMAD with a runtime 1) + one 3-input
+//             min on the ALU pipe (VIMNMX3): 2 relax / 3 instr, exact int32
+//   s32iadd3: the same with the adds as plain add.s32 (ptxas: IADD3 / IMAD.IADD)
+//   s32mix  : per chain 1 VIADDMNMX + (2 IMAD + 1 VIMNMX3): 3 relax / 4 instr
+//             (routes past the VIADDMNMX issue rate for int32)
 // plus the host link (pinned H2D, D2H, both at once), used by the
 // out-of-core roofline. Prints one JSON object on stdout.
 #include <cuda_runtime.h>
@@ -159,6 +164,87 @@ __global__ void k_f32x2b(const int* __restrict__ in, int* __restrict__ out, int 
   out[blockIdx.x * blockDim.x + threadIdx.x] = (int)s;
 }
 
+// int32 forms that keep the adds off the ALU pipe. The adds are inline
+// PTX so that ptxas cannot re-fuse them into VIADDMNMX: mad.lo with a multiplier it cannot
+// prove to be 1 stays an IMAD (FMA pipe); plain add.s32 is left to ptxas.
+__device__ __forceinline__ int mad1(int a, int one, int b) {
+  int r;
+  asm volatile("mad.lo.s32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(one), "r"(b));
+  return r;
+}
+__device__ __forceinline__ int add1(int a, int b) {
+  int r;
+  asm volatile("add.s32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b));
+  return r;
+}
+__global__ void k_s32imad3(const int* __restrict__ in, int* __restrict__ out, int iters) {
+  int x[CH], x2[CH], acc[CH];
+  const int one = in[255] == 12345 ? 2 : 1;  // 1 at run time, unknown to the compiler
+#pragma unroll
+  for (int j = 0; j < CH; ++j) {
+    x[j] = in[(threadIdx.x + j) & 255]; x2[j] = in[(threadIdx.x + j + 3) & 255]; acc[j] = 1 << 29;
+  }
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {  // 4 x 2 = 8 relaxations per chain per iteration, as k_s32
+      const int y0 = it * 8 + u, y1 = it * 8 + u + 4;
+#pragma unroll
+      for (int j = 0; j < CH; ++j) acc[j] = __vimin3_s32(acc[j], mad1(x[j], one, y0), mad1(x2[j], one, y1));
+    }
+  }
+  int s = 0;
+#pragma unroll
+  for (int j = 0; j < CH; ++j) s ^= acc[j];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+__global__ void k_s32iadd3(const int* __restrict__ in, int* __restrict__ out, int iters) {
+  int x[CH], x2[CH], acc[CH];
+#pragma unroll
+  for (int j = 0; j < CH; ++j) {
+    x[j] = in[(threadIdx.x + j) & 255]; x2[j] = in[(threadIdx.x + j + 3) & 255]; acc[j] = 1 << 29;
+  }
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int y0 = it * 8 + u, y1 = it * 8 + u + 4;
+#pragma unroll
+      for (int j = 0; j < CH; ++j) acc[j] = __vimin3_s32(acc[j], add1(x[j], y0), add1(x2[j], y1));
+    }
+  }
+  int s = 0;
+#pragma unroll
+  for (int j = 0; j < CH; ++j) s ^= acc[j];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+// 8 relaxations per chain per iteration: 2 x (1 VIADDMNMX + 2 IMAD + 1 VIMNMX3) + 2 VIADDMNMX
+__global__ void k_s32mix(const int* __restrict__ in, int* __restrict__ out, int iters) {
+  int x[CH], x2[CH], acc[CH];
+  const int one = in[255] == 12345 ? 2 : 1;
+#pragma unroll
+  for (int j = 0; j < CH; ++j) {
+    x[j] = in[(threadIdx.x + j) & 255]; x2[j] = in[(threadIdx.x + j + 3) & 255]; acc[j] = 1 << 29;
+  }
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      const int y0 = it * 8 + u, y1 = it * 8 + u + 2, y2 = it * 8 + u + 4;
+#pragma unroll
+      for (int j = 0; j < CH; ++j) {
+        acc[j] = __viaddmin_s32(x[j], y0, acc[j]);
+        acc[j] = __vimin3_s32(acc[j], mad1(x2[j], one, y1), mad1(x[j], one, y2));
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < CH; ++j) acc[j] = __viaddmin_s32(x2[j], it, acc[j]);
+#pragma unroll
+    for (int j = 0; j < CH; ++j) acc[j] = __viaddmin_s32(x[j], it + 7, acc[j]);
+  }
+  int s = 0;
+#pragma unroll
+  for (int j = 0; j < CH; ++j) s ^= acc[j];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+
 typedef void (*kfn)(const int*, int*, int);
 
 static double run(kfn f, int blocks, int threads, int iters, const int* in, int* out, double relax_per_op) {
@@ -210,7 +296,8 @@ int main(int argc, char** argv) {
   int cfgs[][2] = {{4, 256}, {8, 256}, {16, 128}, {4, 512}};
   struct V { const char* name; kfn f; double rpo; } vs[] = {
     {"s32", k_s32, 1.0}, {"s16x2", k_s16x2, 2.0}, {"f32", k_f32, 1.0}, {"f32x2", k_f32x2, 2.0},
-    {"f32b", k_f32b, 1.0}, {"f32x2b", k_f32x2b, 1.0}};
+    {"f32b", k_f32b, 1.0}, {"f32x2b", k_f32x2b, 1.0}, {"s32imad3", k_s32imad3, 1.0},
+    {"s32iadd3", k_s32iadd3, 1.0}, {"s32mix", k_s32mix, 1.0}};
   CK(cudaMalloc(&out, (size_t)p.multiProcessorCount * 16 * 512 * sizeof(int)));
   for (auto& v : vs) {
     double best = 0;

@@ -30,7 +30,7 @@ def check(got, src, dist):
     assert np.all(np.diag(got) == 0)
 
 
-@pytest.mark.parametrize("schedule", [0, 1], ids=["dataflow", "per_phase"])
+@pytest.mark.parametrize("schedule", [0, 1, 2, 3], ids=["auto", "per_phase", "dataflow128", "small64"])
 @pytest.mark.parametrize("name", FIXTURES)
 def test_golden_fw_i32(lib, name, schedule):
     g, src, dist = load(name)
@@ -39,10 +39,11 @@ def test_golden_fw_i32(lib, name, schedule):
     check(lib.solve(g, cfg=c).astype(np.int64), src, dist)
 
 
+@pytest.mark.parametrize("schedule", [0, 2], ids=["auto", "dataflow128"])
 @pytest.mark.parametrize("name", FIXTURES)
-def test_golden_fw_f32(lib, name):
+def test_golden_fw_f32(lib, name, schedule):
     g, src, dist = load(name, np.float32)
-    got = lib.solve(g, cfg=lib.apsp_config_default(device=0))
+    got = lib.solve(g, cfg=lib.apsp_config_default(device=0, schedule=schedule))
     assert got.dtype == np.float32
     check(got.astype(np.int64), src, dist)  # small integers: exact in fp32
 

@@ -8,7 +8,7 @@ set -u
 mkdir -p gpurun_out
 what=$1; shift
 case $what in
-  tests) python -m pytest tests -m gpu -x -q ${1:+-k "$1"} > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?";
+  tests) python -m pytest tests -m gpu ${PYTEST_X--x} -q ${1:+-k "$1"} > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?";
          tail -5 gpurun_out/pytest_gpu.log ;;
   bench) python bench.py "$@" > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench rc=$?";
          tail -c 600 gpurun_out/bench.json; tail -5 gpurun_out/bench.err ;;
