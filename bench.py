@@ -440,6 +440,22 @@ def run_ours(args):
                                                      if not args.force_ooc else None),
                     "peak_source": peak_src, "avg_launch_ms": p3_ms, "relax_per_launch": p3_relax,
                     "share_of_step": (st_acc[0][2] / steps) / ms_step}
+        if info.mode == apsp.APSP_MODE_OUT_OF_CORE:
+            # host link of the out-of-core step (transfers are part of the time):
+            # every streamed band crosses the link once each way per super-round, plus the init's
+            # D2H of every streamed band (apsp_reinit) -> bytes per direction per step
+            nd = info.n_pad // info.ooc_block
+            link_bytes = float(info.host_bytes) * (nd + 1)
+            lk = pk.get("dpx", {}).get("host_link_gbs", {})
+            lpeak = lk.get("duplex_each_dir") or 47.59
+            roofline["link"] = {"bytes_each_direction_per_step": link_bytes,
+                                "achieved_gbs": link_bytes / (ms_step * 1e-3) / 1e9, "peak_gbs": lpeak,
+                                "link_frac": link_bytes / (ms_step * 1e-3) / 1e9 / lpeak,
+                                "peak_source": "MEASURED_DPX.json host_link_gbs.duplex_each_dir (pinned H2D and "
+                                               "D2H at once, 1 GiB copies)",
+                                "bands": nd, "band_rows": int(info.ooc_block),
+                                "streamed_bytes": int(info.host_bytes),
+                                "resident_bands": int(nd - info.host_bytes // (info.ooc_block * info.n_pad * 4))}
         return {"value": value, "ms_per_step": ms_step, "arith": arith, "clocks": clocks, "roofline": roofline,
                 "steps": steps, "warmup": warmup,
                 "launches_per_step": int(round(st_acc[1][:3].sum() / steps)) + 1,  # + init kernel

@@ -1023,6 +1023,12 @@ apsp_status apsp_local_rows(const apsp_handle* hh, int64_t* row_begin, int64_t* 
     *row_count = h->n;
     return APSP_OK;
   }
+  if (h->mode == APSP_MODE_OUT_OF_CORE) {  // rank r: bands [r nd/P, (r+1) nd/P) (apsp_ooc.cu)
+    const int64_t rb = (int64_t)h->rank * h->rows_per_rank;
+    *row_begin = rb;
+    *row_count = std::max<int64_t>(0, std::min<int64_t>(rb + h->rows_per_rank, h->n) - rb);
+    return APSP_OK;
+  }
   int64_t np;
   return apsp_partition(h->n, h->b, h->world, h->rank, &np, row_begin, row_count);
 }

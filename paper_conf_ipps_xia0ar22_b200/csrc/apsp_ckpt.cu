@@ -51,7 +51,7 @@ void fill_header(const Handle* h, CkptHeader* hd) {
   hd->ooc_block = h->mode == APSP_MODE_OUT_OF_CORE ? (int32_t)h->ooc_B : 0;
   hd->world = h->world;
   hd->rank = h->rank;
-  hd->row_begin = h->mode == APSP_MODE_OUT_OF_CORE ? 0 : h->shards[0].row_begin;
+  hd->row_begin = h->mode == APSP_MODE_OUT_OF_CORE ? ooc_row_begin(h) : h->shards[0].row_begin;
   hd->next_round = h->next_round;
   hd->has_neg = h->has_neg ? 1 : 0;
   hd->neg_cycle = 0;

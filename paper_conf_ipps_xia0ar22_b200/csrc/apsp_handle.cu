@@ -205,6 +205,23 @@ apsp_status setup_device(Handle* h, const apsp_config& cfg) {
   return h->cuda(cudaMemsetAsync(h->d_flag, 0, sizeof(int), h->stream), "memset flag");
 }
 
+// The NCCL communicator of a sharded placement (one per handle).
+static apsp_status create_comm(Handle* h, const apsp_config& cfg) {
+  ncclUniqueId id;
+  if (cfg.nccl_unique_id) {
+    memcpy(&id, cfg.nccl_unique_id, sizeof(id));
+  } else if (h->world == 1) {
+    if (ncclGetUniqueId(&id) != ncclSuccess) return h->fail(APSP_ENCCL, "ncclGetUniqueId failed");
+  } else {
+    return h->fail(APSP_EINVAL, "nccl_unique_id is NULL");
+  }
+  ncclComm_t comm;
+  ncclResult_t r = ncclCommInitRank(&comm, h->world, id, h->rank);
+  if (r != ncclSuccess) return h->fail(APSP_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
+  h->comm = comm;
+  return APSP_OK;
+}
+
 // In-core (1-D block-row shards, packed int16) or out-of-core placement + init.
 static apsp_status init_placement(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, const int32_t* col,
                                   const void* w) {
@@ -226,9 +243,10 @@ static apsp_status init_placement(Handle* h, const apsp_config& cfg, const int64
   const bool need_ooc =
       cfg.force_out_of_core || ((cfg.dist_device ? 0 : mat_bytes) + panel_bytes > budget);
   if (need_ooc) {
-    if (h->world > 1) return h->fail(APSP_ENOMEM, "matrix shard (%lld B) exceeds the device budget (%lld B); "
-                                     "out-of-core x multi-GPU is not supported", mat_bytes, budget);
+    // out of core, on one GPU or replicated over the P ranks' band subsets (apsp_ooc.cu);
+    // the ranks exchange only the finished pivot band of every super-round (NCCL broadcast)
     h->mode = APSP_MODE_OUT_OF_CORE;
+    if (h->use_comm && (st = create_comm(h, cfg))) return st;
     return ooc_setup(h, cfg, budget, row_ptr, col, w);
   }
 
@@ -272,20 +290,7 @@ static apsp_status init_placement(Handle* h, const apsp_config& cfg, const int64
     h->shards.push_back(sh);
   }
 
-  if (h->use_comm) {
-    ncclUniqueId id;
-    if (cfg.nccl_unique_id) {
-      memcpy(&id, cfg.nccl_unique_id, sizeof(id));
-    } else if (h->world == 1) {
-      if (ncclGetUniqueId(&id) != ncclSuccess) return h->fail(APSP_ENCCL, "ncclGetUniqueId failed");
-    } else {
-      return h->fail(APSP_EINVAL, "nccl_unique_id is NULL");
-    }
-    ncclComm_t comm;
-    ncclResult_t r = ncclCommInitRank(&comm, h->world, id, h->rank);
-    if (r != ncclSuccess) return h->fail(APSP_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
-    h->comm = comm;
-  }
+  if (h->use_comm && (st = create_comm(h, cfg))) return st;
 
   if ((st = h->dtype == APSP_I32 ? upload_csr<int>(h, row_ptr, col, w) : upload_csr<float>(h, row_ptr, col, w)))
     return st;

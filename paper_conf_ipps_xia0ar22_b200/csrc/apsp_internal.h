@@ -80,8 +80,7 @@ struct Handle {
   // out-of-core
   int mode = APSP_MODE_INCORE;
   long long ooc_B = 0;
-  void* h_dist = nullptr;   // pinned n_pad x n_pad host matrix
-  void* ooc_dev = nullptr;  // device arena for bands
+  void* ooc_dev = nullptr;  // out-of-core state (apsp_ooc.cu): per-rank band buffers, pinned host bands
   void* ooc_streams[3] = {nullptr, nullptr, nullptr};
   // boundary algorithm (apsp_boundary.cu)
   void* bnd = nullptr;
@@ -155,7 +154,8 @@ apsp_status ooc_setup(Handle* h, const apsp_config& cfg, long long budget, const
                       const int32_t* col, const void* w);
 apsp_status run_out_of_core(Handle* h);
 apsp_status run_out_of_core_range(Handle* h, long long K0, long long K1);
-long long ooc_bands(const Handle* h);
+long long ooc_bands(const Handle* h);      // this process's bands
+long long ooc_row_begin(const Handle* h);  // first padded row of this process's bands
 apsp_status ooc_band_copy(Handle* h, long long I, void* buf, bool to_handle);
 apsp_status ooc_get_rows(Handle* h, long long r0, long long cnt, void* out, long long ld_out);
 void ooc_free(Handle* h);

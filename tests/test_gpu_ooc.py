@@ -106,3 +106,74 @@ def test_ooc_f32_and_reinit(lib):
     fin = np.isfinite(want)
     assert np.array_equal(np.isfinite(a), fin)
     assert np.all(np.abs(a[fin] - want[fin]) <= 1e-5 * np.abs(want[fin]))
+
+
+# ------------------------------------- out of core x P ranks (SURVEY §8(e) last bullet, NEXT-3)
+
+
+@pytest.mark.parametrize("world,n,block", [(2, 1000, 128), (3, 700, 128), (4, 1536, 128), (2, 2048, 256),
+                                           (8, 1024, 128)])
+def test_ooc_virtual_ranks_bit_exact(lib, world, n, block):
+    """Rank r owns bands [r nd/P, (r+1) nd/P) in its own pinned memory; the owner of band K
+    closes it and broadcasts the finished pivot band (here a device copy between virtual
+    ranks, the non-root receive path of the NCCL broadcast); every rank updates its bands."""
+    g = gg.grid_2d(max(2, n // 25), 25, seed=n + world) if world % 2 == 0 else gg.erdos_renyi(n, 4 * n, seed=n)
+    c = ooc_cfg(lib, block)
+    c.world_size = world
+    c.virtual_ranks = 1
+    with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
+        info = lib.apsp_get_info(h)
+        assert info.mode == lib.APSP_MODE_OUT_OF_CORE and info.ooc_block == block
+        assert info.n_pad % (block * world) == 0 and info.host_bytes == info.n_pad ** 2 * 4
+        lib.apsp_fw_blocked(h)
+        got = lib.apsp_get_dist(h)
+        st = lib.apsp_get_phase_stats(h)
+    want, _ = oracle_i32(g)
+    assert np.array_equal(got.astype(np.int64), want)
+    assert abs(sum(st.relax[:3]) - float(info.n_pad) ** 3) < 1
+
+
+def test_ooc_virtual_ranks_resident_negative_f32(lib):
+    # resident bands on every rank (a budget shared by the virtual ranks), negative weights
+    rng = np.random.default_rng(4)
+    g0 = gg.erdos_renyi(1024, 6000, seed=6)
+    p = rng.integers(-300, 300, size=g0.n)
+    s, t, w = g0.arcs()
+    g = gg.csr_from_arcs(g0.n, s, t, (w.astype(np.int64) + p[s] - p[t]).astype(np.int32))
+    c = ooc_cfg(lib, 128, budget_mb=6.4, stream_all=False)  # 2 of each rank's 4 bands resident
+    c.world_size = 2
+    c.virtual_ranks = 1
+    with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
+        info = lib.apsp_get_info(h)
+        assert 0 < info.host_bytes < info.n_pad ** 2 * 4
+        lib.apsp_fw_blocked(h)
+        got = lib.apsp_get_dist(h)
+    want, _ = oracle_i32(g)
+    assert np.array_equal(got.astype(np.int64), want)
+    gc = gg.with_arcs(g0, [900, 30], [30, 900], [-200, 50])
+    c2 = ooc_cfg(lib, 128)
+    c2.world_size, c2.virtual_ranks = 4, 1
+    with lib.apsp_init_from_csr(gc.n, gc.row_ptr, gc.col, gc.w, cfg=c2) as h:
+        with pytest.raises(lib.NegativeCycleError):
+            lib.apsp_fw_blocked(h)
+    gf = gg.erdos_renyi(900, 9000, seed=7, dtype="f32")
+    c3 = ooc_cfg(lib, 128)
+    c3.world_size, c3.virtual_ranks = 3, 1
+    a = lib.solve(gf, cfg=c3)
+    b = lib.solve(gf, cfg=lib.apsp_config_default(device=0, schedule=1))
+    assert np.array_equal(a.view(np.int32), b.view(np.int32))  # same relaxations, same RN adds
+
+
+def test_ooc_virtual_ranks_partial_rounds(lib):
+    """apsp_fw_rounds in whole super-rounds over 2 virtual ranks: the state after super-round
+    K is the FW state with intermediates {0 .. (K+1)B - 1}."""
+    g = gg.erdos_renyi(1024, 5000, seed=12)
+    c = ooc_cfg(lib, 256)
+    c.world_size, c.virtual_ranks = 2, 1
+    with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
+        lib.apsp_fw_rounds(h, 0, 4)  # super-rounds 0 and 1 (B = 256 = 2 rounds of 128)
+        d, _ = oracle.fw_i64(g.row_ptr, g.col, g.w, k_iters=512)
+        assert np.array_equal(lib.apsp_get_dist(h).astype(np.int64), np.where(d == oracle.INF_I64, INF32, d))
+        lib.apsp_fw_blocked(h)
+        want, _ = oracle_i32(g)
+        assert np.array_equal(lib.apsp_get_dist(h).astype(np.int64), want)

@@ -76,8 +76,12 @@ def test_small_f32(lib):
     fin = np.isfinite(want)
     assert np.array_equal(np.isfinite(got), fin)
     assert np.all(np.abs(got[fin] - want[fin]) <= 1e-5 * np.abs(want[fin]))
-    # every relaxation is one RN add of the same operands and an exact min: the schedules agree
-    assert np.array_equal(run(lib, g).view(np.int32), run(lib, g, schedule=1).view(np.int32))
+    # deterministic (each candidate sum is one RN add of operands fixed by the schedule); a
+    # different round depth b (the 128-tile kernels) rounds other partial paths, so across b
+    # the results agree within the tolerance only (R13)
+    assert np.array_equal(run(lib, g).view(np.int32), got.astype(np.float32).view(np.int32))
+    other = run(lib, g, schedule=1).astype(np.float64)
+    assert np.all(np.abs(other[fin] - got[fin]) <= 2e-5 * np.abs(want[fin]))
 
 
 def test_small_forced_at_larger_n_equals_other_schedules(lib):
