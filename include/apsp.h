@@ -360,10 +360,12 @@ apsp_status apsp_synchronize(apsp_handle* h);
 /*
  * apsp_debug_queue — diagnostics for tests: the persistent dataflow kernel's task queue,
  * computed on the host by the same decoder the kernel runs. P = 0: the single-GPU queue;
- * P >= 1: rank q's queue of the sharded kernel (nb % P == 0). Writes up to `cap` tasks as
- * (type, k, i, j) int32 quadruples (type 0 = phase 1 of round k, 1 = row-panel tile (k, j),
- * 2 = column-panel tile (i, k), 3 = phase-3 tile (i, j); i, j global tile indices) and
- * returns the queue length (-1 on bad arguments). No device is touched.
+ * P >= 1: rank q's queue of the sharded kernel (nb % P == 0); P = -1: the small-n kernel's
+ * queue (64-wide tiles, APSP_SCHED_SMALL). Writes up to `cap` tasks as (type, k, i, j) int32
+ * quadruples (type 0 = phase 1 of round k, 1 = row-panel tile (k, j), 2 = column-panel tile
+ * (i, k), 3 = phase-3 tile (i, j), 4 = phase-3 tile (k+1, k+1) of round k fused with phase 1
+ * of round k+1; i, j global tile indices) and returns the queue length (-1 on bad
+ * arguments). No device is touched.
  */
 int64_t apsp_debug_queue(int32_t nb, int32_t P, int32_t q, int64_t delay, int32_t* out, int64_t cap);
 

@@ -1000,6 +1000,15 @@ long long fw_dataflow_work_bytes(int nb, size_t elem) { return fw_dataflow_work_
 // host. P = 0: the single-GPU queue (decode); P >= 1: rank q's sharded queue (decode_sh).
 extern "C" int64_t apsp_debug_queue(int32_t nb, int32_t P, int32_t q, int64_t delay, int32_t* out, int64_t cap) {
   using namespace apsp;
+  if (P == -1) {  // the small-n kernel's queue (apsp_fw_small.cu), nb 64-wide tile rows
+    if (nb <= 0) return -1;
+    std::vector<int4> sq;
+    const long long total = small_queue(nb, &sq);
+    for (long long g = 0; g < total && g < cap; ++g) {
+      out[4 * g] = sq[g].x; out[4 * g + 1] = sq[g].y; out[4 * g + 2] = sq[g].z; out[4 * g + 3] = sq[g].w;
+    }
+    return total;
+  }
   if (nb <= 0 || P < 0 || (P > 0 && (nb % P || q < 0 || q >= P))) return -1;
   const int nl = P > 0 ? nb / P : nb;
   std::vector<long long> seg((size_t)nb + 1);

@@ -13,10 +13,20 @@
 // tasks for the 148 SMs instead of 64. The blocked FW is the same for any b
 // (R7 pads n to a multiple of 128, hence of 64).
 //
-// Structure (the schedule of apsp_fw_dataflow.cu, shared through
-// apsp_df_common.cuh: the same dependency-ordered queue decode(g, nb, delay),
-// the same per-tile flags deps_met / signal_done and double-buffered panel
-// copies), with a simpler engine sized for latency:
+// Structure: the flag protocol of apsp_fw_dataflow.cu (apsp_df_common.cuh: per-tile
+// versions, diagonal / panel readiness, double-buffered panel copies, deps_met /
+// signal_done) with a queue ordered for the critical path and a simpler engine:
+//   * the queue is built on the host (small_queue, at most 32^3 entries) in
+//     segments seg(k) = [P2R(k,k+1), P2C(k+1,k), round k-1's phase-3 tiles on
+//     row / column k+1, F(k), the other panel tiles of round k, the rest of round
+//     k-1's phase 3, round k's phase-3 tiles on row / column k+1], so the chain
+//     P1(k) -> panels (k,k+1), (k+1,k) -> tile (k+1,k+1) -> P1(k+1) is queued
+//     first in every segment; every dependency of an entry lies earlier in the
+//     queue (tests/test_schedule.py simulates it), so a CTA that finishes its
+//     task before taking the next cannot deadlock;
+//   * F(k) fuses P3(k; k+1,k+1) with P1(k+1): the CTA that updates the next
+//     diagonal tile closes it in registers right away (one flag hop and one
+//     tile load less on the chain of every round);
 //   * one CTA of 256 threads per task (one CTA per SM by default), thread
 //     (tx, ty) owns rows 4ty..4ty+3 x columns 4tx..4tx+3 of the 64x64 tile;
 //   * the task's whole depth (64) is staged at once: A^T as As[kk][r] and B as
@@ -29,14 +39,16 @@
 //   * phase 1: the tile in registers, 64 steps, each publishing row / column kk
 //     through a double-buffered shared copy (one barrier per step), the R6
 //     negative-cycle check at the start of every step;
-//   * thread 0 dequeues and decodes the NEXT task and reads its flags while the
-//     CTA computes the current one.
+//   * thread 0 fetches the next queue entry and the index after it while the CTA
+//     computes the current task, and checks the next task's flags right after
+//     publishing the current one.
 #include "apsp_kernels.cuh"
 #include "apsp_df_common.cuh"
 
 #include <cuda_runtime.h>
 #include <cstdint>
 #include <cstring>
+#include <vector>
 
 namespace apsp {
 namespace {
@@ -69,8 +81,8 @@ struct SmArgs {
   int* done3;      // [nb]
   unsigned long long* counter;
   int* negflag;
-  long long total;  // nb^3 tasks
-  long long delay;
+  long long total;   // queue entries
+  const int4* queue; // [total] (type, k, i, j), built on the host (small_queue)
 };
 
 template <typename T>
@@ -86,25 +98,21 @@ __device__ __forceinline__ T* sp_colT(const SmArgs<T>& a, int k, int i) {
   return sp_diag(a, k) + (2ll + a.nb + i) * STE;
 }
 
+enum { T_P3P1 = 4 };  // fused P3(k; k+1,k+1) + P1(k+1)
+
 struct SmSlot {
   long long t;
   Task tk;
   int ready;
 };
 
-// Phase 1: in-place FW closure of the 64x64 tile (P:60 restricted to the block); also writes
-// the closed block D and D^T to the round's panel copy.
+// Phase 1 on a tile held in registers (thread: rows 4ty.., columns 4tx..): in-place FW
+// closure of the 64x64 block (P:60 restricted to it), 64 steps, row / column kk published
+// through a double-buffered shared copy, one barrier per step; R6 check at every step.
 template <typename T>
-__device__ __forceinline__ void small_phase1(const SmArgs<T>& a, const Task& tk, T* rowbuf, T* colbuf) {
+__device__ __forceinline__ void small_close(T (&acc)[4][4], T* rowbuf, T* colbuf, int* negflag) {
   using V4 = typename SV<T>::V4;
   const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
-  T* const tile = a.D + (long long)tk.i * SB * a.ld + (long long)tk.j * SB;
-  T acc[4][4];
-#pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    const V4 v = __ldcg(reinterpret_cast<const V4*>(tile + (long long)(ty * 4 + i) * a.ld + tx * 4));
-    acc[i][0] = v.x; acc[i][1] = v.y; acc[i][2] = v.z; acc[i][3] = v.w;
-  }
   bool neg = false;
   for (int q = 0; q < 16; ++q) {
 #pragma unroll
@@ -131,9 +139,16 @@ __device__ __forceinline__ void small_phase1(const SmArgs<T>& a, const Task& tk,
         for (int j = 0; j < 4; ++j) acc[i][j] = SV<T>::relax(A4[i], B4[j], acc[i][j]);
     }
   }
-  if (neg) *a.negflag = 1;
-  T* const d = sp_diag(a, tk.k);
-  T* const dt = sp_diagT(a, tk.k);
+  if (neg) *negflag = 1;
+}
+
+// the closed diagonal block of round k: into the matrix, D and D^T into the panel copy
+template <typename T>
+__device__ __forceinline__ void small_store_diag(const SmArgs<T>& a, int k, T* tile, const T (&acc)[4][4]) {
+  using V4 = typename SV<T>::V4;
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  T* const d = sp_diag(a, k);
+  T* const dt = sp_diagT(a, k);
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
     V4 v;
@@ -149,16 +164,35 @@ __device__ __forceinline__ void small_phase1(const SmArgs<T>& a, const Task& tk,
   }
 }
 
+// Phase 1 task P1(k): close A(k,k) (PAPER.md:62 step 1)
+template <typename T>
+__device__ __forceinline__ void small_phase1(const SmArgs<T>& a, const Task& tk, T* rowbuf, T* colbuf) {
+  using V4 = typename SV<T>::V4;
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  T* const tile = a.D + (long long)tk.i * SB * a.ld + (long long)tk.j * SB;
+  T acc[4][4];
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const V4 v = __ldcg(reinterpret_cast<const V4*>(tile + (long long)(ty * 4 + i) * a.ld + tx * 4));
+    acc[i][0] = v.x; acc[i][1] = v.y; acc[i][2] = v.z; acc[i][3] = v.w;
+  }
+  small_close(acc, rowbuf, colbuf, a.negflag);
+  small_store_diag(a, tk.k, tile, acc);
+}
+
 // Phase 2 / phase 3 task: C = min(C, A (x) B) with the depth-64 operands of round k.
 //   P2R(k; k,j): A = D (panel copy D^T), B = A(k,j) itself; result also -> row panel copy
 //   P2C(k; i,k): A = A(i,k) itself (transposed on load), B = D; result also -> column panel^T
 //   P3(k; i,j):  A = column panel^T (i), B = row panel (j)
+//   F(k) = P3(k; k+1,k+1) then P1(k+1) on the same registers (fused: closes the tile right away)
 template <typename T>
-__device__ __forceinline__ void small_minplus(const SmArgs<T>& a, const Task& tk, T* As, T* Bs) {
+__device__ __forceinline__ void small_minplus(const SmArgs<T>& a, const Task& tk, T* As, T* Bs, T* rowbuf,
+                                              T* colbuf) {
   using V4 = typename SV<T>::V4;
   const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
   T* const C = a.D + (long long)tk.i * SB * a.ld + (long long)tk.j * SB;
   // operands -> shared memory: 64 rows of 256 B each, 16 B per cp.async, 4 per thread per operand
+  const bool fused = tk.type == T_P3P1;
   const T* Bsrc;
   long long ldb;
   if (tk.type == T_P2R) { Bsrc = C; ldb = a.ld; }
@@ -206,6 +240,11 @@ __device__ __forceinline__ void small_minplus(const SmArgs<T>& a, const Task& tk
 #pragma unroll
       for (int j = 0; j < 4; ++j) acc[i][j] = SV<T>::relax(A4[i], B4[j], acc[i][j]);
   }
+  if (fused) {  // tile (k+1,k+1) after round k: close it as P1(k+1) (R6 check included)
+    small_close(acc, rowbuf, colbuf, a.negflag);
+    small_store_diag(a, tk.k + 1, C, acc);
+    return;
+  }
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
     V4 v;
@@ -224,12 +263,35 @@ __device__ __forceinline__ void small_minplus(const SmArgs<T>& a, const Task& tk
   }
 }
 
-// thread 0: the next task (dequeue + decode); its flags are checked by the caller
+__device__ __forceinline__ Task small_task(const int4 e) {
+  Task t;
+  t.type = e.x; t.k = e.y; t.i = e.z; t.j = e.w;
+  return t;
+}
+
+// dependencies of a queue entry: a fused F(k) needs those of P3(k; k+1,k+1) and of P1(k+1)
+// (the panel copy of parity (k+1) % 2 may be rewritten once round k-1's panel tasks are done)
 template <typename T>
-__device__ __forceinline__ void small_fetch(const SmArgs<T>& a, SmSlot& s) {
-  s.t = (long long)atomicAdd(a.counter, 1ull);
-  s.ready = 0;
-  if (s.t < a.total) s.tk = decode(s.t, a.nb, a.delay);
+__device__ __forceinline__ bool small_deps(const SmArgs<T>& a, const Task& t) {
+  if (t.type != T_P3P1) return deps_met(a, t);
+  Task p3 = t;
+  p3.type = T_P3;
+  if (t.k >= 1 && ld_relaxed(a.done2 + t.k - 1) < 2 * (a.nb - 1)) return false;
+  return deps_met(a, p3);
+}
+
+template <typename T>
+__device__ __forceinline__ void small_signal(const SmArgs<T>& a, const Task& t) {
+  if (t.type != T_P3P1) {
+    signal_done(a, t);
+    return;
+  }
+  // F(k): tile (k+1,k+1) has rounds 0..k+1 applied; round k+1's diagonal is in the panel copy
+  const int k = t.k, nb = a.nb;
+  asm volatile("fence.release.gpu;" ::: "memory");
+  st_relaxed(a.ver + (long long)t.i * nb + t.j, k + 2);
+  st_relaxed(a.diagready + ((k + 1) & 1), k + 2);
+  red_relaxed_add(a.done3 + k, 1);
 }
 
 template <typename T>
@@ -240,41 +302,99 @@ __global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ S
   __shared__ __align__(16) T colbuf[2 * SB];
   __shared__ SmSlot slot[2];
   const int tid = threadIdx.x;
-  if (tid == 0) small_fetch(a, slot[0]);
+  long long idx_next = 0;  // thread 0: queue index of the slot after N (fetched one task ahead)
+  if (tid == 0) {
+    const long long t0 = (long long)atomicAdd(a.counter, 1ull);
+    slot[0].t = t0;
+    slot[0].ready = 0;
+    if (t0 < a.total) slot[0].tk = small_task(a.queue[t0]);
+    slot[1].t = (long long)atomicAdd(a.counter, 1ull);
+    slot[1].ready = 0;
+  }
   __syncthreads();
   for (int it = 0;; ++it) {
     SmSlot& S = slot[it & 1];
     SmSlot& N = slot[(it + 1) & 1];
     if (S.t >= a.total) break;
     const Task tk = S.tk;
+    int4 nq = make_int4(0, 0, 0, 0);
     if (tid == 0) {
       if (!S.ready)
-        while (!deps_met(a, tk)) __nanosleep(32);
-      small_fetch(a, N);  // the next task, decoded while this one runs
+        while (!small_deps(a, tk)) __nanosleep(32);
+      // N's entry and the next queue index: issued now, consumed after this task's work, so
+      // their latency hides under it
+      if (N.t < a.total) nq = a.queue[N.t];
+      idx_next = (long long)atomicAdd(a.counter, 1ull);
     }
-    __syncthreads();  // dependencies met (acquired by thread 0); N published
+    __syncthreads();  // dependencies met (acquired by thread 0)
     if (tk.type == T_P1) small_phase1(a, tk, rowbuf, colbuf);
-    else small_minplus(a, tk, As, Bs);
-    __syncthreads();  // every thread's stores of this task are issued; As / Bs free again
+    else small_minplus(a, tk, As, Bs, rowbuf, colbuf);
+    if (tid == 0 && N.t < a.total) N.tk = small_task(nq);
+    __syncthreads();  // every thread's stores of this task are issued; As / Bs free; N.tk published
     if (tid == 0) {
-      signal_done(a, tk);
+      small_signal(a, tk);
       // the next task's flags, once: if met, it starts without another wait
-      if (N.t < a.total && deps_met(a, N.tk)) N.ready = 1;
+      N.ready = N.t < a.total && small_deps(a, N.tk);
+      S.t = idx_next;  // this slot becomes the one after N (read by the others only after the
+      S.ready = 0;     // next iteration's first barrier)
     }
   }
 }
 
 }  // namespace
 
+// The small kernel's queue (see the header): critical path first in every segment,
+// F(k) = fused P3(k; k+1,k+1) + P1(k+1). Host and test hook (apsp_debug_queue, P = -1).
+long long small_queue(int nb, std::vector<int4>* q) {
+  std::vector<int4> v;
+  auto add = [&](int type, int k, int i, int j) { v.push_back(make_int4(type, k, i, j)); };
+  // round rd's phase 3 on row r and column r, without rows / columns e0, e1 (and without the
+  // tile (r, r) itself if skip_rr)
+  auto p3_rowcol = [&](int rd, int r, int e0, int e1, bool skip_rr) {
+    for (int j = 0; j < nb; ++j)
+      if (j != rd && j != e0 && j != e1 && !(skip_rr && j == r)) add(T_P3, rd, r, j);
+    for (int i = 0; i < nb; ++i)
+      if (i != rd && i != e0 && i != e1 && i != r) add(T_P3, rd, i, r);
+  };
+  add(T_P1, 0, 0, 0);
+  for (int k = 0; k < nb; ++k) {
+    const int k1 = k + 1;
+    if (k1 < nb) {
+      add(T_P2R, k, k, k1);
+      add(T_P2C, k, k1, k);
+      if (k >= 1) p3_rowcol(k - 1, k1, k, -1, false);  // round k-1 (not on row / column k): incl. (k+1,k+1)
+      add(T_P3P1, k, k1, k1);
+    }
+    for (int j = 0; j < nb; ++j)  // the other panel tiles of round k
+      if (j != k && j != k1) add(T_P2R, k, k, j);
+    for (int i = 0; i < nb; ++i)
+      if (i != k && i != k1) add(T_P2C, k, i, k);
+    if (k >= 1)  // the rest of round k-1's phase 3 (rows / columns not in {k-1, k, k+1})
+      for (int i = 0; i < nb; ++i)
+        for (int j = 0; j < nb; ++j)
+          if (i != k - 1 && i != k && j != k - 1 && j != k && i != k1 && j != k1) add(T_P3, k - 1, i, j);
+    if (k1 < nb) p3_rowcol(k, k1, -1, -1, true);  // round k on row / column k+1 ((k+1,k+1) is in F(k))
+  }
+  for (int i = 0; i < nb; ++i)  // the last round's phase 3
+    for (int j = 0; j < nb; ++j)
+      if (i != nb - 1 && j != nb - 1) add(T_P3, nb - 1, i, j);
+  if (q) *q = v;
+  return (long long)v.size();
+}
+
+static long long small_pbuf_bytes(int nb, size_t elem) { return 2ll * (2 + 2 * nb) * STE * (long long)elem; }
+static long long small_flag_bytes(int nb) {
+  return ((2 + (long long)nb * nb + 2 + 4ll * nb + 2ll * nb) * 4 + 15) / 16 * 16;
+}
+
 long long fw_small_work_bytes(int nb, size_t elem) {
-  const long long pb = 2ll * (2 + 2 * nb) * STE * (long long)elem;
-  const long long flags = ((2 + (long long)nb * nb + 2 + 4ll * nb + 2ll * nb) * 4 + 15) / 16 * 16;
-  return pb + flags;
+  return small_pbuf_bytes(nb, elem) + small_flag_bytes(nb) + small_queue(nb, nullptr) * (long long)sizeof(int4);
 }
 
 template <typename T>
 cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag, long long delay, int ctas_per_sm,
                             cudaStream_t s) {
+  (void)delay;  // the small kernel's queue order is fixed (critical path first)
   if (nb <= 0) return cudaSuccess;
   int dev = 0, sms = 0;
   cudaError_t e;
@@ -286,7 +406,8 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
   a.ld = ld;
   a.nb = nb;
   a.pbuf = static_cast<T*>(work);
-  int* f = reinterpret_cast<int*>(static_cast<char*>(work) + 2ll * (2 + 2 * nb) * STE * (long long)sizeof(T));
+  char* const fb = static_cast<char*>(work) + small_pbuf_bytes(nb, sizeof(T));
+  int* f = reinterpret_cast<int*>(fb);
   a.counter = reinterpret_cast<unsigned long long*>(f); f += 2;
   a.ver = f; f += (long long)nb * nb;
   a.diagready = f; f += 2;
@@ -295,10 +416,16 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
   a.done2 = f; f += nb;
   a.done3 = f; f += nb;
   a.negflag = negflag;
-  a.total = (long long)nb * nb * nb;
-  a.delay = delay;
-  const long long flag_bytes = fw_small_work_bytes(nb, sizeof(T)) - 2ll * (2 + 2 * nb) * STE * (long long)sizeof(T);
-  if ((e = cudaMemsetAsync(a.counter, 0, flag_bytes, s)) != cudaSuccess) return e;
+  // the queue: built once per work buffer layout; uploaded on every launch (<= 512 KB,
+  // stream-ordered before the kernel)
+  std::vector<int4> q;
+  a.total = small_queue(nb, &q);
+  int4* dq = reinterpret_cast<int4*>(fb + small_flag_bytes(nb));
+  a.queue = dq;
+  if ((e = cudaMemcpyAsync(dq, q.data(), q.size() * sizeof(int4), cudaMemcpyHostToDevice, s)) != cudaSuccess)
+    return e;
+  if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return e;  // q is a local
+  if ((e = cudaMemsetAsync(a.counter, 0, small_flag_bytes(nb), s)) != cudaSuccess) return e;
   // persistent grid: every CTA must be resident (tasks wait on each other)
   int occ = 0;
   if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fw_small_kernel<T>, SNT, 0)) != cudaSuccess) return e;

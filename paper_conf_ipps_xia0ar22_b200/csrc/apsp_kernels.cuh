@@ -3,6 +3,7 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <cstdint>
+#include <vector>
 
 namespace apsp {
 
@@ -146,6 +147,8 @@ template <typename T>
 cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag, long long delay, int ctas_per_sm,
                             cudaStream_t s);
 long long fw_small_work_bytes(int nb, size_t elem);
+// its task queue (host-built, critical path first; type 4 = fused P3(k; k+1,k+1) + P1(k+1))
+long long small_queue(int nb, std::vector<int4>* q);
 
 // The packed int16 closure (R16) as one persistent dataflow launch
 // (apsp_fw_dataflow16.cu); `work` holds fw_dataflow16_work_bytes(nb) bytes.

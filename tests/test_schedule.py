@@ -10,7 +10,7 @@ import itertools
 import numpy as np
 import pytest
 
-P1, P2R, P2C, P3 = 0, 1, 2, 3
+P1, P2R, P2C, P3, P3P1 = 0, 1, 2, 3, 4
 
 
 def expected_tasks(nb):
@@ -47,6 +47,9 @@ def simulate(nb, queues):
 
     def ready(r, t):
         typ, k, i, j = (int(x) for x in t)
+        if typ == P3P1:  # fused P3(k; k+1,k+1) + P1(k+1) (small-n kernel)
+            return (ready(r, (P3, k, i, j)) and
+                    (k + 1 < 2 or all(done2[x, k - 1] >= cnt2(x, k - 1) for x in range(P))))
         if ver[i, j] < k:
             return False
         if typ == P3:
@@ -66,7 +69,11 @@ def simulate(nb, queues):
             while pos[r] < len(queues[r]) and ready(r, queues[r][pos[r]]):
                 typ, k, i, j = (int(x) for x in queues[r][pos[r]])
                 ver[i, j] = k + 1
-                if typ == P1:
+                if typ == P3P1:
+                    ver[i, j] = k + 2
+                    p1_done.add(k + 1)
+                    done3[r, k] += 1
+                elif typ == P1:
                     p1_done.add(k)
                 elif typ == P2R:
                     p2r_done.add((k, j))
@@ -132,3 +139,33 @@ def test_bad_arguments(lib):
         lib.apsp_debug_queue(10, 3, 0, 1)  # nb % P != 0
     with pytest.raises(ValueError):
         lib.apsp_debug_queue(8, 4, 4, 1)   # q >= P
+
+
+def expand_fused(q):
+    for typ, k, i, j in q.tolist():
+        if typ == P3P1:
+            yield (P3, k, i, j)
+            yield (P1, k + 1, i, j)
+        else:
+            yield (typ, k, i, j)
+
+
+@pytest.mark.parametrize("nb", [1, 2, 3, 4, 5, 8, 16, 23, 32])
+def test_small_kernel_queue_complete_and_deadlock_free(lib, nb):
+    """The 64-tile small-n kernel's host-built queue (apsp_fw_small.cu; critical path first, F(k)
+    fuses P3(k; k+1,k+1) with P1(k+1)): every blocked-FW task once, and an in-order drain with the
+    kernel's exact waits (a fused entry waits for both halves' dependencies)."""
+    q = lib.apsp_debug_queue(nb, -1, 0, 0)
+    assert sorted(expand_fused(q)) == sorted(expected_tasks(nb))
+    assert len(q) == nb ** 3 - (nb - 1)
+    assert simulate(nb, [q])
+    if nb >= 3:  # the chain of round 0 comes first: P2R(0,1), P2C(1,0), then F(0)
+        assert [tuple(x) for x in q[1:4].tolist()] == [(P2R, 0, 0, 1), (P2C, 0, 1, 0), (P3P1, 0, 1, 1)]
+
+
+def test_simulator_rejects_fused_entry_before_its_panels(lib):
+    """Pin of the fused-entry rule: F(0) moved ahead of the panel tiles it reads cannot drain."""
+    q = lib.apsp_debug_queue(6, -1, 0, 0).tolist()
+    f = next(x for x, t in enumerate(q) if t[0] == P3P1 and t[1] == 0)
+    q.insert(1, q.pop(f))
+    assert not simulate(6, [np.array(q)])
