@@ -273,12 +273,12 @@ static apsp_status run_small(Handle* h) {
   }
   int ctas = 1;
   if (const char* e = getenv("APSP_SMALL_CTAS")) ctas = atoi(e);  // tuning experiments only
-  const long long delay = h->df_delay > 0 ? h->df_delay : 0;
   h->ev_begin(2);
-  if ((st = h->cuda(launch_fw_small<T>(static_cast<T*>(h->shards[0].D), h->ld, nb, h->df_work, h->d_flag, delay, ctas,
-                                       h->stream),
+  if ((st = h->cuda(launch_fw_small<T>(static_cast<T*>(h->shards[0].D), h->ld, nb, h->df_work, h->d_flag,
+                                       h->small_queue_loaded, ctas, h->stream),
                     "fw_small")))
     return st;
+  h->small_queue_loaded = true;
   h->ev_end((double)h->n_pad * h->n_pad * h->n_pad);
   return APSP_OK;
 }

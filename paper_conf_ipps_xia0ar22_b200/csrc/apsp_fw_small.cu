@@ -16,14 +16,13 @@
 // Structure: the flag protocol of apsp_fw_dataflow.cu (apsp_df_common.cuh: per-tile
 // versions, diagonal / panel readiness, double-buffered panel copies, deps_met /
 // signal_done) with a queue ordered for the critical path and a simpler engine:
-//   * the queue is built on the host (small_queue, at most 32^3 entries) in
-//     segments seg(k) = [P2R(k,k+1), P2C(k+1,k), round k-1's phase-3 tiles on
-//     row / column k+1, F(k), the other panel tiles of round k, the rest of round
-//     k-1's phase 3, round k's phase-3 tiles on row / column k+1], so the chain
-//     P1(k) -> panels (k,k+1), (k+1,k) -> tile (k+1,k+1) -> P1(k+1) is queued
-//     first in every segment; every dependency of an entry lies earlier in the
-//     queue (tests/test_schedule.py simulates it), so a CTA that finishes its
-//     task before taking the next cannot deadlock;
+//   * the queue is built on the host (small_queue, at most 32^3 entries) by
+//     critical-path list scheduling: tasks in decreasing order of their bottom
+//     level in the dependency graph the kernel waits on, a topological order in
+//     which the chain P1(k) -> panels -> tile (k+1,k+1) -> P1(k+1) comes first and
+//     the bulk of phase 3 fills in behind it; every dependency of an entry lies
+//     earlier in the queue (tests/test_schedule.py simulates it), so a CTA that
+//     finishes its task before taking the next cannot deadlock;
 //   * F(k) fuses P3(k; k+1,k+1) with P1(k+1): the CTA that updates the next
 //     diagonal tile closes it in registers right away (one flag hop and one
 //     tile load less on the chain of every round);
@@ -46,6 +45,7 @@
 #include "apsp_df_common.cuh"
 
 #include <cuda_runtime.h>
+#include <algorithm>
 #include <cstdint>
 #include <cstring>
 #include <vector>
@@ -343,43 +343,80 @@ __global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ S
 
 }  // namespace
 
-// The small kernel's queue (see the header): critical path first in every segment,
-// F(k) = fused P3(k; k+1,k+1) + P1(k+1). Host and test hook (apsp_debug_queue, P = -1).
+// The small kernel's queue: critical-path list scheduling. Every task (k, i, j) of the blocked
+// FW (P1 / P2R / P2C / P3 by position) is a node of the dependency graph the kernel waits on
+// (previous round of the same tile; the diagonal / panel tiles it reads; the panel copies'
+// parity reuse two rounds later); its bottom level = its duration + the longest chain of
+// (hop + duration) after it. Entries are sorted by decreasing bottom level, which is a
+// topological order (every edge strictly decreases it), so the queue is deadlock-free, and the
+// chain phase 1 -> panel tiles -> next diagonal tile is always served first with the bulk
+// filling the gaps. F(k) = P3(k; k+1,k+1) fused with P1(k+1) (one entry, type 4). Durations
+// are model units (a 64^3 min-plus task ~3 us on one SM, phase 1 ~5 us, a flag hop ~1.5 us).
+// Host and test hook (apsp_debug_queue, P = -1).
 long long small_queue(int nb, std::vector<int4>* q) {
-  std::vector<int4> v;
-  auto add = [&](int type, int k, int i, int j) { v.push_back(make_int4(type, k, i, j)); };
-  // round rd's phase 3 on row r and column r, without rows / columns e0, e1 (and without the
-  // tile (r, r) itself if skip_rr)
-  auto p3_rowcol = [&](int rd, int r, int e0, int e1, bool skip_rr) {
-    for (int j = 0; j < nb; ++j)
-      if (j != rd && j != e0 && j != e1 && !(skip_rr && j == r)) add(T_P3, rd, r, j);
+  if (nb <= 0) return 0;
+  const double d13 = 3.0, d1 = 5.0, hop = 1.5;
+  const long long N = (long long)nb * nb * nb;
+  auto id = [&](int k, int i, int j) { return ((long long)k * nb + i) * nb + j; };
+  std::vector<double> bl(N, 0.0);
+  std::vector<double> maxP2(nb + 2, -1.0), maxP1(nb + 2, -1.0);
+  auto dur = [&](int k, int i, int j) { return (i == k && j == k) ? d1 : d13; };
+  for (int k = nb - 1; k >= 0; --k) {
+    auto finish = [&](int i, int j) {  // bl of (k, i, j) from its successors
+      double m = -1.0;
+      if (k + 1 < nb) m = std::max(m, bl[id(k + 1, i, j)]);  // the tile's next round
+      const bool p1 = i == k && j == k, p2r = i == k && j != k, p2c = j == k && i != k;
+      if (p1)
+        for (int x = 0; x < nb; ++x)
+          if (x != k) m = std::max({m, bl[id(k, k, x)], bl[id(k, x, k)]});
+      if (p2r)
+        for (int x = 0; x < nb; ++x)
+          if (x != k) m = std::max(m, bl[id(k, x, j)]);
+      if (p2c)
+        for (int x = 0; x < nb; ++x)
+          if (x != k) m = std::max(m, bl[id(k, i, x)]);
+      if ((p2r || p2c) && k + 2 < nb) m = std::max(m, maxP1[k + 2]);  // done2[k] -> P1(k+2)
+      if (!p1 && !p2r && !p2c && k + 2 < nb) m = std::max(m, maxP2[k + 2]);  // done3[k] -> P2(k+2)
+      bl[id(k, i, j)] = dur(k, i, j) + (m >= 0 ? hop + m : 0.0);
+    };
     for (int i = 0; i < nb; ++i)
-      if (i != rd && i != e0 && i != e1 && i != r) add(T_P3, rd, i, r);
-  };
-  add(T_P1, 0, 0, 0);
-  for (int k = 0; k < nb; ++k) {
-    const int k1 = k + 1;
-    if (k1 < nb) {
-      add(T_P2R, k, k, k1);
-      add(T_P2C, k, k1, k);
-      if (k >= 1) p3_rowcol(k - 1, k1, k, -1, false);  // round k-1 (not on row / column k): incl. (k+1,k+1)
-      add(T_P3P1, k, k1, k1);
-    }
-    for (int j = 0; j < nb; ++j)  // the other panel tiles of round k
-      if (j != k && j != k1) add(T_P2R, k, k, j);
-    for (int i = 0; i < nb; ++i)
-      if (i != k && i != k1) add(T_P2C, k, i, k);
-    if (k >= 1)  // the rest of round k-1's phase 3 (rows / columns not in {k-1, k, k+1})
-      for (int i = 0; i < nb; ++i)
-        for (int j = 0; j < nb; ++j)
-          if (i != k - 1 && i != k && j != k - 1 && j != k && i != k1 && j != k1) add(T_P3, k - 1, i, j);
-    if (k1 < nb) p3_rowcol(k, k1, -1, -1, true);  // round k on row / column k+1 ((k+1,k+1) is in F(k))
+      for (int j = 0; j < nb; ++j)
+        if (i != k && j != k) finish(i, j);
+    for (int x = 0; x < nb; ++x)
+      if (x != k) {
+        finish(k, x);
+        finish(x, k);
+        maxP2[k] = std::max({maxP2[k], bl[id(k, k, x)], bl[id(k, x, k)]});
+      }
+    finish(k, k);
+    maxP1[k] = bl[id(k, k, k)];
   }
-  for (int i = 0; i < nb; ++i)  // the last round's phase 3
-    for (int j = 0; j < nb; ++j)
-      if (i != nb - 1 && j != nb - 1) add(T_P3, nb - 1, i, j);
-  if (q) *q = v;
-  return (long long)v.size();
+  struct E {
+    double key;
+    int4 t;
+  };
+  std::vector<E> e;
+  e.reserve(N);
+  for (int k = 0; k < nb; ++k)
+    for (int i = 0; i < nb; ++i)
+      for (int j = 0; j < nb; ++j) {
+        if (i == k && j == k) {
+          if (k == 0) e.push_back({bl[id(0, 0, 0)], make_int4(T_P1, 0, 0, 0)});
+          continue;  // P1(k >= 1) is fused into F(k-1)
+        }
+        if (k + 1 < nb && i == k + 1 && j == k + 1) {  // F(k): P3 then P1(k+1), no hop in between
+          e.push_back({d13 + bl[id(k + 1, k + 1, k + 1)], make_int4(T_P3P1, k, i, j)});
+          continue;
+        }
+        const int type = i == k ? T_P2R : (j == k ? T_P2C : T_P3);
+        e.push_back({bl[id(k, i, j)], make_int4(type, k, i, j)});
+      }
+  std::stable_sort(e.begin(), e.end(), [](const E& a, const E& b) { return a.key > b.key; });
+  if (q) {
+    q->resize(e.size());
+    for (size_t x = 0; x < e.size(); ++x) (*q)[x] = e[x].t;
+  }
+  return (long long)e.size();
 }
 
 static long long small_pbuf_bytes(int nb, size_t elem) { return 2ll * (2 + 2 * nb) * STE * (long long)elem; }
@@ -392,9 +429,8 @@ long long fw_small_work_bytes(int nb, size_t elem) {
 }
 
 template <typename T>
-cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag, long long delay, int ctas_per_sm,
+cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag, bool queue_loaded, int ctas_per_sm,
                             cudaStream_t s) {
-  (void)delay;  // the small kernel's queue order is fixed (critical path first)
   if (nb <= 0) return cudaSuccess;
   int dev = 0, sms = 0;
   cudaError_t e;
@@ -416,15 +452,18 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
   a.done2 = f; f += nb;
   a.done3 = f; f += nb;
   a.negflag = negflag;
-  // the queue: built once per work buffer layout; uploaded on every launch (<= 512 KB,
-  // stream-ordered before the kernel)
-  std::vector<int4> q;
-  a.total = small_queue(nb, &q);
+  // the queue lives in the work buffer: built and uploaded with the first launch on it
   int4* dq = reinterpret_cast<int4*>(fb + small_flag_bytes(nb));
   a.queue = dq;
-  if ((e = cudaMemcpyAsync(dq, q.data(), q.size() * sizeof(int4), cudaMemcpyHostToDevice, s)) != cudaSuccess)
-    return e;
-  if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return e;  // q is a local
+  if (!queue_loaded) {
+    std::vector<int4> q;
+    a.total = small_queue(nb, &q);
+    if ((e = cudaMemcpyAsync(dq, q.data(), q.size() * sizeof(int4), cudaMemcpyHostToDevice, s)) != cudaSuccess)
+      return e;
+    if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return e;  // q is a local
+  } else {
+    a.total = small_queue(nb, nullptr);
+  }
   if ((e = cudaMemsetAsync(a.counter, 0, small_flag_bytes(nb), s)) != cudaSuccess) return e;
   // persistent grid: every CTA must be resident (tasks wait on each other)
   int occ = 0;
@@ -437,7 +476,7 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
   return cudaGetLastError();
 }
 
-template cudaError_t launch_fw_small<int>(int*, long long, int, void*, int*, long long, int, cudaStream_t);
-template cudaError_t launch_fw_small<float>(float*, long long, int, void*, int*, long long, int, cudaStream_t);
+template cudaError_t launch_fw_small<int>(int*, long long, int, void*, int*, bool, int, cudaStream_t);
+template cudaError_t launch_fw_small<float>(float*, long long, int, void*, int*, bool, int, cudaStream_t);
 
 }  // namespace apsp
