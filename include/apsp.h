@@ -225,7 +225,10 @@ apsp_status apsp_init_johnson(apsp_handle** out, int64_t n, const int64_t* row_p
 
 /*
  * apsp_select — choose the method for a graph as the paper does (§IV,
- * PAPER.md:199-323). Density filter (§IV-C), density = m / n^2:
+ * PAPER.md:199-323). EXPERIMENTAL: the density filter is the selector SURVEY §8(f)
+ * NEXT-4 names; the calibrated cost models behind it are outside the hot-path scope
+ * and are kept as an aid, not a tuned component.
+ * Density filter (§IV-C), density = m / n^2:
  *   > 1 %       blocked FW or Johnson
  *   < 0.01 %    Johnson or the boundary algorithm (only if a partition comp/k is
  *               given; the paper computes one with METIS)

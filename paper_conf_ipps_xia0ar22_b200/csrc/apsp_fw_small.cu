@@ -47,6 +47,7 @@
 #include <cuda_runtime.h>
 #include <algorithm>
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 #include <vector>
 
@@ -355,6 +356,21 @@ __global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ S
 // Host and test hook (apsp_debug_queue, P = -1).
 long long small_queue(int nb, std::vector<int4>* q) {
   if (nb <= 0) return 0;
+  // tuning experiments only: APSP_SMALL_QUEUE=decode (the 128-tile kernel's segment order,
+  // no fusion) or bl_nofuse (list order without fused entries); default: list order + F(k)
+  const char* qv = getenv("APSP_SMALL_QUEUE");
+  const int variant = qv ? (strcmp(qv, "decode") == 0 ? 1 : strcmp(qv, "bl_nofuse") == 0 ? 2 : 0) : 0;
+  if (variant == 1) {
+    const long long total = (long long)nb * nb * nb;
+    if (q) {
+      q->resize(total);
+      for (long long g = 0; g < total; ++g) {
+        const Task t = decode(g, nb, 0);
+        (*q)[g] = make_int4(t.type, t.k, t.i, t.j);
+      }
+    }
+    return total;
+  }
   const double d13 = 3.0, d1 = 5.0, hop = 1.5;
   const long long N = (long long)nb * nb * nb;
   auto id = [&](int k, int i, int j) { return ((long long)k * nb + i) * nb + j; };
@@ -401,10 +417,10 @@ long long small_queue(int nb, std::vector<int4>* q) {
     for (int i = 0; i < nb; ++i)
       for (int j = 0; j < nb; ++j) {
         if (i == k && j == k) {
-          if (k == 0) e.push_back({bl[id(0, 0, 0)], make_int4(T_P1, 0, 0, 0)});
+          if (k == 0 || variant == 2) e.push_back({bl[id(k, k, k)], make_int4(T_P1, k, k, k)});
           continue;  // P1(k >= 1) is fused into F(k-1)
         }
-        if (k + 1 < nb && i == k + 1 && j == k + 1) {  // F(k): P3 then P1(k+1), no hop in between
+        if (variant != 2 && k + 1 < nb && i == k + 1 && j == k + 1) {  // F(k): P3 then P1(k+1), no hop
           e.push_back({d13 + bl[id(k + 1, k + 1, k + 1)], make_int4(T_P3P1, k, i, j)});
           continue;
         }

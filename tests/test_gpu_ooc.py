@@ -43,9 +43,10 @@ def test_ooc_int32_bit_exact(lib, n, block):
 
 def test_ooc_with_resident_bands(lib):
     g = gg.erdos_renyi(1024, 6000, seed=3)
-    # n_pad=1024, B=256: band = 1 MiB; budget leaves room for 2 resident bands
+    # n_pad=1024, B=256: band = 1 MiB; working set = 3 pivot buffers + 3 ring slots + 2 B x B
+    # scratches (6.5 MiB) + CSR; the budget leaves room for 2 resident bands
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w,
-                                cfg=ooc_cfg(lib, 256, budget_mb=6.5, stream_all=False)) as h:
+                                cfg=ooc_cfg(lib, 256, budget_mb=8.7, stream_all=False)) as h:
         info = lib.apsp_get_info(h)
         assert info.mode == lib.APSP_MODE_OUT_OF_CORE
         assert 0 < info.host_bytes < 1024 * 1024 * 4
@@ -81,7 +82,7 @@ def test_ooc_config2_size_mixed_residency(lib):
     g = gg.baseline_config("cfg2_grid16384")
     bb = 2048 * 16384 * 4
     c = ooc_cfg(lib, 2048, stream_all=False)
-    c.device_budget_bytes = 4 * bb + 2048 * 2048 * 4 + 3 * bb + (1 << 20)
+    c.device_budget_bytes = 6 * bb + 2 * 2048 * 2048 * 4 + 3 * bb + (2 << 20)  # working set + 3 bands
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
         info = lib.apsp_get_info(h)
         assert info.mode == lib.APSP_MODE_OUT_OF_CORE and info.host_bytes == 5 * bb
@@ -140,7 +141,7 @@ def test_ooc_virtual_ranks_resident_negative_f32(lib):
     p = rng.integers(-300, 300, size=g0.n)
     s, t, w = g0.arcs()
     g = gg.csr_from_arcs(g0.n, s, t, (w.astype(np.int64) + p[s] - p[t]).astype(np.int32))
-    c = ooc_cfg(lib, 128, budget_mb=6.4, stream_all=False)  # 2 of each rank's 4 bands resident
+    c = ooc_cfg(lib, 128, budget_mb=8.6, stream_all=False)  # 2 of each rank's 4 bands resident
     c.world_size = 2
     c.virtual_ranks = 1
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=c) as h:
