@@ -359,17 +359,26 @@ long long small_queue(int nb, std::vector<int4>* q) {
   // tuning experiments only: APSP_SMALL_QUEUE=decode (the 128-tile kernel's segment order,
   // no fusion) or bl_nofuse (list order without fused entries); default: list order + F(k)
   const char* qv = getenv("APSP_SMALL_QUEUE");
-  const int variant = qv ? (strcmp(qv, "decode") == 0 ? 1 : strcmp(qv, "bl_nofuse") == 0 ? 2 : 0) : 0;
-  if (variant == 1) {
+  const int variant = !qv ? 3
+                          : strcmp(qv, "decode") == 0      ? 1
+                          : strcmp(qv, "bl_nofuse") == 0  ? 2
+                          : strcmp(qv, "decode_fuse") == 0 ? 3
+                                                           : 0;
+  if (variant == 1 || variant == 3) {
+    // the 128-tile kernel's segment order (decode, delay 0); variant 3 fuses the tile (k+1,k+1)
+    // of round k with the P1(k+1) that follows it
+    std::vector<int4> v;
     const long long total = (long long)nb * nb * nb;
-    if (q) {
-      q->resize(total);
-      for (long long g = 0; g < total; ++g) {
-        const Task t = decode(g, nb, 0);
-        (*q)[g] = make_int4(t.type, t.k, t.i, t.j);
-      }
+    for (long long g = 0; g < total; ++g) {
+      const Task t = decode(g, nb, 0);
+      if (variant == 3 && t.type == T_P1 && t.k >= 1) continue;  // inside F(k-1)
+      if (variant == 3 && t.type == T_P3 && t.i == t.k + 1 && t.j == t.k + 1)
+        v.push_back(make_int4(T_P3P1, t.k, t.i, t.j));
+      else
+        v.push_back(make_int4(t.type, t.k, t.i, t.j));
     }
-    return total;
+    if (q) *q = v;
+    return (long long)v.size();
   }
   const double d13 = 3.0, d1 = 5.0, hop = 1.5;
   const long long N = (long long)nb * nb * nb;

@@ -152,15 +152,17 @@ def expand_fused(q):
 
 @pytest.mark.parametrize("nb", [1, 2, 3, 4, 5, 8, 16, 23, 32])
 def test_small_kernel_queue_complete_and_deadlock_free(lib, nb):
-    """The 64-tile small-n kernel's host-built queue (apsp_fw_small.cu; critical path first, F(k)
-    fuses P3(k; k+1,k+1) with P1(k+1)): every blocked-FW task once, and an in-order drain with the
-    kernel's exact waits (a fused entry waits for both halves' dependencies)."""
+    """The 64-tile small-n kernel's host-built queue (apsp_fw_small.cu: the 128-tile kernel's segment
+    order with F(k) = P3(k; k+1,k+1) fused with P1(k+1)): every blocked-FW task once, and an
+    in-order drain with the kernel's exact waits (a fused entry waits for both halves' dependencies)."""
     q = lib.apsp_debug_queue(nb, -1, 0, 0)
     assert sorted(expand_fused(q)) == sorted(expected_tasks(nb))
     assert len(q) == nb ** 3 - (nb - 1)
     assert simulate(nb, [q])
-    if nb >= 3:  # the chain of round 0 comes first: P2R(0,1), P2C(1,0), then F(0)
-        assert [tuple(x) for x in q[1:4].tolist()] == [(P2R, 0, 0, 1), (P2C, 0, 1, 0), (P3P1, 0, 1, 1)]
+    if nb >= 2:  # round 0's panel tiles right after P1(0), then F(0) (the next diagonal tile) first
+        assert sorted(tuple(x) for x in q[1:2 * nb - 1].tolist()) == sorted(
+            t for t in expected_tasks(nb) if t[1] == 0 and t[0] in (P2R, P2C))
+        assert tuple(q[2 * nb - 1].tolist()) == (P3P1, 0, 1, 1)
 
 
 def test_simulator_rejects_fused_entry_before_its_panels(lib):
