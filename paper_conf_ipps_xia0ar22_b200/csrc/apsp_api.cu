@@ -271,10 +271,13 @@ static apsp_status run_small(Handle* h) {
     if ((st = h->cuda(cudaMallocAsync(&h->df_work, wb, h->stream), "cudaMalloc dataflow (small)"))) return st;
     h->device_bytes += wb;
   }
-  int ctas = 1;
+  // CTAs per SM and queue delay measured per size: one CTA per SM up to
+  // n_pad = 1024 (the critical path dominates), two above (more tasks per round in flight)
+  int ctas = h->n_pad <= 1024 ? 1 : 2;
   if (const char* e = getenv("APSP_SMALL_CTAS")) ctas = atoi(e);  // tuning experiments only
+  const long long delay = h->df_delay > 0 ? h->df_delay : kSmallDelay;
   h->ev_begin(2);
-  if ((st = h->cuda(launch_fw_small<T>(static_cast<T*>(h->shards[0].D), h->ld, nb, h->df_work, h->d_flag,
+  if ((st = h->cuda(launch_fw_small<T>(static_cast<T*>(h->shards[0].D), h->ld, nb, h->df_work, h->d_flag, delay,
                                        h->small_queue_loaded, ctas, h->stream),
                     "fw_small")))
     return st;

@@ -1003,7 +1003,7 @@ extern "C" int64_t apsp_debug_queue(int32_t nb, int32_t P, int32_t q, int64_t de
   if (P == -1) {  // the small-n kernel's queue (apsp_fw_small.cu), nb 64-wide tile rows
     if (nb <= 0) return -1;
     std::vector<int4> sq;
-    const long long total = small_queue(nb, &sq);
+    const long long total = small_queue(nb, delay, &sq);
     for (long long g = 0; g < total && g < cap; ++g) {
       out[4 * g] = sq[g].x; out[4 * g + 1] = sq[g].y; out[4 * g + 2] = sq[g].z; out[4 * g + 3] = sq[g].w;
     }

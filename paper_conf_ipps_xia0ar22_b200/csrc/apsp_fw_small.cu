@@ -354,7 +354,7 @@ __global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ S
 // filling the gaps. F(k) = P3(k; k+1,k+1) fused with P1(k+1) (one entry, type 4). Durations
 // are model units (a 64^3 min-plus task ~3 us on one SM, phase 1 ~5 us, a flag hop ~1.5 us).
 // Host and test hook (apsp_debug_queue, P = -1).
-long long small_queue(int nb, std::vector<int4>* q) {
+long long small_queue(int nb, long long delay, std::vector<int4>* q) {
   if (nb <= 0) return 0;
   // tuning experiments only: APSP_SMALL_QUEUE=decode (the 128-tile kernel's segment order,
   // no fusion) or bl_nofuse (list order without fused entries); default: list order + F(k)
@@ -365,12 +365,12 @@ long long small_queue(int nb, std::vector<int4>* q) {
                           : strcmp(qv, "decode_fuse") == 0 ? 3
                                                            : 0;
   if (variant == 1 || variant == 3) {
-    // the 128-tile kernel's segment order (decode, delay 0); variant 3 fuses the tile (k+1,k+1)
+    // the 128-tile kernel's segment order (decode with this queue delay); variant 3 fuses the tile (k+1,k+1)
     // of round k with the P1(k+1) that follows it
     std::vector<int4> v;
     const long long total = (long long)nb * nb * nb;
     for (long long g = 0; g < total; ++g) {
-      const Task t = decode(g, nb, 0);
+      const Task t = decode(g, nb, delay);
       if (variant == 3 && t.type == T_P1 && t.k >= 1) continue;  // inside F(k-1)
       if (variant == 3 && t.type == T_P3 && t.i == t.k + 1 && t.j == t.k + 1)
         v.push_back(make_int4(T_P3P1, t.k, t.i, t.j));
@@ -449,13 +449,13 @@ static long long small_flag_bytes(int nb) {
   return ((2 + (long long)nb * nb + 2 + 4ll * nb + 2ll * nb) * 4 + 15) / 16 * 16;
 }
 
-long long fw_small_work_bytes(int nb, size_t elem) {
-  return small_pbuf_bytes(nb, elem) + small_flag_bytes(nb) + small_queue(nb, nullptr) * (long long)sizeof(int4);
+long long fw_small_work_bytes(int nb, size_t elem) {  // the queue is at most nb^3 entries
+  return small_pbuf_bytes(nb, elem) + small_flag_bytes(nb) + (long long)nb * nb * nb * (long long)sizeof(int4);
 }
 
 template <typename T>
-cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag, bool queue_loaded, int ctas_per_sm,
-                            cudaStream_t s) {
+cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag, long long delay, bool queue_loaded,
+                            int ctas_per_sm, cudaStream_t s) {
   if (nb <= 0) return cudaSuccess;
   int dev = 0, sms = 0;
   cudaError_t e;
@@ -482,12 +482,12 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
   a.queue = dq;
   if (!queue_loaded) {
     std::vector<int4> q;
-    a.total = small_queue(nb, &q);
+    a.total = small_queue(nb, delay, &q);
     if ((e = cudaMemcpyAsync(dq, q.data(), q.size() * sizeof(int4), cudaMemcpyHostToDevice, s)) != cudaSuccess)
       return e;
     if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return e;  // q is a local
   } else {
-    a.total = small_queue(nb, nullptr);
+    a.total = small_queue(nb, delay, nullptr);
   }
   if ((e = cudaMemsetAsync(a.counter, 0, small_flag_bytes(nb), s)) != cudaSuccess) return e;
   // persistent grid: every CTA must be resident (tasks wait on each other)
@@ -501,7 +501,7 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
   return cudaGetLastError();
 }
 
-template cudaError_t launch_fw_small<int>(int*, long long, int, void*, int*, bool, int, cudaStream_t);
-template cudaError_t launch_fw_small<float>(float*, long long, int, void*, int*, bool, int, cudaStream_t);
+template cudaError_t launch_fw_small<int>(int*, long long, int, void*, int*, long long, bool, int, cudaStream_t);
+template cudaError_t launch_fw_small<float>(float*, long long, int, void*, int*, long long, bool, int, cudaStream_t);
 
 }  // namespace apsp

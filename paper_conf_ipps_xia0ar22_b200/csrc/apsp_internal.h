@@ -12,6 +12,8 @@ namespace apsp {
 
 // n_pad up to which APSP_SCHED_AUTO picks the 64-tile small-n kernel (apsp_fw_small.cu)
 constexpr long long kSmallAutoMaxN = 2048;
+// its default queue delay (dataflow_delay = 0): G3R(k-1) tasks queued before round k's panels
+constexpr long long kSmallDelay = 0;
 
 // NVTX range for the duration of a scope (C-ABI entry points, out-of-core
 // super-rounds): shows up in Nsight timelines and `ncu --nvtx` filters; a

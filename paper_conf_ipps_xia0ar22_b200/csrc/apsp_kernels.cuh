@@ -145,11 +145,11 @@ cudaError_t launch_fw_dataflow_sharded(const DFShard* ranks, int nv, int P, int 
 // `work` holds fw_small_work_bytes(nb, elem) bytes (panel copies + flags, zeroed here, + the task
 // queue, uploaded when !queue_loaded).
 template <typename T>
-cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag, bool queue_loaded, int ctas_per_sm,
-                            cudaStream_t s);
+cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag, long long delay, bool queue_loaded,
+                            int ctas_per_sm, cudaStream_t s);
 long long fw_small_work_bytes(int nb, size_t elem);
 // its task queue (host-built, critical path first; type 4 = fused P3(k; k+1,k+1) + P1(k+1))
-long long small_queue(int nb, std::vector<int4>* q);
+long long small_queue(int nb, long long delay, std::vector<int4>* q);
 
 // The packed int16 closure (R16) as one persistent dataflow launch
 // (apsp_fw_dataflow16.cu); `work` holds fw_dataflow16_work_bytes(nb) bytes.

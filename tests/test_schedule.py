@@ -150,16 +150,17 @@ def expand_fused(q):
             yield (typ, k, i, j)
 
 
-@pytest.mark.parametrize("nb", [1, 2, 3, 4, 5, 8, 16, 23, 32])
-def test_small_kernel_queue_complete_and_deadlock_free(lib, nb):
+@pytest.mark.parametrize("nb,delay", [(1, 0), (2, 0), (3, 0), (4, 2), (5, 0), (8, 7), (16, 0), (16, 40), (23, 5),
+                                      (32, 0), (32, 1000)])
+def test_small_kernel_queue_complete_and_deadlock_free(lib, nb, delay):
     """The 64-tile small-n kernel's host-built queue (apsp_fw_small.cu: the 128-tile kernel's segment
     order with F(k) = P3(k; k+1,k+1) fused with P1(k+1)): every blocked-FW task once, and an
     in-order drain with the kernel's exact waits (a fused entry waits for both halves' dependencies)."""
-    q = lib.apsp_debug_queue(nb, -1, 0, 0)
+    q = lib.apsp_debug_queue(nb, -1, 0, delay)
     assert sorted(expand_fused(q)) == sorted(expected_tasks(nb))
     assert len(q) == nb ** 3 - (nb - 1)
     assert simulate(nb, [q])
-    if nb >= 2:  # round 0's panel tiles right after P1(0), then F(0) (the next diagonal tile) first
+    if nb >= 2 and delay == 0:  # round 0's panel tiles right after P1(0), then F(0) (the next diagonal tile) first
         assert sorted(tuple(x) for x in q[1:2 * nb - 1].tolist()) == sorted(
             t for t in expected_tasks(nb) if t[1] == 0 and t[0] in (P2R, P2C))
         assert tuple(q[2 * nb - 1].tolist()) == (P3P1, 0, 1, 1)

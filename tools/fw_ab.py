@@ -26,6 +26,7 @@ def main():
     ap.add_argument("--runs", type=int, default=2)
     ap.add_argument("--modes", nargs="+", default=["dataflow", "per_phase"])
     ap.add_argument("--packed16", action="store_true", help="int32 input solved on the packed int16 path")
+    ap.add_argument("--delay", type=int, default=0, help="apsp_config.dataflow_delay (0 = auto)")
     a = ap.parse_args()
     g = gg.erdos_renyi(a.n, a.deg * a.n, seed=4, dtype=a.dtype)
     out = {"n": a.n, "deg": a.deg, "dtype": a.dtype, "packed16": a.packed16}
@@ -34,6 +35,7 @@ def main():
             continue
         cfg = apsp.apsp_config_default(device=0, timing=1, packed16=int(a.packed16))
         cfg.schedule = legacy
+        cfg.dataflow_delay = a.delay
         with apsp.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=cfg) as h:
             best, best_dev = 1e30, 1e30
             for r in range(a.runs + 1):
