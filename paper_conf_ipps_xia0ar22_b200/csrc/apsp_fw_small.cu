@@ -47,6 +47,7 @@
 #include <cuda_runtime.h>
 #include <algorithm>
 #include <cstdint>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <vector>
@@ -84,6 +85,7 @@ struct SmArgs {
   int* negflag;
   long long total;   // queue entries
   const int4* queue; // [total] (type, k, i, j), built on the host (small_queue)
+  unsigned long long* prof;  // optional [CTAs][16] cycle counters (tuning: APSP_SMALL_PROFILE)
 };
 
 template <typename T>
@@ -313,6 +315,10 @@ __global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ S
     slot[1].ready = 0;
   }
   __syncthreads();
+  // thread 0's cycle counters (a.prof): [0] dependency waits, [1 + type] task bodies, [6 + type]
+  // task counts, [11] publication
+  unsigned long long pr[12] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
+  long long c0 = clock64();
   for (int it = 0;; ++it) {
     SmSlot& S = slot[it & 1];
     SmSlot& N = slot[(it + 1) & 1];
@@ -322,6 +328,11 @@ __global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ S
     if (tid == 0) {
       if (!S.ready)
         while (!small_deps(a, tk)) __nanosleep(32);
+      if (a.prof) {
+        const long long c1 = clock64();
+        pr[0] += c1 - c0;
+        c0 = c1;
+      }
       // N's entry and the next queue index: issued now, consumed after this task's work, so
       // their latency hides under it
       if (N.t < a.total) nq = a.queue[N.t];
@@ -333,13 +344,26 @@ __global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ S
     if (tid == 0 && N.t < a.total) N.tk = small_task(nq);
     __syncthreads();  // every thread's stores of this task are issued; As / Bs free; N.tk published
     if (tid == 0) {
+      if (a.prof) {
+        const long long c1 = clock64();
+        pr[1 + tk.type] += c1 - c0;
+        pr[6 + tk.type] += 1;
+        c0 = c1;
+      }
       small_signal(a, tk);
       // the next task's flags, once: if met, it starts without another wait
       N.ready = N.t < a.total && small_deps(a, N.tk);
       S.t = idx_next;  // this slot becomes the one after N (read by the others only after the
       S.ready = 0;     // next iteration's first barrier)
+      if (a.prof) {
+        const long long c1 = clock64();
+        pr[11] += c1 - c0;
+        c0 = c1;
+      }
     }
   }
+  if (a.prof && tid == 0)
+    for (int x = 0; x < 12; ++x) a.prof[(long long)blockIdx.x * 16 + x] = pr[x];
 }
 
 }  // namespace
@@ -497,8 +521,26 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
   const int per_sm = ctas_per_sm < 1 ? 1 : (ctas_per_sm > occ ? occ : ctas_per_sm);
   long long grid = (long long)sms * per_sm;
   if (grid > a.total) grid = a.total;
+  // APSP_SMALL_PROFILE=1 (tuning only): per-CTA cycle counters, summarised on stderr
+  const bool prof = getenv("APSP_SMALL_PROFILE") != nullptr;
+  if (prof && (e = cudaMalloc(&a.prof, grid * 16 * sizeof(unsigned long long))) != cudaSuccess) return e;
+  if (prof && (e = cudaMemsetAsync(a.prof, 0, grid * 16 * sizeof(unsigned long long), s)) != cudaSuccess) return e;
   fw_small_kernel<T><<<(unsigned)grid, SNT, 0, s>>>(a);
-  return cudaGetLastError();
+  if ((e = cudaGetLastError()) != cudaSuccess || !prof) return e;
+  std::vector<unsigned long long> hp(grid * 16);
+  cudaStreamSynchronize(s);
+  cudaMemcpy(hp.data(), a.prof, hp.size() * 8, cudaMemcpyDeviceToHost);
+  cudaFree(a.prof);
+  double t[12] = {0};
+  for (long long b = 0; b < grid; ++b)
+    for (int x = 0; x < 12; ++x) t[x] += (double)hp[b * 16 + x];
+  const double all = t[0] + t[1] + t[2] + t[3] + t[4] + t[5] + t[11];
+  fprintf(stderr, "[small] CTAs %lld: wait %.1f%% sig %.1f%% | per task (cycles): P1 %.0f P2R %.0f P2C %.0f P3 %.0f F %.0f"
+                  " | counts %.0f %.0f %.0f %.0f %.0f | kernel cycles/CTA %.0f\n",
+          grid, 100 * t[0] / all, 100 * t[11] / all, t[1] / std::max(1.0, t[6]), t[2] / std::max(1.0, t[7]),
+          t[3] / std::max(1.0, t[8]), t[4] / std::max(1.0, t[9]), t[5] / std::max(1.0, t[10]), t[6], t[7], t[8], t[9],
+          t[10], all / grid);
+  return cudaSuccess;
 }
 
 template cudaError_t launch_fw_small<int>(int*, long long, int, void*, int*, long long, bool, int, cudaStream_t);

@@ -277,3 +277,21 @@ def test_boundary_out_of_core_config2_certified(lib):
         for r0 in range(0, g.n, 4096):
             rows = lib.apsp_get_dist(h, r0, 4096)
             assert oracle.certify_rows_i32(g.row_ptr, g.col, g.w, r0, rows, INF32) == (0, -1), r0
+
+
+@pytest.mark.gpu
+@pytest.mark.slow
+def test_boundary_out_of_core_config5_certified(lib):
+    """Config 5 (n = 262144, the 275 GB result exceeds the device) with k = sqrt(n)/4 = 128 grid
+    components: the out-of-core boundary algorithm streams the block rows that do not fit
+    (P:184-197), and EVERY row is proven exact by the oracle's optimality certificate."""
+    g = gg.baseline_config("cfg5_grid262144")
+    comp, k = gg.grid_block_partition(g, 16, 8)
+    assert k == 128
+    with lib.apsp_init_boundary(g.n, g.row_ptr, g.col, g.w, comp, k, cfg=lib.apsp_config_default(device=0)) as h:
+        info = lib.apsp_get_info(h)
+        assert info.ooc_block > 0 and info.host_bytes > 0  # out of core, some block rows streamed
+        lib.apsp_solve(h)
+        for r0 in range(0, g.n, 8192):
+            rows = lib.apsp_get_dist(h, r0, 8192)
+            assert oracle.certify_rows_i32(g.row_ptr, g.col, g.w, r0, rows, INF32) == (0, -1), r0
