@@ -201,6 +201,163 @@ __host__ __device__ Task decode(long long g, int nb, long long delay) {
   return g3l_task(nb, k, g - 1);
 }
 
+// ---- two-round ("pair") schedule of the single-GPU int32 / fp32 kernel ---------------------
+// Rounds are paired (k, k+1), k even. Every tile (i, j) with i, j not in {k, k+1} gets BOTH
+// rounds' phase-3 updates in ONE task (T_PAIR: depth 256, the C tile read and written once per
+// two rounds); the tiles on rows / columns k and k+1 stay single-round tasks. Panel copies are
+// kept for four rounds (parity k % 4), so round k+2's and k+3's panels can be computed while
+// the pairs of (k, k+1) still read theirs. Queue, segment p (k = 2p):
+//   PRL(k-2)  pairs of (k-2, k-1) on rows / columns k and k+1: (k,k) first, then P1(k)
+//   PRB(k-2)  the other pairs of (k-2, k-1) (banded), the first `delay` of them here
+//   G2(k), G3L(k)[(k+1,k+1)], P1(k+1), G3L(k)[rest], G2(k+1), G3K(k+1), PRB(k-2)[delay:]
+// where G3L(k) = round k on row / column k+1 and G3K(k+1) = round k+1 on row / column k.
+// Segment 0 has no PRL / PRB; after the last pair, the tail is its PR (even nb) or, for odd
+// nb, a last single round k = nb-1 (segment [PRL(k-2) with P1(k), PRB, G2(k)] + its phase 3).
+// Every dependency of an entry lies earlier in the queue (tests/test_schedule.py).
+enum { T_PAIR = 5 };
+
+// x-th value of [0, nb) without the (distinct, any order, -1 = none) values e[0..3]
+__host__ __device__ __forceinline__ int skip4(int x, int e0, int e1, int e2, int e3) {
+  int e[4] = {e0, e1, e2, e3};
+  for (int a = 0; a < 4; ++a)  // sort ascending, -1 last
+    for (int b = a + 1; b < 4; ++b) {
+      const bool swap = (e[b] >= 0 && (e[a] < 0 || e[b] < e[a]));
+      if (swap) { const int t = e[a]; e[a] = e[b]; e[b] = t; }
+    }
+  for (int a = 0; a < 4; ++a)
+    if (e[a] >= 0 && x >= e[a]) ++x;
+  return x;
+}
+
+// G3K(k1): round k1 = k+1 on row / column k = k1-1 (tiles (k, j), j != k1; (i, k), i not in {k, k1})
+__host__ __device__ __forceinline__ Task g3k_task(int nb, int k1, long long x) {
+  Task t;
+  t.type = T_P3; t.k = k1;
+  const int k = k1 - 1;
+  if (x < nb - 1) { t.i = k; t.j = skip3((int)x, k1, -1, -1); return t; }
+  x -= nb - 1;
+  t.i = skip3((int)x, k, k1, -1); t.j = k;
+  return t;
+}
+
+// PRL(kp): pairs of (kp, kp+1) on rows / columns L = {k, k+1} < nb (k = kp+2), P1(k) second
+__host__ __device__ __forceinline__ Task prl_task(int nb, int kp, long long x) {
+  Task t;
+  const int k = kp + 2, k1 = k + 1;
+  t.type = T_PAIR; t.k = kp;
+  if (x == 0) { t.i = k; t.j = k; return t; }
+  if (x == 1) { t.type = T_P1; t.k = k; t.i = t.j = k; return t; }
+  x -= 2;
+  const int m = nb - 2;  // indices not in {kp, kp+1}
+  if (x < m - 1) { t.i = k; t.j = skip4((int)x, kp, kp + 1, k, -1); return t; }      // row k
+  x -= m - 1;
+  if (x < m - 1) { t.i = skip4((int)x, kp, kp + 1, k, -1); t.j = k; return t; }      // column k
+  x -= m - 1;
+  if (x < m - 1) { t.i = k1; t.j = skip4((int)x, kp, kp + 1, k, -1); return t; }     // row k+1
+  x -= m - 1;
+  t.i = skip4((int)x, kp, kp + 1, k, k1); t.j = k1;                                  // column k+1
+  return t;
+}
+
+__host__ __device__ __forceinline__ long long pair_prl_size(int nb, int k) {  // PRL(k-2), incl. P1(k)
+  const long long m = nb - 2;
+  return (k + 1 < nb) ? 4 * m - 3 : 2 * m;
+}
+__host__ __device__ __forceinline__ long long pair_singles_size(int nb) { return 8ll * nb - 9; }
+__host__ __device__ __forceinline__ long long pair_seg_size(int nb, int k) {  // segment of pair k/2, k >= 2
+  const long long m = nb - 2, c = (k + 1 < nb) ? 2 : 1;
+  return pair_prl_size(nb, k) + (m - c) * (m - c) + ((k + 1 < nb) ? pair_singles_size(nb) : 2ll * nb - 2);
+}
+__host__ __device__ __forceinline__ long long pair_total(int nb) {
+  if (nb == 1) return 1;
+  const int np = nb / 2;  // pairs; odd nb: + the last single round k = nb - 1
+  long long t = 8ll * nb - 8;  // segment 0: P1(0) + the singles of rounds 0, 1
+  for (int p = 1; p < np; ++p) t += pair_seg_size(nb, 2 * p);
+  if (nb & 1) t += pair_seg_size(nb, nb - 1) + (long long)(nb - 1) * (nb - 1);
+  else t += (long long)(nb - 2) * (nb - 2);
+  return t;
+}
+
+// the singles of pair (k, k+1), k + 1 < nb: G2(k), G3L(k)[0], P1(k+1), G3L(k)[1:], G2(k+1), G3K(k+1)
+__host__ __device__ __forceinline__ Task pair_single(int nb, int k, long long x) {
+  const long long n2 = 2ll * (nb - 1), n3 = 2ll * nb - 3;
+  if (x < n2) return p2_task(nb, k, x);
+  x -= n2;
+  if (x == 0) return g3l_task(nb, k, 0);
+  if (x == 1) { Task t; t.type = T_P1; t.k = k + 1; t.i = t.j = k + 1; return t; }
+  x -= 2;
+  if (x < n3 - 1) return g3l_task(nb, k, x + 1);
+  x -= n3 - 1;
+  if (x < n2) return p2_task(nb, k + 1, x);
+  x -= n2;
+  return g3k_task(nb, k + 1, x);
+}
+
+// PRB(kp): pairs of (kp, kp+1) on tiles with i, j not in {kp, kp+1, kp+2, kp+3 (< nb)}, banded
+__host__ __device__ __forceinline__ Task prb_task(int nb, int kp, long long x) {
+  const int e3 = kp + 3 < nb ? kp + 3 : -1, e2 = kp + 2 < nb ? kp + 2 : -1;
+  const int w = nb - 2 - (e2 >= 0) - (e3 >= 0);
+  int r, c;
+  banded(x, w, w, r, c);
+  Task t;
+  t.type = T_PAIR; t.k = kp;
+  t.i = skip4(r, kp, kp + 1, e2, e3);
+  t.j = skip4(c, kp, kp + 1, e2, e3);
+  return t;
+}
+
+__host__ __device__ Task decode2(long long g, int nb, long long delay) {
+  Task t;
+  if (g == 0) { t.type = T_P1; t.k = 0; t.i = t.j = 0; return t; }
+  if (nb == 1) return t;
+  g -= 1;
+  const long long single = pair_singles_size(nb);
+  if (g < single) return pair_single(nb, 0, g);
+  g -= single;
+  const int np = nb / 2;
+  // middle segments p = 1 .. np-1 (k + 1 < nb) all have the same size
+  const long long sm = np >= 2 ? pair_seg_size(nb, 2) : 0;
+  const bool odd_tail = (nb & 1) != 0;
+  int k;
+  long long off;
+  if (np >= 2 && g < (long long)(np - 1) * sm) {
+    const int p = 1 + (int)(g / sm);
+    k = 2 * p;
+    off = g % sm;
+  } else {
+    g -= (long long)(np - 1) * sm;
+    if (!odd_tail) {  // tail: the pairs of (nb-2, nb-1) on the tiles not in {nb-2, nb-1}
+      const int kp = nb - 2, w = nb - 2;
+      int r, c;
+      banded(g, w, w, r, c);
+      t.type = T_PAIR; t.k = kp; t.i = r; t.j = c;  // i, j < nb - 2: no skip needed
+      return t;
+    }
+    k = nb - 1;  // odd nb: the last single round
+    const long long sl = pair_seg_size(nb, k);
+    if (g >= sl) {  // its phase 3, all (i, j) != k
+      g -= sl;
+      int r, c;
+      banded(g, nb - 1, nb - 1, r, c);
+      t.type = T_P3; t.k = k; t.i = r; t.j = c;  // k = nb - 1: no skip needed
+      return t;
+    }
+    off = g;
+  }
+  // segment of round k (k = 2p, or the odd last single round): PRL(k-2), PRB(k-2)[0:d], singles, PRB[d:]
+  const long long prl = pair_prl_size(nb, k);
+  if (off < prl) return prl_task(nb, k - 2, off);
+  off -= prl;
+  const long long m = nb - 2, c = (k + 1 < nb) ? 2 : 1, prb = (m - c) * (m - c);
+  const long long d = delay < prb ? delay : prb;
+  if (off < d) return prb_task(nb, k - 2, off);
+  off -= d;
+  const long long sing = (k + 1 < nb) ? single : 2ll * nb - 2;
+  if (off < sing) return (k + 1 < nb) ? pair_single(nb, k, off) : p2_task(nb, k, off);
+  off -= sing;
+  return prb_task(nb, k - 2, d + off);
+}
+
 // Dependency test and publication below work on any argument block with the
 // flag fields of DFArgs (nb, ver, diagready, rowready, colready, done2, done3).
 // Dependency test of task t (one thread): up to three flags, read with

@@ -1000,6 +1000,15 @@ long long fw_dataflow_work_bytes(int nb, size_t elem) { return fw_dataflow_work_
 // host. P = 0: the single-GPU queue (decode); P >= 1: rank q's sharded queue (decode_sh).
 extern "C" int64_t apsp_debug_queue(int32_t nb, int32_t P, int32_t q, int64_t delay, int32_t* out, int64_t cap) {
   using namespace apsp;
+  if (P == -2) {  // the two-round ("pair") queue of the single-GPU kernel (decode2)
+    if (nb <= 0) return -1;
+    const long long total = pair_total(nb);
+    for (long long g = 0; g < total && g < cap; ++g) {
+      const Task t = decode2(g, nb, delay);
+      out[4 * g] = t.type; out[4 * g + 1] = t.k; out[4 * g + 2] = t.i; out[4 * g + 3] = t.j;
+    }
+    return total;
+  }
   if (P == -1) {  // the small-n kernel's queue (apsp_fw_small.cu), nb 64-wide tile rows
     if (nb <= 0) return -1;
     std::vector<int4> sq;

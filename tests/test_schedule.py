@@ -10,7 +10,7 @@ import itertools
 import numpy as np
 import pytest
 
-P1, P2R, P2C, P3, P3P1 = 0, 1, 2, 3, 4
+P1, P2R, P2C, P3, P3P1, PAIR = 0, 1, 2, 3, 4, 5
 
 
 def expected_tasks(nb):
@@ -25,9 +25,10 @@ def expected_tasks(nb):
                 yield (P3, k, i, j)
 
 
-def simulate(nb, queues):
+def simulate(nb, queues, par=2):
     """queues[r]: array (total, 4) of rank r (P = len(queues); P = 1 single GPU). One worker
-    per rank, strictly in queue order; returns True iff every queue drains."""
+    per rank, strictly in queue order; returns True iff every queue drains. par: panel-copy
+    parities (2; 4 for the pair schedule, whose round k reuses round k-4's copies)."""
     P = len(queues)
     nl = nb // P
     owner = lambda row: row // nl  # noqa: E731
@@ -49,16 +50,18 @@ def simulate(nb, queues):
         typ, k, i, j = (int(x) for x in t)
         if typ == P3P1:  # fused P3(k; k+1,k+1) + P1(k+1) (small-n kernel)
             return (ready(r, (P3, k, i, j)) and
-                    (k + 1 < 2 or all(done2[x, k - 1] >= cnt2(x, k - 1) for x in range(P))))
+                    (k + 1 < par or all(done2[x, k + 1 - par] >= cnt2(x, k + 1 - par) for x in range(P))))
         if ver[i, j] < k:
             return False
+        if typ == PAIR:  # rounds k and k+1 on one tile (pair schedule)
+            return all((kk, j) in p2r_done and (kk, i) in p2c_done for kk in (k, k + 1))
         if typ == P3:
             return (k, j) in p2r_done and (k, i) in p2c_done
         if typ == P2C:
-            return k in p1_done and (k < 2 or done3[r, k - 2] >= cnt3(r, k - 2))
+            return k in p1_done and (k < par or done3[r, k - par] >= cnt3(r, k - par))
         if typ == P2R:
-            return k in p1_done and (k < 2 or all(done3[x, k - 2] >= cnt3(x, k - 2) for x in range(P)))
-        return k < 2 or all(done2[x, k - 2] >= cnt2(x, k - 2) for x in range(P))
+            return k in p1_done and (k < par or all(done3[x, k - par] >= cnt3(x, k - par) for x in range(P)))
+        return k < par or all(done2[x, k - par] >= cnt2(x, k - par) for x in range(P))
 
     pos = [0] * P
     total = sum(len(q) for q in queues)
@@ -73,6 +76,10 @@ def simulate(nb, queues):
                     ver[i, j] = k + 2
                     p1_done.add(k + 1)
                     done3[r, k] += 1
+                elif typ == PAIR:
+                    ver[i, j] = k + 2
+                    done3[r, k] += 1
+                    done3[r, k + 1] += 1
                 elif typ == P1:
                     p1_done.add(k)
                 elif typ == P2R:
@@ -146,6 +153,9 @@ def expand_fused(q):
         if typ == P3P1:
             yield (P3, k, i, j)
             yield (P1, k + 1, i, j)
+        elif typ == PAIR:
+            yield (P3, k, i, j)
+            yield (P3, k + 1, i, j)
         else:
             yield (typ, k, i, j)
 
@@ -172,3 +182,25 @@ def test_simulator_rejects_fused_entry_before_its_panels(lib):
     f = next(x for x, t in enumerate(q) if t[0] == P3P1 and t[1] == 0)
     q.insert(1, q.pop(f))
     assert not simulate(6, [np.array(q)])
+
+
+@pytest.mark.parametrize("nb,delay", [(1, 0), (2, 0), (3, 0), (4, 0), (5, 3), (6, 8), (7, 100), (8, 1184), (16, 40),
+                                      (33, 5), (70, 1184), (131, 592)])
+def test_pair_queue_complete_and_deadlock_free(lib, nb, delay):
+    """The single-GPU kernel's two-round schedule (decode2): tiles off rows / columns k, k+1 get
+    rounds k and k+1 in one task; panel copies are kept for 4 rounds. Every task of the blocked FW
+    exactly once and an in-order drain under the exact waits (4-parity reuse rule), including the
+    multi-band phase 3 (nb >= 67) and odd nb (a last single round)."""
+    q = lib.apsp_debug_queue(nb, -2, 0, delay)
+    assert sorted(expand_fused(q)) == sorted(expected_tasks(nb))
+    n_pairs = sum(1 for t in q.tolist() if t[0] == PAIR)
+    assert n_pairs == (nb // 2) * (nb - 2) ** 2 if nb >= 2 else n_pairs == 0
+    assert simulate(nb, [q], par=4)
+
+
+def test_pair_queue_needs_four_parities(lib):
+    """Pin of the parity rule: with only two panel-copy parities the pair queue cannot drain
+    (round k+2's panels would overwrite copies the pairs of (k, k+1) still read)."""
+    q = lib.apsp_debug_queue(12, -2, 0, 40)
+    assert simulate(12, [q], par=4)
+    assert not simulate(12, [q], par=2)
