@@ -340,7 +340,7 @@ template <typename T>
 static apsp_status run_dataflow_sharded(Handle* h) {
   const int nb = (int)(h->n_pad / h->b), P = h->world, nl = nb / P;
   const long long wb = fw_dataflow_work_bytes(nb, nl, sizeof(T));
-  const long long pbb = fw_dataflow_pbuf_bytes(nb, nl, sizeof(T)), fbb = fw_dataflow_flag_bytes(nb, nl);
+  const long long pbb = fw_dataflow_pbuf_bytes(nb, nl, sizeof(T), 2), fbb = fw_dataflow_flag_bytes(nb, nl);
   apsp_status st;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);

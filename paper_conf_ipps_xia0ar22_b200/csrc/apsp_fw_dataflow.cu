@@ -58,6 +58,7 @@
 
 #include <cuda_runtime.h>
 #include <climits>
+#include <cstdlib>
 #include <cstdint>
 #include <cstring>
 #include <vector>
@@ -70,6 +71,8 @@ namespace {
 #endif
 constexpr int BM = 128, BN = 128, BK = 32, GNT = 256, GROUPS = DF_GROUPS, STAGES = 3;
 constexpr int CTAS_PER_SM = 2 / GROUPS;  // two groups per SM either way
+// single GPU: the two-round (pair) queue by default (decode2)
+constexpr bool kPairDefault = true;
 // Stage = A chunk stored transposed, As[kk][r] (32 x 128), then B chunk
 // Bs[kk][c] (32 x 128): every operand read is one 16-byte vector per 4 rows or
 // columns (4 shared loads per 64 relaxations); a C half-tile (64 x 128) fits too.
@@ -125,16 +128,18 @@ struct DFArgs {
   // block and the row panel straight into every rank's pbuf (peer stores over NVLink) and
   // raises their flags; owners read every rank's done2/done3 before reusing a parity.
   int P, q, nl;
+  int npar;   // panel-copy parities: 2 (sharded kernel), 4 (single GPU: the pair schedule needs them)
+  int pairq;  // single GPU: 1 = the two-round queue (decode2, T_PAIR tasks), 0 = decode
   const long long* segstart;  // [nb + 1] queue position of segment k (k = nb: the last round's phase 3)
   T* peer_pbuf[kMaxRanks];    // pbuf of every rank (peer_pbuf[q] == pbuf)
   int* peer_base[kMaxRanks];  // flag block of every rank (== its counter address)
 };
 
-// panel copies of round k (parity k % 2), 128x128 tiles with ld 128:
+// panel copies of round k (parity k % npar), 128x128 tiles with ld 128:
 //   D = A(k,k) closed, D^T, row panel A(k,j), column panel A(i,k) transposed
 template <typename T>
 __device__ __forceinline__ T* pb_diag(const DFArgs<T>& a, int k) {
-  return a.pbuf + (long long)(k & 1) * (2 + a.nb + a.nl) * TILE_ELEMS;
+  return a.pbuf + (long long)(k & (a.npar - 1)) * (2 + a.nb + a.nl) * TILE_ELEMS;
 }
 template <typename T>
 __device__ __forceinline__ T* pb_diagT(const DFArgs<T>& a, int k) {
@@ -309,6 +314,54 @@ __device__ void signal_done_sh(const DFArgs<T>& a, const Task& t) {
   }
 }
 
+// Single-GPU dependencies / publication with npar parities (the per-round panel copies of
+// round k are rewritten by round k + npar) and the pair task T_PAIR (rounds k, k+1 of one tile).
+template <typename T>
+__device__ bool deps_single(const DFArgs<T>& a, const Task& t) {
+  const int nb = a.nb, k = t.k, np = a.npar, p = k & (np - 1);
+  // up to five flags: independent relaxed loads first (one round trip), then the tests
+  const int* f0 = a.ver + (long long)t.i * nb + t.j;
+  const int* f1;
+  const int* f2;
+  const int* f3 = f0;
+  const int* f4 = f0;
+  int v1, v2, v3 = INT_MIN, v4 = INT_MIN;
+  if (t.type == T_P1) {
+    f1 = a.done2 + (k >= np ? k - np : 0); v1 = k >= np ? 2 * (nb - 1) : INT_MIN;
+    f2 = f1; v2 = v1;
+  } else if (t.type == T_P3 || t.type == T_PAIR) {
+    f1 = a.rowready + p * nb + t.j; v1 = k + 1;
+    f2 = a.colready + p * nb + t.i; v2 = k + 1;
+    if (t.type == T_PAIR) {
+      const int p1 = (k + 1) & (np - 1);
+      f3 = a.rowready + p1 * nb + t.j; v3 = k + 2;
+      f4 = a.colready + p1 * nb + t.i; v4 = k + 2;
+    }
+  } else {
+    f1 = a.diagready + p; v1 = k + 1;
+    f2 = a.done3 + (k >= np ? k - np : 0); v2 = k >= np ? (nb - 1) * (nb - 1) : INT_MIN;
+  }
+  const int x0 = ld_relaxed(f0), x1 = ld_relaxed(f1), x2 = ld_relaxed(f2), x3 = ld_relaxed(f3), x4 = ld_relaxed(f4);
+  if (x0 >= k && x1 >= v1 && x2 >= v2 && x3 >= v3 && x4 >= v4) {
+    asm volatile("fence.acquire.gpu;" ::: "memory");  // (see deps_met)
+    return true;
+  }
+  return false;
+}
+template <typename T>
+__device__ void signal_single(const DFArgs<T>& a, const Task& t) {
+  const int nb = a.nb, k = t.k, p = k & (a.npar - 1);
+  asm volatile("fence.release.gpu;" ::: "memory");
+  st_relaxed(a.ver + (long long)t.i * nb + t.j, t.type == T_PAIR ? k + 2 : k + 1);
+  switch (t.type) {
+    case T_P1: st_relaxed(a.diagready + p, k + 1); break;
+    case T_P2R: st_relaxed(a.rowready + p * nb + t.j, k + 1); red_relaxed_add(a.done2 + k, 1); break;
+    case T_P2C: st_relaxed(a.colready + p * nb + t.i, k + 1); red_relaxed_add(a.done2 + k, 1); break;
+    case T_PAIR: red_relaxed_add(a.done3 + k, 1); red_relaxed_add(a.done3 + k + 1, 1); break;
+    default: red_relaxed_add(a.done3 + k, 1); break;
+  }
+}
+
 template <bool SH, typename T>
 __device__ __forceinline__ Task decode_any(const DFArgs<T>& a, long long g) {
   // sharded: the segment starts are binary-searched in a shared-memory copy (the kernel
@@ -319,12 +372,12 @@ __device__ __forceinline__ Task decode_any(const DFArgs<T>& a, long long g) {
   if constexpr (SH)
     return decode_sh(g, a.nb, a.nl, a.q, a.delay,
                      reinterpret_cast<const long long*>(smem_raw + GROUPS * STAGES * STAGE_ELEMS * sizeof(T)));
-  else return decode(g, a.nb, a.delay);
+  else return a.pairq ? decode2(g, a.nb, a.delay) : decode(g, a.nb, a.delay);
 }
 template <bool SH, typename T>
 __device__ __forceinline__ bool deps_any(const DFArgs<T>& a, const Task& t) {
   if constexpr (SH) return deps_met_sh(a, t);
-  else return deps_met(a, t);
+  else return deps_single(a, t);
 }
 
 // Phase 1 inside a group: in-place FW closure of one 128x128 tile (the same
@@ -422,6 +475,9 @@ struct GDesc {
   T* Cout2;  // panel copy (ld 128) or nullptr; c2t = 1: written transposed
   int lda, ldb, ldc;
   int a_rows, c2t;
+  const T* A2;  // pair task: round k+1's operands (chunks 4..7), same layout as A / B
+  const T* B2;
+  int nk;    // chunks of depth 32: 4 (one round), 8 (pair task: rounds k and k+1)
   int bulk;  // 1: A and B chunks are contiguous 16 KB blocks (panel copies): one thread copies them
   int bcast; // sharded P2R: Cout2 also goes to every other rank's pbuf (same offset)
 };
@@ -445,7 +501,7 @@ __device__ void fill_desc(const DFArgs<T>& a, const Task& tk, GDesc<T>& d) {
   const int k = tk.k;
   T* const tile = a.D + (long long)(tk.i - a.q * a.nl) * BM * a.ld + (long long)tk.j * BN;
   d.Cin = tile; d.Cout = tile; d.ldc = (int)a.ld;
-  d.a_rows = 0; d.c2t = 0; d.bulk = 0; d.bcast = 0;
+  d.a_rows = 0; d.c2t = 0; d.bulk = 0; d.bcast = 0; d.nk = BM / BK; d.A2 = d.B2 = nullptr;
   if (tk.type == T_P2R) {         // A(k,j) = D (x) A(k,j)
     d.A = pb_diagT(a, k); d.lda = BM; d.B = tile; d.ldb = (int)a.ld; d.Cout2 = pb_row(a, k, tk.j);
     d.bcast = a.P > 1;
@@ -454,6 +510,9 @@ __device__ void fill_desc(const DFArgs<T>& a, const Task& tk, GDesc<T>& d) {
     d.Cout2 = pb_colT(a, k, tk.i); d.c2t = 1;
   } else {                        // A(i,j) = min(A(i,j), A(i,k) (x) A(k,j)) from the panel copies
     d.A = pb_colT(a, k, tk.i); d.lda = BM; d.B = pb_row(a, k, tk.j); d.ldb = BN; d.Cout2 = nullptr;
+    if (tk.type == T_PAIR) {      // then round k+1: min(., A(i,k+1) (x) A(k+1,j)) (min is order-free)
+      d.A2 = pb_colT(a, k + 1, tk.i); d.B2 = pb_row(a, k + 1, tk.j); d.nk = 2 * (BM / BK);
+    }
 #ifndef DF_NOBULK
     d.bulk = 1;
 #endif
@@ -479,7 +538,7 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
                                            int gtid, int g, const DFArgs<T>* args, long long nxt,
                                            Slot<T>* ns, int pref) {
   using V4 = typename DV<T>::V4;
-  constexpr int NK = BM / BK;  // 4 chunks of depth 32
+  const int NK = d->nk;  // 4 chunks of depth 32 (8 for a pair task)
   // fp32: fold the top half of C before the last chunk and issue the next phase-3 task's
   // chunk 0 into the freed stage (measured +1.2 % for fp32, -1.7 % for int32, so int32 keeps
   // the C fetch into both free stages during the last chunk and the fold at the end)
@@ -509,8 +568,11 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         const unsigned bytes = BK * BM * (unsigned)sizeof(T);
         mb_expect_tx(full0 + 8 * stage, 2 * bytes);
-        bulk_g2s(saddr(st), d->A + (long long)c * BK * BM, bytes, full0 + 8 * stage);
-        bulk_g2s(saddr(st + BK * ALD), d->B + (long long)c * BK * BN, bytes, full0 + 8 * stage);
+        const int cr = c & 3;  // chunk within its round (pair tasks: chunks 4..7 from round k+1)
+        const T* const Ar = c < 4 ? d->A : d->A2;
+        const T* const Br = c < 4 ? d->B : d->B2;
+        bulk_g2s(saddr(st), Ar + (long long)cr * BK * BM, bytes, full0 + 8 * stage);
+        bulk_g2s(saddr(st + BK * ALD), Br + (long long)cr * BK * BN, bytes, full0 + 8 * stage);
       }
       return;
     }
@@ -557,7 +619,9 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
   for (int i = 0; i < 8; ++i)
 #pragma unroll
     for (int j = 0; j < 8; ++j) acc[i][j] = DV<T>::inf();
-  const int s_lo = (int)((c0 + 1) % STAGES), s_hi = (int)((c0 + 2) % STAGES);
+  // the C tile goes to the stages of chunks c0+NK-3 and c0+NK-2 (free during the last chunk)
+  const unsigned g_lo = c0 + NK - 3, g_hi = c0 + NK - 2;
+  const int s_lo = (int)(g_lo % STAGES), s_hi = (int)(g_hi % STAGES);
 
 #pragma unroll 1
   for (int c = 0; c < NK; ++c) {
@@ -565,8 +629,8 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
     const int s = (int)(G % STAGES);
     if (!kXpref && c == NK - 1) {
       // C goes to the stages of chunks c0+1 and c0+2 once every warp released them
-      mb_wait(empty0 + 8 * s_lo, ((c0 + 1) / STAGES) & 1);
-      mb_wait(empty0 + 8 * s_hi, ((c0 + 2) / STAGES) & 1);
+      mb_wait(empty0 + 8 * s_lo, (g_lo / STAGES) & 1);
+      mb_wait(empty0 + 8 * s_hi, (g_hi / STAGES) & 1);
       const int ldc = d->ldc;
       const T* cg = d->Cin + (gtid >> 5) * ldc + (gtid & 31) * 4;
       const int cd = (gtid >> 5) * CLD + (gtid & 31) * 4;
@@ -578,14 +642,14 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
       for (int q = 0; q < 8; ++q) cp16(cs_hi + cd + q * 8 * CLD, cg + (64 + q * 8) * ldc);
       cp_commit();
     }
-    // fp32 (kXpref): C rows 0-63 go to stage s_lo as soon as chunk c0+1 released it (start of chunk c0+2),
+    // fp32 (kXpref): C rows 0-63 go to stage s_lo as soon as chunk g_lo released it (start of chunk NK-2),
     // rows 64-127 to s_hi at the start of the last chunk. The top half is folded into the
     // accumulators right before the last chunk (min is order-free), which frees s_lo for the
     // NEXT task's chunk 0 (stage of chunk c0+4): thread 0 issues it then, if that task is a
     // phase-3 task whose dependencies were seen met, so its latency hides under this chunk.
     if (kXpref && c >= NK - 2) {
       const int sC = c == NK - 2 ? s_lo : s_hi;
-      mb_wait(empty0 + 8 * sC, ((c0 + (c == NK - 2 ? 1 : 2)) / STAGES) & 1);
+      mb_wait(empty0 + 8 * sC, ((c == NK - 2 ? g_lo : g_hi) / STAGES) & 1);
       const int ldc = d->ldc;
       const T* cg = d->Cin + ((gtid >> 5) + (c == NK - 2 ? 0 : 64)) * (long long)ldc + (gtid & 31) * 4;
       const int cd = (gtid >> 5) * CLD + (gtid & 31) * 4;
@@ -620,7 +684,7 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
       gbar(g);  // s_lo read by every thread: free for the next task's chunk 0
       if (gtid == 0) {
         int pf = 0;
-        if (ns->t < args->total && ns->ready && ns->tk.type == T_P3 && ns->d.bulk) {
+        if (ns->t < args->total && ns->ready && (ns->tk.type == T_P3 || ns->tk.type == T_PAIR) && ns->d.bulk) {
           asm volatile("fence.proxy.async.global;" ::: "memory");  // acquired panel copies (see load_chunk)
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           const unsigned bytes = BK * BM * (unsigned)sizeof(T);
@@ -839,7 +903,7 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
       }
     } else {
       group_minplus<SH, T>(&S.d, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N, S.pref);
-      chunk += BM / BK;
+      chunk += S.d.nk;
     }
     const long long tc2 = clock64();
     pr[1] += tc2 - tc1;
@@ -850,7 +914,7 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
     // better than deferring it under the next task's first loads)
     if (gtid == SIG) {
       if constexpr (SH) signal_done_sh(a, tk);
-      else signal_done(a, tk);
+      else signal_single(a, tk);
     }
     tc0 = clock64();
     pr[2] += tc0 - tc2;
@@ -863,20 +927,21 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
 
 }  // namespace
 
-// Work-buffer layout of one rank: pbuf (2 parities x (2 + nb + nl) tiles), then the
-// flag block, then (sharded) the nb + 1 segment starts.
+// Work-buffer layout of one rank: pbuf (npar parities x (2 + nb + nl) tiles), then the
+// flag block (sized for 4 parities), then (sharded) the nb + 1 segment starts.
 template <typename T>
-static void df_layout(DFArgs<T>& a, void* work, int nb, int nl) {
+static void df_layout(DFArgs<T>& a, void* work, int nb, int nl, int npar) {
   a.nb = nb;
   a.nl = nl;
+  a.npar = npar;
   a.pbuf = static_cast<T*>(work);
-  char* const fb = static_cast<char*>(work) + fw_dataflow_pbuf_bytes(nb, nl, sizeof(T));
+  char* const fb = static_cast<char*>(work) + fw_dataflow_pbuf_bytes(nb, nl, sizeof(T), npar);
   int* f = reinterpret_cast<int*>(fb);
   a.counter = reinterpret_cast<unsigned long long*>(f); f += 2;  // first: 8-byte aligned
   a.ver = f; f += (long long)nl * nb;
-  a.diagready = f; f += 2;
-  a.rowready = f; f += 2 * nb;
-  a.colready = f; f += 2 * nl;
+  a.diagready = f; f += 4;
+  a.rowready = f; f += 4 * nb;
+  a.colready = f; f += 4 * nl;
   a.done2 = f; f += nb;
   a.done3 = f; f += nb;
   a.segstart = reinterpret_cast<const long long*>(fb + fw_dataflow_flag_bytes(nb, nl));
@@ -896,10 +961,13 @@ cudaError_t launch_fw_dataflow(T* D, long long ld, int nb, void* work, int* negf
   memset(&L, 0, sizeof(L));
   L.nv = 1;
   DFArgs<T>& a = L.r[0];
-  df_layout(a, work, nb, nb);
+  df_layout(a, work, nb, nb, 4);
   a.D = D; a.ld = ld;
   a.negflag = negflag;
-  a.total = (long long)nb * nb * nb;
+  // the two-round (pair) queue: APSP_DF_PAIR=0/1 overrides the default (tuning experiments)
+  a.pairq = kPairDefault && nb >= 4;
+  if (const char* e = getenv("APSP_DF_PAIR")) a.pairq = atoi(e) != 0 && nb >= 2;
+  a.total = a.pairq ? pair_total(nb) : (long long)nb * nb * nb;
   a.delay = delay;
   a.stagger = stagger;
   a.prof = prof;
@@ -948,7 +1016,8 @@ cudaError_t launch_fw_dataflow_sharded(const DFShard* ranks, int nv, int P, int 
   for (int v = 0; v < nv; ++v) {
     DFArgs<T>& a = L.r[v];
     const DFShard& sh = ranks[v];
-    df_layout(a, sh.work, nb, nl);
+    df_layout(a, sh.work, nb, nl, 2);
+    a.pairq = 0;
     a.D = static_cast<T*>(sh.D); a.ld = ld;
     a.negflag = negflag;
     a.P = P; a.q = sh.rank;
@@ -959,7 +1028,7 @@ cudaError_t launch_fw_dataflow_sharded(const DFShard* ranks, int nv, int P, int 
     for (int r = 0; r < P; ++r) {
       a.peer_pbuf[r] = static_cast<T*>(sh.peer_work[r]);
       a.peer_base[r] = reinterpret_cast<int*>(static_cast<char*>(sh.peer_work[r]) +
-                                              fw_dataflow_pbuf_bytes(nb, nl, sizeof(T)));
+                                              fw_dataflow_pbuf_bytes(nb, nl, sizeof(T), 2));
     }
     // blocking copy: `seg` is reused for the next rank (a few KB)
     if ((e = cudaMemcpyAsync(const_cast<long long*>(a.segstart), seg.data(), seg.size() * sizeof(long long),
@@ -981,18 +1050,20 @@ cudaError_t launch_fw_dataflow_sharded(const DFShard* ranks, int nv, int P, int 
   return cudaGetLastError();
 }
 
-long long fw_dataflow_pbuf_bytes(int nb, int nl, size_t elem) {
-  return 2ll * (2 + nb + nl) * TILE_ELEMS * (long long)elem;  // (kept a multiple of 8 bytes)
+long long fw_dataflow_pbuf_bytes(int nb, int nl, size_t elem, int npar) {
+  return (long long)npar * (2 + nb + nl) * TILE_ELEMS * (long long)elem;  // (kept a multiple of 8 bytes)
 }
-long long fw_dataflow_flag_bytes(int nb, int nl) {  // rounded to 16 B: the segment starts (int64) follow
-  return ((((long long)nl * nb + 4ll * nb + 2ll * nl + 4) * 4 + 15) / 16) * 16;
+long long fw_dataflow_flag_bytes(int nb, int nl) {  // 4 parities; rounded to 16 B: the segment starts follow
+  return ((((long long)nl * nb + 6ll * nb + 4ll * nl + 6) * 4 + 15) / 16) * 16;
 }
-long long fw_dataflow_work_bytes(int nb, int nl, size_t elem) {
-  return fw_dataflow_pbuf_bytes(nb, nl, elem) + fw_dataflow_flag_bytes(nb, nl) + 8ll * (nb + 1);
+long long fw_dataflow_work_bytes(int nb, int nl, size_t elem) {  // sharded kernel: 2 parities
+  return fw_dataflow_pbuf_bytes(nb, nl, elem, 2) + fw_dataflow_flag_bytes(nb, nl) + 8ll * (nb + 1);
 }
-long long fw_dataflow_pbuf_bytes(int nb, size_t elem) { return fw_dataflow_pbuf_bytes(nb, nb, elem); }
+long long fw_dataflow_pbuf_bytes(int nb, size_t elem) { return fw_dataflow_pbuf_bytes(nb, nb, elem, 4); }
 long long fw_dataflow_flag_bytes(int nb) { return fw_dataflow_flag_bytes(nb, nb); }
-long long fw_dataflow_work_bytes(int nb, size_t elem) { return fw_dataflow_work_bytes(nb, nb, elem); }
+long long fw_dataflow_work_bytes(int nb, size_t elem) {  // single GPU: 4 parities (pair schedule)
+  return fw_dataflow_pbuf_bytes(nb, nb, elem, 4) + fw_dataflow_flag_bytes(nb, nb) + 8ll * (nb + 1);
+}
 
 }  // namespace apsp
 

@@ -118,7 +118,7 @@ cudaError_t launch_fw_dataflow(T* D, long long ld, int nb, void* work, int* negf
 long long fw_dataflow_pbuf_bytes(int nb, size_t elem);
 long long fw_dataflow_flag_bytes(int nb);
 long long fw_dataflow_work_bytes(int nb, size_t elem);
-long long fw_dataflow_pbuf_bytes(int nb, int nl, size_t elem);
+long long fw_dataflow_pbuf_bytes(int nb, int nl, size_t elem, int npar);
 long long fw_dataflow_flag_bytes(int nb, int nl);
 
 // The same kernel over a 1-D block-row shard (rank q of P owns tile rows

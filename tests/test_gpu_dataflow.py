@@ -107,3 +107,21 @@ def test_dataflow_banded_phase3_order_partial_band(lib):
     srcs = np.array([0, 4500, g.n - 1])
     want = oracle.dijkstra_rows_i64(g.row_ptr, g.col, g.w, srcs)
     assert np.array_equal(a[srcs].astype(np.int64), np.where(want == oracle.INF_I64, INF32, want))
+
+
+@pytest.mark.parametrize("n", [300, 512, 640, 1000, 1152, 2560, 8960])
+def test_pair_schedule_equals_single_round_schedule(lib, monkeypatch, n):
+    """The two-round (pair) queue (decode2: rounds k, k+1 of a tile in one depth-256 task, panel
+    copies kept for 4 rounds; the single-GPU default) against the one-round queue: bit-identical
+    for int32 and fp32 (every candidate sum is the same RN add of the same panel operands; min is
+    exact), and int32 equal to the oracle. Odd and even tile counts, nb >= 67 (multi-band)."""
+    g = gg.erdos_renyi(n, 5 * n, seed=n + 2)
+    gf = gg.erdos_renyi(n, 5 * n, seed=n + 3, dtype="f32")
+    out = {}
+    for pair in ("0", "1"):
+        monkeypatch.setenv("APSP_DF_PAIR", pair)
+        out[pair] = (run(lib, g), run(lib, gf))
+    assert np.array_equal(out["1"][0], out["0"][0])
+    assert np.array_equal(out["1"][1].view(np.int32), out["0"][1].view(np.int32))
+    if n <= 2560:
+        assert np.array_equal(out["1"][0].astype(np.int64), want_i32(g))
