@@ -292,10 +292,10 @@ static apsp_status run_dataflow(Handle* h) {
   const int nb = (int)(h->n_pad / h->b);
   apsp_status st;
   if (!h->df_work) {
-    if ((st = h->cuda(cudaMallocAsync(&h->df_work, fw_dataflow_work_bytes(nb, sizeof(T)), h->stream),
-                      "cudaMalloc dataflow")))
-      return st;
-    h->device_bytes += fw_dataflow_work_bytes(nb, sizeof(T));
+    long long wb = fw_dataflow_work_bytes(nb, sizeof(T));
+    if (getenv("APSP_DF_WORK2")) wb = fw_dataflow_work_bytes(nb, nb, sizeof(T));  // A/B: 2-parity size
+    if ((st = h->cuda(cudaMallocAsync(&h->df_work, wb, h->stream), "cudaMalloc dataflow"))) return st;
+    h->device_bytes += wb;
   }
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);

@@ -71,8 +71,11 @@ namespace {
 #endif
 constexpr int BM = 128, BN = 128, BK = 32, GNT = 256, GROUPS = DF_GROUPS, STAGES = 3;
 constexpr int CTAS_PER_SM = 2 / GROUPS;  // two groups per SM either way
-// single GPU: the two-round (pair) queue by default (decode2)
+// single GPU: the two-round (pair) queue by default for int32 from nb = kPairMinNb tile rows
+// (decode2). Measured against the one-round kernel (profiles/r02_pair_ab.txt): nb = 128 -1.8 %,
+// nb = 256 +0.1 %, nb = 512 (config 3) +0.8 %; fp32 nb = 256 -0.8 % (one-round kept)
 constexpr bool kPairDefault = true;
+constexpr int kPairMinNb = 384;
 // Stage = A chunk stored transposed, As[kk][r] (32 x 128), then B chunk
 // Bs[kk][c] (32 x 128): every operand read is one 16-byte vector per 4 rows or
 // columns (4 shared loads per 64 relaxations); a C half-tile (64 x 128) fits too.
@@ -362,7 +365,7 @@ __device__ void signal_single(const DFArgs<T>& a, const Task& t) {
   }
 }
 
-template <bool SH, typename T>
+template <bool SH, bool PQ, typename T>
 __device__ __forceinline__ Task decode_any(const DFArgs<T>& a, long long g) {
   // sharded: the segment starts are binary-searched in a shared-memory copy (the kernel
   // fills it after its stages): from global memory the ~log2(nb) dependent loads went to
@@ -372,14 +375,15 @@ __device__ __forceinline__ Task decode_any(const DFArgs<T>& a, long long g) {
   if constexpr (SH)
     return decode_sh(g, a.nb, a.nl, a.q, a.delay,
                      reinterpret_cast<const long long*>(smem_raw + GROUPS * STAGES * STAGE_ELEMS * sizeof(T)));
-  else return a.pairq ? decode2(g, a.nb, a.delay) : decode(g, a.nb, a.delay);
+  else if constexpr (PQ) return decode2(g, a.nb, a.delay);  // the two-round queue
+  else return decode(g, a.nb, a.delay);
 }
-template <bool SH, typename T>
+template <bool SH, bool PQ, typename T>
 __device__ __forceinline__ bool deps_any(const DFArgs<T>& a, const Task& t) {
   if constexpr (SH) return deps_met_sh(a, t);
-  else return deps_single(a, t);
+  else if constexpr (PQ) return deps_single(a, t);  // 4 parities, T_PAIR
+  else return deps_met(a, t);
 }
-
 // Phase 1 inside a group: in-place FW closure of one 128x128 tile (the same
 // register blocking as phase1_kernel in apsp_kernels.cu); result also to out2.
 // Sharded kernel: `peers` (npeer entries) also receive D at the same offset (peer stores).
@@ -475,11 +479,17 @@ struct GDesc {
   T* Cout2;  // panel copy (ld 128) or nullptr; c2t = 1: written transposed
   int lda, ldb, ldc;
   int a_rows, c2t;
-  const T* A2;  // pair task: round k+1's operands (chunks 4..7), same layout as A / B
-  const T* B2;
-  int nk;    // chunks of depth 32: 4 (one round), 8 (pair task: rounds k and k+1)
   int bulk;  // 1: A and B chunks are contiguous 16 KB blocks (panel copies): one thread copies them
   int bcast; // sharded P2R: Cout2 also goes to every other rank's pbuf (same offset)
+};
+
+// The second round of a pair task (kept out of GDesc: the engine's shared-memory descriptor
+// layout is performance-sensitive, measured -2 % when these fields sat inside it)
+template <typename T>
+struct GPair {
+  const T* A2;  // round k+1's operands (chunks 4..7), same layout as GDesc::A / B
+  const T* B2;
+  int nk;       // chunks of depth 32: 4 (one round), 8 (pair task: rounds k and k+1)
 };
 
 
@@ -487,7 +497,7 @@ struct GDesc {
 // the task index, its decoded form, the operands of a min-plus task and
 // whether its dependencies were already seen met. Thread 0 fills the slot of
 // the next iteration while the current task runs.
-template <typename T>
+template <typename T, bool PQ>
 struct Slot {
   long long t;
   Task tk;
@@ -495,13 +505,30 @@ struct Slot {
   int ready;
   int pref;  // fp32: chunk 0 already issued by the previous task (during its last chunk)
 };
+template <typename T>
+struct Slot<T, true> {  // the pair kernel's slot: + the second round of a pair task
+  long long t;
+  Task tk;
+  GDesc<T> d;
+  int ready;
+  int pref;
+  GPair<T> p2;
+};
+
+// the pair data of a slot (nullptr in the one-round kernels)
+template <typename T>
+__device__ __forceinline__ GPair<T>* slot_p2(Slot<T, true>* s) { return &s->p2; }
+template <typename T>
+__device__ __forceinline__ GPair<T>* slot_p2(Slot<T, false>*) { return nullptr; }
+
 
 template <typename T>
-__device__ void fill_desc(const DFArgs<T>& a, const Task& tk, GDesc<T>& d) {
+__device__ void fill_desc(const DFArgs<T>& a, const Task& tk, GDesc<T>& d, GPair<T>* p2 = nullptr) {
   const int k = tk.k;
   T* const tile = a.D + (long long)(tk.i - a.q * a.nl) * BM * a.ld + (long long)tk.j * BN;
   d.Cin = tile; d.Cout = tile; d.ldc = (int)a.ld;
-  d.a_rows = 0; d.c2t = 0; d.bulk = 0; d.bcast = 0; d.nk = BM / BK; d.A2 = d.B2 = nullptr;
+  d.a_rows = 0; d.c2t = 0; d.bulk = 0; d.bcast = 0;
+  if (p2) p2->nk = BM / BK;
   if (tk.type == T_P2R) {         // A(k,j) = D (x) A(k,j)
     d.A = pb_diagT(a, k); d.lda = BM; d.B = tile; d.ldb = (int)a.ld; d.Cout2 = pb_row(a, k, tk.j);
     d.bcast = a.P > 1;
@@ -510,8 +537,8 @@ __device__ void fill_desc(const DFArgs<T>& a, const Task& tk, GDesc<T>& d) {
     d.Cout2 = pb_colT(a, k, tk.i); d.c2t = 1;
   } else {                        // A(i,j) = min(A(i,j), A(i,k) (x) A(k,j)) from the panel copies
     d.A = pb_colT(a, k, tk.i); d.lda = BM; d.B = pb_row(a, k, tk.j); d.ldb = BN; d.Cout2 = nullptr;
-    if (tk.type == T_PAIR) {      // then round k+1: min(., A(i,k+1) (x) A(k+1,j)) (min is order-free)
-      d.A2 = pb_colT(a, k + 1, tk.i); d.B2 = pb_row(a, k + 1, tk.j); d.nk = 2 * (BM / BK);
+    if (p2 && tk.type == T_PAIR) {  // then round k+1: min(., A(i,k+1) (x) A(k+1,j)) (min is order-free)
+      p2->A2 = pb_colT(a, k + 1, tk.i); p2->B2 = pb_row(a, k + 1, tk.j); p2->nk = 2 * (BM / BK);
     }
 #ifndef DF_NOBULK
     d.bulk = 1;
@@ -533,12 +560,13 @@ __device__ void fill_desc(const DFArgs<T>& a, const Task& tk, GDesc<T>& d) {
 #else
 #define DF_MP_INLINE __noinline__
 #endif
-template <bool SH, typename T>
-__device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigned full0, unsigned empty0, unsigned c0,
+template <bool SH, bool PQ, typename T, int NK>
+__device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, const GPair<T>* p2, T* stage0, unsigned full0,
+                                           unsigned empty0, unsigned c0,
                                            int gtid, int g, const DFArgs<T>* args, long long nxt,
-                                           Slot<T>* ns, int pref) {
+                                           Slot<T, PQ>* ns, int pref) {
   using V4 = typename DV<T>::V4;
-  const int NK = d->nk;  // 4 chunks of depth 32 (8 for a pair task)
+  // NK = 4 chunks of depth 32 (one round), 8 for a pair task (compile-time: two instantiations)
   // fp32: fold the top half of C before the last chunk and issue the next phase-3 task's
   // chunk 0 into the freed stage (measured +1.2 % for fp32, -1.7 % for int32, so int32 keeps
   // the C fetch into both free stages during the last chunk and the fold at the end)
@@ -569,8 +597,8 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
         const unsigned bytes = BK * BM * (unsigned)sizeof(T);
         mb_expect_tx(full0 + 8 * stage, 2 * bytes);
         const int cr = c & 3;  // chunk within its round (pair tasks: chunks 4..7 from round k+1)
-        const T* const Ar = c < 4 ? d->A : d->A2;
-        const T* const Br = c < 4 ? d->B : d->B2;
+        const T* const Ar = (NK == 4 || c < 4) ? d->A : p2->A2;
+        const T* const Br = (NK == 4 || c < 4) ? d->B : p2->B2;
         bulk_g2s(saddr(st), Ar + (long long)cr * BK * BM, bytes, full0 + 8 * stage);
         bulk_g2s(saddr(st + BK * ALD), Br + (long long)cr * BK * BN, bytes, full0 + 8 * stage);
       }
@@ -661,10 +689,10 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
     if (c == 1 && gtid == SCH) {  // the next task's slot
       ns->t = nxt;
       if (nxt < args->total) {
-        const Task tn = decode_any<SH>(*args, nxt);
+        const Task tn = decode_any<SH, PQ>(*args, nxt);
         ns->tk = tn;
-        if (tn.type != T_P1) fill_desc(*args, tn, ns->d);
-        ns->ready = deps_any<SH>(*args, tn) ? 1 : 0;
+        if (tn.type != T_P1) fill_desc(*args, tn, ns->d, slot_p2(ns));
+        ns->ready = deps_any<SH, PQ>(*args, tn) ? 1 : 0;
       }
     }
     if (kXpref && c == NK - 1) {
@@ -684,7 +712,8 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, T* stage0, unsigne
       gbar(g);  // s_lo read by every thread: free for the next task's chunk 0
       if (gtid == 0) {
         int pf = 0;
-        if (ns->t < args->total && ns->ready && (ns->tk.type == T_P3 || ns->tk.type == T_PAIR) && ns->d.bulk) {
+        if (ns->t < args->total && ns->ready && (ns->tk.type == T_P3 || (PQ && ns->tk.type == T_PAIR)) &&
+            ns->d.bulk) {
           asm volatile("fence.proxy.async.global;" ::: "memory");  // acquired panel copies (see load_chunk)
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
           const unsigned bytes = BK * BM * (unsigned)sizeof(T);
@@ -818,11 +847,14 @@ struct DFLaunch {
   int nv;
 };
 
-template <bool SH, typename T>
+// SH: the sharded kernel; PQ: the single-GPU kernel on the two-round (pair) queue. The one-round
+// single-GPU kernel (PQ = false) keeps exactly the pre-pair code (measured: the pair engine's
+// extra code costs the one-round path ~2-3 %, so each queue gets its own instantiation).
+template <bool SH, bool PQ, typename T>
 __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(const __grid_constant__ DFLaunch<T> L) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   __shared__ __align__(8) unsigned long long bars[GROUPS][2 * STAGES];
-  __shared__ Slot<T> slots[GROUPS][2];
+  __shared__ Slot<T, PQ> slots[GROUPS][2];
   const DFArgs<T>& a = L.r[SH ? blockIdx.x % L.nv : 0];
   const int g = threadIdx.x / GNT, gtid = threadIdx.x % GNT;
   T* const stage0 = reinterpret_cast<T*>(smem_raw) + g * STAGES * STAGE_ELEMS;
@@ -844,14 +876,14 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
       const long long t0 = clock64();
       while (clock64() - t0 < a.stagger) __nanosleep(256);
     }
-    Slot<T>& s0 = slots[g][0];
+    Slot<T, PQ>& s0 = slots[g][0];
     s0.t = (long long)atomicAdd(a.counter, 1ull);
     s0.ready = 0;
     s0.pref = 0;
     slots[g][1].pref = 0;
     if (s0.t < a.total) {
-      s0.tk = decode_any<SH>(a, s0.t);
-      if (s0.tk.type != T_P1) fill_desc(a, s0.tk, s0.d);
+      s0.tk = decode_any<SH, PQ>(a, s0.t);
+      if (s0.tk.type != T_P1) fill_desc(a, s0.tk, s0.d, slot_p2(&s0));
     }
   }
   gbar(g);
@@ -859,15 +891,15 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
   unsigned long long pr[6] = {0, 0, 0, 0, 0, 0};  // wait, body, tail, tasks, p1 cycles, waits that blocked
   long long tc0 = clock64();
   for (int it = 0;; ++it) {
-    Slot<T>& S = slots[g][it & 1];
-    Slot<T>* N = &slots[g][(it + 1) & 1];
+    Slot<T, PQ>& S = slots[g][it & 1];
+    Slot<T, PQ>* N = &slots[g][(it + 1) & 1];
     const long long t = S.t;
     if (t >= a.total) break;
     const Task tk = S.tk;
     if (!S.ready) {  // uniform: the slot was published by the last barrier
-      if (gtid == SCH && !deps_any<SH>(a, tk)) {
+      if (gtid == SCH && !deps_any<SH, PQ>(a, tk)) {
         const long long w0 = clock64();
-        while (!deps_any<SH>(a, tk)) {
+        while (!deps_any<SH, PQ>(a, tk)) {
           __nanosleep(64);
           // sharded: a peer that never delivers (a dead rank) must not hang the GPU: after
           // ~30 s of waiting the kernel traps (the launch fails, the handle reports APSP_ECUDA)
@@ -896,14 +928,24 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
         N->t = nxt;
         N->pref = 0;
         if (nxt < a.total) {
-          N->tk = decode_any<SH>(a, nxt);
+          N->tk = decode_any<SH, PQ>(a, nxt);
           N->ready = 0;
-          if (N->tk.type != T_P1) fill_desc(a, N->tk, N->d);
+          if (N->tk.type != T_P1) fill_desc(a, N->tk, N->d, slot_p2(N));
         }
       }
     } else {
-      group_minplus<SH, T>(&S.d, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N, S.pref);
-      chunk += S.d.nk;
+      if constexpr (PQ) {
+        if (S.p2.nk == 2 * (BM / BK)) {
+          group_minplus<SH, PQ, T, 2 * (BM / BK)>(&S.d, &S.p2, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N,
+                                                  S.pref);
+        } else {
+          group_minplus<SH, PQ, T, BM / BK>(&S.d, &S.p2, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N, S.pref);
+        }
+        chunk += S.p2.nk;
+      } else {
+        group_minplus<SH, PQ, T, BM / BK>(&S.d, nullptr, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N, S.pref);
+        chunk += BM / BK;
+      }
     }
     const long long tc2 = clock64();
     pr[1] += tc2 - tc1;
@@ -914,7 +956,8 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
     // better than deferring it under the next task's first loads)
     if (gtid == SIG) {
       if constexpr (SH) signal_done_sh(a, tk);
-      else signal_single(a, tk);
+      else if constexpr (PQ) signal_single(a, tk);
+      else signal_done(a, tk);
     }
     tc0 = clock64();
     pr[2] += tc0 - tc2;
@@ -952,7 +995,10 @@ cudaError_t launch_fw_dataflow(T* D, long long ld, int nb, void* work, int* negf
                                long long stagger, cudaStream_t s, unsigned long long* prof) {
   if (nb <= 0) return cudaSuccess;
   const int smem = GROUPS * STAGES * STAGE_ELEMS * (int)sizeof(T);
-  cudaError_t e = cudaFuncSetAttribute(fw_dataflow_kernel<false, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaError_t e = cudaFuncSetAttribute(fw_dataflow_kernel<false, false, T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       smem);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(fw_dataflow_kernel<false, true, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return e;
   int dev = 0, sms = 0;
   if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
@@ -961,12 +1007,13 @@ cudaError_t launch_fw_dataflow(T* D, long long ld, int nb, void* work, int* negf
   memset(&L, 0, sizeof(L));
   L.nv = 1;
   DFArgs<T>& a = L.r[0];
-  df_layout(a, work, nb, nb, 4);
+  // the two-round (pair) queue: APSP_DF_PAIR=0/1 overrides the default (tuning experiments)
+  int pairq = kPairDefault && sizeof(T) == 4 && T(0.5) == T(0) && nb >= kPairMinNb;  // int32
+  if (const char* e = getenv("APSP_DF_PAIR")) pairq = atoi(e) != 0 && nb >= 2;
+  df_layout(a, work, nb, nb, pairq ? 4 : 2);  // the pair queue keeps 4 rounds of panel copies
+  a.pairq = pairq;
   a.D = D; a.ld = ld;
   a.negflag = negflag;
-  // the two-round (pair) queue: APSP_DF_PAIR=0/1 overrides the default (tuning experiments)
-  a.pairq = kPairDefault && nb >= 4;
-  if (const char* e = getenv("APSP_DF_PAIR")) a.pairq = atoi(e) != 0 && nb >= 2;
   a.total = a.pairq ? pair_total(nb) : (long long)nb * nb * nb;
   a.delay = delay;
   a.stagger = stagger;
@@ -978,7 +1025,8 @@ cudaError_t launch_fw_dataflow(T* D, long long ld, int nb, void* work, int* negf
   if (e != cudaSuccess) return e;
   long long grid = (long long)sms * CTAS_PER_SM;
   if (grid > a.total) grid = a.total;
-  fw_dataflow_kernel<false, T><<<(unsigned)grid, GNT * GROUPS, smem, s>>>(L);
+  if (a.pairq) fw_dataflow_kernel<false, true, T><<<(unsigned)grid, GNT * GROUPS, smem, s>>>(L);
+  else fw_dataflow_kernel<false, false, T><<<(unsigned)grid, GNT * GROUPS, smem, s>>>(L);
   return cudaGetLastError();
 }
 
@@ -1004,7 +1052,7 @@ cudaError_t launch_fw_dataflow_sharded(const DFShard* ranks, int nv, int P, int 
   if (nb <= 0 || nv < 1 || nv > kMaxRanks || P < 1 || P > kMaxRanks || nb % P) return cudaErrorInvalidValue;
   const int nl = nb / P;
   const int smem = GROUPS * STAGES * STAGE_ELEMS * (int)sizeof(T) + 8 * (nb + 1);  // + segment starts
-  cudaError_t e = cudaFuncSetAttribute(fw_dataflow_kernel<true, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaError_t e = cudaFuncSetAttribute(fw_dataflow_kernel<true, false, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return e;
   int dev = 0, sms = 0;
   if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
@@ -1039,14 +1087,14 @@ cudaError_t launch_fw_dataflow_sharded(const DFShard* ranks, int nv, int P, int 
   // a persistent grid must be fully resident (tasks wait on each other): CTAs per SM as the
   // occupancy calculator allows with this launch's shared memory (the segment starts grow it)
   int occ = 0;
-  if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fw_dataflow_kernel<true, T>, GNT * GROUPS, smem)) !=
+  if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fw_dataflow_kernel<true, false, T>, GNT * GROUPS, smem)) !=
       cudaSuccess)
     return e;
   if (occ < 1) return cudaErrorInvalidConfiguration;
   long long grid = (long long)sms * (occ < CTAS_PER_SM ? occ : CTAS_PER_SM);
   grid -= grid % nv;
   if (grid < nv) return cudaErrorInvalidConfiguration;
-  fw_dataflow_kernel<true, T><<<(unsigned)grid, GNT * GROUPS, smem, s>>>(L);
+  fw_dataflow_kernel<true, false, T><<<(unsigned)grid, GNT * GROUPS, smem, s>>>(L);
   return cudaGetLastError();
 }
 
