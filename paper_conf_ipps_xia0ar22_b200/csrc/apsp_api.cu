@@ -788,10 +788,10 @@ apsp_status apsp_select(int64_t n, const int64_t* row_ptr, const int32_t* col_id
   std::string err;
   int dev = cfg.device;
   if (dev < 0 && cudaGetDevice(&dev) != cudaSuccess) return fail_global(APSP_ECUDA, "no CUDA device");
-  size_t free_b = 0, total_b = 0;
-  if (cudaSetDevice(dev) != cudaSuccess || cudaMemGetInfo(&free_b, &total_b) != cudaSuccess)
-    return fail_global(APSP_ECUDA, "no CUDA device (the library has no CPU path)");
-  const double budget = cfg.device_budget_bytes > 0 ? (double)cfg.device_budget_bytes : (double)free_b - (1 << 30);
+  if (cudaSetDevice(dev) != cudaSuccess) return fail_global(APSP_ECUDA, "no CUDA device (the library has no CPU path)");
+  const long long avail = device_free_bytes(dev, (long long)n * n * 4);
+  if (avail < 0) return fail_global(APSP_ECUDA, "no CUDA device (the library has no CPU path)");
+  const double budget = cfg.device_budget_bytes > 0 ? (double)cfg.device_budget_bytes : (double)avail - (1 << 30);
   const double W = 4.0, mat = dn * dn * W;
   const bool ooc = mat > budget;
   double c_unit = 0, TH = 0;

@@ -176,11 +176,10 @@ apsp_status dupload(Handle* h, std::vector<void*>& keep, T** dst, const T* src, 
 apsp_status plan_placement(Handle* h, const apsp_config& cfg, long long fixed) {
   Bnd* b = B_(h);
   const long long W = h->elem, n_pad = b->n_pad, NB = b->NB_pad;
-  size_t free_b = 0, total_b = 0;
-  apsp_status st;
-  if ((st = h->cuda(cudaMemGetInfo(&free_b, &total_b), "cudaMemGetInfo"))) return st;
-  const long long L = cfg.device_budget_bytes > 0 ? cfg.device_budget_bytes : (long long)free_b - (1ll << 30);
   const long long incore = n_pad * n_pad * W + n_pad * NB * W;  // result + tmp for all block rows
+  const long long avail = device_free_bytes(h->device, fixed + incore);
+  if (avail < 0) return h->fail(APSP_ECUDA, "cudaMemGetInfo failed");
+  const long long L = cfg.device_budget_bytes > 0 ? cfg.device_budget_bytes : avail - (1ll << 30);
   if (!cfg.force_out_of_core && fixed + incore <= L) {
     b->ooc = false;
     b->res_row0 = 0;

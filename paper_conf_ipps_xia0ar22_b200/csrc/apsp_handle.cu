@@ -205,6 +205,24 @@ apsp_status setup_device(Handle* h, const apsp_config& cfg) {
   return h->cuda(cudaMemsetAsync(h->d_flag, 0, sizeof(int), h->stream), "memset flag");
 }
 
+// Device memory a new handle may use. apsp_destroy returns its big buffers to the device's
+// stream-ordered pool, which keeps them cached (no driver round trip for the next handle); but
+// cudaMemGetInfo does not count that cached memory as free, and plain cudaMalloc cannot use it.
+// So when the driver's free memory is short of `want` (the caller's in-core working set) the
+// pool's unused memory is returned to the driver first: without this a handle created after a
+// large one was destroyed would see almost nothing free and fall back to the out-of-core path.
+long long device_free_bytes(int device, long long want) {
+  size_t free_b = 0, total_b = 0;
+  if (cudaMemGetInfo(&free_b, &total_b) != cudaSuccess) return -1;
+  if (want > (long long)free_b - (1ll << 30)) {
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, device) == cudaSuccess && cudaMemPoolTrimTo(pool, 0) == cudaSuccess &&
+        cudaMemGetInfo(&free_b, &total_b) != cudaSuccess)
+      return -1;
+  }
+  return (long long)free_b;
+}
+
 // The NCCL communicator of a sharded placement (one per handle).
 static apsp_status create_comm(Handle* h, const apsp_config& cfg) {
   ncclUniqueId id;
@@ -234,10 +252,10 @@ static apsp_status init_placement(Handle* h, const apsp_config& cfg, const int64
   // two pivot-band panels (double-buffered by round parity)
   const long long panel_bytes =
       (h->world > 1 || h->use_comm) ? 2 * (long long)h->b * h->ld * (long long)h->elem : 0;
-  size_t free_b = 0, total_b = 0;
-  if ((st = h->cuda(cudaMemGetInfo(&free_b, &total_b), "cudaMemGetInfo"))) return st;
+  const long long avail = device_free_bytes(h->device, mat_bytes + panel_bytes);
+  if (avail < 0) return h->fail(APSP_ECUDA, "cudaMemGetInfo failed");
   long long budget = cfg.device_budget_bytes > 0 ? cfg.device_budget_bytes
-                                                 : (long long)free_b - (1ll << 30);  // keep 1 GiB headroom
+                                                 : avail - (1ll << 30);  // keep 1 GiB headroom
   // a caller-owned matrix (cfg.dist_device, checked against mat_bytes by apsp_init_from_csr)
   // keeps the handle in core; only the library's own buffers count against the budget
   const bool need_ooc =

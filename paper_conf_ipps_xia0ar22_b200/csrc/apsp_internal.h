@@ -192,5 +192,7 @@ apsp_status johnson_seconds(const apsp_config& cfg, long long n, const int64_t* 
 apsp_status global_fail(apsp_status st, const char* msg);
 // common device / stream setup of a handle (apsp_handle.cu)
 apsp_status setup_device(Handle* h, const apsp_config& cfg);
+// free device memory, the memory pool trimmed first when it is short of `want` (apsp_handle.cu); -1 on error
+long long device_free_bytes(int device, long long want);
 
 }  // namespace apsp

@@ -514,10 +514,10 @@ apsp_status jn_setup(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, 
     return st;
   graph_bytes += (long long)work_bytes + (j->smem_bits ? 0 : (long long)j->grid * bits_bytes);
 
-  size_t free_b = 0, total_b = 0;
-  if ((st = h->cuda(cudaMemGetInfo(&free_b, &total_b), "cudaMemGetInfo"))) return st;
+  const long long avail = device_free_bytes(h->device, (long long)n * n * h->elem);
+  if (avail < 0) return h->fail(APSP_ECUDA, "cudaMemGetInfo failed");
   const long long budget = cfg.device_budget_bytes > 0 ? cfg.device_budget_bytes - graph_bytes
-                                                       : (long long)free_b - (1ll << 30);
+                                                       : avail - (1ll << 30);
   // sources of this rank (world_size > 1): a contiguous block of result rows; the
   // SSSP instances are independent, so ranks need no communication at all
   {
