@@ -35,9 +35,9 @@
 //   * C is loaded into the accumulators first (min is exact, any order) and
 //     stored once (out of place per tile, so phase 2, where an operand aliases
 //     C, is exact);
-//   * phase 1: the tile in registers, two FW steps per barrier (rows / columns kk,
-//     kk+1 published through a double-buffered shared copy), the R6 negative-cycle
-//     check at every step;
+//   * phase 1: the tile in registers, 64 steps, each publishing row / column kk
+//     through a double-buffered shared copy (one barrier per step), the R6
+//     negative-cycle check at the start of every step;
 //   * thread 0 fetches the next queue entry and the index after it while the CTA
 //     computes the current task, and checks the next task's flags right after
 //     publishing the current one.
@@ -110,62 +110,36 @@ struct SmSlot {
 };
 
 // Phase 1 on a tile held in registers (thread: rows 4ty.., columns 4tx..): in-place FW
-// closure of the 64x64 block (P:60 restricted to it), TWO steps per barrier: the owners publish
-// rows kk, kk+1 and columns kk, kk+1 as they stand before step kk (double-buffered shared
-// copies); every thread then derives row kk+1 and column kk+1 after step kk for its own columns
-// / rows (T[kk+1][c] = min(T[kk+1][c], T[kk+1][kk] + T[kk][c]), likewise the column: the very
-// values sequential FW would produce, one RN add each) and applies steps kk and kk+1 to its
-// block: 40 relaxations per thread and 32 barriers instead of 32 and 64. R6 check at both steps.
+// closure of the 64x64 block (P:60 restricted to it), 64 steps, row / column kk published
+// through a double-buffered shared copy, one barrier per step; R6 check at every step.
 template <typename T>
 __device__ __forceinline__ void small_close(T (&acc)[4][4], T* rowbuf, T* colbuf, int* negflag) {
   using V4 = typename SV<T>::V4;
   const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
   bool neg = false;
-  // rowbuf / colbuf: [parity 2][2 rows or columns][64]
   for (int q = 0; q < 16; ++q) {
 #pragma unroll
-    for (int u = 0; u < 4; u += 2) {
-      const int kk = q * 4 + u, p = (u >> 1) & 1;
-      T* const rb = rowbuf + p * 2 * SB;
-      T* const cb = colbuf + p * 2 * SB;
-      if (ty == q) {  // rows kk, kk+1 (local rows u, u+1 of this thread's 4)
-        V4 x0, x1;
-        x0.x = acc[u][0]; x0.y = acc[u][1]; x0.z = acc[u][2]; x0.w = acc[u][3];
-        x1.x = acc[u + 1][0]; x1.y = acc[u + 1][1]; x1.z = acc[u + 1][2]; x1.w = acc[u + 1][3];
-        *reinterpret_cast<V4*>(&rb[tx * 4]) = x0;
-        *reinterpret_cast<V4*>(&rb[SB + tx * 4]) = x1;
+    for (int u = 0; u < 4; ++u) {
+      const int kk = q * 4 + u, p = u & 1;
+      if (ty == q) {  // row kk
+        V4 x;
+        x.x = acc[u][0]; x.y = acc[u][1]; x.z = acc[u][2]; x.w = acc[u][3];
+        *reinterpret_cast<V4*>(&rowbuf[p * SB + tx * 4]) = x;
       }
-      if (tx == q) {  // columns kk, kk+1
-        V4 y0, y1;
-        y0.x = acc[0][u]; y0.y = acc[1][u]; y0.z = acc[2][u]; y0.w = acc[3][u];
-        y1.x = acc[0][u + 1]; y1.y = acc[1][u + 1]; y1.z = acc[2][u + 1]; y1.w = acc[3][u + 1];
-        *reinterpret_cast<V4*>(&cb[ty * 4]) = y0;
-        *reinterpret_cast<V4*>(&cb[SB + ty * 4]) = y1;
+      if (tx == q) {  // column kk
+        V4 y;
+        y.x = acc[0][u]; y.y = acc[1][u]; y.z = acc[2][u]; y.w = acc[3][u];
+        *reinterpret_cast<V4*>(&colbuf[p * SB + ty * 4]) = y;
       }
       __syncthreads();
-      const T t01 = rb[kk + 1];       // T[kk][kk+1]
-      const T t10 = rb[SB + kk];      // T[kk+1][kk]
-      const V4 a0v = *reinterpret_cast<const V4*>(&cb[ty * 4]);
-      const V4 a1v = *reinterpret_cast<const V4*>(&cb[SB + ty * 4]);
-      const V4 b0v = *reinterpret_cast<const V4*>(&rb[tx * 4]);
-      const V4 b1v = *reinterpret_cast<const V4*>(&rb[SB + tx * 4]);
-      if (tid == 0) {  // R6: D[kk][kk] < 0 at step kk; D[kk+1][kk+1] (after step kk) < 0 at step kk+1
-        const T d0 = rb[kk], d1 = SV<T>::relax(t10, t01, rb[SB + kk + 1]);
-        if (d0 < T(0) || d1 < T(0)) neg = true;
-      }
-      const T a0[4] = {a0v.x, a0v.y, a0v.z, a0v.w}, b0[4] = {b0v.x, b0v.y, b0v.z, b0v.w};
-      T a1[4] = {a1v.x, a1v.y, a1v.z, a1v.w}, b1[4] = {b1v.x, b1v.y, b1v.z, b1v.w};
-#pragma unroll
-      for (int i = 0; i < 4; ++i) a1[i] = SV<T>::relax(a0[i], t01, a1[i]);  // column kk+1 after step kk
-#pragma unroll
-      for (int j = 0; j < 4; ++j) b1[j] = SV<T>::relax(t10, b0[j], b1[j]);  // row kk+1 after step kk
+      if (tid == 0 && rowbuf[p * SB + kk] < T(0)) neg = true;  // R6: D[kk][kk] < 0 -> negative cycle
+      const V4 av = *reinterpret_cast<const V4*>(&colbuf[p * SB + ty * 4]);
+      const V4 bv = *reinterpret_cast<const V4*>(&rowbuf[p * SB + tx * 4]);
+      const T A4[4] = {av.x, av.y, av.z, av.w}, B4[4] = {bv.x, bv.y, bv.z, bv.w};
 #pragma unroll
       for (int i = 0; i < 4; ++i)
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          acc[i][j] = SV<T>::relax(a0[i], b0[j], acc[i][j]);  // step kk
-          acc[i][j] = SV<T>::relax(a1[i], b1[j], acc[i][j]);  // step kk+1
-        }
+        for (int j = 0; j < 4; ++j) acc[i][j] = SV<T>::relax(A4[i], B4[j], acc[i][j]);
     }
   }
   if (neg) *negflag = 1;
@@ -334,8 +308,8 @@ template <typename T>
 __global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ SmArgs<T> a) {
   __shared__ __align__(16) T As[STE];
   __shared__ __align__(16) T Bs[STE];
-  __shared__ __align__(16) T rowbuf[4 * SB];  // [parity][row kk, kk+1][64]
-  __shared__ __align__(16) T colbuf[4 * SB];
+  __shared__ __align__(16) T rowbuf[2 * SB];
+  __shared__ __align__(16) T colbuf[2 * SB];
   __shared__ SmSlot slot[2];
   const int tid = threadIdx.x;
   long long idx_next = 0;  // thread 0: queue index of the slot after N (fetched one task ahead)
