@@ -400,7 +400,9 @@ def run_ours(args):
         clocks = clk.stop()
         ms_step = max_over_ranks(e0.elapsed_time(e1)) / steps
         value = float(n) ** 3 / (ms_step * 1e-3)
-        arith = apsp.ARITH_NAMES[apsp.apsp_get_info(h).arith]
+        info_end = apsp.apsp_get_info(h)
+        arith = apsp.ARITH_NAMES[info_end.arith]
+        kernel_used = apsp.KERNEL_NAMES.get(info_end.kernel, "other")
         apsp.apsp_destroy(h)
         del dist_buf
         # roofline of the dominant kernel: phase-3 min-plus launches
@@ -426,7 +428,8 @@ def run_ours(args):
         tp = os.path.join(ROOT, "profiles", "phase3_traffic.json")
         if os.path.exists(tp) and not ooc_mode:
             try:
-                sched = "dataflow" if dataflow else "legacy"
+                sched = kernel_used if kernel_used in ("dataflow_pair", "small64") else (
+                    "dataflow" if dataflow else "legacy")
                 for tj in json.load(open(tp)).get("captures", []):
                     if (tj.get("workload") == wl and tj.get("arith") == arith
                             and tj.get("schedule", "legacy") == sched):
@@ -437,10 +440,15 @@ def run_ours(args):
         kname = ("%s: all rounds and phases 1-3 in one persistent launch (%s)"
                  % ("fw_dataflow16_kernel" if arith == "s16x2" else "fw_dataflow_kernel", arith) if dataflow
                  else "phase-3 min-plus (%s)" % arith)
+        if kernel_used == "dataflow_pair":
+            kname = ("fw_dataflow_kernel (two-round queue: rounds k, k+1 of each bulk tile in one depth-256 task): "
+                     "all rounds and phases 1-3 in one persistent launch (%s)" % arith)
+        elif kernel_used == "small64":
+            kname = "fw_small_kernel (64x64 tiles): all rounds and phases in one persistent launch (%s)" % arith
         if dataflow and world > 1:
             kname = ("fw_dataflow_kernel<sharded>: this rank's tile rows, all rounds in one persistent launch, "
                      "pivot panels stored into every GPU by their owner (%s)" % arith)
-        roofline = {"bound": "alu", "kernel": kname, "achieved": achieved / 1e12,
+        roofline = {"bound": "alu", "kernel": kname, "kernel_id": kernel_used, "achieved": achieved / 1e12,
                     "peak": peak / 1e12, "unit": "Trelax/s", "frac": achieved / peak, "traffic": traffic,
                     "traffic_unit": "bytes per launch (DRAM read+write)",
                     "algorithmic_bytes_per_launch": (p3_relax * 2 * 128 * 128 * elem / 128 ** 3

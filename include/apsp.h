@@ -411,7 +411,18 @@ typedef struct {
   int32_t packed16_eligible;                   /* packed16 requested and the input allows it */
   int64_t boundary_nodes;                      /* boundary algorithm: boundary nodes, else 0 */
   int64_t edges_scanned;                       /* Johnson: arcs relaxed by the last run, else 0 */
+  int32_t kernel;                              /* APSP_KERNEL_*: what ran the last blocked-FW
+                                                  closure (0 = none yet / other methods) */
+  int32_t pad0;
 } apsp_info;
+
+#define APSP_KERNEL_PER_PHASE 1      /* launch-per-phase rounds (phase1 / min-plus kernels) */
+#define APSP_KERNEL_DATAFLOW 2       /* fw_dataflow_kernel, one round per task */
+#define APSP_KERNEL_DATAFLOW_PAIR 3  /* fw_dataflow_kernel, two rounds per bulk task (decode2) */
+#define APSP_KERNEL_SMALL 4          /* fw_small_kernel, 64x64 tiles */
+#define APSP_KERNEL_DATAFLOW16 5     /* fw_dataflow16_kernel, packed int16 */
+#define APSP_KERNEL_SHARDED 6        /* fw_dataflow_kernel<sharded> */
+#define APSP_KERNEL_OUT_OF_CORE 7    /* the out-of-core band scheduler (min-plus kernels) */
 
 #define APSP_ARITH_I32 0   /* VIADDMNMX (int32 DPX), 1 relaxation / instruction */
 #define APSP_ARITH_S16X2 1 /* VIADDMNMX.S16x2, 2 relaxations / instruction, verified exact */

@@ -74,10 +74,13 @@ class apsp_info(ctypes.Structure):
         ("arith", ctypes.c_int32), ("packed16_eligible", ctypes.c_int32),
         ("boundary_nodes", ctypes.c_int64),
         ("edges_scanned", ctypes.c_int64),
+        ("kernel", ctypes.c_int32), ("pad0", ctypes.c_int32),
     ]
 
 
 APSP_ARITH_I32, APSP_ARITH_S16X2, APSP_ARITH_F32 = 0, 1, 2
+KERNEL_NAMES = {0: "none", 1: "per_phase", 2: "dataflow", 3: "dataflow_pair", 4: "small64", 5: "dataflow16",
+                6: "sharded_dataflow", 7: "out_of_core"}
 ARITH_NAMES = {0: "i32", 1: "s16x2", 2: "f32"}
 
 

@@ -276,6 +276,7 @@ static apsp_status run_small(Handle* h) {
   int ctas = h->n_pad <= 1024 ? 1 : 2;
   if (const char* e = getenv("APSP_SMALL_CTAS")) ctas = atoi(e);  // tuning experiments only
   const long long delay = h->df_delay > 0 ? h->df_delay : kSmallDelay;
+  h->kernel = APSP_KERNEL_SMALL;
   h->ev_begin(2);
   if ((st = h->cuda(launch_fw_small<T>(static_cast<T*>(h->shards[0].D), h->ld, nb, h->df_work, h->d_flag, delay,
                                        h->small_queue_loaded, ctas, h->stream),
@@ -309,10 +310,12 @@ static apsp_status run_dataflow(Handle* h) {
   const size_t prof_bytes = (size_t)sms * 2 * 8 * sizeof(unsigned long long);  // 2 groups per SM
   if (want_prof && (st = h->cuda(cudaMalloc(&prof, prof_bytes), "cudaMalloc prof"))) return st;
   h->ev_begin(2);
+  int used_pair = 0;
   if ((st = h->cuda(launch_fw_dataflow<T>(static_cast<T*>(h->shards[0].D), h->ld, nb, h->df_work, h->d_flag, delay,
-                                          stagger, h->stream, prof),
+                                          stagger, h->stream, prof, &used_pair),
                     "fw_dataflow")))
     return st;
+  h->kernel = used_pair ? APSP_KERNEL_DATAFLOW_PAIR : APSP_KERNEL_DATAFLOW;
   h->ev_end((double)h->n_pad * h->n_pad * h->n_pad);
   if (want_prof) {
     std::vector<unsigned long long> hp(prof_bytes / 8);
@@ -467,6 +470,7 @@ static apsp_status prepare_sharded_peers(Handle* h) {
 }
 
 apsp_status run_incore_rounds(Handle* h, long long k0, long long k1) {
+  h->kernel = APSP_KERNEL_PER_PHASE;  // (the dataflow / sharded paths below set their own)
   if (h->world == 1 && !h->use_comm && !h->virt && h->dataflow && k0 == 0 && k1 == h->n_pad / h->b)
     return h->dtype == APSP_I32 ? run_dataflow<int>(h) : run_dataflow<float>(h);
   if ((h->virt || h->use_comm) && h->dataflow && h->world <= 8 && k0 == 0 && k1 == h->n_pad / h->b) {
@@ -474,8 +478,10 @@ apsp_status run_incore_rounds(Handle* h, long long k0, long long k1) {
     if (!h->virt &&
         (st = h->dtype == APSP_I32 ? prepare_sharded_peers<int>(h) : prepare_sharded_peers<float>(h)))
       return st;
-    if (!h->sh_disabled)
+    if (!h->sh_disabled) {
+      h->kernel = APSP_KERNEL_SHARDED;
       return h->dtype == APSP_I32 ? run_dataflow_sharded<int>(h) : run_dataflow_sharded<float>(h);
+    }
   }
   if (h->world == 1 && !h->use_comm) {  // single GPU: the whole closure, with lookahead
     return h->dtype == APSP_I32
@@ -871,6 +877,7 @@ apsp_status apsp_fw_rounds(apsp_handle* hh, int64_t k_begin, int64_t k_end) {
     if (k_begin % kb || (k_end % kb && k_end != nb))
       return h->fail(APSP_EINVAL, "out of core, rounds run in super-rounds of %lld", kb);
     memset(&h->stats, 0, sizeof(h->stats));
+    h->kernel = APSP_KERNEL_OUT_OF_CORE;
     if ((st = run_out_of_core_range(h, k_begin / kb, (k_end + kb - 1) / kb))) return st;
     h->next_round = k_end;
     return finish_fw(h, k_end == nb);
@@ -897,6 +904,7 @@ apsp_status apsp_fw_blocked(apsp_handle* hh) {
   if (h->mode == APSP_MODE_OUT_OF_CORE) {
     const long long kb = h->ooc_B / h->b;
     if (h->next_round % kb) return h->fail(APSP_ESTATE, "out of core, rounds run in super-rounds of %lld", kb);
+    h->kernel = APSP_KERNEL_OUT_OF_CORE;
     if ((st = run_out_of_core_range(h, h->next_round / kb, nb / kb))) return st;
     h->next_round = nb;
     return finish_fw(h, true);
@@ -1059,6 +1067,7 @@ apsp_status apsp_get_info(const apsp_handle* hh, apsp_info* info) {
   if (h->result16) info->dist_device = h->d16;
   info->boundary_nodes = bnd_boundary_nodes(h);
   info->edges_scanned = jn_edges(h);
+  info->kernel = h->kernel;
   return APSP_OK;
 }
 

@@ -992,7 +992,7 @@ static void df_layout(DFArgs<T>& a, void* work, int nb, int nl, int npar) {
 
 template <typename T>
 cudaError_t launch_fw_dataflow(T* D, long long ld, int nb, void* work, int* negflag, long long delay,
-                               long long stagger, cudaStream_t s, unsigned long long* prof) {
+                               long long stagger, cudaStream_t s, unsigned long long* prof, int* used_pair) {
   if (nb <= 0) return cudaSuccess;
   const int smem = GROUPS * STAGES * STAGE_ELEMS * (int)sizeof(T);
   cudaError_t e = cudaFuncSetAttribute(fw_dataflow_kernel<false, false, T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1012,6 +1012,7 @@ cudaError_t launch_fw_dataflow(T* D, long long ld, int nb, void* work, int* negf
   if (const char* e = getenv("APSP_DF_PAIR")) pairq = atoi(e) != 0 && nb >= 2;
   df_layout(a, work, nb, nb, pairq ? 4 : 2);  // the pair queue keeps 4 rounds of panel copies
   a.pairq = pairq;
+  if (used_pair) *used_pair = pairq;
   a.D = D; a.ld = ld;
   a.negflag = negflag;
   a.total = a.pairq ? pair_total(nb) : (long long)nb * nb * nb;
@@ -1155,8 +1156,8 @@ template cudaError_t launch_fw_dataflow_sharded<int>(const DFShard*, int, int, i
 template cudaError_t launch_fw_dataflow_sharded<float>(const DFShard*, int, int, int, long long, int*, long long,
                                                        cudaStream_t);
 template cudaError_t launch_fw_dataflow<int>(int*, long long, int, void*, int*, long long, long long, cudaStream_t,
-                                             unsigned long long*);
+                                             unsigned long long*, int*);
 template cudaError_t launch_fw_dataflow<float>(float*, long long, int, void*, int*, long long, long long,
-                                               cudaStream_t, unsigned long long*);
+                                               cudaStream_t, unsigned long long*, int*);
 
 }  // namespace apsp

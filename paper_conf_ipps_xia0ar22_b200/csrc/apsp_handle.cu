@@ -330,6 +330,7 @@ static apsp_status run_dataflow16(Handle* h) {
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const long long delay = h->df_delay > 0 ? h->df_delay : 4ll * fw_dataflow16_ctas_per_sm() * sms;
+  h->kernel = APSP_KERNEL_DATAFLOW16;
   h->ev_begin(2);
   if ((st = h->cuda(launch_fw_dataflow16(h->d16, h->ld, nb, h->df_work, delay, h->stream), "fw_dataflow16")))
     return st;
@@ -350,8 +351,9 @@ apsp_status enqueue_fw16(Handle* h) {
   if (h->fell_back16) return run_fw16_int32(h);
   if (h->dataflow) {  // default: every round in one persistent launch (apsp_fw_dataflow16.cu)
     if ((st = run_dataflow16(h))) return st;
-  } else if ((st = fw_closure<short>(h, h->d16, h->ld, h->n_pad, 0, nb, h->stream))) {
-    return st;
+  } else {
+    h->kernel = APSP_KERNEL_PER_PHASE;
+    if ((st = fw_closure<short>(h, h->d16, h->ld, h->n_pad, 0, nb, h->stream))) return st;
   }
   if (!h->h_max16 && (st = h->cuda(cudaHostAlloc(&h->h_max16, sizeof(int), cudaHostAllocDefault), "cudaHostAlloc")))
     return st;
@@ -407,6 +409,7 @@ static apsp_status run_fw16_int32(Handle* h) {
     return st;
   h->result16 = false;
   h->arith = APSP_ARITH_I32;
+  h->kernel = APSP_KERNEL_PER_PHASE;
   return fw_closure<int>(h, static_cast<int*>(sh.D), h->ld, h->n_pad, 0, nb, h->stream);
 }
 

@@ -92,6 +92,7 @@ struct Handle {
   bool dataflow = true;     // apsp_config.schedule (APSP_SCHED_PER_PHASE: launch per phase)
   bool small = false;       // dataflow with 64x64 tiles (apsp_fw_small.cu): small n, APSP_SCHED_SMALL
   bool small_queue_loaded = false;  // its task queue is in df_work
+  int kernel = 0;           // APSP_KERNEL_* of the last blocked-FW closure (apsp_info.kernel)
   long long df_delay = 0;   // apsp_config.dataflow_delay (0 = auto)
   void* df_work = nullptr;
   // sharded dataflow kernel (multi-GPU / virtual ranks): per-rank work buffers

@@ -114,7 +114,8 @@ extern int g_minplus_variant;
 // group of every CTA waits before its first task.
 template <typename T>
 cudaError_t launch_fw_dataflow(T* D, long long ld, int nb, void* work, int* negflag, long long delay,
-                               long long stagger, cudaStream_t s, unsigned long long* prof = nullptr);
+                               long long stagger, cudaStream_t s, unsigned long long* prof = nullptr,
+                               int* used_pair = nullptr);
 long long fw_dataflow_pbuf_bytes(int nb, size_t elem);
 long long fw_dataflow_flag_bytes(int nb);
 long long fw_dataflow_work_bytes(int nb, size_t elem);

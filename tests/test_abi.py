@@ -179,3 +179,14 @@ def test_dist_device_too_small_or_misaligned_is_refused(lib):
         with pytest.raises(lib.ApspError) as e:
             call()
         assert e.value.status == lib.APSP_EINVAL
+
+
+def test_kernel_ids_match_header(lib):
+    hdr = open(os.path.join(ROOT, "include", "apsp.h")).read()
+    ids = {int(v): k for k, v in re.findall(r"#define APSP_KERNEL_([A-Z0-9_]+) (\d+)", hdr)}
+    assert sorted(ids) == list(range(1, 8))
+    names = {"PER_PHASE": "per_phase", "DATAFLOW": "dataflow", "DATAFLOW_PAIR": "dataflow_pair", "SMALL": "small64",
+             "DATAFLOW16": "dataflow16", "SHARDED": "sharded_dataflow", "OUT_OF_CORE": "out_of_core"}
+    for v, k in ids.items():
+        assert lib.KERNEL_NAMES[v] == names[k]
+    assert [f[0] for f in lib.apsp_info._fields_][-2:] == ["kernel", "pad0"]

@@ -125,3 +125,23 @@ def test_pair_schedule_equals_single_round_schedule(lib, monkeypatch, n):
     assert np.array_equal(out["1"][1].view(np.int32), out["0"][1].view(np.int32))
     if n <= 2560:
         assert np.array_equal(out["1"][0].astype(np.int64), want_i32(g))
+
+
+def test_kernel_reported_per_placement(lib, monkeypatch):
+    """apsp_info.kernel names what ran the closure (the bench's roofline reads it): the small-n
+    kernel at n <= 2048, the one-round dataflow kernel above, the pair kernel when selected,
+    launch-per-phase, packed16, the sharded kernel, out of core."""
+    def kernel_of(g, **kw):
+        with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=lib.apsp_config_default(device=0, **kw)) as h:
+            lib.apsp_fw_blocked(h)
+            return lib.KERNEL_NAMES[lib.apsp_get_info(h).kernel]
+    small, big = gg.erdos_renyi(1000, 5000, seed=1), gg.erdos_renyi(3000, 15000, seed=2)
+    assert kernel_of(small) == "small64"
+    assert kernel_of(big) == "dataflow"
+    monkeypatch.setenv("APSP_DF_PAIR", "1")
+    assert kernel_of(big) == "dataflow_pair"
+    monkeypatch.delenv("APSP_DF_PAIR")
+    assert kernel_of(big, schedule=1) == "per_phase"
+    assert kernel_of(big, packed16=1) == "dataflow16"
+    assert kernel_of(big, world_size=2, virtual_ranks=1, schedule=2) == "sharded_dataflow"
+    assert kernel_of(small, force_out_of_core=1, ooc_block=256) == "out_of_core"
