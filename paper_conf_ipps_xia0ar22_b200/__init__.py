@@ -79,6 +79,8 @@ class apsp_info(ctypes.Structure):
 
 
 APSP_ARITH_I32, APSP_ARITH_S16X2, APSP_ARITH_F32 = 0, 1, 2
+(APSP_KERNEL_PER_PHASE, APSP_KERNEL_DATAFLOW, APSP_KERNEL_DATAFLOW_PAIR, APSP_KERNEL_SMALL, APSP_KERNEL_DATAFLOW16,
+ APSP_KERNEL_SHARDED, APSP_KERNEL_OUT_OF_CORE) = range(1, 8)
 KERNEL_NAMES = {0: "none", 1: "per_phase", 2: "dataflow", 3: "dataflow_pair", 4: "small64", 5: "dataflow16",
                 6: "sharded_dataflow", 7: "out_of_core"}
 ARITH_NAMES = {0: "i32", 1: "s16x2", 2: "f32"}
