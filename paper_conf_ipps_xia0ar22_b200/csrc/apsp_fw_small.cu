@@ -350,6 +350,9 @@ __global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ S
     else small_minplus(a, tk, As, Bs, rowbuf, colbuf);
     if (tid == 0 && N.t < a.total) N.tk = small_task(nq);
     __syncthreads();  // every thread's stores of this task are issued; As / Bs free; N.tk published
+    // publication (release fence + flags) by warp 1 while thread 0 checks the next task's flags:
+    // two L2 round trips in parallel instead of one after the other
+    if (tid == 32) small_signal(a, tk);
     if (tid == 0) {
       if (a.prof) {
         const long long c1 = clock64();
@@ -357,7 +360,6 @@ __global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ S
         pr[6 + tk.type] += 1;
         c0 = c1;
       }
-      small_signal(a, tk);
       // the next task's flags, once: if met, it starts without another wait
       N.ready = N.t < a.total && small_deps(a, N.tk);
       S.t = idx_next;  // this slot becomes the one after N (read by the others only after the

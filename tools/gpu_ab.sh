@@ -1,0 +1,33 @@
+#!/bin/bash
+# A/B timing recipes for one B200 (device time via tools/fw_ab.py / tools/ooc_ab.py), output in
+# gpurun_out/ab_<what>.txt:
+#   tools/gpu_ab.sh small   64-tile small-n kernel vs the 128-tile kernels, n = 1024 .. 4096, CTAs per SM
+#   tools/gpu_ab.sh pair    two-round (pair) queue vs one-round queue, int32 n = 16384 / 32768 / 65536, fp32
+#   tools/gpu_ab.sh ooc     out of core, every band streamed (n = 16384 / 32768, 1 and 2 virtual ranks)
+mkdir -p gpurun_out
+what=$1
+out=gpurun_out/ab_$what.txt
+case $what in
+  small)
+    { for n in 1024 1536 2048 3072 4096; do
+        echo "== n=$n"; python tools/fw_ab.py --n $n --deg 8 --dtype i32 --runs 20 --modes small dataflow per_phase
+      done
+      for c in 1 2 3; do echo "== n=1024 ctas=$c"; APSP_SMALL_CTAS=$c python tools/fw_ab.py --n 1024 --deg 8 --runs 20 --modes small; done
+      echo "== n=1024 profile"; APSP_SMALL_PROFILE=1 python tools/fw_ab.py --n 1024 --deg 8 --runs 3 --modes small
+    } > $out 2>&1 ;;
+  pair)
+    { for n in 16384 32768 65536; do
+        r=3; d=4; [ $n -gt 16384 ] && r=2; [ $n -gt 32768 ] && r=1 && d=16
+        for p in 0 1; do echo "== pair=$p n=$n"; APSP_DF_PAIR=$p python tools/fw_ab.py --n $n --deg $d --dtype i32 --runs $r --modes dataflow; done
+      done
+      for p in 0 1; do echo "== pair=$p f32 n=32768"; APSP_DF_PAIR=$p python tools/fw_ab.py --n 32768 --deg 64 --dtype f32 --runs 2 --modes dataflow; done
+    } > $out 2>&1 ;;
+  ooc)
+    { python tools/ooc_ab.py --n 16384 --block 2048 --stream-all --runs 2
+      python tools/ooc_ab.py --n 16384 --block 4096 --stream-all --runs 2
+      python tools/ooc_ab.py --n 32768 --block 4096 --stream-all --runs 1
+      python tools/ooc_ab.py --n 32768 --block 4096 --stream-all --runs 1 --world 2
+    } > $out 2>&1 ;;
+  *) echo "usage: tools/gpu_ab.sh small|pair|ooc"; exit 2 ;;
+esac
+cat $out | grep -vE "^\s*$" | tail -40
