@@ -12,8 +12,8 @@ case $what in
     { for n in 1024 1536 2048 3072 4096; do
         echo "== n=$n"; python tools/fw_ab.py --n $n --deg 8 --dtype i32 --runs 20 --modes small dataflow per_phase
       done
-      for c in 1 2 3; do echo "== n=1024 ctas=$c"; APSP_SMALL_CTAS=$c python tools/fw_ab.py --n 1024 --deg 8 --runs 20 --modes small; done
-      echo "== n=1024 profile"; APSP_SMALL_PROFILE=1 python tools/fw_ab.py --n 1024 --deg 8 --runs 3 --modes small
+      for c in 1 2 3; do echo "== n=1024 ctas=$c"; APSP_SMALL_CTAS=$c python tools/fw_ab.py --n 1024 --deg 8 --dtype i32 --runs 20 --modes small; done
+      echo "== n=1024 profile"; APSP_SMALL_PROFILE=1 python tools/fw_ab.py --n 1024 --deg 8 --dtype i32 --runs 3 --modes small
     } > $out 2>&1 ;;
   pair)
     { for n in 16384 32768 65536; do
