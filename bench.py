@@ -73,6 +73,8 @@ def parse():
     ap.add_argument("--packed16-e2e", action="store_true", help="also time the packed16 leg end to end")
     ap.add_argument("--no-ooc-leg", action="store_true",
                     help="skip the out-of-core leg (every band streamed from pinned host memory, B = 4096)")
+    ap.add_argument("--no-boundary-leg", action="store_true",
+                    help="skip the boundary-algorithm leg (2-D grid of the same n, k = sqrt(n)/4, out of core)")
     ap.add_argument("--rendezvous-only", action="store_true",
                     help="launcher check: init the process group (gloo), barrier, print the rank, exit")
     return ap.parse_args()
@@ -638,6 +640,61 @@ def run_ours(args):
                     "lookahead; step = apsp_reinit (init + D2H of every band) + apsp_fw_blocked; bit-exact in "
                     "tests/test_gpu_ooc.py" % (args.ooc_block or 4096)}
 
+    # the boundary algorithm (eq. (1), Alg. 3) out of core on a small-separator graph of
+    # the same n: a sqrt(n) x sqrt(n) 2-D grid (cfg2/cfg5's recipe) split into the paper's
+    # k = sqrt(n)/4 components, every block row of the result streamed to pinned host
+    # memory through two N_row buffers (transfers inside the solve), beside the
+    # blocked-FW out-of-core step of the same n (dense FW cost does not depend on the structure)
+    def boundary_timed():
+        side = int(round(n ** 0.5))
+        if side * side != n:
+            return {"skipped": "n=%d is not a square" % n}
+        gb = gg.grid_2d(side, side, seed=3, name="grid%d" % n)
+        blocks = max(1, int(round((side / 4) ** 0.5)))  # blocks x blocks components, k ~ sqrt(n)/4
+        comp, k = gg.grid_block_partition(gb, blocks, blocks)
+        cfg = apsp.apsp_config_default(device=local, timing=1)
+        cfg.stream = stream.cuda_stream
+        cfg.force_out_of_core = 1
+        h = apsp.apsp_init_boundary(n, gb.row_ptr, gb.col, gb.w, comp, k, cfg=cfg)
+        try:
+            steps = min(args.steps, 5)
+            for _ in range(min(args.warmup, 2)):
+                apsp.apsp_reinit(h)
+                apsp.apsp_solve(h)
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            for _ in range(steps):
+                apsp.apsp_reinit(h)
+                apsp.apsp_solve(h)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            ms = e0.elapsed_time(e1) / steps
+            info = apsp.apsp_get_info(h)
+            st = apsp.apsp_get_phase_stats(h)
+        finally:
+            apsp.apsp_destroy(h)
+        link = float(info.host_bytes)
+        lk = peaks().get("dpx", {}).get("host_link_gbs", {})
+        d2h = lk.get("d2h") or 0.0
+        out = {"workload": "grid %dx%d, seed 3, int32 U{1..100}, k = %d components (%dx%d blocks)" %
+                           (side, side, k, blocks, blocks),
+               "ms_per_solve": ms, "steps": steps, "boundary_nodes": int(info.boundary_nodes),
+               "relaxations_per_solve": float(sum(st.relax[:3])),
+               "out_of_core": bool(info.ooc_block > 0), "buffer_rows": int(info.ooc_block),
+               "host_bytes_per_solve": int(link), "link_gbs": link / (ms * 1e-3) / 1e9,
+               "link_frac_d2h": (link / (ms * 1e-3) / 1e9 / d2h) if d2h else None,
+               "note": "apsp_init_boundary (force_out_of_core: nothing resident, every block row crosses the "
+                       "link) + apsp_reinit + apsp_solve per step; bit-exact in tests/test_boundary.py"}
+        if alt_ooc and "ms_per_step" in alt_ooc:
+            out["fw_out_of_core_ms_per_step_same_n"] = alt_ooc["ms_per_step"]
+            out["speedup_vs_fw_out_of_core"] = alt_ooc["ms_per_step"] / ms
+        return out
+
+    alt_bnd = None
+    if world == 1 and not is_f and not args.force_ooc and not args.no_boundary_leg:
+        alt_bnd = guarded(boundary_timed)
+
     # Johnson's algorithm on the same graph (batched Near-Far SSSP): the
     # paper's method for sparse graphs; a different algorithm (O(n m) work, not n^3), so it is
     # reported as time per APSP beside the FW step, not as the metric
@@ -679,6 +736,7 @@ def run_ours(args):
             "packed16": alt16,
             "out_of_core": alt_ooc,
             "johnson": alt_jn,
+            "boundary": alt_bnd,
             "relax_per_step_rank0": main_run["relax_per_step_rank0"],
             "phase_ms_per_step_rank0": main_run["phase_ms_per_step_rank0"],
         }
