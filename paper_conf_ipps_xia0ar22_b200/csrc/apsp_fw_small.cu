@@ -86,6 +86,7 @@ struct SmArgs {
   long long total;   // queue entries
   const int4* queue; // [total] (type, k, i, j), built on the host (small_queue)
   unsigned long long* prof;  // optional [CTAs][16] cycle counters (tuning: APSP_SMALL_PROFILE)
+  int close_v;               // phase-1 variant: 1 small_close_defer, 0 small_close (APSP_SMALL_CLOSE)
 };
 
 template <typename T>
@@ -145,6 +146,101 @@ __device__ __forceinline__ void small_close(T (&acc)[4][4], T* rowbuf, T* colbuf
   if (neg) *negflag = 1;
 }
 
+// The closure with the bulk of each step deferred past the next barrier: in step kk a thread
+// relaxes only its elements of row / column kk+1 (the owners store them into the other buffer
+// for step kk+1), and the rest of its 4x4 block for step kk right after the barrier of step
+// kk+1, while that step's row / column loads are in flight. The per-step chain is then barrier
+// -> loads -> 7 relaxations -> stores; per element the steps still apply in order (the deferred
+// rest of step kk precedes step kk+1's relaxations of the same registers). One barrier per step:
+// the other buffer was last read before this step's barrier (WAR) and is read after the next.
+// Steps are a template on kk mod 4 with the first and last steps peeled, so a step body has no
+// branch and ptxas schedules across it.
+template <typename T, int U, bool REST, bool CRIT>
+__device__ __forceinline__ void close_step(T (&acc)[4][4], T (&pa)[4], T (&pb)[4], T* rowbuf, T* colbuf, int kk,
+                                           bool& neg) {
+  using V4 = typename SV<T>::V4;
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  constexpr int p = U & 1, nu = (U + 1) & 3;  // buffer; row / column kk+1 within a 4x4 block
+  __syncthreads();
+  const V4 av = *reinterpret_cast<const V4*>(&colbuf[p * SB + ty * 4]);
+  const V4 bv = *reinterpret_cast<const V4*>(&rowbuf[p * SB + tx * 4]);
+  const T dkk = rowbuf[p * SB + kk];
+  if (REST) {  // rest of step kk-1: every element outside row / column U (= (kk-1)+1 mod 4)
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        if (i != U && j != U) acc[i][j] = SV<T>::relax(pa[i], pb[j], acc[i][j]);
+  }
+  const T A4[4] = {av.x, av.y, av.z, av.w}, B4[4] = {bv.x, bv.y, bv.z, bv.w};
+  if (CRIT) {
+    const int owner = (kk + 1) >> 2;  // ty (row kk+1) / tx (column kk+1) of its owners
+#pragma unroll
+    for (int j = 0; j < 4; ++j) acc[nu][j] = SV<T>::relax(A4[nu], B4[j], acc[nu][j]);
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+      if (i != nu) acc[i][nu] = SV<T>::relax(A4[i], B4[nu], acc[i][nu]);
+    if (ty == owner) {
+      V4 x;
+      x.x = acc[nu][0]; x.y = acc[nu][1]; x.z = acc[nu][2]; x.w = acc[nu][3];
+      *reinterpret_cast<V4*>(&rowbuf[(p ^ 1) * SB + tx * 4]) = x;
+    }
+    if (tx == owner) {
+      V4 y;
+      y.x = acc[0][nu]; y.y = acc[1][nu]; y.z = acc[2][nu]; y.w = acc[3][nu];
+      *reinterpret_cast<V4*>(&colbuf[(p ^ 1) * SB + ty * 4]) = y;
+    }
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      pa[i] = A4[i];
+      pb[i] = B4[i];
+    }
+  } else {
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j) acc[i][j] = SV<T>::relax(A4[i], B4[j], acc[i][j]);
+  }
+  neg |= dkk < T(0);  // R6: D[kk][kk] < 0 -> negative cycle (every thread reads it: a broadcast)
+}
+
+template <typename T>
+__device__ __forceinline__ void small_close_defer(T (&acc)[4][4], T* rowbuf, T* colbuf, int* negflag) {
+  using V4 = typename SV<T>::V4;
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  bool neg = false;
+  if (ty == 0) {
+    V4 x;
+    x.x = acc[0][0]; x.y = acc[0][1]; x.z = acc[0][2]; x.w = acc[0][3];
+    *reinterpret_cast<V4*>(&rowbuf[tx * 4]) = x;
+  }
+  if (tx == 0) {
+    V4 y;
+    y.x = acc[0][0]; y.y = acc[1][0]; y.z = acc[2][0]; y.w = acc[3][0];
+    *reinterpret_cast<V4*>(&colbuf[ty * 4]) = y;
+  }
+  T pa[4], pb[4];  // step kk-1's column / row values for its deferred rest
+  close_step<T, 0, false, true>(acc, pa, pb, rowbuf, colbuf, 0, neg);
+  for (int q = 0; q < 15; ++q) {  // steps 1 .. 60
+    const int kk = 4 * q + 1;
+    close_step<T, 1, true, true>(acc, pa, pb, rowbuf, colbuf, kk, neg);
+    close_step<T, 2, true, true>(acc, pa, pb, rowbuf, colbuf, kk + 1, neg);
+    close_step<T, 3, true, true>(acc, pa, pb, rowbuf, colbuf, kk + 2, neg);
+    close_step<T, 0, true, true>(acc, pa, pb, rowbuf, colbuf, kk + 3, neg);
+  }
+  close_step<T, 1, true, true>(acc, pa, pb, rowbuf, colbuf, 61, neg);
+  close_step<T, 2, true, true>(acc, pa, pb, rowbuf, colbuf, 62, neg);
+  close_step<T, 3, true, false>(acc, pa, pb, rowbuf, colbuf, 63, neg);
+  if (neg) *negflag = 1;
+}
+
+// phase 1 of the tile in registers: small_close_defer (default) or small_close (APSP_SMALL_CLOSE=0)
+template <typename T>
+__device__ __forceinline__ void small_close_any(const SmArgs<T>& a, T (&acc)[4][4], T* rowbuf, T* colbuf) {
+  if (a.close_v) small_close_defer(acc, rowbuf, colbuf, a.negflag);
+  else small_close(acc, rowbuf, colbuf, a.negflag);
+}
+
 // the closed diagonal block of round k: into the matrix, D and D^T into the panel copy
 template <typename T>
 __device__ __forceinline__ void small_store_diag(const SmArgs<T>& a, int k, T* tile, const T (&acc)[4][4]) {
@@ -179,7 +275,7 @@ __device__ __forceinline__ void small_phase1(const SmArgs<T>& a, const Task& tk,
     const V4 v = __ldcg(reinterpret_cast<const V4*>(tile + (long long)(ty * 4 + i) * a.ld + tx * 4));
     acc[i][0] = v.x; acc[i][1] = v.y; acc[i][2] = v.z; acc[i][3] = v.w;
   }
-  small_close(acc, rowbuf, colbuf, a.negflag);
+  small_close_any(a, acc, rowbuf, colbuf);
   small_store_diag(a, tk.k, tile, acc);
 }
 
@@ -251,7 +347,7 @@ __device__ __forceinline__ void small_minplus(const SmArgs<T>& a, const Task& tk
       for (int j = 0; j < 4; ++j) acc[i][j] = SV<T>::relax(A4[i], B4[j], acc[i][j]);
   }
   if (fused) {  // tile (k+1,k+1) after round k: close it as P1(k+1) (R6 check included)
-    small_close(acc, rowbuf, colbuf, a.negflag);
+    small_close_any(a, acc, rowbuf, colbuf);
     small_store_diag(a, tk.k + 1, C, acc);
     return;
   }
@@ -510,6 +606,8 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
   a.done2 = f; f += nb;
   a.done3 = f; f += nb;
   a.negflag = negflag;
+  const char* cv = getenv("APSP_SMALL_CLOSE");  // phase-1 variant A/B (tuning only)
+  a.close_v = cv ? atoi(cv) : 1;
   // the queue lives in the work buffer: built and uploaded with the first launch on it
   int4* dq = reinterpret_cast<int4*>(fb + small_flag_bytes(nb));
   a.queue = dq;

@@ -2,6 +2,7 @@
 # A/B timing recipes for one B200 (device time via tools/fw_ab.py / tools/ooc_ab.py), output in
 # gpurun_out/ab_<what>.txt:
 #   tools/gpu_ab.sh small   64-tile small-n kernel vs the 128-tile kernels, n = 1024 .. 4096, CTAs per SM
+#   tools/gpu_ab.sh close   small-n phase 1: deferred-bulk closure (default) vs one barrier per step
 #   tools/gpu_ab.sh pair    two-round (pair) queue vs one-round queue, int32 n = 16384 / 32768 / 65536, fp32
 #   tools/gpu_ab.sh ooc     out of core, every band streamed (n = 16384 / 32768, 1 and 2 virtual ranks)
 mkdir -p gpurun_out
@@ -14,6 +15,12 @@ case $what in
       done
       for c in 1 2 3; do echo "== n=1024 ctas=$c"; APSP_SMALL_CTAS=$c python tools/fw_ab.py --n 1024 --deg 8 --dtype i32 --runs 20 --modes small; done
       echo "== n=1024 profile"; APSP_SMALL_PROFILE=1 python tools/fw_ab.py --n 1024 --deg 8 --dtype i32 --runs 3 --modes small
+    } > $out 2>&1 ;;
+  close)
+    { for n in 1024 1536 2048; do for v in 0 1 0 1; do
+        echo "== close_v=$v n=$n"; APSP_SMALL_CLOSE=$v python tools/fw_ab.py --n $n --deg 8 --dtype i32 --runs 20 --modes small
+      done; done
+      for v in 0 1; do echo "== close_v=$v profile"; APSP_SMALL_CLOSE=$v APSP_SMALL_PROFILE=1 python tools/fw_ab.py --n 1024 --deg 8 --dtype i32 --runs 3 --modes small; done
     } > $out 2>&1 ;;
   pair)
     { for n in 16384 32768 65536; do
