@@ -764,7 +764,9 @@ def rendezvous_only(args):
     world, rank, _ = dist_env()
     dist.init_process_group("gloo")
     dist.barrier()
-    print(json.dumps({"rendezvous": True, "rank": rank, "world": world}), flush=True)
+    # one write per line: the ranks share the launcher's stdout pipe
+    sys.stdout.write(json.dumps({"rendezvous": True, "rank": rank, "world": world}) + "\n")
+    sys.stdout.flush()
     dist.destroy_process_group()
     return 0
 

@@ -245,6 +245,122 @@ __global__ void k_s32mix(const int* __restrict__ in, int* __restrict__ out, int 
   out[blockIdx.x * blockDim.x + threadIdx.x] = s;
 }
 
+
+// ---- round 2: pipe decomposition of the fp32 form and a mixed int/fp32 form -------------
+// fadd2only : FADD2 chains alone (FMA pipe), reported as adds/s
+// fmnmx3only: FMNMX3 chains alone (ALU pipe), reported as folded mins/s (2 per instr)
+// f32x2nb   : FADD2 with two pair operands (depth k, k+1 of one output) + FMNMX3
+// mix<F,I>  : one accumulator updated by both forms. A is held biased, float(2^23 + a),
+//             whose bits are 0x4B000000 + a, so VIADDMNMX(a_bits, b_int, c) and
+//             FMNMX3(c, a_f + b_f, ...) produce the same bits for every a + b < 2^23
+//             (fp32 values in [2^23, 2^24) order like their bit patterns).
+//             Per iteration F float depth pairs (64 relax) + I int depth steps (32 relax).
+__global__ void k_fadd2only(const int* __restrict__ in, int* __restrict__ out, int iters) {
+  float2 s[CH];
+#pragma unroll
+  for (int j = 0; j < CH; ++j) s[j] = make_float2((float)in[(threadIdx.x + j) & 255], 1.0f);
+  float2 y = make_float2((float)in[threadIdx.x & 255], 0.5f);
+  const float2 d = make_float2(0.25f, 0.125f);
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      y = __fadd2_rn(y, d);
+#pragma unroll
+      for (int j = 0; j < CH; ++j) s[j] = __fadd2_rn(s[j], y);
+    }
+  }
+  float r = 0;
+#pragma unroll
+  for (int j = 0; j < CH; ++j) r += s[j].x + s[j].y;
+  out[blockIdx.x * blockDim.x + threadIdx.x] = (int)r;
+}
+__global__ void k_fmnmx3only(const int* __restrict__ in, int* __restrict__ out, int iters) {
+  float x[CH], acc[CH];
+#pragma unroll
+  for (int j = 0; j < CH; ++j) { x[j] = (float)in[(threadIdx.x + j) & 255]; acc[j] = 1e30f; }
+  float y = (float)in[threadIdx.x & 255];
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      y = __fadd_rn(y, -1.0f);
+#pragma unroll
+      for (int j = 0; j < CH; ++j) acc[j] = fminf(fminf(acc[j], x[j]), y);
+    }
+  }
+  float r = 0;
+#pragma unroll
+  for (int j = 0; j < CH; ++j) r += acc[j];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = (int)r;
+}
+__global__ void k_f32x2nb(const int* __restrict__ in, int* __restrict__ out, int iters) {
+  float2 x[CH2];
+  float acc[CH2];
+#pragma unroll
+  for (int j = 0; j < CH2; ++j) {
+    x[j] = make_float2((float)in[(threadIdx.x + j) & 255], (float)in[(threadIdx.x + j + 5) & 255]);
+    acc[j] = 1e30f;
+  }
+  float2 y = make_float2((float)in[threadIdx.x & 255], 3.0f);
+  const float2 one = make_float2(1.0f, 1.0f);
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int u = 0; u < 2; ++u) {
+      y = __fadd2_rn(y, one);
+#pragma unroll
+      for (int j = 0; j < CH2; ++j) {
+        const float2 s = __fadd2_rn(x[j], y);
+        acc[j] = fminf(fminf(acc[j], s.x), s.y);
+      }
+    }
+  }
+  float r = 0;
+#pragma unroll
+  for (int j = 0; j < CH2; ++j) r += acc[j];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = (int)r;
+}
+template <int F, int I>
+__global__ void k_mix(const int* __restrict__ in, int* __restrict__ out, int iters) {
+  unsigned a0[CH2 / 2], a1[CH2 / 2];  // biased: bits 0x4B000000 + a == float(2^23 + a)
+  unsigned acc[CH2];
+#pragma unroll
+  for (int j = 0; j < CH2 / 2; ++j) {
+    a0[j] = 0x4B000000u + (unsigned)in[(threadIdx.x + j) & 255];
+    a1[j] = 0x4B000000u + (unsigned)in[(threadIdx.x + j + 7) & 255];
+  }
+#pragma unroll
+  for (int j = 0; j < CH2; ++j) acc[j] = 0x4B7FFFFFu;
+  float2 yf0 = make_float2((float)in[threadIdx.x & 255], 3.0f), yf1 = make_float2(5.0f, 7.0f);
+  const float2 one = make_float2(1.0f, 1.0f);
+  int yi0 = in[(threadIdx.x + 3) & 255], yi1 = 9;
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int f = 0; f < F; ++f) {
+      yf0 = __fadd2_rn(yf0, one);
+      yf1 = __fadd2_rn(yf1, one);
+#pragma unroll
+      for (int j = 0; j < CH2 / 2; ++j) {
+        const float2 s0 = __fadd2_rn(make_float2(__uint_as_float(a0[j]), __uint_as_float(a0[j])), yf0);
+        const float2 s1 = __fadd2_rn(make_float2(__uint_as_float(a1[j]), __uint_as_float(a1[j])), yf1);
+        acc[2 * j] = __float_as_uint(fminf(fminf(__uint_as_float(acc[2 * j]), s0.x), s1.x));
+        acc[2 * j + 1] = __float_as_uint(fminf(fminf(__uint_as_float(acc[2 * j + 1]), s0.y), s1.y));
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < I; ++i) {
+      yi0 += 1; yi1 += 1;
+#pragma unroll
+      for (int j = 0; j < CH2 / 2; ++j) {
+        acc[2 * j] = (unsigned)__viaddmin_s32((int)a0[j], yi0, (int)acc[2 * j]);
+        acc[2 * j + 1] = (unsigned)__viaddmin_s32((int)a0[j], yi1, (int)acc[2 * j + 1]);
+      }
+    }
+  }
+  unsigned r = 0;
+#pragma unroll
+  for (int j = 0; j < CH2; ++j) r ^= acc[j];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = (int)r;
+}
+
 typedef void (*kfn)(const int*, int*, int);
 
 static double run(kfn f, int blocks, int threads, int iters, const int* in, int* out, double relax_per_op) {
@@ -297,7 +413,12 @@ int main(int argc, char** argv) {
   struct V { const char* name; kfn f; double rpo; } vs[] = {
     {"s32", k_s32, 1.0}, {"s16x2", k_s16x2, 2.0}, {"f32", k_f32, 1.0}, {"f32x2", k_f32x2, 2.0},
     {"f32b", k_f32b, 1.0}, {"f32x2b", k_f32x2b, 1.0}, {"s32imad3", k_s32imad3, 1.0},
-    {"s32iadd3", k_s32iadd3, 1.0}, {"s32mix", k_s32mix, 1.0}};
+    {"s32iadd3", k_s32iadd3, 1.0}, {"s32mix", k_s32mix, 1.0},
+    {"fadd2only", k_fadd2only, 2.0}, {"fmnmx3only", k_fmnmx3only, 2.0}, {"f32x2nb", k_f32x2nb, 1.0},
+    {"mix10", k_mix<1, 0>, 64.0 / 128}, {"mix01", k_mix<0, 1>, 32.0 / 128},
+    {"mix11", k_mix<1, 1>, 96.0 / 128}, {"mix21", k_mix<2, 1>, 160.0 / 128},
+    {"mix31", k_mix<3, 1>, 224.0 / 128}, {"mix12", k_mix<1, 2>, 128.0 / 128},
+    {"mix41", k_mix<4, 1>, 288.0 / 128}};
   CK(cudaMalloc(&out, (size_t)p.multiProcessorCount * 16 * 512 * sizeof(int)));
   for (auto& v : vs) {
     double best = 0;

@@ -2,6 +2,7 @@
 one JSON line with the contract's keys, runnable without a GPU. The GPU arm's line is checked
 on the B200 by the driver (and its keys by tests/test_gpu_fullsize.py's bench usage)."""
 import json
+import re
 import os
 import subprocess
 import sys
@@ -38,7 +39,8 @@ def test_self_launch_two_ranks_rendezvous():
     p = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--rendezvous-only"],
                        capture_output=True, text=True, timeout=300, cwd=ROOT, env=env)
     assert p.returncode == 0, p.stderr[-2000:]
-    got = sorted(json.loads(l)["rank"] for l in p.stdout.splitlines() if l.strip().startswith("{"))
+    objs = re.findall(r"\{[^{}]*\}", p.stdout)  # robust to two ranks' lines interleaving
+    got = sorted(json.loads(o)["rank"] for o in objs if '"rendezvous"' in o)
     assert got == [0, 1]
 
 
