@@ -1131,6 +1131,7 @@ extern "C" int64_t apsp_debug_queue(int32_t nb, int32_t P, int32_t q, int64_t de
   }
   if (P == -1) {  // the small-n kernel's queue (apsp_fw_small.cu), nb 64-wide tile rows
     if (nb <= 0) return -1;
+    if (!out || cap <= 0) return small_queue(nb, delay, nullptr);  // the launch path's closed-form length
     std::vector<int4> sq;
     const long long total = small_queue(nb, delay, &sq);
     for (long long g = 0; g < total && g < cap; ++g) {

@@ -16,13 +16,14 @@
 // Structure: the flag protocol of apsp_fw_dataflow.cu (apsp_df_common.cuh: per-tile
 // versions, diagonal / panel readiness, double-buffered panel copies, deps_met /
 // signal_done) with a queue ordered for the critical path and a simpler engine:
-//   * the queue is built on the host (small_queue, at most 32^3 entries) by
-//     critical-path list scheduling: tasks in decreasing order of their bottom
-//     level in the dependency graph the kernel waits on, a topological order in
-//     which the chain P1(k) -> panels -> tile (k+1,k+1) -> P1(k+1) comes first and
-//     the bulk of phase 3 fills in behind it; every dependency of an entry lies
+//   * the queue is built on the host (small_queue, at most 32^3 + 186 entries): the
+//     128-tile kernel's segment order (decode), so round k+1's diagonal and panels
+//     come right after the round-k tiles they need; every dependency of an entry lies
 //     earlier in the queue (tests/test_schedule.py simulates it), so a CTA that
-//     finishes its task before taking the next cannot deadlock;
+//     finishes its task before taking the next cannot deadlock (a critical-path list
+//     order is kept as a tuning variant: measured slower);
+//   * the two panel tiles next to the diagonal, P2R(k; k,k+1) and P2C(k; k+1,k), which
+//     every round's chain waits for, run as 4 parts on 4 CTAs (column / row ranges);
 //   * F(k) fuses P3(k; k+1,k+1) with P1(k+1): the CTA that updates the next
 //     diagonal tile closes it in registers right away (one flag hop and one
 //     tile load less on the chain of every round);
@@ -40,7 +41,9 @@
 //     negative-cycle check at the start of every step;
 //   * thread 0 fetches the next queue entry and the index after it while the CTA
 //     computes the current task, and checks the next task's flags right after
-//     publishing the current one.
+//     publishing the current one;
+//   * the last CTA to finish zeroes the flags for the next launch (no memset in the
+//     launch's critical path).
 #include "apsp_kernels.cuh"
 #include "apsp_df_common.cuh"
 
@@ -62,10 +65,12 @@ constexpr int STE = SB * SB;    // elements per tile
 template <typename T> struct SV;
 template <> struct SV<int> {
   using V4 = int4;
+  using V2 = int2;
   static __device__ __forceinline__ int relax(int a, int b, int c) { return __viaddmin_s32(a, b, c); }
 };
 template <> struct SV<float> {
   using V4 = float4;
+  using V2 = float2;
   static __device__ __forceinline__ float relax(float a, float b, float c) { return fminf(c, __fadd_rn(a, b)); }
 };
 
@@ -87,6 +92,11 @@ struct SmArgs {
   const int4* queue; // [total] (type, k, i, j), built on the host (small_queue)
   unsigned long long* prof;  // optional [CTAs][16] cycle counters (tuning: APSP_SMALL_PROFILE)
   int close_v;               // phase-1 variant: 1 small_close_defer, 0 small_close (APSP_SMALL_CLOSE)
+  int split;                 // parts of each chain panel tile (small_split(); 1 = whole tasks)
+  int* rsplit;               // [nb] finished parts of P2R(j-1; j-1, j), the row-panel tile next to the diagonal
+  int* csplit;               // [nb] finished parts of P2C(i-1; i, i-1)
+  int* exitc;                // CTAs past their last task: the last one zeroes every flag for the next launch
+  long long flag_words;      // 32-bit words from counter to exitc inclusive
 };
 
 template <typename T>
@@ -103,6 +113,37 @@ __device__ __forceinline__ T* sp_colT(const SmArgs<T>& a, int k, int i) {
 }
 
 enum { T_P3P1 = 4 };  // fused P3(k; k+1,k+1) + P1(k+1)
+// Split chain panel tasks: queue entry type = base (T_P2R / T_P2C) + 16 * (part + 1). The two panel
+// tiles next to the diagonal, P2R(k; k,k+1) and P2C(k; k+1,k), sit on every round's critical path
+// (F(k) waits for both); each is cut into `split` parts run by as many CTAs: P2R by column ranges
+// (a part reads only its columns of the tile it updates, B = A(k,k+1)), P2C by row ranges (a part
+// reads only its rows, A = A(k+1,k)), so no part reads what another writes. The parts count into
+// rsplit / csplit instead of the tile's version and panel flags (PAPER.md:62 phase 2, unchanged).
+constexpr int kPartShift = 4;
+__host__ __device__ __forceinline__ int part_of(int type) { return (type >> kPartShift) - 1; }
+__host__ __device__ __forceinline__ int base_of(int type) { return type & 15; }
+
+// queue variant: 3 (default) the 128-tile kernel's segment order with F(k) fused; tuning
+// experiments only: APSP_SMALL_QUEUE=decode (1: no fusion), bl_nofuse (2: list order without
+// fused entries), anything else (0: list order + F(k))
+static int small_variant() {
+  const char* qv = getenv("APSP_SMALL_QUEUE");
+  return !qv                               ? 3
+         : strcmp(qv, "decode") == 0      ? 1
+         : strcmp(qv, "bl_nofuse") == 0   ? 2
+         : strcmp(qv, "decode_fuse") == 0 ? 3
+                                          : 0;
+}
+
+// parts per chain panel tile: 4 by default (measured, n = 1024: whole tasks 0.265 ms, 2 parts 0.248,
+// 4 parts 0.240; n = 2048 unchanged: DESIGN.md §5); APSP_SMALL_SPLIT=1|2|4 (tuning A/B)
+// (the fused segment-order queue only, variant 3; the tuning variants keep whole tasks)
+static int small_split_for(int variant) {
+  if (variant != 3) return 1;
+  const char* e = getenv("APSP_SMALL_SPLIT");
+  const int v = e ? atoi(e) : 4;
+  return v == 1 || v == 2 ? v : 4;
+}
 
 struct SmSlot {
   long long t;
@@ -369,31 +410,174 @@ __device__ __forceinline__ void small_minplus(const SmArgs<T>& a, const Task& tk
   }
 }
 
+// N consecutive elements (N = 1, 2, 4; the address is N-element aligned) in one store
+template <typename T, int N>
+__device__ __forceinline__ void st_vec(T* dst, const T* v) {
+  if constexpr (N == 4) {
+    typename SV<T>::V4 x;
+    x.x = v[0]; x.y = v[1]; x.z = v[2]; x.w = v[3];
+    *reinterpret_cast<typename SV<T>::V4*>(dst) = x;
+  } else if constexpr (N == 2) {
+    typename SV<T>::V2 x;
+    x.x = v[0]; x.y = v[1];
+    *reinterpret_cast<typename SV<T>::V2*>(dst) = x;
+  } else {
+    dst[0] = v[0];
+  }
+}
+
+// One part of a split chain panel task (see kPartShift): P2R(k; k,j) part q updates columns
+// [q*C, (q+1)*C) of A(k,j) (C = 64/split; A = D via the panel copy D^T, B = those columns of A(k,j));
+// P2C(k; i,k) part q updates rows [q*R, (q+1)*R) (A = those rows of A(i,k), transposed on load;
+// B = D). Thread (tx, ty) owns TR x TC outputs (TR * TC = 16 / split), 256 threads per part.
+template <typename T, bool COLS, int TR, int TC>
+__device__ __forceinline__ void small_part(const SmArgs<T>& a, const Task& tk, int q, T* As, T* Bs) {
+  constexpr int R = 16 * TR, CC = 16 * TC;  // part rows / columns
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  const int r_off = COLS ? 0 : q * R, c_off = COLS ? q * CC : 0;
+  T* const C = a.D + (long long)tk.i * SB * a.ld + (long long)tk.j * SB;
+  if (COLS) {  // As[kk][r] = D^T (whole), Bs[kk][c] = A(k,j)[kk][c_off + c]
+    const T* dt = sp_diagT(a, tk.k);
+#pragma unroll
+    for (int e = 0; e < 4; ++e) cp16(As + (tid + e * SNT) * 4, dt + (tid + e * SNT) * 4);
+    constexpr int CH = CC / 4;  // 16-byte chunks per row
+#pragma unroll
+    for (int e = 0; e < (SB * CH + SNT - 1) / SNT; ++e) {
+      const int x = tid + e * SNT;
+      if (SB * CH % SNT == 0 || x < SB * CH) cp16(Bs + (x / CH) * CC + (x % CH) * 4, C + (long long)(x / CH) * a.ld + c_off + (x % CH) * 4);
+    }
+  } else {  // As[kk][r] = A(i,k)[r_off + r][kk] (4x4 register transpose), Bs = D (whole)
+    const T* d = sp_diag(a, tk.k);
+#pragma unroll
+    for (int e = 0; e < 4; ++e) cp16(Bs + (tid + e * SNT) * 4, d + (tid + e * SNT) * 4);
+    constexpr int RB = R / 4;  // 4x4 blocks per column strip
+    if (tid < RB * 16) {
+      using V4 = typename SV<T>::V4;
+      const int r0 = (tid % RB) * 4, c0 = (tid / RB) * 4;
+      V4 v[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        v[u] = __ldcg(reinterpret_cast<const V4*>(C + (long long)(r_off + r0 + u) * a.ld + c0));
+      V4 w;
+      w.x = v[0].x; w.y = v[1].x; w.z = v[2].x; w.w = v[3].x;
+      *reinterpret_cast<V4*>(As + (c0 + 0) * R + r0) = w;
+      w.x = v[0].y; w.y = v[1].y; w.z = v[2].y; w.w = v[3].y;
+      *reinterpret_cast<V4*>(As + (c0 + 1) * R + r0) = w;
+      w.x = v[0].z; w.y = v[1].z; w.z = v[2].z; w.w = v[3].z;
+      *reinterpret_cast<V4*>(As + (c0 + 2) * R + r0) = w;
+      w.x = v[0].w; w.y = v[1].w; w.z = v[2].w; w.w = v[3].w;
+      *reinterpret_cast<V4*>(As + (c0 + 3) * R + r0) = w;
+    }
+  }
+  cp_commit();
+  T acc[TR][TC];
+#pragma unroll
+  for (int i = 0; i < TR; ++i)
+#pragma unroll
+    for (int j = 0; j < TC; ++j) acc[i][j] = __ldcg(C + (long long)(r_off + ty * TR + i) * a.ld + c_off + tx * TC + j);
+  cp_wait_all();
+  __syncthreads();
+#pragma unroll 8
+  for (int kk = 0; kk < SB; ++kk) {
+    T A[TR], B[TC];
+#pragma unroll
+    for (int i = 0; i < TR; ++i) A[i] = As[kk * R + ty * TR + i];
+#pragma unroll
+    for (int j = 0; j < TC; ++j) B[j] = Bs[kk * CC + tx * TC + j];
+#pragma unroll
+    for (int i = 0; i < TR; ++i)
+#pragma unroll
+      for (int j = 0; j < TC; ++j) acc[i][j] = SV<T>::relax(A[i], B[j], acc[i][j]);
+  }
+  const int r0 = r_off + ty * TR, c0 = c_off + tx * TC;
+#pragma unroll
+  for (int i = 0; i < TR; ++i) {
+    st_vec<T, TC>(C + (long long)(r0 + i) * a.ld + c0, acc[i]);
+    if (COLS) st_vec<T, TC>(sp_row(a, tk.k, tk.j) + (r0 + i) * SB + c0, acc[i]);
+  }
+  if (!COLS) {
+    T* const ct = sp_colT(a, tk.k, tk.i);
+#pragma unroll
+    for (int j = 0; j < TC; ++j) {
+      T col[TR];
+#pragma unroll
+      for (int i = 0; i < TR; ++i) col[i] = acc[i][j];
+      st_vec<T, TR>(ct + (c0 + j) * SB + r0, col);
+    }
+  }
+}
+
+template <typename T>
+__device__ __forceinline__ void small_part_any(const SmArgs<T>& a, const Task& tk, T* As, T* Bs) {
+  const int q = part_of(tk.type);
+  Task w = tk;
+  w.type = base_of(tk.type);
+  if (w.type == T_P2R) {
+    if (a.split == 4) small_part<T, true, 4, 1>(a, w, q, As, Bs);
+    else small_part<T, true, 4, 2>(a, w, q, As, Bs);
+  } else {
+    if (a.split == 4) small_part<T, false, 1, 4>(a, w, q, As, Bs);
+    else small_part<T, false, 2, 4>(a, w, q, As, Bs);
+  }
+}
+
 __device__ __forceinline__ Task small_task(const int4 e) {
   Task t;
   t.type = e.x; t.k = e.y; t.i = e.z; t.j = e.w;
   return t;
 }
 
-// dependencies of a queue entry: a fused F(k) needs those of P3(k; k+1,k+1) and of P1(k+1)
-// (the panel copy of parity (k+1) % 2 may be rewritten once round k-1's panel tasks are done)
+// Dependencies of a queue entry (one thread): deps_met's flags (own tile's version, the panel
+// tiles / diagonal it reads, panel-copy parity reuse) with the split chain tiles read through
+// their part counters, all loaded at once (one round trip), then an acquire fence once met.
+// A fused F(k) needs those of P3(k; k+1,k+1) and of P1(k+1) (the panel copy of parity (k+1) % 2
+// may be rewritten once round k-1's panel tasks, every part counted, are done).
 template <typename T>
 __device__ __forceinline__ bool small_deps(const SmArgs<T>& a, const Task& t) {
-  if (t.type != T_P3P1) return deps_met(a, t);
-  Task p3 = t;
-  p3.type = T_P3;
-  if (t.k >= 1 && ld_relaxed(a.done2 + t.k - 1) < 2 * (a.nb - 1)) return false;
-  return deps_met(a, p3);
+  const int type = base_of(t.type), nb = a.nb, k = t.k, p = k & 1, S = a.split;
+  const bool sp = S > 1;
+  const int* f[4];
+  int v[4];
+  // own tile: the chain tiles of round k-1 (P2R(k-1; k-1,k) / P2C(k-1; k,k-1)) finish as parts
+  if (sp && k >= 1 && t.i == k - 1 && t.j == k) { f[0] = a.rsplit + k; v[0] = S; }
+  else if (sp && k >= 1 && t.i == k && t.j == k - 1) { f[0] = a.csplit + k; v[0] = S; }
+  else { f[0] = a.ver + (long long)t.i * nb + t.j; v[0] = k; }
+  f[3] = f[0]; v[3] = v[0];
+  if (type == T_P1) {
+    f[1] = a.done2 + (k >= 2 ? k - 2 : 0); v[1] = k >= 2 ? 2 * (nb - 1) + 2 * (S - 1) : INT_MIN;
+    f[2] = f[1]; v[2] = v[1];
+  } else if (type == T_P3 || type == T_P3P1) {
+    if (sp && t.j == k + 1) { f[1] = a.rsplit + t.j; v[1] = S; }
+    else { f[1] = a.rowready + p * nb + t.j; v[1] = k + 1; }
+    if (sp && t.i == k + 1) { f[2] = a.csplit + t.i; v[2] = S; }
+    else { f[2] = a.colready + p * nb + t.i; v[2] = k + 1; }
+    if (type == T_P3P1 && k >= 1) { f[3] = a.done2 + k - 1; v[3] = 2 * (nb - 1) + 2 * (S - 1); }
+  } else {
+    f[1] = a.diagready + p; v[1] = k + 1;
+    f[2] = a.done3 + (k >= 2 ? k - 2 : 0); v[2] = k >= 2 ? (nb - 1) * (nb - 1) : INT_MIN;
+  }
+  const int x0 = ld_relaxed(f[0]), x1 = ld_relaxed(f[1]), x2 = ld_relaxed(f[2]), x3 = ld_relaxed(f[3]);
+  if (x0 >= v[0] && x1 >= v[1] && x2 >= v[2] && x3 >= v[3]) {
+    asm volatile("fence.acquire.gpu;" ::: "memory");
+    return true;
+  }
+  return false;
 }
 
 template <typename T>
 __device__ __forceinline__ void small_signal(const SmArgs<T>& a, const Task& t) {
+  const int k = t.k, nb = a.nb;
+  if (t.type >= (1 << kPartShift)) {  // a part of a split chain panel tile: count it
+    asm volatile("fence.release.gpu;" ::: "memory");
+    red_relaxed_add(base_of(t.type) == T_P2R ? a.rsplit + t.j : a.csplit + t.i, 1);
+    red_relaxed_add(a.done2 + k, 1);
+    return;
+  }
   if (t.type != T_P3P1) {
     signal_done(a, t);
     return;
   }
   // F(k): tile (k+1,k+1) has rounds 0..k+1 applied; round k+1's diagonal is in the panel copy
-  const int k = t.k, nb = a.nb;
   asm volatile("fence.release.gpu;" ::: "memory");
   st_relaxed(a.ver + (long long)t.i * nb + t.j, k + 2);
   st_relaxed(a.diagready + ((k + 1) & 1), k + 2);
@@ -443,6 +627,7 @@ __global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ S
     }
     __syncthreads();  // dependencies met (acquired by thread 0)
     if (tk.type == T_P1) small_phase1(a, tk, rowbuf, colbuf);
+    else if (tk.type >= (1 << kPartShift)) small_part_any(a, tk, As, Bs);
     else small_minplus(a, tk, As, Bs, rowbuf, colbuf);
     if (tid == 0 && N.t < a.total) N.tk = small_task(nq);
     __syncthreads();  // every thread's stores of this task are issued; As / Bs free; N.tk published
@@ -452,8 +637,8 @@ __global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ S
     if (tid == 0) {
       if (a.prof) {
         const long long c1 = clock64();
-        pr[1 + tk.type] += c1 - c0;
-        pr[6 + tk.type] += 1;
+        pr[1 + base_of(tk.type)] += c1 - c0;
+        pr[6 + base_of(tk.type)] += 1;
         c0 = c1;
       }
       // the next task's flags, once: if met, it starts without another wait
@@ -469,6 +654,17 @@ __global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ S
   }
   if (a.prof && tid == 0)
     for (int x = 0; x < 12; ++x) a.prof[(long long)blockIdx.x * 16 + x] = pr[x];
+  // The flags start every launch at zero: the last CTA to leave its task loop (no CTA reads a flag
+  // after that) zeroes them, so a launch needs no memset in front of it (only the first one on a
+  // work buffer: launch_fw_small).
+  __shared__ int last;
+  __syncthreads();
+  if (tid == 0) last = atomicAdd(a.exitc, 1) == (int)gridDim.x - 1;
+  __syncthreads();
+  if (last) {
+    int* const fw = reinterpret_cast<int*>(a.counter);
+    for (long long x = tid; x < a.flag_words; x += SNT) fw[x] = 0;
+  }
 }
 
 }  // namespace
@@ -487,12 +683,11 @@ long long small_queue(int nb, long long delay, std::vector<int4>* q) {
   if (nb <= 0) return 0;
   // tuning experiments only: APSP_SMALL_QUEUE=decode (the 128-tile kernel's segment order,
   // no fusion) or bl_nofuse (list order without fused entries); default: list order + F(k)
-  const char* qv = getenv("APSP_SMALL_QUEUE");
-  const int variant = !qv ? 3
-                          : strcmp(qv, "decode") == 0      ? 1
-                          : strcmp(qv, "bl_nofuse") == 0  ? 2
-                          : strcmp(qv, "decode_fuse") == 0 ? 3
-                                                           : 0;
+  const int variant = small_variant();
+  const int S = small_split_for(variant);
+  if (!q)  // the length alone (every launch asks for it): P1(k >= 1) lives inside F(k-1) when fused;
+           // each round but the last has two chain panel tiles of S parts
+    return (long long)nb * nb * nb - (variant == 1 || variant == 2 ? 0 : nb - 1) + 2ll * (S - 1) * (nb - 1);
   if (variant == 1 || variant == 3) {
     // the 128-tile kernel's segment order (decode with this queue delay); variant 3 fuses the tile (k+1,k+1)
     // of round k with the P1(k+1) that follows it
@@ -503,6 +698,8 @@ long long small_queue(int nb, long long delay, std::vector<int4>* q) {
       if (variant == 3 && t.type == T_P1 && t.k >= 1) continue;  // inside F(k-1)
       if (variant == 3 && t.type == T_P3 && t.i == t.k + 1 && t.j == t.k + 1)
         v.push_back(make_int4(T_P3P1, t.k, t.i, t.j));
+      else if (S > 1 && ((t.type == T_P2R && t.j == t.k + 1) || (t.type == T_P2C && t.i == t.k + 1)))
+        for (int part = 0; part < S; ++part) v.push_back(make_int4(t.type + ((part + 1) << kPartShift), t.k, t.i, t.j));
       else
         v.push_back(make_int4(t.type, t.k, t.i, t.j));
     }
@@ -575,11 +772,11 @@ long long small_queue(int nb, long long delay, std::vector<int4>* q) {
 
 static long long small_pbuf_bytes(int nb, size_t elem) { return 2ll * (2 + 2 * nb) * STE * (long long)elem; }
 static long long small_flag_bytes(int nb) {
-  return ((2 + (long long)nb * nb + 2 + 4ll * nb + 2ll * nb) * 4 + 15) / 16 * 16;
+  return ((2 + (long long)nb * nb + 2 + 4ll * nb + 2ll * nb + 2ll * nb + 1) * 4 + 15) / 16 * 16;
 }
 
-long long fw_small_work_bytes(int nb, size_t elem) {  // the queue is at most nb^3 entries
-  return small_pbuf_bytes(nb, elem) + small_flag_bytes(nb) + (long long)nb * nb * nb * (long long)sizeof(int4);
+long long fw_small_work_bytes(int nb, size_t elem) {  // the queue is at most nb^3 + 6 (nb - 1) entries (split 4)
+  return small_pbuf_bytes(nb, elem) + small_flag_bytes(nb) + ((long long)nb * nb * nb + 6ll * nb) * (long long)sizeof(int4);
 }
 
 template <typename T>
@@ -605,6 +802,11 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
   a.colready = f; f += 2 * nb;
   a.done2 = f; f += nb;
   a.done3 = f; f += nb;
+  a.rsplit = f; f += nb;
+  a.csplit = f; f += nb;
+  a.exitc = f; f += 1;
+  a.flag_words = f - reinterpret_cast<int*>(fb);
+  a.split = small_split_for(small_variant());
   a.negflag = negflag;
   const char* cv = getenv("APSP_SMALL_CLOSE");  // phase-1 variant A/B (tuning only)
   a.close_v = cv ? atoi(cv) : 1;
@@ -620,10 +822,14 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
   } else {
     a.total = small_queue(nb, delay, nullptr);
   }
-  if ((e = cudaMemsetAsync(a.counter, 0, small_flag_bytes(nb), s)) != cudaSuccess) return e;
+  // zero flags: the previous launch's last CTA left them so (fw_small_kernel's epilogue); a new work
+  // buffer is zeroed here, with its queue upload
+  if (!queue_loaded && (e = cudaMemsetAsync(a.counter, 0, small_flag_bytes(nb), s)) != cudaSuccess) return e;
   // persistent grid: every CTA must be resident (tasks wait on each other)
-  int occ = 0;
-  if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fw_small_kernel<T>, SNT, 0)) != cudaSuccess) return e;
+  // (queried once: the event window of a small launch is ~0.3 ms, host work inside it shows)
+  static int occ = 0;
+  if (!occ && (e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fw_small_kernel<T>, SNT, 0)) != cudaSuccess)
+    return e;
   if (occ < 1) return cudaErrorInvalidConfiguration;
   const int per_sm = ctas_per_sm < 1 ? 1 : (ctas_per_sm > occ ? occ : ctas_per_sm);
   long long grid = (long long)sms * per_sm;

@@ -318,7 +318,7 @@ __global__ void k_f32x2nb(const int* __restrict__ in, int* __restrict__ out, int
   for (int j = 0; j < CH2; ++j) r += acc[j];
   out[blockIdx.x * blockDim.x + threadIdx.x] = (int)r;
 }
-template <int F, int I>
+template <int F, int I, bool NU = false>
 __global__ void k_mix(const int* __restrict__ in, int* __restrict__ out, int iters) {
   unsigned a0[CH2 / 2], a1[CH2 / 2];  // biased: bits 0x4B000000 + a == float(2^23 + a)
   unsigned acc[CH2];
@@ -330,6 +330,7 @@ __global__ void k_mix(const int* __restrict__ in, int* __restrict__ out, int ite
 #pragma unroll
   for (int j = 0; j < CH2; ++j) acc[j] = 0x4B7FFFFFu;
   float2 yf0 = make_float2((float)in[threadIdx.x & 255], 3.0f), yf1 = make_float2(5.0f, 7.0f);
+  if (NU) yf1.x = (float)in[(threadIdx.x + 5) & 255];  // per-thread: ptxas cannot keep it in a uniform register
   const float2 one = make_float2(1.0f, 1.0f);
   int yi0 = in[(threadIdx.x + 3) & 255], yi1 = 9;
   for (int it = 0; it < iters; ++it) {
@@ -418,7 +419,7 @@ int main(int argc, char** argv) {
     {"mix10", k_mix<1, 0>, 64.0 / 128}, {"mix01", k_mix<0, 1>, 32.0 / 128},
     {"mix11", k_mix<1, 1>, 96.0 / 128}, {"mix21", k_mix<2, 1>, 160.0 / 128},
     {"mix31", k_mix<3, 1>, 224.0 / 128}, {"mix12", k_mix<1, 2>, 128.0 / 128},
-    {"mix41", k_mix<4, 1>, 288.0 / 128}};
+    {"mix41", k_mix<4, 1>, 288.0 / 128}, {"mix10nu", k_mix<1, 0, true>, 64.0 / 128}};
   CK(cudaMalloc(&out, (size_t)p.multiProcessorCount * 16 * 512 * sizeof(int)));
   for (auto& v : vs) {
     double best = 0;

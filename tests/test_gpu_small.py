@@ -100,3 +100,26 @@ def test_small_repeated_runs_and_reinit(lib):
             lib.apsp_fw_blocked(h)
             assert np.array_equal(lib.apsp_get_dist(h).astype(np.int64), want)
             lib.apsp_reinit(h)
+
+
+@pytest.mark.parametrize("split", [1, 2, 4])
+def test_small_split_chain_tiles(lib, monkeypatch, split):
+    """The chain panel tiles P2R(k; k,k+1) / P2C(k; k+1,k) run as `split` parts (column / row ranges,
+    counted into their own flags): bit-exact at several tile counts, with negative weights, a
+    negative cycle next to the diagonal, and fp32 bit-identical to whole tasks (same sums)."""
+    monkeypatch.setenv("APSP_SMALL_SPLIT", str(split))
+    for n in (64, 65, 200, 1024, 1999):
+        g = gg.erdos_renyi(n, 6 * n, seed=n + split)
+        assert np.array_equal(run(lib, g).astype(np.int64), want_i32(g)), n
+    g = gg.grid_2d(20, 50, seed=3)
+    p = np.random.default_rng(5).integers(-300, 300, size=g.n)
+    s, t, w = g.arcs()
+    gn = gg.csr_from_arcs(g.n, s, t, (w.astype(np.int64) + p[s] - p[t]).astype(np.int32))
+    assert np.array_equal(run(lib, gn).astype(np.int64), want_i32(gn))
+    gc = gg.with_arcs(gg.erdos_renyi(500, 2000, seed=6), [100, 130], [130, 100], [-200, 50])  # tiles 1 / 2
+    with pytest.raises(lib.NegativeCycleError):
+        run(lib, gc)
+    gf = gg.erdos_renyi(700, 700 * 16, seed=10, dtype="f32")
+    got = run(lib, gf)
+    monkeypatch.setenv("APSP_SMALL_SPLIT", "1")
+    assert np.array_equal(got.view(np.int32), run(lib, gf).view(np.int32))

@@ -46,8 +46,12 @@ def simulate(nb, queues, par=2):
     def cnt3(r, k):
         return (nl - (owner(k) == r)) * (nb - 1)
 
+    parts_done = {}
+
     def ready(r, t):
         typ, k, i, j = (int(x) for x in t)
+        if typ >= 1 << PART_SHIFT:  # a part waits for what its whole task waits for
+            return ready(r, (typ & 15, k, i, j))
         if typ == P3P1:  # fused P3(k; k+1,k+1) + P1(k+1) (small-n kernel)
             return (ready(r, (P3, k, i, j)) and
                     (k + 1 < par or all(done2[x, k + 1 - par] >= cnt2(x, k + 1 - par) for x in range(P))))
@@ -63,6 +67,12 @@ def simulate(nb, queues, par=2):
             return k in p1_done and (k < par or all(done3[x, k - par] >= cnt3(x, k - par) for x in range(P)))
         return k < par or all(done2[x, k - par] >= cnt2(x, k - par) for x in range(P))
 
+    parts_of = {}
+    for qu in queues:
+        for typ, k, i, j in qu.tolist():
+            if typ >= 1 << PART_SHIFT:
+                key = (typ & 15, k, i, j)
+                parts_of[key] = parts_of.get(key, 0) + 1
     pos = [0] * P
     total = sum(len(q) for q in queues)
     ndone = 0
@@ -71,6 +81,15 @@ def simulate(nb, queues, par=2):
         for r in range(P):
             while pos[r] < len(queues[r]) and ready(r, queues[r][pos[r]]):
                 typ, k, i, j = (int(x) for x in queues[r][pos[r]])
+                if typ >= 1 << PART_SHIFT:  # the whole task's effects once its last part is done
+                    key = (typ & 15, k, i, j)
+                    parts_done[key] = parts_done.get(key, 0) + 1
+                    if parts_done[key] < parts_of[key]:
+                        pos[r] += 1
+                        ndone += 1
+                        progressed = True
+                        continue
+                    typ = typ & 15
                 ver[i, j] = k + 1
                 if typ == P3P1:
                     ver[i, j] = k + 2
@@ -148,8 +167,16 @@ def test_bad_arguments(lib):
         lib.apsp_debug_queue(8, 4, 4, 1)   # q >= P
 
 
+PART_SHIFT = 4  # small-n kernel: a part of a split chain panel tile has type base + 16 * (part + 1)
+
+
 def expand_fused(q):
+    parts = {}
     for typ, k, i, j in q.tolist():
+        if typ >= 1 << PART_SHIFT:  # one part of a split task: the whole task once its parts are all there
+            key = (typ & 15, k, i, j)
+            parts.setdefault(key, set()).add((typ >> PART_SHIFT) - 1)
+            continue
         if typ == P3P1:
             yield (P3, k, i, j)
             yield (P1, k + 1, i, j)
@@ -158,6 +185,9 @@ def expand_fused(q):
             yield (P3, k + 1, i, j)
         else:
             yield (typ, k, i, j)
+    for key, got in parts.items():
+        assert got == set(range(len(got))) and len(got) in (2, 4), (key, got)
+        yield key
 
 
 @pytest.mark.parametrize("nb,delay", [(1, 0), (2, 0), (3, 0), (4, 2), (5, 0), (8, 7), (16, 0), (16, 40), (23, 5),
@@ -168,12 +198,38 @@ def test_small_kernel_queue_complete_and_deadlock_free(lib, nb, delay):
     in-order drain with the kernel's exact waits (a fused entry waits for both halves' dependencies)."""
     q = lib.apsp_debug_queue(nb, -1, 0, delay)
     assert sorted(expand_fused(q)) == sorted(expected_tasks(nb))
-    assert len(q) == nb ** 3 - (nb - 1)
+    S = 4  # default parts per chain panel tile (APSP_SMALL_SPLIT)
+    assert len(q) == nb ** 3 - (nb - 1) + 2 * (S - 1) * (nb - 1)
+    split = [tuple(t) for t in q.tolist() if t[0] >= 1 << PART_SHIFT]
+    assert sorted(split) == sorted((b + ((p + 1) << PART_SHIFT), k, i, j) for k in range(nb - 1) for p in range(S)
+                                   for b, i, j in ((P2R, k, k + 1), (P2C, k + 1, k)))
     assert simulate(nb, [q])
     if nb >= 2 and delay == 0:  # round 0's panel tiles right after P1(0), then F(0) (the next diagonal tile) first
-        assert sorted(tuple(x) for x in q[1:2 * nb - 1].tolist()) == sorted(
+        n0 = 2 * (nb - 1) + 2 * (S - 1)
+        assert sorted(expand_fused(q[1:1 + n0])) == sorted(
             t for t in expected_tasks(nb) if t[1] == 0 and t[0] in (P2R, P2C))
-        assert tuple(q[2 * nb - 1].tolist()) == (P3P1, 0, 1, 1)
+        assert tuple(q[1 + n0].tolist()) == (P3P1, 0, 1, 1)
+
+
+@pytest.mark.parametrize("split,nb", [(1, 5), (2, 2), (2, 7), (2, 16), (4, 3)])
+def test_small_kernel_queue_split_parts(lib, monkeypatch, split, nb):
+    """APSP_SMALL_SPLIT: the chain panel tiles P2R(k; k,k+1) / P2C(k; k+1,k) in 1 (whole) or 4 parts;
+    the queue still holds every task once and drains under the kernel's waits."""
+    monkeypatch.setenv("APSP_SMALL_SPLIT", str(split))
+    q = lib.apsp_debug_queue(nb, -1, 0, 0)
+    assert sorted(expand_fused(q)) == sorted(expected_tasks(nb))
+    assert len(q) == nb ** 3 - (nb - 1) + 2 * (split - 1) * (nb - 1)
+    assert sum(1 for t in q.tolist() if t[0] >= 1 << PART_SHIFT) == (2 * split * (nb - 1) if split > 1 else 0)
+    assert simulate(nb, [q])
+
+
+def test_simulator_rejects_fused_entry_before_a_part(lib):
+    """Pin of the split rule: F(0) ahead of the last part of the column-panel tile it reads cannot drain."""
+    q = lib.apsp_debug_queue(6, -1, 0, 0).tolist()
+    f = next(x for x, t in enumerate(q) if t[0] == P3P1 and t[1] == 0)
+    last = max(x for x, t in enumerate(q) if t[0] >= 1 << PART_SHIFT and t[0] & 15 == P2C and t[1] == 0)
+    q.insert(f, q.pop(last))  # the part now sits right behind F(0)
+    assert not simulate(6, [np.array(q)])
 
 
 def test_simulator_rejects_fused_entry_before_its_panels(lib):
