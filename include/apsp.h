@@ -136,7 +136,17 @@ typedef struct {
                                    2 = TMA persistent (an A/B experiment, measured slower) */
   int32_t dataflow_delay;       /* dataflow kernel queue delay (phase-3 tasks of round k-1
                                    queued before round k's panels); 0 = auto */
-  int32_t reserved[4];          /* must be 0 (APSP_EINVAL otherwise) */
+  int32_t exact_f32;            /* 1 = int32 inputs with weights in [0, W] and
+                                   2 (n - 1) W <= 2^24 are closed by the fp32 engine
+                                   (FADD2 + FMNMX3 instead of VIADDMNMX): every candidate
+                                   sum of the blocked FW is an integer of magnitude <= 2^24,
+                                   so each fp32 add is exact and the int32 output is
+                                   bit-exact (R25, a proof before the run, no
+                                   check after it). Single-GPU in-core 128-tile dataflow
+                                   schedule only (n_pad > 2048); ignored elsewhere and for
+                                   graphs outside the bound. apsp_info.arith reports
+                                   APSP_ARITH_F32_EXACT when it applies */
+  int32_t reserved[3];          /* must be 0 (APSP_EINVAL otherwise) */
 } apsp_config;
 
 /* Fill *cfg with defaults (struct_size set, device -1, world 1, rank 0). */
@@ -413,7 +423,7 @@ typedef struct {
   int64_t edges_scanned;                       /* Johnson: arcs relaxed by the last run, else 0 */
   int32_t kernel;                              /* APSP_KERNEL_*: what ran the last blocked-FW
                                                   closure (0 = none yet / other methods) */
-  int32_t pad0;
+  int32_t exact_f32_eligible;                  /* exact_f32 requested and the input allows it */
 } apsp_info;
 
 #define APSP_KERNEL_PER_PHASE 1      /* launch-per-phase rounds (phase1 / min-plus kernels) */
@@ -428,6 +438,9 @@ typedef struct {
 #define APSP_ARITH_S16X2 1 /* VIADDMNMX.S16x2, 2 relaxations / instruction, verified exact */
 #define APSP_ARITH_F32 2   /* fp32: FADD2 (one A value against a column pair) + FMNMX3
                               (two depth steps folded into one accumulator update) */
+#define APSP_ARITH_F32_EXACT 3 /* int32 distances closed by the fp32 engine (apsp_config.exact_f32,
+                                  R25): the matrix converted to fp32 in place before the
+                                  closure and back after it; bit-exact by the a priori bound */
 
 apsp_status apsp_get_info(const apsp_handle* h, apsp_info* info);
 

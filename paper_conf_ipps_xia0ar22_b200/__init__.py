@@ -60,7 +60,8 @@ class apsp_config(ctypes.Structure):
         ("force_nccl", ctypes.c_int32),
         ("minplus_variant", ctypes.c_int32),
         ("dataflow_delay", ctypes.c_int32),
-        ("reserved", ctypes.c_int32 * 4),
+        ("exact_f32", ctypes.c_int32),
+        ("reserved", ctypes.c_int32 * 3),
     ]
 
 
@@ -74,16 +75,16 @@ class apsp_info(ctypes.Structure):
         ("arith", ctypes.c_int32), ("packed16_eligible", ctypes.c_int32),
         ("boundary_nodes", ctypes.c_int64),
         ("edges_scanned", ctypes.c_int64),
-        ("kernel", ctypes.c_int32), ("pad0", ctypes.c_int32),
+        ("kernel", ctypes.c_int32), ("exact_f32_eligible", ctypes.c_int32),
     ]
 
 
-APSP_ARITH_I32, APSP_ARITH_S16X2, APSP_ARITH_F32 = 0, 1, 2
+APSP_ARITH_I32, APSP_ARITH_S16X2, APSP_ARITH_F32, APSP_ARITH_F32_EXACT = 0, 1, 2, 3
 (APSP_KERNEL_PER_PHASE, APSP_KERNEL_DATAFLOW, APSP_KERNEL_DATAFLOW_PAIR, APSP_KERNEL_SMALL, APSP_KERNEL_DATAFLOW16,
  APSP_KERNEL_SHARDED, APSP_KERNEL_OUT_OF_CORE) = range(1, 8)
 KERNEL_NAMES = {0: "none", 1: "per_phase", 2: "dataflow", 3: "dataflow_pair", 4: "small64", 5: "dataflow16",
                 6: "sharded_dataflow", 7: "out_of_core"}
-ARITH_NAMES = {0: "i32", 1: "s16x2", 2: "f32"}
+ARITH_NAMES = {0: "i32", 1: "s16x2", 2: "f32", 3: "f32_exact"}
 
 
 class apsp_selection(ctypes.Structure):

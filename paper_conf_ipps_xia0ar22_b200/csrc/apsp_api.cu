@@ -288,7 +288,7 @@ static apsp_status run_small(Handle* h) {
 }
 
 template <typename T>
-static apsp_status run_dataflow(Handle* h) {
+static apsp_status run_dataflow(Handle* h, bool timed = true) {
   if (h->small) return run_small<T>(h);
   const int nb = (int)(h->n_pad / h->b);
   apsp_status st;
@@ -309,14 +309,14 @@ static apsp_status run_dataflow(Handle* h) {
   const bool want_prof = getenv("APSP_DF_PROFILE") != nullptr;
   const size_t prof_bytes = (size_t)sms * 2 * 8 * sizeof(unsigned long long);  // 2 groups per SM
   if (want_prof && (st = h->cuda(cudaMalloc(&prof, prof_bytes), "cudaMalloc prof"))) return st;
-  h->ev_begin(2);
+  if (timed) h->ev_begin(2);
   int used_pair = 0;
   if ((st = h->cuda(launch_fw_dataflow<T>(static_cast<T*>(h->shards[0].D), h->ld, nb, h->df_work, h->d_flag, delay,
                                           stagger, h->stream, prof, &used_pair),
                     "fw_dataflow")))
     return st;
   h->kernel = used_pair ? APSP_KERNEL_DATAFLOW_PAIR : APSP_KERNEL_DATAFLOW;
-  h->ev_end((double)h->n_pad * h->n_pad * h->n_pad);
+  if (timed) h->ev_end((double)h->n_pad * h->n_pad * h->n_pad);
   if (want_prof) {
     std::vector<unsigned long long> hp(prof_bytes / 8);
     cudaStreamSynchronize(h->stream);
@@ -469,10 +469,30 @@ static apsp_status prepare_sharded_peers(Handle* h) {
   return APSP_OK;
 }
 
+// R25 (apsp_config.exact_f32): an int32 matrix whose every candidate sum is an integer of
+// magnitude <= 2^24 (checked at init: weights in [0, W], 2 (n - 1) W <= 2^24) is closed by the
+// fp32 engine: converted to fp32 in place (APSP_INF_I32 -> +inf), one fp32 dataflow launch,
+// converted back. Each fp32 add then returns the exact integer sum and min is exact, so the
+// result is the int32 APSP bit for bit. The two conversions are inside the closure's event.
+static apsp_status run_dataflow_f32x(Handle* h) {
+  const long long count = h->rows_per_rank * h->ld;
+  int* const D = static_cast<int*>(h->shards[0].D);
+  apsp_status st;
+  h->ev_begin(2);
+  if ((st = h->cuda(launch_i32_to_f32(D, count, h->stream), "i32 -> f32"))) return st;
+  if ((st = run_dataflow<float>(h, false))) return st;
+  if ((st = h->cuda(launch_f32_to_i32(reinterpret_cast<float*>(D), count, h->stream), "f32 -> i32"))) return st;
+  h->ev_end((double)h->n_pad * h->n_pad * h->n_pad);
+  h->arith = APSP_ARITH_F32_EXACT;
+  return APSP_OK;
+}
+
 apsp_status run_incore_rounds(Handle* h, long long k0, long long k1) {
   h->kernel = APSP_KERNEL_PER_PHASE;  // (the dataflow / sharded paths below set their own)
-  if (h->world == 1 && !h->use_comm && !h->virt && h->dataflow && k0 == 0 && k1 == h->n_pad / h->b)
+  if (h->world == 1 && !h->use_comm && !h->virt && h->dataflow && k0 == 0 && k1 == h->n_pad / h->b) {
+    if (h->modef32x && !h->small) return run_dataflow_f32x(h);
     return h->dtype == APSP_I32 ? run_dataflow<int>(h) : run_dataflow<float>(h);
+  }
   if ((h->virt || h->use_comm) && h->dataflow && h->world <= 8 && k0 == 0 && k1 == h->n_pad / h->b) {
     apsp_status st;
     if (!h->virt &&
@@ -602,6 +622,7 @@ static apsp_status load_config(const apsp_config* cfg_in, apsp_config* cfg) {
   if (cfg->minplus_variant < 0 || cfg->minplus_variant > 2)
     return fail_global(APSP_EINVAL, "apsp_config.minplus_variant must be 0, 1 or 2");
   if (cfg->dataflow_delay < 0) return fail_global(APSP_EINVAL, "apsp_config.dataflow_delay < 0");
+  if (cfg->exact_f32 != 0 && cfg->exact_f32 != 1) return fail_global(APSP_EINVAL, "apsp_config.exact_f32 must be 0 or 1");
   if (cfg->dist_device_bytes < 0) return fail_global(APSP_EINVAL, "apsp_config.dist_device_bytes < 0");
   return APSP_OK;
 }
@@ -980,6 +1001,8 @@ apsp_status apsp_load_csr(apsp_handle* hh, const int64_t* row_ptr, const int32_t
   h->max_abs_w = maxabs;
   // packed16 handle (R16): int16 again if this graph is eligible, else straight to int32
   if (h->mode16) h->fell_back16 = has_neg || maxabs > 8191;
+  h->modef32x = f32x_eligible(h);  // R25: decided per graph
+  if (h->dtype == APSP_I32 && !h->mode16) h->arith = h->modef32x ? APSP_ARITH_F32_EXACT : APSP_ARITH_I32;
   return load_csr(h, row_ptr, col_idx, weights);
 }
 
@@ -1068,6 +1091,7 @@ apsp_status apsp_get_info(const apsp_handle* hh, apsp_info* info) {
   info->boundary_nodes = bnd_boundary_nodes(h);
   info->edges_scanned = jn_edges(h);
   info->kernel = h->kernel;
+  info->exact_f32_eligible = h->modef32x ? 1 : 0;
   return APSP_OK;
 }
 

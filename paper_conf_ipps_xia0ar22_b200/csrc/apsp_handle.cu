@@ -99,6 +99,20 @@ apsp_status load_csr(Handle* h, const int64_t* row_ptr, const int32_t* col, cons
   return run_init(h);
 }
 
+// R25: every candidate sum a + b of the blocked FW is a sum of two restricted shortest-path
+// lengths (phase 3: panel entries final for the round; phases 1-2: FW within a tile),
+// each of at most n - 1 arcs of weight in [0, W], so |a + b| <= 2 (n - 1) W. With that <= 2^24
+// every sum is an integer fp32 represents exactly, one RN add returns it, and min is exact: the
+// fp32 closure equals the int32 one. Non-negative weights (no negative cycles, no drift below 0),
+// single-GPU in-core 128-tile dataflow schedule (the path run_dataflow_f32x takes).
+bool f32x_eligible(const Handle* h) {
+  if (!h->want_f32x || h->dtype != APSP_I32 || h->has_neg || h->mode16) return false;
+  if (h->mode != APSP_MODE_INCORE || h->world != 1 || h->virt || h->use_comm || !h->dataflow || h->small)
+    return false;
+  const double bound = 2.0 * (double)(h->n > 0 ? h->n - 1 : 0) * (double)h->max_abs_w;
+  return bound <= 16777216.0;
+}
+
 // a1: CSR -> dense for every local shard, from the device CSR.
 apsp_status run_init(Handle* h) {
   apsp_status st;
@@ -288,6 +302,11 @@ static apsp_status init_placement(Handle* h, const apsp_config& cfg, const int64
     if ((st = run_init(h))) return st;
     return h->cuda(cudaStreamSynchronize(h->stream), "init sync");
   }
+
+  // R25 exact fp32 closure (apsp_config.exact_f32): decided per graph (f32x_eligible)
+  h->want_f32x = cfg.exact_f32 == 1;
+  h->modef32x = f32x_eligible(h);
+  if (h->modef32x) h->arith = APSP_ARITH_F32_EXACT;
 
   if (cfg.dist_device) {
     h->dist_external = true;

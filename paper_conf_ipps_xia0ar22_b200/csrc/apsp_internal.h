@@ -63,6 +63,9 @@ struct Handle {
   cudaStream_t copy_stream = nullptr;
   cudaEvent_t copy_ev[4] = {nullptr, nullptr, nullptr, nullptr};  // widened[2], copied[2]
   int arith = APSP_ARITH_I32;
+  // R25 exact-fp32 closure of an int32 matrix (apsp_config.exact_f32 and the bound holds)
+  bool modef32x = false;
+  bool want_f32x = false;   // apsp_config.exact_f32 (re-checked against each graph loaded)
   // placement
   int device = 0;
   int world = 1, rank = 0;
@@ -138,6 +141,8 @@ struct Handle {
 
 apsp_status init_handle(Handle* h, const apsp_config& cfg, const int64_t* row_ptr, const int32_t* col,
                         const void* w);
+// R25: may this handle's current graph be closed by the fp32 engine exactly? (apsp_handle.cu)
+bool f32x_eligible(const Handle* h);
 void delete_handle(Handle* h);
 apsp_status run_init(Handle* h);
 apsp_status run_fw16(Handle* h);  // packed int16 closure, verify, int32 fallback

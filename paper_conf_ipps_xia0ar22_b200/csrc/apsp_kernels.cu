@@ -642,6 +642,46 @@ cudaError_t launch_canonicalize_i32(int* D, long long ld, long long rows, long l
   return cudaGetLastError();
 }
 
+// R25 (apsp_config.exact_f32): an int32 matrix to fp32 and back, in place, 16 B per thread and
+// step (count is a multiple of 4: n_pad is a multiple of 128). APSP_INF_I32 <-> +inf; every
+// other value is an integer of magnitude <= 2^24, exact in fp32 both ways.
+__global__ void i32_to_f32_kernel(int4* D, long long count4) {
+  const int INF = 0x3FFFFFFF;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < count4;
+       i += (long long)gridDim.x * blockDim.x) {
+    const int4 v = D[i];
+    float4 f;
+    f.x = v.x == INF ? __int_as_float(0x7f800000) : (float)v.x;
+    f.y = v.y == INF ? __int_as_float(0x7f800000) : (float)v.y;
+    f.z = v.z == INF ? __int_as_float(0x7f800000) : (float)v.z;
+    f.w = v.w == INF ? __int_as_float(0x7f800000) : (float)v.w;
+    reinterpret_cast<float4*>(D)[i] = f;
+  }
+}
+__global__ void f32_to_i32_kernel(float4* D, long long count4) {
+  const int INF = 0x3FFFFFFF;
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < count4;
+       i += (long long)gridDim.x * blockDim.x) {
+    const float4 f = D[i];
+    int4 v;
+    v.x = isinf(f.x) ? INF : __float2int_rn(f.x);
+    v.y = isinf(f.y) ? INF : __float2int_rn(f.y);
+    v.z = isinf(f.z) ? INF : __float2int_rn(f.z);
+    v.w = isinf(f.w) ? INF : __float2int_rn(f.w);
+    reinterpret_cast<int4*>(D)[i] = v;
+  }
+}
+cudaError_t launch_i32_to_f32(int* D, long long count, cudaStream_t s) {
+  if (count <= 0) return cudaSuccess;
+  i32_to_f32_kernel<<<148 * 8, 256, 0, s>>>(reinterpret_cast<int4*>(D), count / 4);
+  return cudaGetLastError();
+}
+cudaError_t launch_f32_to_i32(float* D, long long count, cudaStream_t s) {
+  if (count <= 0) return cudaSuccess;
+  f32_to_i32_kernel<<<148 * 8, 256, 0, s>>>(reinterpret_cast<float4*>(D), count / 4);
+  return cudaGetLastError();
+}
+
 // ------------------------------------------------------ batched min-plus --
 
 template <typename T>

@@ -75,6 +75,11 @@ cudaError_t launch_init_rows(T* D, long long ld, long long n_pad, long long row_
 // weights, reading R5). rows x cols block at ld.
 cudaError_t launch_canonicalize_i32(int* D, long long ld, long long rows, long long cols, cudaStream_t s);
 
+// R25 (apsp_config.exact_f32): count int32 entries to fp32 in place (APSP_INF_I32 -> +inf) and
+// back (+inf -> APSP_INF_I32); count % 4 == 0, 16-byte aligned.
+cudaError_t launch_i32_to_f32(int* D, long long count, cudaStream_t s);
+cudaError_t launch_f32_to_i32(float* D, long long count, cudaStream_t s);
+
 // Per-device kernel attributes (dynamic shared memory opt-in). Call once per
 // device before the first launch.
 cudaError_t configure_kernels();

@@ -137,7 +137,7 @@ def test_config_named_fields_and_reserved(lib):
     (checked before any device work, so APSP_EINVAL even without a GPU)."""
     names = [f[0] for f in lib.apsp_config._fields_]
     for f in ("dist_device", "dist_device_bytes", "schedule", "no_lookahead", "ooc_stream_all", "force_nccl",
-              "minplus_variant", "dataflow_delay", "reserved"):
+              "minplus_variant", "dataflow_delay", "exact_f32", "reserved"):
         assert f in names, f
     hdr = open(os.path.join(ROOT, "include", "apsp.h")).read()
     body = hdr[hdr.index("typedef struct {\n  int32_t struct_size;"):hdr.index("} apsp_config;")]
@@ -145,7 +145,8 @@ def test_config_named_fields_and_reserved(lib):
     assert re.findall(r"\b(\w+)(?:\[\d+\])?;", body) == names  # same order as the C struct
     assert (lib.APSP_SCHED_AUTO, lib.APSP_SCHED_PER_PHASE, lib.APSP_SCHED_DATAFLOW) == (0, 1, 2)
     g = gg.erdos_renyi(20, 60, seed=1)
-    for field, val in (("reserved", 1), ("schedule", 7), ("minplus_variant", 3), ("dataflow_delay", -1)):
+    for field, val in (("reserved", 1), ("schedule", 7), ("minplus_variant", 3), ("dataflow_delay", -1),
+                       ("exact_f32", 2)):
         cfg = lib.apsp_config_default()
         if field == "reserved":
             cfg.reserved[2] = val
@@ -189,4 +190,4 @@ def test_kernel_ids_match_header(lib):
              "DATAFLOW16": "dataflow16", "SHARDED": "sharded_dataflow", "OUT_OF_CORE": "out_of_core"}
     for v, k in ids.items():
         assert lib.KERNEL_NAMES[v] == names[k]
-    assert [f[0] for f in lib.apsp_info._fields_][-2:] == ["kernel", "pad0"]
+    assert [f[0] for f in lib.apsp_info._fields_][-2:] == ["kernel", "exact_f32_eligible"]

@@ -26,6 +26,7 @@ def main():
     ap.add_argument("--runs", type=int, default=2)
     ap.add_argument("--modes", nargs="+", default=["dataflow", "per_phase"])
     ap.add_argument("--packed16", action="store_true", help="int32 input solved on the packed int16 path")
+    ap.add_argument("--exact-f32", action="store_true", help="int32 input closed by the fp32 engine (R25)")
     ap.add_argument("--delay", type=int, default=0, help="apsp_config.dataflow_delay (0 = auto)")
     a = ap.parse_args()
     g = gg.erdos_renyi(a.n, a.deg * a.n, seed=4, dtype=a.dtype)
@@ -33,7 +34,7 @@ def main():
     for name, legacy in (("dataflow", 2), ("per_phase", 1), ("small", 3), ("auto", 0)):
         if name not in a.modes:
             continue
-        cfg = apsp.apsp_config_default(device=0, timing=1, packed16=int(a.packed16))
+        cfg = apsp.apsp_config_default(device=0, timing=1, packed16=int(a.packed16), exact_f32=int(a.exact_f32))
         cfg.schedule = legacy
         cfg.dataflow_delay = a.delay
         with apsp.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=cfg) as h:
