@@ -419,7 +419,9 @@ int main(int argc, char** argv) {
     {"mix10", k_mix<1, 0>, 64.0 / 128}, {"mix01", k_mix<0, 1>, 32.0 / 128},
     {"mix11", k_mix<1, 1>, 96.0 / 128}, {"mix21", k_mix<2, 1>, 160.0 / 128},
     {"mix31", k_mix<3, 1>, 224.0 / 128}, {"mix12", k_mix<1, 2>, 128.0 / 128},
-    {"mix41", k_mix<4, 1>, 288.0 / 128}, {"mix10nu", k_mix<1, 0, true>, 64.0 / 128}};
+    {"mix41", k_mix<4, 1>, 288.0 / 128}, {"mix10nu", k_mix<1, 0, true>, 64.0 / 128},
+    {"mix11nu", k_mix<1, 1, true>, 96.0 / 128}, {"mix21nu", k_mix<2, 1, true>, 160.0 / 128},
+    {"mix12nu", k_mix<1, 2, true>, 128.0 / 128}};
   CK(cudaMalloc(&out, (size_t)p.multiProcessorCount * 16 * 512 * sizeof(int)));
   for (auto& v : vs) {
     double best = 0;
