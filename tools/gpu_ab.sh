@@ -5,6 +5,8 @@
 #   tools/gpu_ab.sh close   small-n phase 1: deferred-bulk closure (default) vs one barrier per step
 #   tools/gpu_ab.sh pair    two-round (pair) queue vs one-round queue, int32 n = 16384 / 32768 / 65536, fp32
 #   tools/gpu_ab.sh ooc     out of core, every band streamed (n = 16384 / 32768, 1 and 2 virtual ranks)
+#   tools/gpu_ab.sh split   small-n chain panel tiles in 1 / 2 / 4 parts (APSP_SMALL_SPLIT), n = 1024 / 2048
+#   tools/gpu_ab.sh exact   int32 engine vs exact_f32 (R25) at n = 16384 / 65536
 mkdir -p gpurun_out
 what=$1
 out=gpurun_out/ab_$what.txt
@@ -35,6 +37,20 @@ case $what in
       python tools/ooc_ab.py --n 32768 --block 4096 --stream-all --runs 1
       python tools/ooc_ab.py --n 32768 --block 4096 --stream-all --runs 1 --world 2
     } > $out 2>&1 ;;
-  *) echo "usage: tools/gpu_ab.sh small|pair|ooc"; exit 2 ;;
+  split)
+    { timeout 600 python -m pytest tests/test_gpu_small.py -q -x 2>&1 | tail -3
+      for rep in 1 2; do for s in 1 2 4; do for n in 1024 2048; do
+        echo "== split=$s n=$n"; APSP_SMALL_SPLIT=$s timeout 120 python tools/fw_ab.py --n $n --deg 8 --dtype i32 --runs 30 --modes small
+      done; done; done
+      for s in 1 2 4; do echo "== split=$s profile"
+        APSP_SMALL_SPLIT=$s APSP_SMALL_PROFILE=1 timeout 120 python tools/fw_ab.py --n 1024 --deg 8 --dtype i32 --runs 3 --modes small
+      done
+    } > $out 2>&1 ;;
+  exact)
+    { for n in 16384 65536; do for x in "" "--exact-f32"; do
+        echo "== n=$n $x"; timeout 300 python tools/fw_ab.py --n $n --deg 16 --dtype i32 --runs 2 --modes dataflow $x
+      done; done
+    } > $out 2>&1 ;;
+  *) echo "usage: tools/gpu_ab.sh small|close|pair|ooc|split|exact"; exit 2 ;;
 esac
 cat $out | grep -vE "^\s*$" | tail -40
