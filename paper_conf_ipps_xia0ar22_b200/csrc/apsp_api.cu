@@ -279,10 +279,9 @@ static apsp_status run_small(Handle* h) {
   h->kernel = APSP_KERNEL_SMALL;
   h->ev_begin(2);
   if ((st = h->cuda(launch_fw_small<T>(static_cast<T*>(h->shards[0].D), h->ld, nb, h->df_work, h->d_flag, delay,
-                                       h->small_queue_loaded, ctas, h->stream),
+                                       &h->small_queue_key, ctas, h->stream),
                     "fw_small")))
     return st;
-  h->small_queue_loaded = true;
   h->ev_end((double)h->n_pad * h->n_pad * h->n_pad);
   return APSP_OK;
 }

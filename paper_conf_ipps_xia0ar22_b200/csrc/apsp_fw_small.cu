@@ -780,7 +780,7 @@ long long fw_small_work_bytes(int nb, size_t elem) {  // the queue is at most nb
 }
 
 template <typename T>
-cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag, long long delay, bool queue_loaded,
+cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag, long long delay, long long* queue_key,
                             int ctas_per_sm, cudaStream_t s) {
   if (nb <= 0) return cudaSuccess;
   int dev = 0, sms = 0;
@@ -806,7 +806,12 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
   a.csplit = f; f += nb;
   a.exitc = f; f += 1;
   a.flag_words = f - reinterpret_cast<int*>(fb);
-  a.split = small_split_for(small_variant());
+  const int variant = small_variant();
+  a.split = small_split_for(variant);
+  // the queue in the work buffer was built for (variant, split, delay) = *queue_key (-1: none yet);
+  // another configuration (tuning switches changed between launches) rebuilds it
+  const long long key = ((long long)variant << 60) | ((long long)a.split << 56) | (delay & ((1ll << 56) - 1));
+  const bool queue_loaded = *queue_key == key;
   a.negflag = negflag;
   const char* cv = getenv("APSP_SMALL_CLOSE");  // phase-1 variant A/B (tuning only)
   a.close_v = cv ? atoi(cv) : 1;
@@ -819,12 +824,16 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
     if ((e = cudaMemcpyAsync(dq, q.data(), q.size() * sizeof(int4), cudaMemcpyHostToDevice, s)) != cudaSuccess)
       return e;
     if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return e;  // q is a local
+    *queue_key = -1;  // set once the flags are zeroed too, below
   } else {
     a.total = small_queue(nb, delay, nullptr);
   }
   // zero flags: the previous launch's last CTA left them so (fw_small_kernel's epilogue); a new work
   // buffer is zeroed here, with its queue upload
-  if (!queue_loaded && (e = cudaMemsetAsync(a.counter, 0, small_flag_bytes(nb), s)) != cudaSuccess) return e;
+  if (!queue_loaded) {
+    if ((e = cudaMemsetAsync(a.counter, 0, small_flag_bytes(nb), s)) != cudaSuccess) return e;
+    *queue_key = key;
+  }
   // persistent grid: every CTA must be resident (tasks wait on each other)
   // (queried once: the event window of a small launch is ~0.3 ms, host work inside it shows)
   static int occ = 0;
@@ -856,7 +865,7 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
   return cudaSuccess;
 }
 
-template cudaError_t launch_fw_small<int>(int*, long long, int, void*, int*, long long, bool, int, cudaStream_t);
-template cudaError_t launch_fw_small<float>(float*, long long, int, void*, int*, long long, bool, int, cudaStream_t);
+template cudaError_t launch_fw_small<int>(int*, long long, int, void*, int*, long long, long long*, int, cudaStream_t);
+template cudaError_t launch_fw_small<float>(float*, long long, int, void*, int*, long long, long long*, int, cudaStream_t);
 
 }  // namespace apsp

@@ -94,7 +94,7 @@ struct Handle {
   // single-GPU in-core dataflow kernel (apsp_fw_dataflow.cu)
   bool dataflow = true;     // apsp_config.schedule (APSP_SCHED_PER_PHASE: launch per phase)
   bool small = false;       // dataflow with 64x64 tiles (apsp_fw_small.cu): small n, APSP_SCHED_SMALL
-  bool small_queue_loaded = false;  // its task queue is in df_work
+  long long small_queue_key = -1;   // configuration of the task queue in df_work (-1: none)
   int kernel = 0;           // APSP_KERNEL_* of the last blocked-FW closure (apsp_info.kernel)
   long long df_delay = 0;   // apsp_config.dataflow_delay (0 = auto)
   void* df_work = nullptr;

@@ -148,10 +148,11 @@ cudaError_t launch_fw_dataflow_sharded(const DFShard* ranks, int nv, int P, int 
 
 // The whole single-GPU blocked FW for small n with 64x64 tiles (apsp_fw_small.cu): the
 // dataflow schedule above at b = 64 (nb = n_pad / 64 rounds), one 256-thread CTA per task.
-// `work` holds fw_small_work_bytes(nb, elem) bytes (panel copies + flags, zeroed here, + the task
-// queue, uploaded when !queue_loaded).
+// `work` holds fw_small_work_bytes(nb, elem) bytes (panel copies + flags + the task queue). *queue_key
+// (-1 for a new work buffer) names the queue configuration already in `work`; on a mismatch the
+// queue is rebuilt and uploaded and the flags zeroed (afterwards each launch's last CTA re-zeroes them).
 template <typename T>
-cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag, long long delay, bool queue_loaded,
+cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag, long long delay, long long* queue_key,
                             int ctas_per_sm, cudaStream_t s);
 long long fw_small_work_bytes(int nb, size_t elem);
 // its task queue (host-built, critical path first; type 4 = fused P3(k; k+1,k+1) + P1(k+1))

@@ -123,3 +123,17 @@ def test_small_split_chain_tiles(lib, monkeypatch, split):
     got = run(lib, gf)
     monkeypatch.setenv("APSP_SMALL_SPLIT", "1")
     assert np.array_equal(got.view(np.int32), run(lib, gf).view(np.int32))
+
+
+def test_small_queue_rebuilt_when_its_configuration_changes(lib, monkeypatch):
+    """One handle, the split switched between runs: the queue in the work buffer is rebuilt for the
+    new configuration (its key), and every run stays exact; repeated runs reuse it (flags re-zeroed
+    by the previous launch's last CTA)."""
+    g = gg.erdos_renyi(1000, 5000, seed=12)
+    want = want_i32(g)
+    with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=lib.apsp_config_default(device=0)) as h:
+        for split in ("4", "4", "1", "2", "2", "4"):
+            monkeypatch.setenv("APSP_SMALL_SPLIT", split)
+            lib.apsp_reinit(h)
+            lib.apsp_fw_blocked(h)
+            assert np.array_equal(lib.apsp_get_dist(h).astype(np.int64), want), split
