@@ -17,6 +17,11 @@ Launch: `python bench.py --gpus N` without torchrun re-executes itself under
 `python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1`; under
 torchrun (WORLD_SIZE set) every rank runs directly.
 
+Legs beside the headline on one GPU (each guarded; skip flags --no-packed16, --no-exact-f32-leg,
+--no-ooc-leg, --no-boundary-leg, --no-johnson): packed16 (R16), exact_f32 (R25: the int32 graph
+closed by the fp32 engine under the 2(n-1)W <= 2^24 bound), the same workload fully out of core,
+the boundary algorithm on a grid of the same n, Johnson's algorithm.
+
 `--impl reference` times the CPU oracle (oracle/, plain C + OpenMP) on a bounded
 sample of the same workload (the reference arm of this paper-only tier).
 """

@@ -750,10 +750,12 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, const GPair<T>* p2
           const V4 a1 = *reinterpret_cast<const V4*>(as + (kk + 1) * ALD + 64 * h + ty * 4);
           const float x0[4] = {a0.x, a0.y, a0.z, a0.w};
           const float x1[4] = {a1.x, a1.y, a1.z, a1.w};
+#ifndef APSP_F32_JP_OUTER
+#define APSP_F32_JP_OUTER 0  // A/B build switch: column pair outer (the pair operand repeats back to back)
+#endif
 #pragma unroll
-          for (int i = 0; i < 4; ++i)
-#pragma unroll
-            for (int jp = 0; jp < 4; ++jp) {
+          for (int u = 0; u < 16; ++u) {
+              const int i = APSP_F32_JP_OUTER ? (u & 3) : (u >> 2), jp = APSP_F32_JP_OUTER ? (u >> 2) : (u & 3);
               const float2 s0 = __fadd2_rn(make_float2(x0[i], x0[i]), p0[jp]);
               const float2 s1 = __fadd2_rn(make_float2(x1[i], x1[i]), p1[jp]);
               float& c0 = acc[4 * h + i][2 * jp];
