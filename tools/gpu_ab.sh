@@ -7,6 +7,8 @@
 #   tools/gpu_ab.sh ooc     out of core, every band streamed (n = 16384 / 32768, 1 and 2 virtual ranks)
 #   tools/gpu_ab.sh split   small-n chain panel tiles in 1 / 2 / 4 parts (APSP_SMALL_SPLIT), n = 1024 / 2048
 #   tools/gpu_ab.sh exact   int32 engine vs exact_f32 (R25) at n = 16384 / 65536
+#   tools/gpu_ab.sh variant NAME [DTYPE]  default build vs build/var_NAME (tools/build_variant.py), dataflow
+#                           kernel, n = 16384 / 32768, alternating twice
 mkdir -p gpurun_out
 what=$1
 out=gpurun_out/ab_$what.txt
@@ -51,6 +53,14 @@ case $what in
         echo "== n=$n $x"; timeout 300 python tools/fw_ab.py --n $n --deg 16 --dtype i32 --runs 2 --modes dataflow $x
       done; done
     } > $out 2>&1 ;;
-  *) echo "usage: tools/gpu_ab.sh small|close|pair|ooc|split|exact"; exit 2 ;;
+  variant)
+    v=$2; dt=${3:-f32}; out=gpurun_out/ab_variant_${v}_${dt}.txt
+    { for rep in 1 2; do for n in 16384 32768; do
+        r=5; [ $n -gt 16384 ] && r=2
+        echo "== default n=$n"; timeout 300 python tools/fw_ab.py --n $n --deg 64 --dtype $dt --runs $r --modes dataflow
+        echo "== $v n=$n"; (cd build/var_$v && timeout 300 python tools/fw_ab.py --n $n --deg 64 --dtype $dt --runs $r --modes dataflow)
+      done; done
+    } > $out 2>&1 ;;
+  *) echo "usage: tools/gpu_ab.sh small|close|pair|ooc|split|exact|variant"; exit 2 ;;
 esac
 cat $out | grep -vE "^\s*$" | tail -40
