@@ -751,10 +751,31 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, const GPair<T>* p2
           const float x0[4] = {a0.x, a0.y, a0.z, a0.w};
           const float x1[4] = {a1.x, a1.y, a1.z, a1.w};
 #ifndef APSP_F32_JP_OUTER
-#define APSP_F32_JP_OUTER 0  // A/B build switch: column pair outer (the pair operand repeats back to back)
+#define APSP_F32_JP_OUTER 2
 #endif
+          // column pair outer, the four sums of each depth step first: the FADD2s of one pair
+          // operand run back to back, so its 64-bit operand comes from the operand reuse cache
+          // (fewer register-file reads, which bound this instruction stream: DESIGN.md §5 pipe
+          // decomposition). Measured at n = 16384 / 32768 (fp32 ER, profiles/r02_f32_order_ab.txt):
+          // row outer (0) 1.849e13, pair outer (1) 1.861e13, pair outer with the sums grouped (2,
+          // default) 1.876-1.880e13.
 #pragma unroll
-          for (int u = 0; u < 16; ++u) {
+          for (int u = 0; u < 16; u += (APSP_F32_JP_OUTER == 2 ? 4 : 1)) {
+            if constexpr (APSP_F32_JP_OUTER == 2) {
+              const int jp = u >> 2;
+              float2 s0[4], s1[4];
+#pragma unroll
+              for (int i = 0; i < 4; ++i) s0[i] = __fadd2_rn(make_float2(x0[i], x0[i]), p0[jp]);
+#pragma unroll
+              for (int i = 0; i < 4; ++i) s1[i] = __fadd2_rn(make_float2(x1[i], x1[i]), p1[jp]);
+#pragma unroll
+              for (int i = 0; i < 4; ++i) {
+                float& c0 = acc[4 * h + i][2 * jp];
+                float& c1 = acc[4 * h + i][2 * jp + 1];
+                c0 = fminf(fminf(c0, s0[i].x), s1[i].x);
+                c1 = fminf(fminf(c1, s0[i].y), s1[i].y);
+              }
+            } else {
               const int i = APSP_F32_JP_OUTER ? (u & 3) : (u >> 2), jp = APSP_F32_JP_OUTER ? (u >> 2) : (u & 3);
               const float2 s0 = __fadd2_rn(make_float2(x0[i], x0[i]), p0[jp]);
               const float2 s1 = __fadd2_rn(make_float2(x1[i], x1[i]), p1[jp]);
@@ -763,6 +784,7 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, const GPair<T>* p2
               c0 = fminf(fminf(c0, s0.x), s1.x);
               c1 = fminf(fminf(c1, s0.y), s1.y);
             }
+          }
         }
       }
     } else {

@@ -99,14 +99,22 @@ __device__ __forceinline__ void relax_two_steps(T (&acc)[8][8], const T (&a)[8][
                           make_float2(b01.z, b01.w)};
     const float2 p1[4] = {make_float2(b10.x, b10.y), make_float2(b10.z, b10.w), make_float2(b11.x, b11.y),
                           make_float2(b11.z, b11.w)};
+    // column pair outer, the four sums of each depth step grouped: the pair operand of
+    // back-to-back FADD2s comes from the operand reuse cache (as in apsp_fw_dataflow.cu)
 #pragma unroll
-    for (int i = 0; i < 8; ++i)
+    for (int jp = 0; jp < 4; ++jp)
 #pragma unroll
-      for (int jp = 0; jp < 4; ++jp) {
-        const float2 s0 = __fadd2_rn(make_float2(a[i][0], a[i][0]), p0[jp]);
-        const float2 s1 = __fadd2_rn(make_float2(a[i][1], a[i][1]), p1[jp]);
-        acc[i][2 * jp] = fminf(fminf(acc[i][2 * jp], s0.x), s1.x);
-        acc[i][2 * jp + 1] = fminf(fminf(acc[i][2 * jp + 1], s0.y), s1.y);
+      for (int h = 0; h < 2; ++h) {
+        float2 s0[4], s1[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) s0[i] = __fadd2_rn(make_float2(a[4 * h + i][0], a[4 * h + i][0]), p0[jp]);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) s1[i] = __fadd2_rn(make_float2(a[4 * h + i][1], a[4 * h + i][1]), p1[jp]);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          acc[4 * h + i][2 * jp] = fminf(fminf(acc[4 * h + i][2 * jp], s0[i].x), s1[i].x);
+          acc[4 * h + i][2 * jp + 1] = fminf(fminf(acc[4 * h + i][2 * jp + 1], s0[i].y), s1[i].y);
+        }
       }
   } else {
 #pragma unroll
