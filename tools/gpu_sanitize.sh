@@ -11,5 +11,5 @@ san memcheck "" memcheck
 san initcheck "" initcheck
 san racecheck "barrier,ooc,johnson,boundary" racecheck_barrier
 san synccheck "barrier,ooc,johnson,boundary" synccheck_barrier
-san racecheck "dataflow" racecheck_dataflow
+san racecheck "dataflow,small" racecheck_dataflow
 san synccheck "dataflow" synccheck_dataflow

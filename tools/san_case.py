@@ -54,6 +54,15 @@ def main():
     if want("ooc"):
         same(run(gb, force_out_of_core=1, ooc_block=256, minplus_variant=1), run(gb, minplus_variant=1, schedule=1), "out of core vs in core")
         same(run(gb, world_size=2, virtual_ranks=1, minplus_variant=1), run(gb, minplus_variant=1, schedule=1), "2 virtual ranks vs 1 GPU")
+    if want("small"):  # 64-tile kernel: split chain panel tiles, flags re-zeroed by the last CTA between runs
+        with apsp.apsp_init_from_csr(n, g.row_ptr, g.col, g.w, cfg=apsp.apsp_config_default(device=0)) as h:
+            for _ in range(2):
+                apsp.apsp_reinit(h)
+                apsp.apsp_fw_blocked(h)
+                same(apsp.apsp_get_dist(h), run(g, schedule=1), "small kernel (split parts), repeated run")
+    if want("exact"):  # R25: int32 in fp32 arithmetic (128-tile dataflow kernel: n_pad > 2048)
+        gx = gg.erdos_renyi(2100, 8400, seed=6)
+        same(run(gx, exact_f32=1), run(gx, schedule=1), "exact_f32 vs int32 per-phase")
     if want("neg"):
         same(run(gn), run(gn, schedule=1), "negative weights (canonicalize)")
     if want("johnson"):
