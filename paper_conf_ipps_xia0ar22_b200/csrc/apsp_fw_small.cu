@@ -95,6 +95,8 @@ struct SmArgs {
   int split;                 // parts of each chain panel tile (small_split(); 1 = whole tasks)
   int* rsplit;               // [nb] finished parts of P2R(j-1; j-1, j), the row-panel tile next to the diagonal
   int* csplit;               // [nb] finished parts of P2C(i-1; i, i-1)
+  int early_pub;             // F(k): diagready published before the matrix tile is stored (APSP_SMALL_EARLYPUB)
+  int spin;                  // dependency polls back to back, no __nanosleep between them (APSP_SMALL_SPIN)
   int* exitc;                // CTAs past their last task: the last one zeroes every flag for the next launch
   long long flag_words;      // 32-bit words from counter to exitc inclusive
 };
@@ -282,7 +284,20 @@ __device__ __forceinline__ void small_close_any(const SmArgs<T>& a, T (&acc)[4][
   else small_close(acc, rowbuf, colbuf, a.negflag);
 }
 
-// the closed diagonal block of round k: into the matrix, D and D^T into the panel copy
+// a thread's 4x4 block of a tile of the matrix (ld elements per row)
+template <typename T>
+__device__ __forceinline__ void small_store_tile(T* tile, long long ld, const T (&acc)[4][4]) {
+  using V4 = typename SV<T>::V4;
+  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    V4 v;
+    v.x = acc[i][0]; v.y = acc[i][1]; v.z = acc[i][2]; v.w = acc[i][3];
+    *reinterpret_cast<V4*>(tile + (long long)(ty * 4 + i) * ld + tx * 4) = v;
+  }
+}
+
+// the closed diagonal block of round k: into the matrix (tile != nullptr), D and D^T into the panel copy
 template <typename T>
 __device__ __forceinline__ void small_store_diag(const SmArgs<T>& a, int k, T* tile, const T (&acc)[4][4]) {
   using V4 = typename SV<T>::V4;
@@ -293,7 +308,7 @@ __device__ __forceinline__ void small_store_diag(const SmArgs<T>& a, int k, T* t
   for (int i = 0; i < 4; ++i) {
     V4 v;
     v.x = acc[i][0]; v.y = acc[i][1]; v.z = acc[i][2]; v.w = acc[i][3];
-    *reinterpret_cast<V4*>(tile + (long long)(ty * 4 + i) * a.ld + tx * 4) = v;
+    if (tile) *reinterpret_cast<V4*>(tile + (long long)(ty * 4 + i) * a.ld + tx * 4) = v;
     *reinterpret_cast<V4*>(d + (ty * 4 + i) * SB + tx * 4) = v;
   }
 #pragma unroll
@@ -389,6 +404,19 @@ __device__ __forceinline__ void small_minplus(const SmArgs<T>& a, const Task& tk
   }
   if (fused) {  // tile (k+1,k+1) after round k: close it as P1(k+1) (R6 check included)
     small_close_any(a, acc, rowbuf, colbuf);
+    if (a.early_pub) {
+      // round k+1's panel tasks need only the panel copies D / D^T: publish them before the
+      // matrix tile is stored, so the release fence does not wait for those 16 KB (the
+      // kernel loop's publication after the task repeats diagready with ver and done3)
+      small_store_diag(a, tk.k + 1, static_cast<T*>(nullptr), acc);
+      __syncthreads();
+      if (threadIdx.x == 32) {
+        asm volatile("fence.release.gpu;" ::: "memory");
+        st_relaxed(a.diagready + ((tk.k + 1) & 1), tk.k + 2);
+      }
+      small_store_tile(C, a.ld, acc);
+      return;
+    }
     small_store_diag(a, tk.k + 1, C, acc);
     return;
   }
@@ -614,7 +642,8 @@ __global__ void __launch_bounds__(SNT) fw_small_kernel(const __grid_constant__ S
     int4 nq = make_int4(0, 0, 0, 0);
     if (tid == 0) {
       if (!S.ready)
-        while (!small_deps(a, tk)) __nanosleep(32);
+        while (!small_deps(a, tk))
+          if (!a.spin) __nanosleep(32);
       if (a.prof) {
         const long long c1 = clock64();
         pr[0] += c1 - c0;
@@ -813,6 +842,10 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
   const long long key = ((long long)variant << 60) | ((long long)a.split << 56) | (delay & ((1ll << 56) - 1));
   const bool queue_loaded = *queue_key == key;
   a.negflag = negflag;
+  const char* ep = getenv("APSP_SMALL_EARLYPUB");  // A/B (tuning only)
+  a.early_pub = ep ? atoi(ep) : 1;  // measured n = 1024: 0.2377-0.2389 ms vs 0.2419-0.2448
+  const char* sp = getenv("APSP_SMALL_SPIN");  // A/B (tuning only)
+  a.spin = sp ? atoi(sp) : 0;
   const char* cv = getenv("APSP_SMALL_CLOSE");  // phase-1 variant A/B (tuning only)
   a.close_v = cv ? atoi(cv) : 1;
   // the queue lives in the work buffer: built and uploaded with the first launch on it
