@@ -406,5 +406,54 @@ __device__ void signal_done(const Args& a, const Task& t) {
   }
 }
 
+// Dependencies / publication with a.npar panel-copy parities (the copies of round k are
+// rewritten by round k + npar) and the pair task T_PAIR (rounds k, k+1 of one tile): any argument
+// block with DFArgs' flag fields plus npar (the packed16 kernel; the int32 kernel keeps its own
+// copies, deps_single / signal_single, whose code layout it was measured with).
+template <class Args>
+__device__ bool deps_np(const Args& a, const Task& t) {
+  const int nb = a.nb, k = t.k, np = a.npar, p = k & (np - 1);
+  const int* f0 = a.ver + (long long)t.i * nb + t.j;
+  const int* f1;
+  const int* f2;
+  const int* f3 = f0;
+  const int* f4 = f0;
+  int v1, v2, v3 = INT_MIN, v4 = INT_MIN;
+  if (t.type == T_P1) {
+    f1 = a.done2 + (k >= np ? k - np : 0); v1 = k >= np ? 2 * (nb - 1) : INT_MIN;
+    f2 = f1; v2 = v1;
+  } else if (t.type == T_P3 || t.type == T_PAIR) {
+    f1 = a.rowready + p * nb + t.j; v1 = k + 1;
+    f2 = a.colready + p * nb + t.i; v2 = k + 1;
+    if (t.type == T_PAIR) {
+      const int p1 = (k + 1) & (np - 1);
+      f3 = a.rowready + p1 * nb + t.j; v3 = k + 2;
+      f4 = a.colready + p1 * nb + t.i; v4 = k + 2;
+    }
+  } else {
+    f1 = a.diagready + p; v1 = k + 1;
+    f2 = a.done3 + (k >= np ? k - np : 0); v2 = k >= np ? (nb - 1) * (nb - 1) : INT_MIN;
+  }
+  const int x0 = ld_relaxed(f0), x1 = ld_relaxed(f1), x2 = ld_relaxed(f2), x3 = ld_relaxed(f3), x4 = ld_relaxed(f4);
+  if (x0 >= k && x1 >= v1 && x2 >= v2 && x3 >= v3 && x4 >= v4) {
+    asm volatile("fence.acquire.gpu;" ::: "memory");  // (see deps_met)
+    return true;
+  }
+  return false;
+}
+template <class Args>
+__device__ void signal_np(const Args& a, const Task& t) {
+  const int nb = a.nb, k = t.k, p = k & (a.npar - 1);
+  asm volatile("fence.release.gpu;" ::: "memory");
+  st_relaxed(a.ver + (long long)t.i * nb + t.j, t.type == T_PAIR ? k + 2 : k + 1);
+  switch (t.type) {
+    case T_P1: st_relaxed(a.diagready + p, k + 1); break;
+    case T_P2R: st_relaxed(a.rowready + p * nb + t.j, k + 1); red_relaxed_add(a.done2 + k, 1); break;
+    case T_P2C: st_relaxed(a.colready + p * nb + t.i, k + 1); red_relaxed_add(a.done2 + k, 1); break;
+    case T_PAIR: red_relaxed_add(a.done3 + k, 1); red_relaxed_add(a.done3 + k + 1, 1); break;
+    default: red_relaxed_add(a.done3 + k, 1); break;
+  }
+}
+
 }  // namespace
 }  // namespace apsp

@@ -25,6 +25,7 @@
 #include <cuda_runtime.h>
 #include <climits>
 #include <cstdint>
+#include <cstdlib>
 
 namespace apsp {
 namespace {
@@ -38,6 +39,10 @@ constexpr int B_HALVES = BK * BN;                            // Bs[kk][c], int16
 constexpr int STAGE_BYTES = A_WORDS * 4 + B_HALVES * 2;      // 24 KB
 constexpr long long T16 = (long long)BM * BN * 2;            // int16 tile
 constexpr long long T32 = (long long)BM * BN * 4;            // dup-word tile
+// the two-round (pair) queue by default: n = 16384 3.248e13 vs 3.193e13 one-round, n = 65536
+// 3.346e13 vs 3.217e13 (the int16 tasks are twice as fast as int32 ones, so the
+// per-task cost the pairs halve weighs twice as much)
+constexpr bool kPair16Default = true;
 constexpr int SIG = 32, SCH = 64;
 static_assert(64 * BN * 2 <= STAGE_BYTES, "half an int16 C tile must fit one stage");
 
@@ -61,10 +66,12 @@ struct DFArgs16 {
   long long total;
   long long delay;
   unsigned long long* prof;
+  int npar;   // panel-copy parities: 2, or 4 with the pair queue (round k's copies live until round k+4)
+  int pairq;  // 1 = the two-round queue (decode2, T_PAIR: rounds k, k+1 of one tile in one depth-256 task)
 };
 
 __device__ __forceinline__ unsigned char* pb_base(const DFArgs16& a, int k) {
-  return a.pbuf + (long long)(k & 1) * (T16 + T32 + (long long)a.nb * (T16 + T32));
+  return a.pbuf + (long long)(k & (a.npar - 1)) * (T16 + T32 + (long long)a.nb * (T16 + T32));
 }
 __device__ __forceinline__ short* pb_diag16(const DFArgs16& a, int k) { return reinterpret_cast<short*>(pb_base(a, k)); }
 __device__ __forceinline__ unsigned* pb_diagTd(const DFArgs16& a, int k) {
@@ -148,6 +155,9 @@ __device__ __noinline__ void group_phase1_16(short* tile, long long ld, short* d
 struct GDesc16 {
   const void* A;  // a_rows = 0: dup words [kk][r] (ld 128 words); 1: int16 tile rows r (ld lda), dup'ed on load
   const short* B; // int16 rows kk of 128 columns (ld ldb)
+  const void* A2; // pair task: round k+1's panel copies (chunks 4..7), same layout as A / B
+  const short* B2;
+  int nk;         // chunks of depth 32: 4 (one round), 8 (pair task)
   const short* Cin;
   short* Cout;
   void* Cout2;    // c2 = 1: int16 copy (ld 128); c2 = 2: dup words transposed [c][r]; 0: none
@@ -167,7 +177,7 @@ __device__ void fill_desc16(const DFArgs16& a, const Task& tk, GDesc16& d) {
   const int k = tk.k;
   short* const tile = a.D + (long long)tk.i * BM * a.ld + (long long)tk.j * BN;
   d.Cin = tile; d.Cout = tile; d.ldc = (int)a.ld;
-  d.a_rows = 0; d.bulk = 0;
+  d.a_rows = 0; d.bulk = 0; d.nk = BM / BK; d.A2 = nullptr; d.B2 = nullptr;
   if (tk.type == T_P2R) {         // A(k,j) = D (x) A(k,j)
     d.A = pb_diagTd(a, k); d.lda = BM; d.B = tile; d.ldb = (int)a.ld;
     d.Cout2 = pb_row16(a, k, tk.j); d.c2 = 1;
@@ -177,6 +187,9 @@ __device__ void fill_desc16(const DFArgs16& a, const Task& tk, GDesc16& d) {
   } else {                        // phase 3 from the panel copies
     d.A = pb_colTd(a, k, tk.i); d.lda = BM; d.B = pb_row16(a, k, tk.j); d.ldb = BN;
     d.Cout2 = nullptr; d.c2 = 0; d.bulk = 1;
+    if (tk.type == T_PAIR) {      // then round k+1: min(., A(i,k+1) (x) A(k+1,j)) (min is order-free)
+      d.A2 = pb_colTd(a, k + 1, tk.i); d.B2 = pb_row16(a, k + 1, tk.j); d.nk = 2 * (BM / BK);
+    }
   }
 }
 
@@ -188,7 +201,7 @@ __device__ void fill_desc16(const DFArgs16& a, const Task& tk, GDesc16& d) {
 __device__ __forceinline__ void group_minplus16(const GDesc16* d, unsigned char* stage0, unsigned full0, unsigned empty0,
                                             unsigned c0, int gtid, int g, const DFArgs16* args, long long nxt,
                                             Slot16* ns) {
-  constexpr int NK = BM / BK;
+  const int NK = d->nk;  // 4 chunks of depth 32 (8 for a pair task)
   const int lane = gtid & 31;
   const int tx = gtid & 15, ty = gtid >> 4;
   const bool bulk = d->bulk;
@@ -201,12 +214,14 @@ __device__ __forceinline__ void group_minplus16(const GDesc16* d, unsigned char*
         if (wait_G >= 0) mb_wait(empty0 + 8 * stage, ((unsigned)wait_G / STAGES) & 1);
         // generic -> async proxy: stage (shared::cta) and, once per task, the panel copies other
         // CTAs wrote with generic stores and this CTA acquired before the task (global)
-        if (c == 0) asm volatile("fence.proxy.async.global;" ::: "memory");
+        if (c == 0 || c == 4) asm volatile("fence.proxy.async.global;" ::: "memory");
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         mb_expect_tx(full0 + 8 * stage, A_WORDS * 4 + B_HALVES * 2);
-        bulk_g2s(saddr(sa), static_cast<const unsigned*>(d->A) + (long long)c * A_WORDS, A_WORDS * 4,
-                 full0 + 8 * stage);
-        bulk_g2s(saddr(sb), d->B + (long long)c * B_HALVES, B_HALVES * 2, full0 + 8 * stage);
+        const int cr = c & 3;  // chunk within its round (pair tasks: chunks 4..7 from round k+1)
+        const unsigned* const Ar = static_cast<const unsigned*>(c < 4 ? d->A : d->A2);
+        const short* const Br = c < 4 ? d->B : d->B2;
+        bulk_g2s(saddr(sa), Ar + (long long)cr * A_WORDS, A_WORDS * 4, full0 + 8 * stage);
+        bulk_g2s(saddr(sb), Br + (long long)cr * B_HALVES, B_HALVES * 2, full0 + 8 * stage);
       }
       return;
     }
@@ -250,15 +265,17 @@ __device__ __forceinline__ void group_minplus16(const GDesc16* d, unsigned char*
   for (int i = 0; i < 8; ++i)
 #pragma unroll
     for (int p = 0; p < 4; ++p) acc[i][p] = 0x7FFF7FFFu;
-  const int s_lo = (int)((c0 + 1) % STAGES), s_hi = (int)((c0 + 2) % STAGES);
+  // the C tile goes to the stages of chunks c0+NK-3 and c0+NK-2 (free during the last chunk)
+  const unsigned g_lo = c0 + NK - 3, g_hi = c0 + NK - 2;
+  const int s_lo = (int)(g_lo % STAGES), s_hi = (int)(g_hi % STAGES);
 
 #pragma unroll 1
   for (int c = 0; c < NK; ++c) {
     const unsigned G = c0 + c;
     const int s = (int)(G % STAGES);
     if (c == NK - 1) {  // C (int16 128 x 256 B) into the two stages free during the last chunk
-      mb_wait(empty0 + 8 * s_lo, ((c0 + 1) / STAGES) & 1);
-      mb_wait(empty0 + 8 * s_hi, ((c0 + 2) / STAGES) & 1);
+      mb_wait(empty0 + 8 * s_lo, (g_lo / STAGES) & 1);
+      mb_wait(empty0 + 8 * s_hi, (g_hi / STAGES) & 1);
       const int ldc = d->ldc;
       short* const cs_lo = reinterpret_cast<short*>(stage0 + s_lo * STAGE_BYTES);
       short* const cs_hi = reinterpret_cast<short*>(stage0 + s_hi * STAGE_BYTES);
@@ -273,10 +290,10 @@ __device__ __forceinline__ void group_minplus16(const GDesc16* d, unsigned char*
     if (c == 1 && gtid == SCH) {
       ns->t = nxt;
       if (nxt < args->total) {
-        const Task tn = decode(nxt, args->nb, args->delay);
+        const Task tn = args->pairq ? decode2(nxt, args->nb, args->delay) : decode(nxt, args->nb, args->delay);
         ns->tk = tn;
         if (tn.type != T_P1) fill_desc16(*args, tn, ns->d);
-        ns->ready = deps_met(*args, tn) ? 1 : 0;
+        ns->ready = deps_np(*args, tn) ? 1 : 0;
       }
     }
     mb_wait(full0 + 8 * s, (G / STAGES) & 1);
@@ -379,7 +396,7 @@ __global__ void __launch_bounds__(GNT, CTAS_PER_SM) fw_dataflow16_kernel(const _
     s0.t = (long long)atomicAdd(a.counter, 1ull);
     s0.ready = 0;
     if (s0.t < a.total) {
-      s0.tk = decode(s0.t, a.nb, a.delay);
+      s0.tk = a.pairq ? decode2(s0.t, a.nb, a.delay) : decode(s0.t, a.nb, a.delay);
       if (s0.tk.type != T_P1) fill_desc16(a, s0.tk, s0.d);
     }
   }
@@ -394,8 +411,8 @@ __global__ void __launch_bounds__(GNT, CTAS_PER_SM) fw_dataflow16_kernel(const _
     if (t >= a.total) break;
     const Task tk = S.tk;
     if (!S.ready) {
-      if (gtid == SCH && !deps_met(a, tk)) {
-        while (!deps_met(a, tk)) __nanosleep(64);
+      if (gtid == SCH && !deps_np(a, tk)) {
+        while (!deps_np(a, tk)) __nanosleep(64);
         pr[5]++;
       }
       gbar(g);
@@ -410,21 +427,21 @@ __global__ void __launch_bounds__(GNT, CTAS_PER_SM) fw_dataflow16_kernel(const _
       if (gtid == SCH) {
         N->t = nxt;
         if (nxt < a.total) {
-          N->tk = decode(nxt, a.nb, a.delay);
+          N->tk = a.pairq ? decode2(nxt, a.nb, a.delay) : decode(nxt, a.nb, a.delay);
           N->ready = 0;
           if (N->tk.type != T_P1) fill_desc16(a, N->tk, N->d);
         }
       }
     } else {
       group_minplus16(&S.d, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N);
-      chunk += BM / BK;
+      chunk += S.d.nk;
     }
     const long long tc2 = clock64();
     pr[1] += tc2 - tc1;
     if (tk.type == T_P1) pr[4] += tc2 - tc1;
     pr[3]++;
     gbar(g);
-    if (gtid == SIG) signal_done(a, tk);
+    if (gtid == SIG) signal_np(a, tk);
     tc0 = clock64();
     pr[2] += tc0 - tc2;
   }
@@ -436,7 +453,7 @@ __global__ void __launch_bounds__(GNT, CTAS_PER_SM) fw_dataflow16_kernel(const _
 
 }  // namespace
 
-long long fw_dataflow16_pbuf_bytes(int nb) { return 2ll * (T16 + T32 + (long long)nb * (T16 + T32)); }
+long long fw_dataflow16_pbuf_bytes(int nb) { return 4ll * (T16 + T32 + (long long)nb * (T16 + T32)); }  // 4 parities
 long long fw_dataflow16_work_bytes(int nb) { return fw_dataflow16_pbuf_bytes(nb) + fw_dataflow_flag_bytes(nb); }
 int fw_dataflow16_ctas_per_sm() { return CTAS_PER_SM; }
 
@@ -455,12 +472,17 @@ cudaError_t launch_fw_dataflow16(short* D, long long ld, int nb, void* work, lon
   int* f = reinterpret_cast<int*>(static_cast<char*>(work) + fw_dataflow16_pbuf_bytes(nb));
   a.counter = reinterpret_cast<unsigned long long*>(f); f += 2;
   a.ver = f; f += (long long)nb * nb;
-  a.diagready = f; f += 2;
-  a.rowready = f; f += 2 * nb;
-  a.colready = f; f += 2 * nb;
+  a.diagready = f; f += 4;  // (the flag block is sized for 4 parities: fw_dataflow_flag_bytes)
+  a.rowready = f; f += 4 * nb;
+  a.colready = f; f += 4 * nb;
   a.done2 = f; f += nb;
   a.done3 = f; f += nb;
-  a.total = (long long)nb * nb * nb;
+  // the two-round (pair) queue: APSP_DF16_PAIR=0/1 overrides the default (A/B)
+  int pairq = kPair16Default && nb >= 2;
+  if (const char* ev = getenv("APSP_DF16_PAIR")) pairq = atoi(ev) != 0 && nb >= 2;
+  a.pairq = pairq;
+  a.npar = pairq ? 4 : 2;
+  a.total = pairq ? pair_total(nb) : (long long)nb * nb * nb;
   a.delay = delay;
   a.prof = prof;
   e = cudaMemsetAsync(a.counter, 0, fw_dataflow_flag_bytes(nb), s);

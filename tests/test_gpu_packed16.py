@@ -131,3 +131,20 @@ def test_packed16_dataflow_matches_per_phase_grid(lib):
     want = oracle.dijkstra_rows_i64(g.row_ptr, g.col, g.w, rows)
     want = np.where(want == oracle.INF_I64, INF32, want)
     assert np.array_equal(a[rows].astype(np.int64), want)
+
+
+@pytest.mark.parametrize("pair", ["0", "1"])
+def test_packed16_pair_and_one_round_queues(lib, monkeypatch, pair):
+    """fw_dataflow16_kernel on the two-round queue (decode2: rounds k, k+1 of a bulk tile in one
+    depth-256 task, 4 panel-copy parities; the default) and on the one-round queue
+    (APSP_DF16_PAIR=0): bit-exact at odd and even round counts (a last single round), a ragged
+    tail, and the 8191/8192 fallback boundary's int16 side."""
+    monkeypatch.setenv("APSP_DF16_PAIR", pair)
+    for n, seed in ((129, 1), (640, 2), (1000, 3), (1300, 4)):
+        g = gg.erdos_renyi(n, 5 * n, seed=seed)
+        d, _, _, arith = run16(lib, g)
+        assert arith == lib.APSP_ARITH_S16X2
+        assert np.array_equal(d.astype(np.int64), want_i32(g)), n
+    g = gg.grid_2d(40, 64, seed=12, hi=60)
+    d, _, _, _ = run16(lib, g)
+    assert np.array_equal(d.astype(np.int64), want_i32(g))
