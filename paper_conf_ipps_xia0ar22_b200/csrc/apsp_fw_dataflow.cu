@@ -566,7 +566,10 @@ __device__ DF_MP_INLINE void group_minplus(const GDesc<T>* d, const GPair<T>* p2
                                            int gtid, int g, const DFArgs<T>* args, long long nxt,
                                            Slot<T, PQ>* ns, int pref) {
   using V4 = typename DV<T>::V4;
-  // NK = 4 chunks of depth 32 (one round), 8 for a pair task (compile-time: two instantiations)
+  // NK = 4 chunks of depth 32 (one round), 8 for a pair task (compile-time: two instantiations);
+  // NK = 0: the pair task's runtime depth (one engine copy, APSP_DF_PQ_ONE_ENGINE A/B builds)
+  const int nkc = NK ? NK : p2->nk;
+#define NK nkc
   // fp32: fold the top half of C before the last chunk and issue the next phase-3 task's
   // chunk 0 into the freed stage (measured +1.2 % for fp32, -1.7 % for int32, so int32 keeps
   // the C fetch into both free stages during the last chunk and the fold at the end)
@@ -871,6 +874,8 @@ struct DFLaunch {
   int nv;
 };
 
+#undef NK
+
 // SH: the sharded kernel; PQ: the single-GPU kernel on the two-round (pair) queue. The one-round
 // single-GPU kernel (PQ = false) keeps exactly the pre-pair code (measured: the pair engine's
 // extra code costs the one-round path ~2-3 %, so each queue gets its own instantiation).
@@ -959,12 +964,16 @@ __global__ void __launch_bounds__(GNT * GROUPS, CTAS_PER_SM) fw_dataflow_kernel(
       }
     } else {
       if constexpr (PQ) {
+#ifdef APSP_DF_PQ_ONE_ENGINE
+        group_minplus<SH, PQ, T, 0>(&S.d, &S.p2, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N, S.pref);
+#else
         if (S.p2.nk == 2 * (BM / BK)) {
           group_minplus<SH, PQ, T, 2 * (BM / BK)>(&S.d, &S.p2, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N,
                                                   S.pref);
         } else {
           group_minplus<SH, PQ, T, BM / BK>(&S.d, &S.p2, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N, S.pref);
         }
+#endif
         chunk += S.p2.nk;
       } else {
         group_minplus<SH, PQ, T, BM / BK>(&S.d, nullptr, stage0, full0, empty0, chunk, gtid, g, &a, nxt, N, S.pref);
