@@ -43,6 +43,9 @@ constexpr long long T32 = (long long)BM * BN * 4;            // dup-word tile
 // 3.346e13 vs 3.217e13 (the int16 tasks are twice as fast as int32 ones, so the
 // per-task cost the pairs halve weighs twice as much)
 constexpr bool kPair16Default = true;
+// ... from nb = 128 on: below, the pair queue's longer chain per round costs more than the halved
+// per-task overhead saves (n = 4096: 3.30 vs 2.64-2.71 ms; n = 8192: 18.2 vs 17.5 ms)
+constexpr int kPair16MinNb = 128;
 constexpr int SIG = 32, SCH = 64;
 static_assert(64 * BN * 2 <= STAGE_BYTES, "half an int16 C tile must fit one stage");
 
@@ -478,7 +481,7 @@ cudaError_t launch_fw_dataflow16(short* D, long long ld, int nb, void* work, lon
   a.done2 = f; f += nb;
   a.done3 = f; f += nb;
   // the two-round (pair) queue: APSP_DF16_PAIR=0/1 overrides the default (A/B)
-  int pairq = kPair16Default && nb >= 2;
+  int pairq = kPair16Default && nb >= kPair16MinNb;
   if (const char* ev = getenv("APSP_DF16_PAIR")) pairq = atoi(ev) != 0 && nb >= 2;
   a.pairq = pairq;
   a.npar = pairq ? 4 : 2;
