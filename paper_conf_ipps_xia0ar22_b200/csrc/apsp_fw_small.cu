@@ -137,14 +137,18 @@ static int small_variant() {
                                           : 0;
 }
 
-// parts per chain panel tile: 4 by default (measured, n = 1024: whole tasks 0.265 ms, 2 parts 0.248,
-// 4 parts 0.240; n = 2048 unchanged: DESIGN.md §5); APSP_SMALL_SPLIT=1|2|4 (tuning A/B)
-// (the fused segment-order queue only, variant 3; the tuning variants keep whole tasks)
-static int small_split_for(int variant) {
+// parts per chain panel tile, by size (measured, device time of 30 runs, three alternations,
+// profiles/r02_small_split_ab.txt / r02_small_split8.txt / r02_small_split16.txt):
+//   n = 1024 (nb 16): whole 0.265, 2 parts 0.248, 4 0.239, 8 0.230, 16 0.228 ms
+//   n = 1536 (nb 24): 4 parts 0.436, 8 0.428, 16 0.435 ms;  n = 2048 (nb 32): 4 0.750, 8 0.758, 16 0.778 ms
+// APSP_SMALL_SPLIT=1|2|4|8|16 overrides (tuning A/B); the fused segment-order queue only (variant 3)
+static int small_split_for(int variant, int nb) {
   if (variant != 3) return 1;
-  const char* e = getenv("APSP_SMALL_SPLIT");
-  const int v = e ? atoi(e) : 4;
-  return v == 1 || v == 2 ? v : 4;
+  if (const char* e = getenv("APSP_SMALL_SPLIT")) {
+    const int v = atoi(e);
+    return v == 1 || v == 2 || v == 4 || v == 8 || v == 16 ? v : 8;
+  }
+  return nb <= 16 ? 16 : nb <= 24 ? 8 : 4;
 }
 
 struct SmSlot {
@@ -457,11 +461,12 @@ __device__ __forceinline__ void st_vec(T* dst, const T* v) {
 // One part of a split chain panel task (see kPartShift): P2R(k; k,j) part q updates columns
 // [q*C, (q+1)*C) of A(k,j) (C = 64/split; A = D via the panel copy D^T, B = those columns of A(k,j));
 // P2C(k; i,k) part q updates rows [q*R, (q+1)*R) (A = those rows of A(i,k), transposed on load;
-// B = D). Thread (tx, ty) owns TR x TC outputs (TR * TC = 16 / split), 256 threads per part.
-template <typename T, bool COLS, int TR, int TC>
+// B = D). 256 threads in a GX x (256 / GX) grid; thread (tx, ty) owns TR x TC outputs.
+template <typename T, bool COLS, int TR, int TC, int GX = 16>
 __device__ __forceinline__ void small_part(const SmArgs<T>& a, const Task& tk, int q, T* As, T* Bs) {
-  constexpr int R = 16 * TR, CC = 16 * TC;  // part rows / columns
-  const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+  constexpr int GY = SNT / GX;
+  constexpr int R = GY * TR, CC = GX * TC;  // part rows / columns
+  const int tid = threadIdx.x, tx = tid % GX, ty = tid / GX;
   const int r_off = COLS ? 0 : q * R, c_off = COLS ? q * CC : 0;
   T* const C = a.D + (long long)tk.i * SB * a.ld + (long long)tk.j * SB;
   if (COLS) {  // As[kk][r] = D^T (whole), Bs[kk][c] = A(k,j)[kk][c_off + c]
@@ -541,10 +546,14 @@ __device__ __forceinline__ void small_part_any(const SmArgs<T>& a, const Task& t
   Task w = tk;
   w.type = base_of(tk.type);
   if (w.type == T_P2R) {
-    if (a.split == 4) small_part<T, true, 4, 1>(a, w, q, As, Bs);
+    if (a.split == 16) small_part<T, true, 1, 1, 4>(a, w, q, As, Bs);       // 64 rows x 4 columns
+    else if (a.split == 8) small_part<T, true, 2, 1, 8>(a, w, q, As, Bs);   // 64 rows x 8 columns
+    else if (a.split == 4) small_part<T, true, 4, 1>(a, w, q, As, Bs);
     else small_part<T, true, 4, 2>(a, w, q, As, Bs);
   } else {
-    if (a.split == 4) small_part<T, false, 1, 4>(a, w, q, As, Bs);
+    if (a.split == 16) small_part<T, false, 1, 1, 64>(a, w, q, As, Bs);     // 4 rows x 64 columns
+    else if (a.split == 8) small_part<T, false, 1, 2, 32>(a, w, q, As, Bs); // 8 rows x 64 columns
+    else if (a.split == 4) small_part<T, false, 1, 4>(a, w, q, As, Bs);
     else small_part<T, false, 2, 4>(a, w, q, As, Bs);
   }
 }
@@ -713,7 +722,7 @@ long long small_queue(int nb, long long delay, std::vector<int4>* q) {
   // tuning experiments only: APSP_SMALL_QUEUE=decode (the 128-tile kernel's segment order,
   // no fusion) or bl_nofuse (list order without fused entries); default: list order + F(k)
   const int variant = small_variant();
-  const int S = small_split_for(variant);
+  const int S = small_split_for(variant, nb);
   if (!q)  // the length alone (every launch asks for it): P1(k >= 1) lives inside F(k-1) when fused;
            // each round but the last has two chain panel tiles of S parts
     return (long long)nb * nb * nb - (variant == 1 || variant == 2 ? 0 : nb - 1) + 2ll * (S - 1) * (nb - 1);
@@ -804,8 +813,8 @@ static long long small_flag_bytes(int nb) {
   return ((2 + (long long)nb * nb + 2 + 4ll * nb + 2ll * nb + 2ll * nb + 1) * 4 + 15) / 16 * 16;
 }
 
-long long fw_small_work_bytes(int nb, size_t elem) {  // the queue is at most nb^3 + 6 (nb - 1) entries (split 4)
-  return small_pbuf_bytes(nb, elem) + small_flag_bytes(nb) + ((long long)nb * nb * nb + 6ll * nb) * (long long)sizeof(int4);
+long long fw_small_work_bytes(int nb, size_t elem) {  // the queue is at most nb^3 + 30 (nb - 1) entries (split 16)
+  return small_pbuf_bytes(nb, elem) + small_flag_bytes(nb) + ((long long)nb * nb * nb + 30ll * nb) * (long long)sizeof(int4);
 }
 
 template <typename T>
@@ -836,10 +845,10 @@ cudaError_t launch_fw_small(T* D, long long ld, int nb, void* work, int* negflag
   a.exitc = f; f += 1;
   a.flag_words = f - reinterpret_cast<int*>(fb);
   const int variant = small_variant();
-  a.split = small_split_for(variant);
+  a.split = small_split_for(variant, nb);
   // the queue in the work buffer was built for (variant, split, delay) = *queue_key (-1: none yet);
   // another configuration (tuning switches changed between launches) rebuilds it
-  const long long key = ((long long)variant << 60) | ((long long)a.split << 56) | (delay & ((1ll << 56) - 1));
+  const long long key = ((long long)variant << 58) | ((long long)a.split << 52) | (delay & ((1ll << 52) - 1));
   const bool queue_loaded = *queue_key == key;
   a.negflag = negflag;
   const char* ep = getenv("APSP_SMALL_EARLYPUB");  // A/B (tuning only)

@@ -102,7 +102,7 @@ def test_small_repeated_runs_and_reinit(lib):
             lib.apsp_reinit(h)
 
 
-@pytest.mark.parametrize("split", [1, 2, 4])
+@pytest.mark.parametrize("split", [1, 2, 4, 8, 16])
 def test_small_split_chain_tiles(lib, monkeypatch, split):
     """The chain panel tiles P2R(k; k,k+1) / P2C(k; k+1,k) run as `split` parts (column / row ranges,
     counted into their own flags): bit-exact at several tile counts, with negative weights, a
@@ -132,7 +132,7 @@ def test_small_queue_rebuilt_when_its_configuration_changes(lib, monkeypatch):
     g = gg.erdos_renyi(1000, 5000, seed=12)
     want = want_i32(g)
     with lib.apsp_init_from_csr(g.n, g.row_ptr, g.col, g.w, cfg=lib.apsp_config_default(device=0)) as h:
-        for split in ("4", "4", "1", "2", "2", "4"):
+        for split in ("8", "8", "1", "2", "2", "16", "4"):
             monkeypatch.setenv("APSP_SMALL_SPLIT", split)
             lib.apsp_reinit(h)
             lib.apsp_fw_blocked(h)

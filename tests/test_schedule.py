@@ -186,7 +186,7 @@ def expand_fused(q):
         else:
             yield (typ, k, i, j)
     for key, got in parts.items():
-        assert got == set(range(len(got))) and len(got) in (2, 4), (key, got)
+        assert got == set(range(len(got))) and len(got) in (2, 4, 8, 16), (key, got)
         yield key
 
 
@@ -198,7 +198,7 @@ def test_small_kernel_queue_complete_and_deadlock_free(lib, nb, delay):
     in-order drain with the kernel's exact waits (a fused entry waits for both halves' dependencies)."""
     q = lib.apsp_debug_queue(nb, -1, 0, delay)
     assert sorted(expand_fused(q)) == sorted(expected_tasks(nb))
-    S = 4  # default parts per chain panel tile (APSP_SMALL_SPLIT)
+    S = 16 if nb <= 16 else 8 if nb <= 24 else 4  # default parts per chain panel tile (small_split_for)
     assert len(q) == nb ** 3 - (nb - 1) + 2 * (S - 1) * (nb - 1)
     split = [tuple(t) for t in q.tolist() if t[0] >= 1 << PART_SHIFT]
     assert sorted(split) == sorted((b + ((p + 1) << PART_SHIFT), k, i, j) for k in range(nb - 1) for p in range(S)
@@ -211,7 +211,7 @@ def test_small_kernel_queue_complete_and_deadlock_free(lib, nb, delay):
         assert tuple(q[1 + n0].tolist()) == (P3P1, 0, 1, 1)
 
 
-@pytest.mark.parametrize("split,nb", [(1, 5), (2, 2), (2, 7), (2, 16), (4, 3)])
+@pytest.mark.parametrize("split,nb", [(1, 5), (2, 2), (2, 7), (2, 16), (4, 3), (4, 16), (16, 2), (16, 9)])
 def test_small_kernel_queue_split_parts(lib, monkeypatch, split, nb):
     """APSP_SMALL_SPLIT: the chain panel tiles P2R(k; k,k+1) / P2C(k; k+1,k) in 1 (whole) or 4 parts;
     the queue still holds every task once and drains under the kernel's waits."""
