@@ -23,7 +23,8 @@
 //     finishes its task before taking the next cannot deadlock (a critical-path list
 //     order is kept as a tuning variant: measured slower);
 //   * the two panel tiles next to the diagonal, P2R(k; k,k+1) and P2C(k; k+1,k), which
-//     every round's chain waits for, run as 4 parts on 4 CTAs (column / row ranges);
+//     every round's chain waits for, run as 16, 8 or 4 parts on as many CTAs (column / row
+//     ranges; small_split_for);
 //   * F(k) fuses P3(k; k+1,k+1) with P1(k+1): the CTA that updates the next
 //     diagonal tile closes it in registers right away (one flag hop and one
 //     tile load less on the chain of every round);
