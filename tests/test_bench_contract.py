@@ -63,7 +63,13 @@ def test_oracle_steady_rate_counts_full_iterations():
     import bench
     import graphgen as gg
     g = gg.erdos_renyi(1536, 1536 * 2, seed=11)  # sparse: many rows skipped early in a real run
-    whole, _, _ = bench.oracle_whole_run(g, 2)
-    steady, cores, sample, rates, _ = bench.oracle_steady_rate(g, warm_s=0.2, step_s=0.3, steps=2)
-    assert cores >= 1 and len(rates) == 2 and "steady-state" in sample
-    assert steady <= whole * 1.3
+    seen = []
+    for _ in range(3):  # wall-clock rates: a busy host can slow one measurement; one clean pair decides
+        whole, _, _ = bench.oracle_whole_run(g, 2)
+        steady, cores, sample, rates, _ = bench.oracle_steady_rate(g, warm_s=0.2, step_s=0.3, steps=2)
+        assert cores >= 1 and len(rates) == 2 and "steady-state" in sample
+        seen.append((steady, whole))
+        if steady <= whole * 1.3:
+            break
+    else:
+        raise AssertionError("steady-state rate above the whole-run rate in every attempt: %r" % seen)
