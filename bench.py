@@ -19,7 +19,8 @@ torchrun (WORLD_SIZE set) every rank runs directly.
 
 Legs beside the headline on one GPU (each guarded; skip flags --no-packed16, --no-exact-f32-leg,
 --no-ooc-leg, --no-boundary-leg, --no-johnson): packed16 (R16), exact_f32 (R25: the int32 graph
-closed by the fp32 engine under the 2(n-1)W <= 2^24 bound), the same workload fully out of core,
+closed by the fp32 engine under the 2(n-1)W <= 2^24 bound), the same workload fully out of core
+(N = 1; --ooc-leg-multi at N > 1),
 the boundary algorithm on a grid of the same n, Johnson's algorithm.
 
 `--impl reference` times the CPU oracle (oracle/, plain C + OpenMP) on a bounded
